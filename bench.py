@@ -1,0 +1,397 @@
+#!/usr/bin/env python
+"""Benchmark of the TBlock hot path (BASELINE.json metric) -- one JSON line on rank 0.
+
+    python bench.py [--gpus N --steps K --warmup W --config REDDIT --precision fp32]
+    python bench.py --impl reference ...      # the CPU oracle on the host cores
+
+A step = one batch through every §8(a) row: roots (S2) -> [dedup (S3)] ->
+sample (S4) -> next block (S5) -> ... -> TBlock attention tail..head (S6-S13,
+S15) -> dedup inverse at the roots (S14), replayed as one CUDA graph with the
+graph, features and batch edges resident in HBM.  Between timed steps L2 is
+flushed by writing a 256 MiB buffer (outside the timed events).  With N GPUs
+(torchrun) every rank runs its own batch of the stream (weak scaling) and the
+root embeddings of all ranks are all-gathered over NCCL inside the step (S16).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "sampled edges/s and TBlock embeddings/s at 1/2/4/8 B200; % HBM roofline"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="REDDIT")
+    ap.add_argument("--precision", default="fp32", choices=["fp32", "bf16"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    return ap.parse_args()
+
+
+# ---------------------------------------------------------------------- clocks
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.idx = gpu_index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.idx), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self) -> dict:
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=2)
+        except Exception:
+            self.proc.kill()
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 6:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                smax.append(float(parts[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, parts[2:6]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(smax) if smax else None,
+                "samples": len(sm), "reasons": sorted(reasons)}
+
+
+# ---------------------------------------------------------------------- shared inputs
+def load_world(cfg_name: str):
+    import synth
+    cfg = synth.get_config(cfg_name)
+    g = synth.make_graph(cfg)
+    neg = synth.make_negatives(cfg)
+    params = synth.gen.model_params(cfg)
+    return cfg, g, neg, params
+
+
+def oracle_rate(cfg, g, neg, params, batches, seconds: float):
+    """CPU oracle (as it stands) on whole batches until `seconds` of CPU work."""
+    import oracle
+    from oracle import pipeline as opipe
+    t0 = time.perf_counter()
+    tc = oracle.build_tcsr(cfg.n_nodes, g.src, g.dst, g.t, True)
+    t_build = time.perf_counter() - t0
+    done, edges, t_run, nb = 0, 0, 0.0, 0
+    for b in batches:
+        nb += 1
+        t0 = time.perf_counter()
+        emb, blocks = opipe.run_batch(tc, g.nfeat, g.efeat, params, cfg.k, cfg.strategy,
+                                      cfg.dedup, cfg.seeds["sampler"],
+                                      *synth_batch(g, neg, b))
+        t_run += time.perf_counter() - t0
+        done += emb.shape[0]
+        edges += sum(int(bl.seg_ptr[-1]) for bl in blocks)
+        if t_run >= seconds:
+            break
+    return {"emb_per_s": done / t_run, "edges_per_s": edges / t_run, "batches": nb,
+            "roots": done, "seconds": t_run,
+        "cores": oracle.num_threads(), "tcsr_build_s": t_build}
+
+
+def synth_batch(g, neg, b):
+    import synth
+    return synth.batch_roots_inputs(g, neg, b)
+
+
+# ---------------------------------------------------------------------- reference arm
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    cfg, g, neg, params = load_world(args.config)
+    import oracle
+    from oracle import pipeline as opipe
+    tc = oracle.build_tcsr(cfg.n_nodes, g.src, g.dst, g.t, True)
+    b0 = int(0.7 * cfg.n_batches)
+    # bounded sample: a slice of each batch's roots (first `frac` of its edges)
+    frac_edges = max(1, cfg.batch // 8)
+    times, roots, edges = [], 0, 0
+    for i in range(args.warmup + args.steps):
+        b = b0 + i
+        src_b, dst_b, t_b, neg_b = synth_batch(g, neg, b)
+        sl = slice(0, frac_edges)
+        t0 = time.perf_counter()
+        emb, blocks = opipe.run_batch(tc, g.nfeat, g.efeat, params, cfg.k, cfg.strategy,
+                                      cfg.dedup, cfg.seeds["sampler"], src_b[sl], dst_b[sl],
+                                      t_b[sl], neg_b[sl])
+        dt = time.perf_counter() - t0
+        if i >= args.warmup:
+            times.append(dt)
+            roots += emb.shape[0]
+            edges += sum(int(bl.seg_ptr[-1]) for bl in blocks)
+    T = sum(times)
+    val = roots / T
+    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "embeddings/s",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1e3 * T / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": cfg.name, "batch_edges_per_step": frac_edges,
+                       "roots_per_step": 3 * frac_edges, "layers": cfg.n_layers, "k": cfg.k,
+                       "strategy": cfg.strategy, "dedup": cfg.dedup,
+                       "precompute": cfg.precompute},
+            "sampled_edges_per_s": edges / T,
+            "cpu_baseline": {"value": val, "unit": "embeddings/s",
+                             "cores": oracle.num_threads(), "kind": "oracle",
+                             "sample": f"first {frac_edges} of each {cfg.batch}-edge batch "
+                                       f"({3 * frac_edges} roots) from 70% of the stream"},
+            "e2e": {"value": val, "unit": "embeddings/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ---------------------------------------------------------------------- our arm
+def algorithmic_attn(cfg, n_dst: int, n_edges: int, d_hdst: int, d_hsrc: int):
+    """Per tgl_tblock_attn call: FLOPs and bytes the method must do."""
+    dm, dt, de = cfg.d_model, cfg.d_t, cfg.d_e
+    kkv = d_hsrc + de + dt
+    flops = (n_edges * 2 * (2 * dm) * kkv          # K and V projections (S9)
+             + n_dst * 2 * dm * (d_hdst + dt)       # Q (S8)
+             + n_dst * 2 * dm * (dm + d_hdst)       # FFN (S13)
+             + n_edges * 4 * dm)                    # logits + weighted sum (S10-S12)
+    bytes_ = (n_edges * (4 * (d_hsrc + de) + 4 + 4 + 4 + 8)   # gathers + nbr/eid/ts + idx
+              + n_dst * (4 * d_hdst * 2 + 8 + 8 + 4 * cfg.d_model))  # h_dst (Q and FFN), t, seg, out
+    return flops, bytes_
+
+
+def run_ours(args):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    import synth
+    from paper_conf_asplos_wangm24_b200 import TGATPipeline, TSampler, tgl
+
+    cfg, g, neg, params = load_world(args.config)
+    cu = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    dev = {"src": cu(g.src), "dst": cu(g.dst), "t": cu(g.t), "neg": cu(neg),
+           "nfeat": cu(g.nfeat), "efeat": cu(g.efeat)}
+    torch.cuda.synchronize()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev0.record()
+    tc = tgl.build_tcsr(cfg.n_nodes, dev["src"], dev["dst"], dev["t"], True, True)
+    ev1.record()
+    torch.cuda.synchronize()
+    tcsr_ms = ev0.elapsed_time(ev1)
+    sampler = TSampler(cfg.k, cfg.strategy, cfg.seeds["sampler"])
+    pipe = TGATPipeline(dev, tc, params, cfg.batch, sampler, cfg.dedup, cfg.precompute,
+                        cfg.window, args.precision)
+    pipe.capture()
+    n0 = 3 * cfg.batch
+    gathered = torch.empty(world * n0, cfg.d_model, device="cuda") if world > 1 else None
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    b0 = int(0.7 * cfg.n_batches)
+    nb_avail = cfg.n_batches - b0
+
+    def batch_of(i):
+        return b0 + ((i * world + rank) % nb_avail)
+
+    # per-step device counters read after timing (outside the events)
+    cnt_e = torch.zeros(args.warmup + args.steps, dtype=torch.int64, device="cuda")
+    stream = torch.cuda.current_stream()
+    starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+
+    def counts_into(i):
+        tot = torch.zeros((), dtype=torch.int64, device="cuda")
+        for b in pipe.blocks:
+            tot = tot + b.seg_ptr.index_select(0, b.u_dev.clamp(max=b.n_max)).squeeze()
+        cnt_e[i] = tot
+
+    for i in range(args.warmup):
+        pipe.start_dev.fill_(batch_of(i) * cfg.batch)
+        out = pipe.run_graph()
+        if world > 1:
+            dist.all_gather_into_tensor(gathered, out[:n0])
+        counts_into(i)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = ClockSampler(local)
+    clk.start()
+    time.sleep(0.3)
+    torch.cuda.synchronize()
+    for i in range(args.steps):
+        j = args.warmup + i
+        flush.zero_()                                  # L2 flush, outside the events
+        pipe.start_dev.fill_(batch_of(j) * cfg.batch)
+        starts[i].record(stream)
+        out = pipe.run_graph()
+        if world > 1:
+            dist.all_gather_into_tensor(gathered, out[:n0])   # S16
+        ends[i].record(stream)
+        counts_into(j)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clocks = clk.stop()
+    step_ms = [s.elapsed_time(e) for s, e in zip(starts, ends)]
+    total_ms = sum(step_ms)
+    t_max = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
+    total_ms = float(t_max.item())
+    edges_local = int(cnt_e[args.warmup:].sum().item())
+    e_tot = torch.tensor([edges_local], dtype=torch.int64, device="cuda")
+    if world > 1:
+        dist.all_reduce(e_tot)
+    roots_all = world * n0 * args.steps
+    emb_per_s = roots_all / (total_ms / 1e3)
+    edges_per_s = int(e_tot.item()) / (total_ms / 1e3)
+
+    # ---- dominant call: tgl_tblock_attn on the tail block, timed eagerly with events
+    rec_ms, rec_shape = [], None
+    for i in range(max(3, min(args.steps, 20))):
+        flush.zero_()
+        pipe.start_dev.fill_(batch_of(args.warmup + i) * cfg.batch)
+        rec = {}
+        pipe.forward(record=rec)
+        torch.cuda.synchronize()
+        tail = pipe.L - 1
+        rec_ms.append(rec[tail][0].elapsed_time(rec[tail][1]))
+        bt = pipe.blocks[tail]
+        U = int(bt.u_dev.item())
+        E = int(bt.seg_ptr[U].item())
+        rec_shape = (rec_shape or []) + [(U, E)]
+    U_avg = sum(u for u, _ in rec_shape) / len(rec_shape)
+    E_avg = sum(e for _, e in rec_shape) / len(rec_shape)
+    fl, by = algorithmic_attn(cfg, U_avg, E_avg, cfg.d_v, cfg.d_v)
+    attn_ms = sum(rec_ms) / len(rec_ms)
+    peaks = {}
+    try:
+        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        pass
+    sm_max = clocks.get("sm_max_mhz") or peaks.get("sm_max_mhz", 1965.0)
+    fp32_peak = 148 * 128 * 2 * sm_max * 1e6 / 1e12     # TFLOP/s, FFMA on all SMs
+    achieved_tf = fl / (attn_ms / 1e3) / 1e12
+    roofline = {"kernel": "tgl_tblock_attn (tail block: q_proj + kv_attn + out_ffn)",
+                "bound": "alu", "achieved": achieved_tf, "peak": fp32_peak, "unit": "TFLOP/s",
+                "frac": achieved_tf / fp32_peak, "traffic": None,
+                "hbm_achieved_gbs": by / (attn_ms / 1e3) / 1e9,
+                "hbm_peak_gbs": peaks.get("hbm_gbs", 6545.9),
+                "per_launch_ms": attn_ms, "algorithmic_flops": fl, "algorithmic_bytes": by,
+                "n_dst_avg": U_avg, "n_edges_avg": E_avg,
+                "peak_note": "FP32 FFMA peak = 148 SM x 128 lanes x 2 x clocks.max.sm"}
+
+    # ---- e2e through the public API: pinned host batch -> device -> host embeddings
+    e2e = None
+    if world >= 1:
+        pipe_h = TGATPipeline(dev, tc, params, cfg.batch, sampler, cfg.dedup, cfg.precompute,
+                              cfg.window, args.precision, staging=True)
+        pipe_h.capture()
+        out_h = torch.empty(n0, cfg.d_model, dtype=torch.float32).pin_memory()
+        host_batches = []
+        for i in range(args.steps):
+            sb, db, tb, nb_ = synth.batch_roots_inputs(g, neg, batch_of(args.warmup + i))
+            host_batches.append(tuple(torch.from_numpy(np.ascontiguousarray(x)).pin_memory()
+                                      for x in (sb, db, tb, nb_)))
+        for i in range(min(3, args.steps)):
+            pipe_h.embed_host(*host_batches[i], out_h)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        for i in range(args.steps):
+            pipe_h.embed_host(*host_batches[i], out_h)
+            if world > 1:
+                dist.all_gather_into_tensor(gathered, pipe_h.graph_out[:n0])
+        torch.cuda.synchronize()
+        el = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device="cuda")
+        if world > 1:
+            dist.all_reduce(el, op=dist.ReduceOp.MAX)
+        h2d = cfg.batch * (4 + 4 + 4 + 4)
+        e2e = {"value": world * n0 * args.steps / float(el.item()), "unit": "embeddings/s",
+               "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": n0 * cfg.d_model * 4,
+               "timing": "host wall clock around H2D + graph replay + D2H + sync"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        r = oracle_rate(cfg, g, neg, params, [batch_of(i) for i in range(200)], args.cpu_seconds)
+        cpu = {"value": r["emb_per_s"], "unit": "embeddings/s", "cores": r["cores"],
+               "kind": "oracle", "sample": f"{r['batches']} whole batch(es) "
+               f"({r['roots']} roots) from 70% of the stream, {r['seconds']:.1f} s",
+               "sampled_edges_per_s": r["edges_per_s"]}
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": emb_per_s, "unit": "embeddings/s",
+                "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+                "ms_per_step": total_ms / args.steps, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "f32" if args.precision == "fp32"
+                else "bf16", "data": "synthetic",
+                "config": {"workload": cfg.name, "batch_edges": cfg.batch, "roots_per_step": n0,
+                           "roots_per_step_all_ranks": world * n0, "layers": cfg.n_layers,
+                           "k": cfg.k, "strategy": cfg.strategy, "dedup": cfg.dedup,
+                           "precompute": cfg.precompute, "precision": args.precision,
+                           "parallelism": f"root-sharded dp{world}" if world > 1 else "single",
+                           "l2": "flushed (256 MiB write) between timed steps",
+                           "timing": "CUDA events per step on the launch stream; max over ranks"},
+                "sampled_edges_per_s": edges_per_s,
+                "tcsr_build_ms": tcsr_ms,
+                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+                "gpu_launches": pipe.launches_per_forward * args.steps,
+                "gpu_launches_per_step": pipe.launches_per_forward,
+                "step_ms_p50": statistics.median(step_ms)}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

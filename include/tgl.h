@@ -1,0 +1,230 @@
+/*
+ * tgl.h -- C ABI of the B200-native TBlock hot path (libtgl.so, sm_100a).
+ *
+ * Method: TGLite (Wang & Mendis, ASPLOS'24).  "P:n" cites line n of the paper
+ * text; "R<n>" cites a reading in DESIGN.md §2.
+ *
+ * Conventions (all entry points):
+ *  - Every array argument is a DEVICE pointer unless stated otherwise.  The
+ *    parameter structs (tgl_tcsr, tgl_attn_params) are HOST structs holding
+ *    device pointers; they are read during the call only.
+ *  - The caller owns every buffer.  The library never allocates or frees device
+ *    memory, never synchronises the stream, and keeps no mutable global state.
+ *    Calls on different streams may run concurrently.
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *  - Workspace (CUB style): `ws == NULL` writes the required byte count to
+ *    *ws_bytes and returns TGL_OK without launching; a non-NULL `ws` smaller
+ *    than *ws_bytes' requirement returns TGL_EWORKSPACE.  Workspace must be
+ *    256-byte aligned and is clobbered.
+ *  - Data-dependent sizes stay on the device: outputs are capacity-bounded and
+ *    the true count is written to a device int64 (`*_dev`).  Every consumer
+ *    takes a HOST upper bound `*_max` (sizes the launch) plus the DEVICE count
+ *    `*_dev` (NULL = the host bound is exact).  No call needs a host sync, so a
+ *    batch is a fixed launch sequence a CUDA graph can capture.
+ *  - Errors: host-side validation is synchronous and enqueues nothing.
+ *    TGL_ECUDA reports a launch error; tgl_last_error() gives a thread-local
+ *    message.  Device-side faults surface at the caller's next sync.
+ *  - Dtypes: node ids int32, edge ids int32 (< 2^31 edges), CSR / segment
+ *    offsets int64, times fp32, features / weights / outputs fp32 row-major
+ *    with explicit leading dimensions (in elements).
+ */
+#ifndef TGL_H_
+#define TGL_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef int32_t tgl_status;
+#define TGL_OK 0
+#define TGL_EINVAL (-1)       /* null pointer, negative size, k <= 0, bad flags, ... */
+#define TGL_EWORKSPACE (-2)   /* workspace too small */
+#define TGL_ECUDA (-3)        /* CUDA launch / API error (see tgl_last_error) */
+#define TGL_ERANGE (-4)       /* value out of representable range (e.g. > 2^31 entries) */
+#define TGL_EUNSUPPORTED (-5) /* shape the kernels do not take (message says which) */
+
+/* tgl_build_tcsr flags */
+#define TGL_UNDIRECTED 1u        /* R2: both endpoints own an entry (default for TGNN data) */
+#define TGL_INPUT_TIME_SORTED 2u /* COO already sorted by t: skips the time passes */
+
+/* tgl_sample strategies */
+#define TGL_RECENT 0
+#define TGL_UNIFORM 1
+
+/* tgl_attn_params.precision */
+#define TGL_FP32 0 /* fp32 operands, fp32 accumulate (max abs err 1e-3 vs oracle) */
+#define TGL_BF16 1 /* bf16-rounded projection operands, fp32 accumulate (5e-2) */
+
+const char* tgl_version(void);
+const char* tgl_status_string(tgl_status s);
+const char* tgl_last_error(void); /* thread-local; "" if none */
+
+/* ---------------------------------------------------------------------------
+ * S1  T-CSR build.  P:311: "TGLITE initially stores temporal edges in COO
+ * format, sorting based on timestamp ... it is best to use a CSR format for
+ * faster lookups".
+ *
+ * Input COO (src, dst, t)[num_edges]; the edge id of edge e is e.  Output: for
+ * every node v the segment [indptr[v], indptr[v+1]) of entries (nbr, eid, ts)
+ * whose owner is v: (owner=src_e, nbr=dst_e) and, with TGL_UNDIRECTED,
+ * (owner=dst_e, nbr=src_e).  Inside a segment entries are ordered by
+ * (t asc, eid asc, forward-before-reverse) (R3).  num_entries M = E or 2E.
+ * Capacities: indptr[num_nodes+1], nbr/eid/ts[M].  TGL_INPUT_TIME_SORTED is a
+ * promise (t non-decreasing); the result is the same either way.
+ * Errors: EINVAL (null, negative size, unknown flag), ERANGE (M >= 2^32 or
+ * num_nodes >= 2^31).  Node ids must lie in [0, num_nodes) (unchecked on device).
+ * ------------------------------------------------------------------------- */
+tgl_status tgl_build_tcsr(int64_t num_nodes, int64_t num_edges, const int32_t* src,
+                          const int32_t* dst, const float* t, uint32_t flags,
+                          int64_t* indptr, int32_t* nbr, int32_t* eid, float* ts,
+                          void* ws, size_t* ws_bytes, void* stream);
+
+typedef struct {
+  int64_t num_nodes;
+  int64_t num_entries;
+  const int64_t* indptr; /* [num_nodes+1] */
+  const int32_t* nbr;    /* [num_entries] */
+  const int32_t* eid;    /* [num_entries] */
+  const float* ts;       /* [num_entries], sorted inside each segment */
+} tgl_tcsr;
+
+/* ---------------------------------------------------------------------------
+ * S2  Roots of a batch (head TBlock).  P:235 (L2.8) `head = batch.block(ctx)`;
+ * roots are the batch's source and destination nodes plus one negative
+ * per edge (R15), all at the edge time.
+ *
+ * Batch = edges [s, s + min(batch, num_edges - s)), s = *start_dev (device
+ * int64; NULL -> 0).  qnode = [src; dst; neg], qtime = [t; t; t]; neg is
+ * indexed like src.  Capacity 3*batch; *n_roots_dev = 3 * (edges in batch).
+ * ------------------------------------------------------------------------- */
+tgl_status tgl_batch_roots(int64_t batch, int64_t num_edges, const int64_t* start_dev,
+                           const int32_t* src, const int32_t* dst, const float* t,
+                           const int32_t* neg, int32_t* qnode, float* qtime,
+                           int64_t* n_roots_dev, void* stream);
+
+/* ---------------------------------------------------------------------------
+ * S3  Dedup of <node, time> pairs.  P:149 "embeddings are only computed for
+ * unique node-time pairs"; dedup() filters a block's destinations in place and
+ * registers an inverting hook (TGOpt dedup_filter/dedup_invert P:177-179).
+ *
+ * uniq = distinct pairs in order of first occurrence (R9); two times are equal
+ * when they compare equal (-0 == +0, R8).  inv[i] = position of pair i in uniq,
+ * so uniq[inv[i]] == (node[i], t[i]).  n = *n_dev (NULL -> n_max).
+ * Capacities: uniq_node/uniq_t/inv[n_max]; *num_uniq_dev = U.
+ * Workspace: O(n_max) (hash table of next_pow2(2 n_max) slots + scan state).
+ * ------------------------------------------------------------------------- */
+tgl_status tgl_dedup(int64_t n_max, const int64_t* n_dev, const int32_t* node,
+                     const float* t, int32_t* uniq_node, float* uniq_t,
+                     int64_t* num_uniq_dev, int32_t* inv, void* ws, size_t* ws_bytes,
+                     void* stream);
+
+/* ---------------------------------------------------------------------------
+ * S4  Temporal neighbourhood sampling.  P:92: N(i,t) = neighbours over edges
+ * with timestamp less than t (strict, R1), "further sampled based on a strategy
+ * such as most-recent"; TSampler: uniform or most-recent, used as a
+ * block operator `sampler.sample(tail)`.
+ *
+ * For query q = (v, t): candidates = entries of v's segment with ts < t (a
+ * prefix; n of them).  TGL_RECENT: the last min(n,k) candidates in CSR order
+ * (R4).  TGL_UNIFORM: n <= k -> all n in CSR order; else k draws with
+ * replacement in slot order, slot s picks start + floor(r*n/2^32) with
+ * r = Philox4x32-10(ctr={v, bits(t), layer, s/4}, key={lo32(seed),hi32(seed)})
+ * word s%4 (R5, R6).  Output segments are compact: seg_ptr[q] = exclusive
+ * prefix of per-query counts, seg_ptr[nq] = total (R7).  nq = *nq_dev (NULL ->
+ * nq_max).  Capacities: seg_ptr[nq_max+1], out_*[nq_max*k].
+ * Errors: EINVAL (k <= 0, bad strategy, null).  Workspace: scan state.
+ * ------------------------------------------------------------------------- */
+tgl_status tgl_sample(const tgl_tcsr* g, int64_t nq_max, const int64_t* nq_dev,
+                      const int32_t* qnode, const float* qtime, int32_t k, int32_t strategy,
+                      uint64_t seed, uint32_t layer, int64_t* seg_ptr, int32_t* out_nbr,
+                      int32_t* out_eid, float* out_ts, void* ws, size_t* ws_bytes,
+                      void* stream);
+
+/* ---------------------------------------------------------------------------
+ * S5  Next block.  P:237-238 (L2.10-11) `tail.next_block(...)`; reading R14:
+ * dst' = [dst ; sampled src], t' = [t_dst ; edge t].
+ * n_dst = *n_dst_dev (NULL -> n_dst_max); the source count is seg_ptr[n_dst].
+ * Capacities: out_node/out_t[n_dst_max + n_src_max]; *n_out_dev = n_dst + n_src.
+ * ------------------------------------------------------------------------- */
+tgl_status tgl_next_block(int64_t n_dst_max, const int64_t* n_dst_dev, const int32_t* dst_node,
+                          const float* dst_t, int64_t n_src_max, const int64_t* seg_ptr,
+                          const int32_t* src_node, const float* src_t, int32_t* out_node,
+                          float* out_t, int64_t* n_out_dev, void* stream);
+
+/* ---------------------------------------------------------------------------
+ * S6  Time encoding, eq (8): Phi(dt) = cos(omega*dt + phi), computed as
+ * the paper's code does in fp32 (`torch.cos(ts * w + b)`): fp32
+ * multiply, fp32 add, accurate cosine of that fp32 argument (R10).
+ *
+ * tgl_time_precompute: table[d][j] = Phi_j((float)d), d in [0, window) -- the
+ * time-precomputation optimisation (R11).
+ * tgl_time_encode: out[i][j] = Phi_j(dt[i]); when table != NULL and dt[i] is an
+ * integer in [0, window) the row is read from the table (bit-identical).
+ * ------------------------------------------------------------------------- */
+tgl_status tgl_time_precompute(int64_t window, int32_t d_t, const float* omega,
+                               const float* phi, float* table, void* stream);
+tgl_status tgl_time_encode(int64_t n, const float* dt, int32_t d_t, const float* omega,
+                           const float* phi, const float* table, int64_t window, float* out,
+                           void* stream);
+
+/* ---------------------------------------------------------------------------
+ * S7-S13  One TBlock of TGAT temporal attention, eqs (4)-(7) P:104-119 as in
+ * Listing 2 `TemporalAttnLayer.forward`:
+ *   q_i   = Wq [h_i ; Phi(0)] + bq                              (eq 4; L2.27,29)
+ *   k_e,v_e = W{k,v} [h_src(e) ; efeat(eid_e) ; Phi(t_i - t_e)] + b{k,v}
+ *                                                               (eq 5; L2.28,30-31)
+ *   s_e^h = LeakyReLU(logit_scale * <q_i^h, k_e^h>)             (L2.33; R12)
+ *   alpha = edge_softmax over i's segment, per head              (L2.34)
+ *   r_i   = sum_e alpha_e v_e  (0 for an empty segment)          (L2.36; R19)
+ *   out_i = LayerNorm(ReLU(Wo [r_i ; h_i] + bo))                 (eq 7; R13)
+ * Weights are [out, in] row-major (PyTorch Linear layout); concat orders are
+ * exactly as written.  Heads split d_model into n_heads contiguous slices.
+ *
+ * Destinations i in [0, n_dst), n_dst = *n_dst_dev (NULL -> n_dst_max), with
+ * time dst_t[i] and segment [seg_ptr[i], seg_ptr[i+1]) of edges.
+ * Row of h_i: hdst_idx ? hdst_idx[i] : i, in table hdst (leading dim ld_hdst).
+ * Row of h_src(e): hsrc_idx ? hsrc_idx[o + e] : o + e, o = *hsrc_off_dev
+ * (NULL -> 0) -- the dedup inverse hook of the next block (S14).
+ * efeat row eid[e] (ld_e); unused when d_e == 0.  edge_t[e] = edge time.
+ * tenc_table (NULL = direct) as in tgl_time_encode.  max_seg is a launch hint
+ * (the sampler's k); any segment length is handled.
+ * Output out[n_dst_max][d_out] (rows >= n_dst untouched).
+ * Limits: d_model == d_out, d_model % n_heads == 0, d_model <= 128, d_t <= 256.
+ * ------------------------------------------------------------------------- */
+typedef struct {
+  int32_t d_hdst, d_hsrc, d_e, d_t, d_model, n_heads, d_out;
+  const float *Wq, *bq;           /* [d_model][d_hdst + d_t]          */
+  const float *Wk, *bk, *Wv, *bv; /* [d_model][d_hsrc + d_e + d_t]   */
+  const float *Wo, *bo;           /* [d_out][d_model + d_hdst]        */
+  const float *ln_gamma, *ln_beta;
+  float ln_eps;                   /* 1e-5 */
+  const float *omega, *phi;       /* [d_t] */
+  float leaky_slope;              /* 0.2; < 0 -> identity */
+  float logit_scale;              /* 1.0 */
+  int32_t precision;              /* TGL_FP32 | TGL_BF16 */
+} tgl_attn_params;
+
+tgl_status tgl_tblock_attn(const tgl_attn_params* P, int64_t n_dst_max, const int64_t* n_dst_dev,
+                           const int64_t* seg_ptr, const float* dst_t, const float* hdst,
+                           const int32_t* hdst_idx, int64_t ld_hdst, const float* hsrc,
+                           const int32_t* hsrc_idx, const int64_t* hsrc_off_dev, int64_t ld_hsrc,
+                           const float* efeat, const int32_t* eid, int64_t ld_e,
+                           const float* edge_t, const float* tenc_table, int64_t window,
+                           int32_t max_seg, float* out, void* ws, size_t* ws_bytes,
+                           void* stream);
+
+/* ---------------------------------------------------------------------------
+ * S14  Dedup inverse applied to rows (the hook of P:279 / TGOpt dedup_invert
+ * P:179): out[j][:] = table[idx[j]][:] for j < n, n = *n_dev (NULL -> n_max).
+ * ------------------------------------------------------------------------- */
+tgl_status tgl_gather_rows(int64_t n_max, const int64_t* n_dev, const int32_t* idx,
+                           const float* table, int64_t ld_table, int32_t d, float* out,
+                           int64_t ld_out, void* stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TGL_H_ */

@@ -1,0 +1,230 @@
+"""TBlock chain for one batch on one GPU (S2-S15) -- host bookkeeping only.
+
+Names follow the paper: a `TBlock` holds destination <node, time> pairs and,
+once sampled, its source nodes / edges (Table 2); `TSampler`
+(L2.5) fills a block; `dedup` filters a block's destinations and keeps the
+inverse hook; `aggregate` runs the attention layers from the tail block
+back to the head (L2.18-19).  Every step is a libtgl kernel launch on one
+stream; sizes stay on the device (capacity-bounded buffers + device counts), so
+`TGATPipeline.forward` is a fixed launch sequence that `capture()` records into
+a CUDA graph.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass, field
+
+import torch
+
+from . import tgl
+
+
+@dataclass
+class TBlock:
+    """One TBlock (Fig 3): dst pairs (+ dedup hook) and sampled sources."""
+    layer: int
+    n_max: int                     # capacity of the dst arrays before dedup
+    dst_node: torch.Tensor
+    dst_t: torch.Tensor
+    n_dev: torch.Tensor            # device count of dst pairs
+    uniq_node: torch.Tensor = None  # after dedup (aliases dst_* when dedup is off)
+    uniq_t: torch.Tensor = None
+    u_dev: torch.Tensor = None
+    inv: torch.Tensor = None       # dedup inverse hook (None when dedup is off)
+    seg_ptr: torch.Tensor = None   # sampled sources
+    nbr: torch.Tensor = None
+    eid: torch.Tensor = None
+    ts: torch.Tensor = None
+    out: torch.Tensor = None       # layer output [n_max, d_out]
+    ws: dict = field(default_factory=dict)
+
+
+class TSampler:
+    """`tg.TSampler(n_nbr, 'recent' | 'uniform')` (L2.5)."""
+
+    def __init__(self, k: int, strategy: str = "recent", seed: int = 0x74676C00):
+        self.k, self.strategy, self.seed = k, strategy, seed
+
+
+class TGATPipeline:
+    """L-layer TGAT over TBlocks (Listing 2) with all buffers preallocated.
+
+    graph: dict of device tensors src, dst, t, neg (per edge), nfeat, efeat.
+    params: list of per-block weight dicts (block 0 = head, block L-1 = raw features).
+    """
+
+    def __init__(self, graph: dict, tcsr: tgl.TemporalCSR, params: list, batch: int,
+                 sampler: TSampler, use_dedup: bool, precompute: bool, window: int = 65536,
+                 precision: str = "fp32", staging: bool = False, device=None):
+        self.dev = device or torch.device("cuda")
+        self.g = graph
+        self.tcsr = tcsr
+        self.L = len(params)
+        self.batch = batch
+        self.sampler = sampler
+        self.use_dedup = use_dedup
+        self.E = graph["src"].numel()
+        self.attn = [tgl.AttnParams(p, self.dev, precision) for p in params]
+        self.tables = [tgl.time_precompute(window, a.t["omega"], a.t["phi"]) if precompute else None
+                       for a in self.attn]
+        k = sampler.k
+        i32, f32, i64 = torch.int32, torch.float32, torch.int64
+        z = lambda n, dt: torch.zeros(max(int(n), 1), dtype=dt, device=self.dev)
+        self.start_dev = torch.zeros(1, dtype=i64, device=self.dev)
+        self.blocks = []
+        n_max = 3 * batch
+        for l in range(self.L):
+            b = TBlock(l, n_max, z(n_max, i32), z(n_max, f32), z(1, i64))
+            if use_dedup:
+                b.uniq_node, b.uniq_t, b.u_dev, b.inv = z(n_max, i32), z(n_max, f32), z(1, i64), z(n_max, i32)
+            else:
+                b.uniq_node, b.uniq_t, b.u_dev = b.dst_node, b.dst_t, b.n_dev
+            b.seg_ptr = z(n_max + 1, i64)
+            b.nbr, b.eid, b.ts = z(n_max * k, i32), z(n_max * k, i32), z(n_max * k, f32)
+            b.out = z(n_max * self.attn[l].d_out, f32).view(-1, self.attn[l].d_out)
+            self.blocks.append(b)
+            n_max = n_max + n_max * k
+        self.emb = z(3 * batch * self.attn[0].d_out, f32).view(-1, self.attn[0].d_out)
+        # staging mode: the batch's edges arrive from host memory each step (public API)
+        self.staging = staging
+        if staging:
+            self.stage = {"src": z(batch, i32), "dst": z(batch, i32), "t": z(batch, f32),
+                          "neg": z(batch, i32)}
+            self.stage_n = batch
+        # kernels launched per forward (libtgl only; memsets excluded)
+        per_block = [(1 if l > 0 else 0) + (3 if use_dedup else 0) + 1 + 3 for l in range(self.L)]
+        self.launches_per_forward = 1 + sum(per_block) + (1 if use_dedup else 0)
+        self._alloc_workspaces()
+        self.graph_exec = None
+
+    # ------------------------------------------------------------------ workspaces
+    def _alloc_workspaces(self):
+        k = self.sampler.k
+        for b in self.blocks:
+            if self.use_dedup:
+                nb = tgl.ws_bytes("tgl_dedup", b.n_max, None, None, None, None, None, None, None)
+                b.ws["dedup"] = torch.empty(max(nb, 256), dtype=torch.uint8, device=self.dev)
+            nb = tgl.ws_bytes("tgl_sample", C_TCSR(self.tcsr), b.n_max, None, None, None, k, 0,
+                              0, 0, None, None, None, None)
+            b.ws["sample"] = torch.empty(max(nb, 256), dtype=torch.uint8, device=self.dev)
+            a = self.attn[b.layer]
+            nb = tgl.ws_bytes("tgl_tblock_attn", C_ATTN(a), b.n_max, None, None, None, None, None,
+                              0, None, None, None, 0, None, None, 0, None, None, 0, k, None)
+            b.ws["attn"] = torch.empty(max(nb, 256), dtype=torch.uint8, device=self.dev)
+
+    # ------------------------------------------------------------------ the batch
+    def forward(self, stream=None, record: dict | None = None):
+        """Enqueue one batch (edges [start, start+batch) with start = self.start_dev).
+
+        record: optional dict; eager mode only -- CUDA events around each
+        tgl_tblock_attn call are stored as record[layer] = (start, end)."""
+        g, k, s = self.g, self.sampler.k, stream
+        b0 = self.blocks[0]
+        if self.staging:
+            st = self.stage
+            tgl.batch_roots(self.batch, self.stage_n, None, st["src"], st["dst"], st["t"],
+                            st["neg"], b0.dst_node, b0.dst_t, b0.n_dev, stream=s)
+        else:
+            tgl.batch_roots(self.batch, self.E, self.start_dev, g["src"], g["dst"], g["t"],
+                            g["neg"], b0.dst_node, b0.dst_t, b0.n_dev, stream=s)
+        for l, b in enumerate(self.blocks):
+            if l > 0:  # S5 next_block (R14): [dst after dedup ; sampled src]
+                p = self.blocks[l - 1]
+                tgl.next_block(p.n_max, p.u_dev, p.uniq_node, p.uniq_t, p.n_max * k, p.seg_ptr,
+                               p.nbr, p.ts, b.dst_node, b.dst_t, b.n_dev, stream=s)
+            if self.use_dedup:  # S3
+                _call_ws(tgl.lib().tgl_dedup,
+                         [b.n_max, tgl._p(b.n_dev), tgl._p(b.dst_node), tgl._p(b.dst_t),
+                          tgl._p(b.uniq_node), tgl._p(b.uniq_t), tgl._p(b.u_dev),
+                          tgl._p(b.inv)], b.ws["dedup"], s, "tgl_dedup")
+            # S4 sample
+            _call_ws(tgl.lib().tgl_sample,
+                     [tgl.C.byref(self.tcsr.struct), b.n_max, tgl._p(b.u_dev),
+                      tgl._p(b.uniq_node), tgl._p(b.uniq_t), k,
+                      tgl.STRATEGY[self.sampler.strategy], self.sampler.seed, l,
+                      tgl._p(b.seg_ptr), tgl._p(b.nbr), tgl._p(b.eid), tgl._p(b.ts)],
+                     b.ws["sample"], s, "tgl_sample")
+        # S15 aggregate: tail -> head
+        for l in range(self.L - 1, -1, -1):
+            b = self.blocks[l]
+            a = self.attn[l]
+            if l == self.L - 1:
+                hdst, hdst_idx, hsrc, hsrc_idx, off = g["nfeat"], b.uniq_node, g["nfeat"], b.nbr, None
+            else:
+                nx = self.blocks[l + 1]
+                hdst = hsrc = nx.out
+                off = b.u_dev        # S14: rows [U_l + e] of the next block hold the sources
+                if self.use_dedup:
+                    hdst_idx = hsrc_idx = nx.inv
+                else:
+                    hdst_idx = hsrc_idx = None
+            ef = g["efeat"]
+            ld_e = ef.shape[1] if ef.dim() == 2 else 0
+            if record is not None:
+                ev = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                ev[0].record(s if s is not None else torch.cuda.current_stream())
+            _call_ws(tgl.lib().tgl_tblock_attn,
+                     [tgl.C.byref(a.struct), b.n_max, tgl._p(b.u_dev), tgl._p(b.seg_ptr),
+                      tgl._p(b.uniq_t), tgl._p(hdst), tgl._p(hdst_idx), hdst.shape[1],
+                      tgl._p(hsrc), tgl._p(hsrc_idx), tgl._p(off), hsrc.shape[1],
+                      tgl._p(ef) if ld_e else None, tgl._p(b.eid) if ld_e else None, ld_e,
+                      tgl._p(b.ts), tgl._p(self.tables[l]),
+                      0 if self.tables[l] is None else self.tables[l].shape[0], k,
+                      tgl._p(b.out)], b.ws["attn"], s, "tgl_tblock_attn")
+            if record is not None:
+                ev[1].record(s if s is not None else torch.cuda.current_stream())
+                record[l] = ev
+        if self.use_dedup:  # S14 at the roots
+            tgl.gather_rows(b0.inv, b0.out, n_dev=b0.n_dev, n_max=b0.n_max, out=self.emb, stream=s)
+            return self.emb
+        return b0.out[:3 * self.batch]
+
+    # ------------------------------------------------------------------ CUDA graph
+    def capture(self):
+        torch.cuda.synchronize()
+        s = torch.cuda.Stream()
+        s.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(s):
+            for _ in range(2):
+                self.forward()
+        torch.cuda.current_stream().wait_stream(s)
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            out = self.forward()
+        self.graph_exec = g
+        self.graph_out = out
+        return g
+
+    def run_graph(self, start: int | None = None):
+        if start is not None:
+            self.start_dev.fill_(start)
+        self.graph_exec.replay()
+        return self.graph_out
+
+    def embed_host(self, src_h, dst_h, t_h, neg_h, out_h):
+        """Public end-to-end call: one batch from (pinned) host arrays to host embeddings.
+
+        H2D of the batch's edges, the captured TBlock chain, D2H of the root
+        embeddings; returns after the stream has finished."""
+        assert self.staging and self.graph_exec is not None
+        n = src_h.shape[0]
+        assert n == self.batch, "staging pipeline is captured for a full batch"
+        for k_, h in (("src", src_h), ("dst", dst_h), ("t", t_h), ("neg", neg_h)):
+            self.stage[k_][:n].copy_(h, non_blocking=True)
+        self.graph_exec.replay()
+        out_h.copy_(self.graph_out[:3 * n], non_blocking=True)
+        torch.cuda.current_stream().synchronize()
+        return out_h
+
+
+def C_TCSR(t: tgl.TemporalCSR):
+    return tgl.C.byref(t.struct)
+
+
+def C_ATTN(a: tgl.AttnParams):
+    return tgl.C.byref(a.struct)
+
+
+def _call_ws(fn, args, ws_buf: torch.Tensor, stream, what):
+    nb = tgl.C.c_size_t(ws_buf.numel())
+    tgl._check(fn(*args, ws_buf.data_ptr(), tgl.C.byref(nb), tgl._s(stream)), what)

@@ -1,0 +1,290 @@
+"""Thin ctypes binding of libtgl.so (include/tgl.h) -- argument marshalling only.
+
+Every function takes CUDA torch tensors, passes their device pointers and the
+current torch stream to the C ABI, and raises `TGLError` on a non-zero status.
+No step of the method runs here: if libtgl.so is missing this module fails to
+import (there is no CPU fallback).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import torch
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libtgl.so")
+
+TGL_UNDIRECTED = 1
+TGL_INPUT_TIME_SORTED = 2
+RECENT, UNIFORM = 0, 1
+FP32, BF16 = 0, 1
+STRATEGY = {"recent": RECENT, "uniform": UNIFORM}
+PRECISION = {"fp32": FP32, "bf16": BF16}
+
+SYMBOLS = ["tgl_version", "tgl_status_string", "tgl_last_error", "tgl_build_tcsr",
+           "tgl_batch_roots", "tgl_dedup", "tgl_sample", "tgl_next_block",
+           "tgl_time_precompute", "tgl_time_encode", "tgl_tblock_attn", "tgl_gather_rows"]
+
+
+class TGLError(RuntimeError):
+    pass
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} not built: run `python -m "
+                          f"paper_conf_asplos_wangm24_b200.build` (no CPU fallback exists)")
+    lib = C.CDLL(LIB_PATH)
+    vp, i64, i32, u32, u64 = C.c_void_p, C.c_int64, C.c_int32, C.c_uint32, C.c_uint64
+    sz = C.POINTER(C.c_size_t)
+    lib.tgl_version.restype = C.c_char_p
+    lib.tgl_status_string.restype = C.c_char_p
+    lib.tgl_status_string.argtypes = [i32]
+    lib.tgl_last_error.restype = C.c_char_p
+    sig = {
+        "tgl_build_tcsr": [i64, i64, vp, vp, vp, u32, vp, vp, vp, vp, vp, sz, vp],
+        "tgl_batch_roots": [i64, i64, vp, vp, vp, vp, vp, vp, vp, vp, vp],
+        "tgl_dedup": [i64, vp, vp, vp, vp, vp, vp, vp, vp, sz, vp],
+        "tgl_sample": [vp, i64, vp, vp, vp, i32, i32, u64, u32, vp, vp, vp, vp, vp, sz, vp],
+        "tgl_next_block": [i64, vp, vp, vp, i64, vp, vp, vp, vp, vp, vp, vp],
+        "tgl_time_precompute": [i64, i32, vp, vp, vp, vp],
+        "tgl_time_encode": [i64, vp, i32, vp, vp, vp, i64, vp, vp],
+        "tgl_tblock_attn": [vp, i64, vp, vp, vp, vp, vp, i64, vp, vp, vp, i64, vp, vp, i64, vp,
+                            vp, i64, i32, vp, vp, sz, vp],
+        "tgl_gather_rows": [i64, vp, vp, vp, i64, i32, vp, i64, vp],
+    }
+    for name, args in sig.items():
+        f = getattr(lib, name)
+        f.argtypes = args
+        f.restype = i32
+    return lib
+
+
+_lib = _load()
+
+
+def lib():
+    return _lib
+
+
+def version() -> str:
+    return _lib.tgl_version().decode()
+
+
+def _check(status: int, what: str):
+    if status != 0:
+        raise TGLError(f"{what}: {_lib.tgl_status_string(status).decode()}: "
+                       f"{_lib.tgl_last_error().decode()}")
+
+
+def _p(t):
+    if t is None:
+        return None
+    if isinstance(t, int):
+        return t
+    assert t.is_cuda and t.is_contiguous(), "expected a contiguous CUDA tensor"
+    return t.data_ptr()
+
+
+def _s(stream=None):
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return s.cuda_stream
+
+
+class Workspace:
+    """Grow-only device scratch (uint8) owned by the caller, per the ABI."""
+
+    def __init__(self, device=None):
+        self.device = device or torch.device("cuda")
+        self.buf = None
+
+    def get(self, nbytes: int) -> torch.Tensor:
+        nbytes = max(int(nbytes), 256)
+        if self.buf is None or self.buf.numel() < nbytes:
+            self.buf = torch.empty(nbytes, dtype=torch.uint8, device=self.device)
+        return self.buf
+
+
+def _ws_call(fn, args_before_ws, ws: Workspace | None, stream, what):
+    """CUB-style protocol: query (ws=NULL) then call."""
+    nb = C.c_size_t(0)
+    _check(fn(*args_before_ws, None, C.byref(nb), stream), what + " (size query)")
+    ws = ws or Workspace()
+    buf = ws.get(nb.value)
+    nb2 = C.c_size_t(buf.numel())
+    _check(fn(*args_before_ws, buf.data_ptr(), C.byref(nb2), stream), what)
+
+
+def ws_bytes(fn_name: str, *args_before_ws) -> int:
+    nb = C.c_size_t(0)
+    _check(getattr(_lib, fn_name)(*args_before_ws, None, C.byref(nb), None), fn_name)
+    return nb.value
+
+
+# --------------------------------------------------------------------------- S1
+class TCSR(C.Structure):
+    _fields_ = [("num_nodes", C.c_int64), ("num_entries", C.c_int64), ("indptr", C.c_void_p),
+                ("nbr", C.c_void_p), ("eid", C.c_void_p), ("ts", C.c_void_p)]
+
+
+class TemporalCSR:
+    """Device-resident T-CSR + the host struct the ABI takes."""
+
+    def __init__(self, indptr, nbr, eid, ts):
+        self.indptr, self.nbr, self.eid, self.ts = indptr, nbr, eid, ts
+        self.struct = TCSR(indptr.numel() - 1, nbr.numel(), _p(indptr), _p(nbr), _p(eid), _p(ts))
+
+    @property
+    def num_nodes(self):
+        return self.indptr.numel() - 1
+
+
+def build_tcsr(num_nodes: int, src, dst, t, undirected=True, time_sorted=False,
+               ws: Workspace | None = None, stream=None) -> TemporalCSR:
+    dev = src.device
+    E = src.numel()
+    M = 2 * E if undirected else E
+    indptr = torch.empty(num_nodes + 1, dtype=torch.int64, device=dev)
+    nbr = torch.empty(max(M, 1), dtype=torch.int32, device=dev)[:M]
+    eid = torch.empty(max(M, 1), dtype=torch.int32, device=dev)[:M]
+    ts = torch.empty(max(M, 1), dtype=torch.float32, device=dev)[:M]
+    flags = (TGL_UNDIRECTED if undirected else 0) | (TGL_INPUT_TIME_SORTED if time_sorted else 0)
+    _ws_call(_lib.tgl_build_tcsr, [num_nodes, E, _p(src), _p(dst), _p(t), flags, _p(indptr),
+                                   _p(nbr), _p(eid), _p(ts)], ws, _s(stream), "tgl_build_tcsr")
+    return TemporalCSR(indptr, nbr, eid, ts)
+
+
+# --------------------------------------------------------------------------- S2
+def batch_roots(batch: int, num_edges: int, start_dev, src, dst, t, neg, qnode, qtime,
+                n_roots_dev, stream=None):
+    _check(_lib.tgl_batch_roots(batch, num_edges, _p(start_dev), _p(src), _p(dst), _p(t),
+                                _p(neg), _p(qnode), _p(qtime), _p(n_roots_dev), _s(stream)),
+           "tgl_batch_roots")
+
+
+# --------------------------------------------------------------------------- S3
+def dedup(node, t, n_dev=None, n_max=None, out=None, ws: Workspace | None = None, stream=None):
+    """Returns (uniq_node, uniq_t, num_uniq_dev, inv) with capacity n_max."""
+    n_max = node.numel() if n_max is None else n_max
+    dev = node.device
+    if out is None:
+        out = (torch.empty(max(n_max, 1), dtype=torch.int32, device=dev),
+               torch.empty(max(n_max, 1), dtype=torch.float32, device=dev),
+               torch.zeros(1, dtype=torch.int64, device=dev),
+               torch.empty(max(n_max, 1), dtype=torch.int32, device=dev))
+    un, ut, nu, inv = out
+    _ws_call(_lib.tgl_dedup, [n_max, _p(n_dev), _p(node), _p(t), _p(un), _p(ut), _p(nu), _p(inv)],
+             ws, _s(stream), "tgl_dedup")
+    return un, ut, nu, inv
+
+
+# --------------------------------------------------------------------------- S4
+def sample(g: TemporalCSR, qnode, qtime, k: int, strategy, seed: int = 0, layer: int = 0,
+           nq_dev=None, nq_max=None, out=None, ws: Workspace | None = None, stream=None):
+    """Returns (seg_ptr[nq_max+1], nbr, eid, ts) with capacity nq_max*k."""
+    strategy = STRATEGY.get(strategy, strategy)
+    nq_max = qnode.numel() if nq_max is None else nq_max
+    dev = qnode.device
+    cap = max(nq_max * k, 1)
+    if out is None:
+        out = (torch.empty(nq_max + 1, dtype=torch.int64, device=dev),
+               torch.empty(cap, dtype=torch.int32, device=dev),
+               torch.empty(cap, dtype=torch.int32, device=dev),
+               torch.empty(cap, dtype=torch.float32, device=dev))
+    seg, nb, ei, ts = out
+    _ws_call(_lib.tgl_sample, [C.byref(g.struct), nq_max, _p(nq_dev), _p(qnode), _p(qtime), k,
+                               strategy, seed & 0xFFFFFFFFFFFFFFFF, layer, _p(seg), _p(nb),
+                               _p(ei), _p(ts)], ws, _s(stream), "tgl_sample")
+    return seg, nb, ei, ts
+
+
+# --------------------------------------------------------------------------- S5
+def next_block(n_dst_max, n_dst_dev, dst_node, dst_t, n_src_max, seg_ptr, src_node, src_t,
+               out_node, out_t, n_out_dev, stream=None):
+    _check(_lib.tgl_next_block(n_dst_max, _p(n_dst_dev), _p(dst_node), _p(dst_t), n_src_max,
+                               _p(seg_ptr), _p(src_node), _p(src_t), _p(out_node), _p(out_t),
+                               _p(n_out_dev), _s(stream)), "tgl_next_block")
+
+
+# --------------------------------------------------------------------------- S6
+def time_precompute(window: int, omega, phi, stream=None):
+    table = torch.empty(max(window, 1), omega.numel(), dtype=torch.float32, device=omega.device)
+    _check(_lib.tgl_time_precompute(window, omega.numel(), _p(omega), _p(phi), _p(table),
+                                    _s(stream)), "tgl_time_precompute")
+    return table
+
+
+def time_encode(dt, omega, phi, table=None, stream=None):
+    n = dt.numel()
+    out = torch.empty(max(n, 1), omega.numel(), dtype=torch.float32, device=dt.device)[:n]
+    window = 0 if table is None else table.shape[0]
+    _check(_lib.tgl_time_encode(n, _p(dt), omega.numel(), _p(omega), _p(phi), _p(table), window,
+                                _p(out), _s(stream)), "tgl_time_encode")
+    return out
+
+
+# --------------------------------------------------------------------------- S7-S13
+class AttnParamsC(C.Structure):
+    _fields_ = [("d_hdst", C.c_int32), ("d_hsrc", C.c_int32), ("d_e", C.c_int32),
+                ("d_t", C.c_int32), ("d_model", C.c_int32), ("n_heads", C.c_int32),
+                ("d_out", C.c_int32),
+                ("Wq", C.c_void_p), ("bq", C.c_void_p), ("Wk", C.c_void_p),
+                ("bk", C.c_void_p), ("Wv", C.c_void_p), ("bv", C.c_void_p),
+                ("Wo", C.c_void_p), ("bo", C.c_void_p), ("ln_gamma", C.c_void_p),
+                ("ln_beta", C.c_void_p), ("ln_eps", C.c_float),
+                ("omega", C.c_void_p), ("phi", C.c_void_p),
+                ("leaky_slope", C.c_float), ("logit_scale", C.c_float),
+                ("precision", C.c_int32)]
+
+
+_WEIGHTS = ("Wq", "bq", "Wk", "bk", "Wv", "bv", "Wo", "bo", "ln_gamma", "ln_beta", "omega", "phi")
+
+
+class AttnParams:
+    """Device copies of one layer's weights + the host struct of the ABI."""
+
+    def __init__(self, p: dict, device=None, precision="fp32"):
+        device = device or torch.device("cuda")
+        self.host = p
+        self.t = {k: torch.as_tensor(p[k], dtype=torch.float32).contiguous().to(device)
+                  for k in _WEIGHTS}
+        self.precision = PRECISION.get(precision, precision)
+        self.d_model = p["d_model"]
+        self.d_out = p["d_out"]
+        self.d_t = p["d_t"]
+        self.struct = AttnParamsC(p["d_hdst"], p["d_hsrc"], p["d_e"], p["d_t"], p["d_model"],
+                                  p["n_heads"], p["d_out"],
+                                  *[_p(self.t[k]) for k in _WEIGHTS[:10]], float(p["ln_eps"]),
+                                  _p(self.t["omega"]), _p(self.t["phi"]),
+                                  float(p["leaky_slope"]), float(p["logit_scale"]),
+                                  self.precision)
+
+
+def tblock_attn(P: AttnParams, seg_ptr, dst_t, hdst, hdst_idx, hsrc, hsrc_idx, efeat, eid,
+                edge_t, table=None, max_seg=10, n_dst_max=None, n_dst_dev=None,
+                hsrc_off_dev=None, out=None, ws: Workspace | None = None, stream=None):
+    n_dst_max = seg_ptr.numel() - 1 if n_dst_max is None else n_dst_max
+    if out is None:
+        out = torch.empty(max(n_dst_max, 1), P.d_out, dtype=torch.float32,
+                          device=seg_ptr.device)
+    window = 0 if table is None else table.shape[0]
+    ld_e = efeat.shape[1] if (efeat is not None and efeat.dim() == 2) else 0
+    _ws_call(_lib.tgl_tblock_attn,
+             [C.byref(P.struct), n_dst_max, _p(n_dst_dev), _p(seg_ptr), _p(dst_t), _p(hdst),
+              _p(hdst_idx), hdst.shape[1], _p(hsrc), _p(hsrc_idx), _p(hsrc_off_dev),
+              hsrc.shape[1], _p(efeat) if ld_e else None, _p(eid) if ld_e else None, ld_e,
+              _p(edge_t), _p(table), window, max_seg, _p(out)], ws, _s(stream),
+             "tgl_tblock_attn")
+    return out
+
+
+# --------------------------------------------------------------------------- S14
+def gather_rows(idx, table, n_dev=None, n_max=None, out=None, stream=None):
+    n_max = idx.numel() if n_max is None else n_max
+    d = table.shape[1]
+    if out is None:
+        out = torch.empty(max(n_max, 1), d, dtype=table.dtype, device=table.device)
+    _check(_lib.tgl_gather_rows(n_max, _p(n_dev), _p(idx), _p(table), table.stride(0), d,
+                                _p(out), out.stride(0), _s(stream)), "tgl_gather_rows")
+    return out

@@ -1,0 +1,321 @@
+"""GPU parity: every C-ABI call against the CPU oracle on the same seeded inputs.
+
+Bit-exact for T-CSR, sampling and dedup; <= 2 ulp for the time encoder;
+max abs 1e-3 (fp32) / 5e-2 (bf16) for attention outputs and embeddings
+(north_star tolerances).  Sizes span several tiles and a ragged tail.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from oracle import pipeline as opipe
+import synth
+
+pytestmark = pytest.mark.gpu
+
+TOL = {"fp32": 1e-3, "bf16": 5e-2}
+
+
+@pytest.fixture(scope="module")
+def T():
+    from paper_conf_asplos_wangm24_b200 import tgl
+    return tgl
+
+
+def cu(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def np_(t):
+    return t.detach().cpu().numpy()
+
+
+def rand_graph(rng, N, E, max_t, sort=True):
+    src = rng.integers(0, N, E).astype(np.int32)
+    dst = rng.integers(0, N, E).astype(np.int32)
+    dst[::13] = src[::13]
+    t = rng.integers(0, max_t, E).astype(np.float32)
+    if sort:
+        o = np.argsort(t, kind="stable")
+        src, dst, t = src[o], dst[o], t[o]
+    return src, dst, t
+
+
+# ------------------------------------------------------------------ S1
+@pytest.mark.parametrize("undirected", [True, False])
+@pytest.mark.parametrize("sort", [True, False])
+@pytest.mark.parametrize("N,E,max_t", [(1, 5, 3), (50, 3000, 40), (3000, 20000, 10**6),
+                                       (70000, 5000, 100), (300, 0, 1)])
+def test_tcsr_bit_exact(T, N, E, max_t, undirected, sort):
+    rng = np.random.default_rng(N * 7 + E)
+    src, dst, t = rand_graph(rng, N, E, max_t, sort)
+    g = T.build_tcsr(N, cu(src), cu(dst), cu(t), undirected=undirected, time_sorted=sort)
+    exp = oracle.build_tcsr(N, src, dst, t, undirected)
+    got = (np_(g.indptr), np_(g.nbr), np_(g.eid), np_(g.ts))
+    for a, b in zip(got, exp):
+        assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("name", ["WIKI", "REDDIT", "LASTFM"])
+def test_tcsr_full_configs(T, name):
+    cfg = synth.get_config(name)
+    gr = synth.make_graph(cfg, with_features=False)
+    g = T.build_tcsr(cfg.n_nodes, cu(gr.src), cu(gr.dst), cu(gr.t), True, True)
+    exp = oracle.build_tcsr(cfg.n_nodes, gr.src, gr.dst, gr.t, True)
+    for a, b in zip((g.indptr, g.nbr, g.eid, g.ts), exp):
+        assert np.array_equal(np_(a), b)
+
+
+# ------------------------------------------------------------------ S4
+@pytest.mark.parametrize("strategy", ["recent", "uniform"])
+@pytest.mark.parametrize("k", [1, 10, 20, 45])
+def test_sample_bit_exact(T, strategy, k):
+    rng = np.random.default_rng(k)
+    N, E = 400, 60000
+    src, dst, t = rand_graph(rng, N, E, 5000)
+    src[:20000] = 7  # one huge segment (multi-round search)
+    o = np.argsort(t, kind="stable")
+    src, dst, t = src[o], dst[o], t[o]
+    g = T.build_tcsr(N, cu(src), cu(dst), cu(t), True, True)
+    tc = oracle.build_tcsr(N, src, dst, t, True)
+    nq = 3001
+    qn = rng.integers(0, N, nq).astype(np.int32)
+    qn[::5] = 7
+    qt = rng.uniform(-10, 5100, nq).astype(np.float32)
+    qt[::17] = np.nan
+    qt[::19] = 0.0
+    qt[1::19] = -0.0
+    qt[::23] = t[rng.integers(0, E, len(qt[::23]))]   # exact ties
+    sid = 0x74676C00 + k
+    seg, nb, ei, ts = T.sample(g, cu(qn), cu(qt), k, strategy, seed=sid, layer=1)
+    es, en, ee, et = oracle.sample(tc, qn, qt, k, opipe.STRATEGY[strategy], sid, 1)
+    m = int(es[-1])
+    assert np.array_equal(np_(seg), es)
+    assert np.array_equal(np_(nb)[:m], en)
+    assert np.array_equal(np_(ei)[:m], ee)
+    assert np.array_equal(np_(ts)[:m], et)
+
+
+def test_sample_device_count_and_empty(T):
+    rng = np.random.default_rng(3)
+    src, dst, t = rand_graph(rng, 100, 5000, 1000)
+    g = T.build_tcsr(100, cu(src), cu(dst), cu(t), True, True)
+    tc = oracle.build_tcsr(100, src, dst, t, True)
+    qn = rng.integers(0, 100, 500).astype(np.int32)
+    qt = rng.uniform(0, 1000, 500).astype(np.float32)
+    for nq in (0, 1, 31, 32, 33, 499):
+        ndev = torch.tensor([nq], dtype=torch.int64, device="cuda")
+        seg, nb, ei, ts = T.sample(g, cu(qn), cu(qt), 10, "uniform", seed=1, nq_dev=ndev)
+        es, en, ee, et = oracle.sample(tc, qn[:nq], qt[:nq], 10, 1, 1, 0)
+        assert np.array_equal(np_(seg)[:nq + 1], es)
+        assert np.array_equal(np_(nb)[:int(es[-1])], en)
+
+
+# ------------------------------------------------------------------ S3
+@pytest.mark.parametrize("n", [0, 1, 2047, 2048, 2049, 20000, 200001])
+def test_dedup_bit_exact(T, n):
+    rng = np.random.default_rng(n + 1)
+    node = rng.integers(0, max(2, n // 8), n).astype(np.int32)
+    t = rng.integers(0, 50, n).astype(np.float32)
+    if n > 10:
+        t[::7] = -0.0
+        t[::11] = 0.0
+    un, ut, nu, inv = T.dedup(cu(node), cu(t)) if n else T.dedup(
+        torch.zeros(1, dtype=torch.int32, device="cuda"),
+        torch.zeros(1, dtype=torch.float32, device="cuda"), n_max=0)
+    eu, eut, einv = oracle.dedup(node, t)
+    U = int(np_(nu)[0])
+    assert U == len(eu)
+    assert np.array_equal(np_(un)[:U], eu)
+    assert np.array_equal(np_(ut)[:U].view(np.uint32), eut.view(np.uint32))
+    assert np.array_equal(np_(inv)[:n], einv)
+
+
+def test_dedup_device_count(T):
+    rng = np.random.default_rng(9)
+    node = rng.integers(0, 300, 10000).astype(np.int32)
+    t = rng.integers(0, 30, 10000).astype(np.float32)
+    ndev = torch.tensor([6001], dtype=torch.int64, device="cuda")
+    un, ut, nu, inv = T.dedup(cu(node), cu(t), n_dev=ndev)
+    eu, eut, einv = oracle.dedup(node[:6001], t[:6001])
+    U = int(np_(nu)[0])
+    assert U == len(eu) and np.array_equal(np_(un)[:U], eu)
+    assert np.array_equal(np_(inv)[:6001], einv)
+
+
+# ------------------------------------------------------------------ S6
+def ulp_diff(a, b):
+    a = a.astype(np.float32)
+    b = b.astype(np.float32)
+    sp = np.spacing(np.maximum(np.abs(a), np.abs(b)))
+    return np.abs(a.astype(np.float64) - b) / sp
+
+
+def test_time_encode_ulp_and_table(T):
+    cfg = synth.get_config("LASTFM")
+    for random_phi in (False, True):
+        omega, phi = synth.make_time_params(cfg, random_phi, seed=4)
+        rng = np.random.default_rng(5)
+        dt = np.concatenate([np.arange(0, 70000, 7, dtype=np.float32),
+                             rng.uniform(0, 1.4e8, 20000).astype(np.float32),
+                             np.array([0.5, -0.0, 65535, 65536, 3.3e-3], np.float32)])
+        o, p = cu(omega), cu(phi)
+        direct = np_(T.time_encode(cu(dt), o, p))
+        exp = oracle.time_encode(dt, omega, phi)
+        assert ulp_diff(direct, exp).max() <= 2.0
+        tab = T.time_precompute(65536, o, p)
+        assert np.array_equal(np_(tab).view(np.uint32),
+                              np_(T.time_encode(cu(np.arange(65536, dtype=np.float32)), o, p)).view(np.uint32))
+        with_tab = np_(T.time_encode(cu(dt), o, p, table=tab))
+        assert np.array_equal(with_tab.view(np.uint32), direct.view(np.uint32))
+
+
+# ------------------------------------------------------------------ S7-S13
+def attn_case(rng, n_dst, kmax, d_h, d_e, empty=True, long_every=0):
+    from dataclasses import replace
+    cfg = replace(synth.get_config("REDDIT"), d_e=d_e)
+    p = synth.make_layer_params(cfg, 0, d_h, d_h, random_ln=True, random_phi=True)
+    lens = rng.integers(0 if empty else 1, kmax + 1, n_dst)
+    if long_every:
+        lens[::long_every] = 300          # segments longer than one 128-row chunk
+    seg = np.zeros(n_dst + 1, np.int64)
+    seg[1:] = np.cumsum(lens)
+    E = int(seg[-1])
+    N = 500
+    nfeat = rng.uniform(-1, 1, (N, d_h)).astype(np.float32)
+    efeat = rng.uniform(-1, 1, (2000, max(d_e, 1))).astype(np.float32)[:, :d_e]
+    dst_node = rng.integers(0, N, n_dst).astype(np.int32)
+    dst_t = rng.integers(10**5, 2 * 10**6, n_dst).astype(np.float32)
+    src_node = rng.integers(0, N, E).astype(np.int32)
+    eid = rng.integers(0, 2000, E).astype(np.int32)
+    gap = rng.integers(1, 200000, E)
+    gap[::3] = rng.integers(1, 60000, len(gap[::3]))
+    edge_t = (np.repeat(dst_t, lens) - gap).astype(np.float32)
+    return p, seg, dst_t, nfeat, dst_node, src_node, efeat, eid, edge_t
+
+
+@pytest.mark.parametrize("precision", ["fp32", "bf16"])
+@pytest.mark.parametrize("n_dst,kmax,d_h,d_e,long_every", [(1, 10, 172, 172, 0),
+                                                          (777, 10, 172, 172, 0),
+                                                          (300, 20, 128, 128, 0),
+                                                          (200, 10, 100, 0, 0),
+                                                          (150, 10, 24, 12, 7)])
+def test_attention_vs_oracle(T, precision, n_dst, kmax, d_h, d_e, long_every):
+    rng = np.random.default_rng(n_dst + kmax)
+    p, seg, dst_t, nfeat, dn, sn, ef, eid, et = attn_case(rng, n_dst, kmax, d_h, d_e,
+                                                          long_every=long_every)
+    exp = oracle.tblock_attn(p, seg, dst_t, nfeat, dn, nfeat, sn, ef, eid, et)
+    P = T.AttnParams(p, precision=precision)
+    tab = T.time_precompute(65536, P.t["omega"], P.t["phi"])
+    for table in (None, tab):
+        got = T.tblock_attn(P, cu(seg), cu(dst_t), cu(nfeat), cu(dn), cu(nfeat), cu(sn),
+                            cu(ef) if d_e else None, cu(eid) if d_e else None, cu(et),
+                            table=table, max_seg=kmax)
+        err = np.abs(np_(got)[:n_dst] - exp).max()
+        assert err <= TOL[precision], err
+
+
+def test_attention_offsets_and_identity(T):
+    """hdst_idx = NULL (identity), hsrc rows at a device offset (the S14 layout)."""
+    rng = np.random.default_rng(11)
+    p, seg, dst_t, nfeat, dn, sn, ef, eid, et = attn_case(rng, 90, 10, 100, 172)
+    E = int(seg[-1])
+    table = rng.uniform(-1, 1, (90 + E + 5, 100)).astype(np.float32)
+    off = 90
+    exp = oracle.tblock_attn(p, seg, dst_t, table, None, table, np.arange(off, off + E), ef, eid, et)
+    P = T.AttnParams(p)
+    offd = torch.tensor([off], dtype=torch.int64, device="cuda")
+    nd = torch.tensor([90], dtype=torch.int64, device="cuda")
+    got = T.tblock_attn(P, cu(seg), cu(dst_t), cu(table), None, cu(table), None, cu(ef),
+                        cu(eid), cu(et), max_seg=10, n_dst_max=90, n_dst_dev=nd,
+                        hsrc_off_dev=offd)
+    assert np.abs(np_(got)[:90] - exp).max() <= 1e-3
+
+
+# ------------------------------------------------------------------ pipeline (all rows)
+def _world(name, n_edges=None, dedup=None, strategy=None):
+    from dataclasses import replace
+    cfg = synth.get_config(name)
+    if n_edges:
+        cfg = cfg.scaled(n_edges)
+    if dedup is not None:
+        cfg = replace(cfg, dedup=dedup)
+    if strategy is not None:
+        cfg = replace(cfg, strategy=strategy)
+    g = synth.make_graph(cfg)
+    neg = synth.make_negatives(cfg)
+    params = synth.gen.model_params(cfg)
+    return cfg, g, neg, params
+
+
+def _gpu_pipeline(T, cfg, g, neg, params, precision="fp32"):
+    from paper_conf_asplos_wangm24_b200 import TGATPipeline, TSampler
+    dev = {"src": cu(g.src), "dst": cu(g.dst), "t": cu(g.t), "neg": cu(neg),
+           "nfeat": cu(g.nfeat), "efeat": cu(g.efeat)}
+    tc = T.build_tcsr(cfg.n_nodes, dev["src"], dev["dst"], dev["t"], True, True)
+    pipe = TGATPipeline(dev, tc, params, cfg.batch,
+                        TSampler(cfg.k, cfg.strategy, cfg.seeds["sampler"]), cfg.dedup,
+                        cfg.precompute, cfg.window, precision)
+    return pipe
+
+
+@pytest.mark.parametrize("name", ["WIKI", "REDDIT"])
+def test_pipeline_full_config_vs_oracle(T, name):
+    cfg, g, neg, params = _world(name)
+    pipe = _gpu_pipeline(T, cfg, g, neg, params)
+    tc = oracle.build_tcsr(cfg.n_nodes, g.src, g.dst, g.t, True)
+    nb = cfg.n_batches
+    for b in (int(0.7 * nb), nb - 1):
+        pipe.start_dev.fill_(b * cfg.batch)
+        emb = pipe.forward()
+        torch.cuda.synchronize()
+        exp, blocks = opipe.run_batch(tc, g.nfeat, g.efeat, params, cfg.k, cfg.strategy,
+                                      cfg.dedup, cfg.seeds["sampler"],
+                                      *synth.batch_roots_inputs(g, neg, b))
+        # bit-exact block structure
+        for gb, ob in zip(pipe.blocks, blocks):
+            U = len(ob.uniq_node)
+            assert int(np_(gb.u_dev)[0]) == U
+            assert np.array_equal(np_(gb.uniq_node)[:U], ob.uniq_node)
+            assert np.array_equal(np_(gb.seg_ptr)[:U + 1], ob.seg_ptr)
+            m = int(ob.seg_ptr[-1])
+            assert np.array_equal(np_(gb.nbr)[:m], ob.nbr)
+            assert np.array_equal(np_(gb.eid)[:m], ob.eid)
+            if ob.inv is not None:
+                assert np.array_equal(np_(gb.inv)[:len(ob.inv)], ob.inv)
+        n0 = 3 * cfg.batch
+        err = np.abs(np_(emb)[:n0] - exp).max()
+        assert err <= 1e-3, err
+
+
+def test_pipeline_dedup_on_off_and_graph_replay(T):
+    """Semantics preservation on the GPU and CUDA-graph replay == eager."""
+    cfg, g, neg, params = _world("REDDIT", n_edges=60000)
+    from dataclasses import replace
+    p_on = _gpu_pipeline(T, cfg, g, neg, params)
+    p_off = _gpu_pipeline(T, replace(cfg, dedup=False), g, neg, params)
+    b = 80
+    p_on.start_dev.fill_(b * cfg.batch)
+    p_off.start_dev.fill_(b * cfg.batch)
+    e_on = np_(p_on.forward()).copy()
+    e_off = np_(p_off.forward())[:3 * cfg.batch]
+    assert np.abs(e_on - e_off).max() <= 1e-4
+    p_on.capture()
+    e_g = np_(p_on.run_graph(b * cfg.batch))
+    assert np.array_equal(e_g, e_on)
+
+
+def test_pipeline_lastfm_sampled_roots(T):
+    """LastFM-shaped (k=20, heavy skew): roots checked one by one with the recursive oracle."""
+    cfg, g, neg, params = _world("LASTFM")
+    pipe = _gpu_pipeline(T, cfg, g, neg, params)
+    tc = oracle.build_tcsr(cfg.n_nodes, g.src, g.dst, g.t, True)
+    b = int(0.7 * cfg.n_batches)
+    pipe.start_dev.fill_(b * cfg.batch)
+    emb = np_(pipe.forward())
+    qn, qt = opipe.roots(*synth.batch_roots_inputs(g, neg, b))
+    pick = np.random.default_rng(0).choice(len(qn), 24, replace=False)
+    exp = oracle.embed_recursive(tc, g.nfeat, g.efeat, params, cfg.k, opipe.STRATEGY[cfg.strategy],
+                                 cfg.seeds["sampler"], qn[pick], qt[pick])
+    assert np.abs(emb[pick] - exp).max() <= 1e-3
