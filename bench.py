@@ -36,7 +36,7 @@ def parse():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="REDDIT")
-    ap.add_argument("--precision", default="fp32", choices=["fp32", "bf16"])
+    ap.add_argument("--precision", default="fp32", choices=["fp32", "bf16", "fp32_simt"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     return ap.parse_args()
@@ -311,16 +311,23 @@ def run_ours(args):
     except Exception:
         pass
     sm_max = clocks.get("sm_max_mhz") or peaks.get("sm_max_mhz", 1965.0)
-    fp32_peak = 148 * 128 * 2 * sm_max * 1e6 / 1e12     # TFLOP/s, FFMA on all SMs
     achieved_tf = fl / (attn_ms / 1e3) / 1e12
-    roofline = {"kernel": "tgl_tblock_attn (tail block: q_proj + kv_attn + out_ffn)",
-                "bound": "alu", "achieved": achieved_tf, "peak": fp32_peak, "unit": "TFLOP/s",
-                "frac": achieved_tf / fp32_peak, "traffic": None,
+    if args.precision == "fp32_simt":
+        peak = 148 * 128 * 2 * sm_max * 1e6 / 1e12     # TFLOP/s, FFMA on all SMs
+        bound, note = "alu", "FP32 FFMA peak = 148 SM x 128 lanes x 2 x clocks.max.sm (derived)"
+    else:
+        peak = peaks.get("bf16_tflops", 1613.6)
+        bound = "tensor"
+        note = ("measured cuBLAS bf16 burst peak (MEASURED_PEAKS.json); fp32 mode issues 3 bf16 "
+                "MMA passes per algorithmic FLOP, so frac <= 1/3 by construction"
+                if args.precision == "fp32" else "measured cuBLAS bf16 burst peak")
+    roofline = {"kernel": "tgl_tblock_attn on the tail block (pack + q + kv + ffn kernels)",
+                "bound": bound, "achieved": achieved_tf, "peak": peak, "unit": "TFLOP/s",
+                "frac": achieved_tf / peak, "traffic": None,
                 "hbm_achieved_gbs": by / (attn_ms / 1e3) / 1e9,
                 "hbm_peak_gbs": peaks.get("hbm_gbs", 6545.9),
                 "per_launch_ms": attn_ms, "algorithmic_flops": fl, "algorithmic_bytes": by,
-                "n_dst_avg": U_avg, "n_edges_avg": E_avg,
-                "peak_note": "FP32 FFMA peak = 148 SM x 128 lanes x 2 x clocks.max.sm"}
+                "n_dst_avg": U_avg, "n_edges_avg": E_avg, "peak_note": note}
 
     # ---- e2e through the public API: pinned host batch -> device -> host embeddings
     e2e = None
@@ -365,8 +372,8 @@ def run_ours(args):
         line = {"metric": METRIC, "value": emb_per_s, "unit": "embeddings/s",
                 "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
                 "ms_per_step": total_ms / args.steps, "higher_is_better": True,
-                "scaling": "weak", "vs_baseline": None, "dtype": "f32" if args.precision == "fp32"
-                else "bf16", "data": "synthetic",
+                "scaling": "weak", "vs_baseline": None, "dtype": {"fp32": "f32 (3-pass bf16 tensor-core split)",
+                                             "bf16": "bf16", "fp32_simt": "f32"}[args.precision], "data": "synthetic",
                 "config": {"workload": cfg.name, "batch_edges": cfg.batch, "roots_per_step": n0,
                            "roots_per_step_all_ranks": world * n0, "layers": cfg.n_layers,
                            "k": cfg.k, "strategy": cfg.strategy, "dedup": cfg.dedup,

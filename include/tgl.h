@@ -57,6 +57,7 @@ typedef int32_t tgl_status;
 /* tgl_attn_params.precision */
 #define TGL_FP32 0 /* fp32 operands, fp32 accumulate (max abs err 1e-3 vs oracle) */
 #define TGL_BF16 1 /* bf16-rounded projection operands, fp32 accumulate (5e-2) */
+#define TGL_FP32_SIMT 2 /* fp32 FFMA on CUDA cores (exact fp32 products; slow reference mode) */
 
 const char* tgl_version(void);
 const char* tgl_status_string(tgl_status s);
@@ -192,7 +193,11 @@ tgl_status tgl_time_encode(int64_t n, const float* dt, int32_t d_t, const float*
  * tenc_table (NULL = direct) as in tgl_time_encode.  max_seg is a launch hint
  * (the sampler's k); any segment length is handled.
  * Output out[n_dst_max][d_out] (rows >= n_dst untouched).
- * Limits: d_model == d_out, d_model % n_heads == 0, d_model <= 128, d_t <= 256.
+ * Limits: d_model == d_out, d_model % n_heads == 0, n_heads <= 2, d_t <= 256;
+ * TGL_FP32 / TGL_BF16 run on the tensor cores (tcgen05) and need d_model == 100;
+ * TGL_FP32_SIMT takes any d_model <= 128.
+ * Precision: TGL_FP32 splits every fp32 operand into bf16 hi + lo and runs three
+ * MMA passes (hi*hi + lo*hi + hi*lo) with fp32 accumulation; TGL_BF16 one pass.
  * ------------------------------------------------------------------------- */
 typedef struct {
   int32_t d_hdst, d_hsrc, d_e, d_t, d_model, n_heads, d_out;

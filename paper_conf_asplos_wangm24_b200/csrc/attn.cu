@@ -430,6 +430,18 @@ __global__ void __launch_bounds__(kAttnThreads, 1) kv_attn_kernel(AttnArgs a) {
   }
 }
 
+// tensor-core implementation (attn_tc.cu)
+size_t tc_attn_ws_bytes(const tgl_attn_params* P, int64_t n_dst_max, size_t* o_q, size_t* o_r,
+                        size_t* o_wq, size_t* o_wkv, size_t* o_wo);
+bool tc_attn_supported(const tgl_attn_params* P);
+tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int64_t* n_dst_dev,
+                          const int64_t* seg_ptr, const float* dst_t, const float* hdst,
+                          const int32_t* hdst_idx, int64_t ld_hdst, const float* hsrc,
+                          const int32_t* hsrc_idx, const int64_t* hsrc_off_dev, int64_t ld_hsrc,
+                          const float* efeat, const int32_t* eid, int64_t ld_e,
+                          const float* edge_t, const float* table, int64_t window,
+                          int32_t max_seg, float* out, void* ws, cudaStream_t s);
+
 }  // namespace tgl
 
 using namespace tgl;
@@ -453,13 +465,25 @@ extern "C" tgl_status tgl_tblock_attn(const tgl_attn_params* P, int64_t n_dst_ma
               kMaxModel);
     return TGL_EUNSUPPORTED;
   }
-  TGL_REQUIRE(P->precision == TGL_FP32 || P->precision == TGL_BF16, "unknown precision");
+  TGL_REQUIRE(P->precision == TGL_FP32 || P->precision == TGL_BF16 ||
+                  P->precision == TGL_FP32_SIMT,
+              "unknown precision");
+  const bool use_tc = P->precision != TGL_FP32_SIMT;
+  if (use_tc && !tc_attn_supported(P)) {
+    set_error("tensor-core path needs d_model == d_out == 100 (use TGL_FP32_SIMT otherwise)");
+    return TGL_EUNSUPPORTED;
+  }
   WsLayout L;
   const int64_t nrows = n_dst_max > 0 ? n_dst_max : 1;
   const size_t o_q = L.take(sizeof(float) * kQLd * nrows);
   const size_t o_r = L.take(sizeof(float) * kQLd * nrows);
+  size_t need = L.off;
+  if (use_tc) {
+    size_t a0, a1, a2, a3, a4;
+    need = tc_attn_ws_bytes(P, n_dst_max, &a0, &a1, &a2, &a3, &a4);
+  }
   bool query = false;
-  TGL_TRY(ws_protocol(ws, ws_bytes, L.off, &query));
+  TGL_TRY(ws_protocol(ws, ws_bytes, need, &query));
   if (query) return TGL_OK;
   if (n_dst_max == 0) return TGL_OK;
   TGL_REQUIRE(seg_ptr && dst_t && hdst && hsrc && edge_t && out, "null pointer");
@@ -495,6 +519,10 @@ extern "C" tgl_status tgl_tblock_attn(const tgl_attn_params* P, int64_t n_dst_ma
   int dpb = kKvBM / ms;
   a.dpb = dpb < 1 ? 1 : (dpb > kMaxDpb ? kMaxDpb : dpb);
   cudaStream_t s = as_stream(stream);
+  if (use_tc)
+    return tc_attn_launch(P, n_dst_max, n_dst_dev, seg_ptr, dst_t, hdst, hdst_idx, ld_hdst, hsrc,
+                          hsrc_idx, hsrc_off_dev, ld_hsrc, efeat, eid, ld_e, edge_t,
+                          a.table, window, max_seg, out, ws, s);
   const unsigned g64 = (unsigned)ceil_div(n_dst_max, kTBM);
   q_proj_kernel<<<g64, kAttnThreads, 0, s>>>(a);
   TGL_TRY(launch_check("q_proj"));

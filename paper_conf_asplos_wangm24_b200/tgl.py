@@ -18,9 +18,9 @@ LIB_PATH = os.path.join(_PKG, "libtgl.so")
 TGL_UNDIRECTED = 1
 TGL_INPUT_TIME_SORTED = 2
 RECENT, UNIFORM = 0, 1
-FP32, BF16 = 0, 1
+FP32, BF16, FP32_SIMT = 0, 1, 2
 STRATEGY = {"recent": RECENT, "uniform": UNIFORM}
-PRECISION = {"fp32": FP32, "bf16": BF16}
+PRECISION = {"fp32": FP32, "bf16": BF16, "fp32_simt": FP32_SIMT}
 
 SYMBOLS = ["tgl_version", "tgl_status_string", "tgl_last_error", "tgl_build_tcsr",
            "tgl_batch_roots", "tgl_dedup", "tgl_sample", "tgl_next_block",

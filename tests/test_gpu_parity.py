@@ -14,7 +14,7 @@ import synth
 
 pytestmark = pytest.mark.gpu
 
-TOL = {"fp32": 1e-3, "bf16": 5e-2}
+TOL = {"fp32": 1e-3, "bf16": 5e-2, "fp32_simt": 1e-3}
 
 
 @pytest.fixture(scope="module")
@@ -195,7 +195,7 @@ def attn_case(rng, n_dst, kmax, d_h, d_e, empty=True, long_every=0):
     return p, seg, dst_t, nfeat, dst_node, src_node, efeat, eid, edge_t
 
 
-@pytest.mark.parametrize("precision", ["fp32", "bf16"])
+@pytest.mark.parametrize("precision", ["fp32", "bf16", "fp32_simt"])
 @pytest.mark.parametrize("n_dst,kmax,d_h,d_e,long_every", [(1, 10, 172, 172, 0),
                                                           (777, 10, 172, 172, 0),
                                                           (300, 20, 128, 128, 0),
