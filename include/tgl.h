@@ -209,8 +209,19 @@ typedef struct {
   const float *omega, *phi;       /* [d_t] */
   float leaky_slope;              /* 0.2; < 0 -> identity */
   float logit_scale;              /* 1.0 */
-  int32_t precision;              /* TGL_FP32 | TGL_BF16 */
+  int32_t precision;              /* TGL_FP32 | TGL_BF16 | TGL_FP32_SIMT */
+  const void* packed;             /* optional tgl_attn_pack() output for these weights and
+                                     this precision; NULL = pack inside every call */
 } tgl_attn_params;
+
+/* Weight layout transform for the tensor-core path, done once per layer (the
+ * weights are constant across batches): Wq, [Wk;Wv], Wo -> bf16 hi/lo pairs in the
+ * swizzled shared-memory image the kernels stream with bulk copies.  `packed`
+ * (device, >= tgl_attn_packed_bytes(P) bytes, 256-aligned) is owned by the caller
+ * and must be re-packed if the weights change.  EUNSUPPORTED for shapes the
+ * tensor-core path does not take. */
+size_t tgl_attn_packed_bytes(const tgl_attn_params* P);
+tgl_status tgl_attn_pack(const tgl_attn_params* P, void* packed, size_t bytes, void* stream);
 
 tgl_status tgl_tblock_attn(const tgl_attn_params* P, int64_t n_dst_max, const int64_t* n_dst_dev,
                            const int64_t* seg_ptr, const float* dst_t, const float* hdst,

@@ -63,7 +63,7 @@ class TGATPipeline:
         self.sampler = sampler
         self.use_dedup = use_dedup
         self.E = graph["src"].numel()
-        self.attn = [tgl.AttnParams(p, self.dev, precision) for p in params]
+        self.attn = [tgl.AttnParams(p, self.dev, precision, pack=True) for p in params]
         self.tables = [tgl.time_precompute(window, a.t["omega"], a.t["phi"]) if precompute else None
                        for a in self.attn]
         k = sampler.k

@@ -432,7 +432,7 @@ __global__ void __launch_bounds__(kAttnThreads, 1) kv_attn_kernel(AttnArgs a) {
 
 // tensor-core implementation (attn_tc.cu)
 size_t tc_attn_ws_bytes(const tgl_attn_params* P, int64_t n_dst_max, size_t* o_q, size_t* o_r,
-                        size_t* o_wq, size_t* o_wkv, size_t* o_wo);
+                        size_t* o_pack);
 bool tc_attn_supported(const tgl_attn_params* P);
 tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int64_t* n_dst_dev,
                           const int64_t* seg_ptr, const float* dst_t, const float* hdst,
@@ -479,8 +479,8 @@ extern "C" tgl_status tgl_tblock_attn(const tgl_attn_params* P, int64_t n_dst_ma
   const size_t o_r = L.take(sizeof(float) * kQLd * nrows);
   size_t need = L.off;
   if (use_tc) {
-    size_t a0, a1, a2, a3, a4;
-    need = tc_attn_ws_bytes(P, n_dst_max, &a0, &a1, &a2, &a3, &a4);
+    size_t a0, a1, a2;
+    need = tc_attn_ws_bytes(P, n_dst_max, &a0, &a1, &a2);
   }
   bool query = false;
   TGL_TRY(ws_protocol(ws, ws_bytes, need, &query));

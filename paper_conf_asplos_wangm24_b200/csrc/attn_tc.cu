@@ -128,7 +128,28 @@ struct Args {
   int split;           // 1 = 3-pass fp32 mode
 };
 
-// Per-CTA shared-memory image (dynamic, 1024-aligned base).
+__device__ __forceinline__ uint8_t* align1024(uint8_t* p) {
+  return reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(p) + 1023) & ~uintptr_t(1023));
+}
+
+// ------------------------------------------------------------------ warp-specialized CTA
+// 15 warps: 0-3 epilogue (TMEM lane quarter = warp), 4 MMA issuer, 5 row-descriptor
+// builder, 6 weight loader (bulk copies), 7-14 producers (gather -> bf16 hi/lo ->
+// swizzled smem).  Rings: A (gathered rows) 2 stages, W (weights) 2 stages,
+// row descriptors 3 slots, TMEM accumulators 2.  mbarriers only in the steady state.
+constexpr int kEpiWarps = 4;
+constexpr int kMmaWarp = 4;
+constexpr int kDescWarp = 5;
+constexpr int kWWarp = 6;
+constexpr int kProdWarp0 = 7;
+constexpr int kProdWarps = 8;
+constexpr int kProdThreads = kProdWarps * 32;
+constexpr int kWsThreads = (kProdWarp0 + kProdWarps) * 32;   // 480
+constexpr int kAStages = 2;
+constexpr int kWStages = 2;
+constexpr int kDSlots = 3;
+constexpr int kBarEpi = 2;    // named barrier id for the 4 epilogue warps
+
 struct RowDesc {
   const float* p0[kBM];
   const float* p1[kBM];
@@ -137,15 +158,38 @@ struct RowDesc {
   int rdst[kBM];
 };
 
-template <int NP>
-struct Smem {
-  static constexpr int kWChunk = 2 * NP * 128;
-  static constexpr int kStage = 2 * kAPart + kWChunk;   // A_hi, A_lo, W (hi|lo)
-  static constexpr int kStages = 2;
-  static constexpr int kPipe = kStages * kStage;
+struct Bars {
+  uint64_t afull[kAStages], aempty[kAStages];
+  uint64_t wfull[kWStages], wempty[kWStages];
+  uint64_t dfull[kDSlots], dempty[kDSlots];
+  uint64_t tfull[2], tempty[2];
 };
 
-__device__ __forceinline__ void load8(const float* p, int lc, int d, float (&x)[8]) {
+template <int NP>
+struct Pipe {
+  static constexpr int kAStage = 2 * kAPart;        // A_hi | A_lo
+  static constexpr int kWStage = 2 * NP * 128;      // W_hi | W_lo
+  static constexpr int kBytes = kAStages * kAStage + kWStages * kWStage;
+  static __device__ __forceinline__ uint8_t* a(uint8_t* pipe, uint32_t s) {
+    return pipe + s * kAStage;
+  }
+  static __device__ __forceinline__ uint8_t* w(uint8_t* pipe, uint32_t s) {
+    return pipe + kAStages * kAStage + s * kWStage;
+  }
+};
+
+__device__ __forceinline__ void named_bar(int id, int n) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+// wait for the (u-1)-th completion of a ring slot (no wait on first use)
+__device__ __forceinline__ void wait_free(uint64_t* bar, uint32_t u) {
+  if (u >= 1) mbar_wait(bar, (u - 1) & 1u);
+}
+
+__device__ __forceinline__ void load8(const float* p, int lc, int d, float* x) {
   if (p != nullptr && lc + 8 <= d && ((reinterpret_cast<uintptr_t>(p + lc) & 15) == 0)) {
     const float4 a = __ldg(reinterpret_cast<const float4*>(p + lc));
     const float4 b = __ldg(reinterpret_cast<const float4*>(p + lc + 4));
@@ -157,472 +201,626 @@ __device__ __forceinline__ void load8(const float* p, int lc, int d, float (&x)[
   }
 }
 
-// Producer: rows' 64-wide K chunk c -> swizzled bf16 hi (and lo) tiles.
-__device__ __forceinline__ void gather_chunk(int c, const Seg3& sg, bool split, uint8_t* a_hi,
-                                             uint8_t* a_lo, const RowDesc& rd, int rows,
-                                             const float* s_omega, const float* s_phi,
-                                             const float* table) {
-  const int t = threadIdx.x;
-  const int r = t >> 1, jb = (t & 1) * 4;
-  const uint32_t hi_base = smem_u32(a_hi), lo_base = smem_u32(a_lo);
+// producer thread pt (0..255): row pt/2, 16-byte groups jb..jb+3 of a 64-wide chunk
+__device__ __forceinline__ void load_chunk(int c, const Seg3& sg, const RowDesc& rd, int r, int jb,
+                                           const float* s_omega, const float* s_phi,
+                                           const float* table, float* x) {
 #pragma unroll
   for (int jj = 0; jj < 4; ++jj) {
-    const int j = jb + jj;
-    const int kp = c * kChunk + j * 8;
-    float x[8];
+    float* y = x + jj * 8;
+    const int kp = c * kChunk + (jb + jj) * 8;
 #pragma unroll
-    for (int e = 0; e < 8; ++e) x[e] = 0.f;
-    if (r < rows && kp < sg.kpad) {
-      if (kp < sg.p0) {
-        load8(rd.p0[r], kp, sg.d0, x);
-      } else if (kp < sg.p0 + sg.p1) {
-        load8(rd.p1[r], kp - sg.p0, sg.d1, x);
+    for (int e = 0; e < 8; ++e) y[e] = 0.f;
+    if (rd.rdst[r] < 0 || kp >= sg.kpad) continue;
+    if (kp < sg.p0) {
+      load8(rd.p0[r], kp, sg.d0, y);
+    } else if (kp < sg.p0 + sg.p1) {
+      load8(rd.p1[r], kp - sg.p0, sg.d1, y);
+    } else {
+      const int j0 = kp - sg.p0 - sg.p1;
+      const int trow = rd.trow[r];
+      if (trow >= 0) {
+        load8(table + (int64_t)trow * sg.d2, j0, sg.d2, y);
       } else {
-        const int j0 = kp - sg.p0 - sg.p1;
-        const int trow = rd.trow[r];
-        if (trow >= 0) {
-          load8(table + (int64_t)trow * sg.d2, j0, sg.d2, x);
-        } else {
-          const float dt = rd.dt[r];
+        const float dt = rd.dt[r];
 #pragma unroll
-          for (int e = 0; e < 8; ++e)
-            if (j0 + e < sg.d2) x[e] = tenc_direct(dt, s_omega[j0 + e], s_phi[j0 + e]);
-        }
+        for (int e = 0; e < 8; ++e)
+          if (j0 + e < sg.d2) y[e] = tenc_direct(dt, s_omega[j0 + e], s_phi[j0 + e]);
       }
     }
+  }
+}
+
+__device__ __forceinline__ void store_chunk(const float* x, uint8_t* a_hi, uint8_t* a_lo, int r,
+                                            int jb, bool split) {
+  const uint32_t hb = smem_u32(a_hi), lb = smem_u32(a_lo);
+#pragma unroll
+  for (int jj = 0; jj < 4; ++jj) {
     uint32_t h[4], l[4];
 #pragma unroll
-    for (int e = 0; e < 4; ++e) split2(x[2 * e], x[2 * e + 1], h[e], l[e]);
-    const uint32_t off = sw128_off(r, j);
-    st_shared_v4(hi_base + off, h[0], h[1], h[2], h[3]);
-    if (split) st_shared_v4(lo_base + off, l[0], l[1], l[2], l[3]);
+    for (int e = 0; e < 4; ++e) split2(x[jj * 8 + 2 * e], x[jj * 8 + 2 * e + 1], h[e], l[e]);
+    const uint32_t off = sw128_off(r, jb + jj);
+    st_shared_v4(hb + off, h[0], h[1], h[2], h[3]);
+    if (split) st_shared_v4(lb + off, l[0], l[1], l[2], l[3]);
   }
 }
 
-// One M-tile of 128 rows: all K chunks through the 2-stage pipeline.  All threads
-// gather; thread 0 moves W chunks (bulk copy) and issues the MMAs.  On return the
-// accumulator in TMEM is complete and visible (after tc_fence_after).
+// ---- tile schedules (every role walks the same sequence) --------------------------
+struct DenseSched {   // q / ffn: tile = 128 consecutive destinations
+  int64_t n, tile, stride;
+  __device__ DenseSched(int64_t n_) : n(n_), tile(blockIdx.x), stride(gridDim.x) {}
+  __device__ bool next(int64_t& i0, int& rows) {
+    const int64_t ntiles = (n + kBM - 1) / kBM;
+    if (tile >= ntiles) return false;
+    i0 = tile * kBM;
+    rows = (int)((n - i0) < kBM ? (n - i0) : kBM);
+    tile += stride;
+    return true;
+  }
+};
+
+struct GroupSched {   // kv: groups of `dpb` destinations, each cut into 128-row tiles
+  const int64_t* seg_ptr;
+  int64_t n, groups, g, stride;
+  int dpb;
+  int64_t d0, e1, c0;
+  int nd;
+  __device__ GroupSched(const int64_t* sp, int64_t n_, int dpb_)
+      : seg_ptr(sp), n(n_), groups((n_ + dpb_ - 1) / dpb_), g(blockIdx.x), stride(gridDim.x),
+        dpb(dpb_), d0(0), e1(0), c0(0), nd(0) {}
+  __device__ bool next_group() {
+    if (g >= groups) return false;
+    d0 = g * dpb;
+    nd = (int)((n - d0) < dpb ? (n - d0) : dpb);
+    c0 = seg_ptr[d0];
+    e1 = seg_ptr[d0 + nd];
+    g += stride;
+    return true;
+  }
+  __device__ bool next_tile(int64_t& t0, int& rows) {
+    if (c0 >= e1) return false;
+    t0 = c0;
+    rows = (int)((e1 - c0) < kBM ? (e1 - c0) : kBM);
+    c0 += kBM;
+    return true;
+  }
+  // flat walk over tiles (for roles that do not care about group boundaries)
+  __device__ bool next(int64_t& t0, int& rows) {
+    while (!next_tile(t0, rows))
+      if (!next_group()) return false;
+    return true;
+  }
+};
+
+// ---- roles ------------------------------------------------------------------------
 template <int NP, int N>
-__device__ __forceinline__ void mainloop(const Seg3& sg, bool split, uint8_t* pipe,
-                                         const uint8_t* wpack, uint64_t* w_bar,
-                                         uint64_t* mma_bar, uint32_t tmem_d, uint32_t& it,
-                                         const RowDesc& rd, int rows, const float* s_omega,
-                                         const float* s_phi, const float* table) {
-  using S = Smem<NP>;
+__device__ __forceinline__ void mma_tile(const Seg3& sg, bool split, uint8_t* pipe, Bars& B,
+                                         uint32_t tmem_acc, uint32_t& ait, uint32_t& wit,
+                                         uint32_t tt) {
+  using PP = Pipe<NP>;
   constexpr uint32_t idesc = idesc_bf16(kBM, N);
-  uint32_t last_stage = 0, last_parity = 0;
-  for (int c = 0; c < sg.nchunks; ++c) {
-    const uint32_t s = it & 1u;
-    uint8_t* st = pipe + s * S::kStage;
-    uint8_t* a_hi = st;
-    uint8_t* a_lo = st + kAPart;
-    uint8_t* w = st + 2 * kAPart;
-    if (it >= 2) mbar_wait(&mma_bar[s], ((it - 2) >> 1) & 1u);
-    if (threadIdx.x == 0) {
-      mbar_arrive_expect_tx(&w_bar[s], S::kWChunk);
-      bulk_g2s(w, wpack + (size_t)c * S::kWChunk, S::kWChunk, &w_bar[s]);
-    }
-    gather_chunk(c, sg, split, a_hi, a_lo, rd, rows, s_omega, s_phi, table);
-    fence_proxy_async_smem();
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      mbar_wait(&w_bar[s], (it >> 1) & 1u);
-      tc_fence_after();
-      const int rem = sg.kpad - c * kChunk;
-      const int nk = rem >= kChunk ? 4 : (rem + 15) / 16;
-      const uint32_t ahb = smem_u32(a_hi), alb = smem_u32(a_lo), whb = smem_u32(w);
-      const uint32_t wlb = whb + NP * 128;
-      for (int ks = 0; ks < nk; ++ks) {
-        const uint64_t ah = desc_sw128(ahb + ks * 32), bh = desc_sw128(whb + ks * 32);
-        mma_bf16(tmem_d, ah, bh, idesc, (c | ks) != 0);
-        if (split) {
-          const uint64_t al = desc_sw128(alb + ks * 32), bl = desc_sw128(wlb + ks * 32);
-          mma_bf16(tmem_d, al, bh, idesc, 1u);
-          mma_bf16(tmem_d, ah, bl, idesc, 1u);
-        }
-      }
-      mma_commit(&mma_bar[s]);
-    }
-    last_stage = s;
-    last_parity = (it >> 1) & 1u;
-    ++it;
-  }
-  mbar_wait(&mma_bar[last_stage], last_parity);
+  wait_free(&B.tempty[tt & 1u], tt >> 1);    // epilogue drained this accumulator
   tc_fence_after();
+  for (int c = 0; c < sg.nchunks; ++c, ++ait, ++wit) {
+    const uint32_t sa = ait % kAStages, sw = wit % kWStages;
+    mbar_wait(&B.afull[sa], (ait / kAStages) & 1u);
+    mbar_wait(&B.wfull[sw], (wit / kWStages) & 1u);
+    tc_fence_after();
+    const uint32_t ahb = smem_u32(PP::a(pipe, sa)), alb = ahb + kAPart;
+    const uint32_t whb = smem_u32(PP::w(pipe, sw)), wlb = whb + NP * 128;
+    const int rem = sg.kpad - c * kChunk;
+    const int nk = rem >= kChunk ? 4 : (rem + 15) / 16;
+    for (int ks = 0; ks < nk; ++ks) {
+      const uint64_t ah = desc_sw128(ahb + ks * 32), bh = desc_sw128(whb + ks * 32);
+      mma_bf16(tmem_acc, ah, bh, idesc, (c | ks) != 0);
+      if (split) {
+        mma_bf16(tmem_acc, desc_sw128(alb + ks * 32), bh, idesc, 1u);
+        mma_bf16(tmem_acc, ah, desc_sw128(wlb + ks * 32), idesc, 1u);
+      }
+    }
+    mma_commit(&B.aempty[sa]);
+    mma_commit(&B.wempty[sw]);
+  }
+  mma_commit(&B.tfull[tt & 1u]);
 }
 
-__device__ __forceinline__ uint8_t* align1024(uint8_t* p) {
-  return reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(p) + 1023) & ~uintptr_t(1023));
+template <int NP>
+__device__ __forceinline__ void wload_tile(const Seg3& sg, uint8_t* pipe, Bars& B,
+                                           const uint8_t* wpack, uint32_t& wit) {
+  using PP = Pipe<NP>;
+  for (int c = 0; c < sg.nchunks; ++c, ++wit) {
+    const uint32_t sw = wit % kWStages;
+    wait_free(&B.wempty[sw], wit / kWStages);
+    mbar_arrive_expect_tx(&B.wfull[sw], PP::kWStage);
+    bulk_g2s(PP::w(pipe, sw), wpack + (size_t)c * PP::kWStage, PP::kWStage, &B.wfull[sw]);
+  }
 }
 
-// common prologue: barriers + TMEM allocation
-template <int NCOLS>
-__device__ __forceinline__ uint32_t prologue(uint64_t* w_bar, uint64_t* mma_bar, uint32_t* s_tmem) {
+template <int NP>
+__device__ __forceinline__ void produce_tile(const Seg3& sg, bool split, uint8_t* pipe, Bars& B,
+                                             uint32_t& ait, const RowDesc& rd,
+                                             const float* s_omega, const float* s_phi,
+                                             const float* table) {
+  using PP = Pipe<NP>;
+  const int pt = threadIdx.x - kProdWarp0 * 32;
+  const int r = pt >> 1, jb = (pt & 1) * 4;
+  const int lane = threadIdx.x & 31;
+  float cur[32], nxt[32];
+  load_chunk(0, sg, rd, r, jb, s_omega, s_phi, table, cur);
+  for (int c = 0; c < sg.nchunks; ++c, ++ait) {
+    const uint32_t sa = ait % kAStages;
+    if (c + 1 < sg.nchunks) load_chunk(c + 1, sg, rd, r, jb, s_omega, s_phi, table, nxt);
+    wait_free(&B.aempty[sa], ait / kAStages);
+    uint8_t* st = PP::a(pipe, sa);
+    store_chunk(cur, st, st + kAPart, r, jb, split);
+    fence_proxy_async_smem();
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&B.afull[sa]);
+#pragma unroll
+    for (int i = 0; i < 32; ++i) cur[i] = nxt[i];
+  }
+}
+
+__device__ __forceinline__ void ws_init(Bars& B, uint32_t* s_tmem, uint32_t ncols) {
   if (threadIdx.x == 0) {
-    for (int i = 0; i < 2; ++i) {
-      mbar_init(&w_bar[i], 1);
-      mbar_init(&mma_bar[i], 1);
+    for (int s = 0; s < kAStages; ++s) {
+      mbar_init(&B.afull[s], kProdWarps);
+      mbar_init(&B.aempty[s], 1);
+    }
+    for (int s = 0; s < kWStages; ++s) {
+      mbar_init(&B.wfull[s], 1);
+      mbar_init(&B.wempty[s], 1);
+    }
+    for (int s = 0; s < kDSlots; ++s) {
+      mbar_init(&B.dfull[s], 1);
+      mbar_init(&B.dempty[s], kProdWarps + kEpiWarps);
+    }
+    for (int a = 0; a < 2; ++a) {
+      mbar_init(&B.tfull[a], 1);
+      mbar_init(&B.tempty[a], kEpiWarps);
     }
     fence_mbar_init();
   }
-  if ((threadIdx.x >> 5) == 0) tmem_alloc(s_tmem, NCOLS);
+  if ((threadIdx.x >> 5) == kMmaWarp) tmem_alloc(s_tmem, ncols);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
-  return *s_tmem;
 }
 
-template <int NCOLS>
-__device__ __forceinline__ void epilogue_teardown(uint32_t tmem) {
+__device__ __forceinline__ void ws_teardown(uint32_t tmem, uint32_t ncols) {
   tc_fence_before();
   __syncthreads();
-  if ((threadIdx.x >> 5) == 0) tmem_dealloc(tmem, NCOLS);
+  if ((threadIdx.x >> 5) == kMmaWarp) tmem_dealloc(tmem, ncols);
 }
 
-// ------------------------------------------------------------------ S8: q projection
+// per-warp arrive (all lanes done with a resource)
+__device__ __forceinline__ void warp_arrive(uint64_t* bar) {
+  __syncwarp();
+  if ((threadIdx.x & 31) == 0) mbar_arrive(bar);
+}
+
+// ------------------------------------------------------------------ S8 / S13 (dense rows)
 constexpr int kNPq = 104;   // d_model padded to a multiple of 8 (rows of Wq / Wo)
 
-__global__ void __launch_bounds__(kThreads, 1) q_kernel(Args a) {
+template <bool kFfn>
+__global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* pipe = align1024(smem_raw);
-  using S = Smem<kNPq>;
-  __shared__ uint64_t w_bar[2], mma_bar[2];
+  __shared__ Bars B;
   __shared__ uint32_t s_tmem;
-  __shared__ RowDesc rd;
+  __shared__ RowDesc rd[kDSlots];
   __shared__ float s_omega[256], s_phi[256];
+  constexpr uint32_t kCols = 128;
   const tgl_attn_params& P = a.P;
   const int64_t n = dev_count(a.n_dst_dev, a.n_dst_max);
-  const int64_t tiles = (n + kBM - 1) / kBM;
-  const uint32_t tmem = prologue<128>(w_bar, mma_bar, &s_tmem);
+  const Seg3& sg = kFfn ? a.so : a.sq;
+  const uint8_t* wpack = kFfn ? a.wo : a.wq;
+  const bool split = a.split != 0;
   for (int j = threadIdx.x; j < P.d_t; j += blockDim.x) {
     s_omega[j] = P.omega[j];
     s_phi[j] = P.phi[j];
   }
-  uint32_t it = 0;
-  const int dm = P.d_model;
+  ws_init(B, &s_tmem, 2 * kCols);
+  const uint32_t tmem = s_tmem;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int q4 = warp & 3, half = warp >> 2;
-  const int HC = (dm + 1) / 2;
-  for (int64_t tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
-    const int64_t i0 = tile * kBM;
-    const int rows = (int)((n - i0) < kBM ? (n - i0) : kBM);
-    if (threadIdx.x < kBM) {
-      const int r = threadIdx.x;
-      const float* p0 = nullptr;
-      if (r < rows) {
-        const int64_t i = i0 + r;
-        const int64_t row = a.hdst_idx ? (int64_t)a.hdst_idx[i] : i;
-        p0 = a.hdst + row * a.ld_hdst;
+  DenseSched sched(n);
+  int64_t i0;
+  int rows;
+  uint32_t tt = 0;
+  if (warp == kDescWarp) {                           // ---------------- row descriptors
+    for (; sched.next(i0, rows); ++tt) {
+      const uint32_t ds = tt % kDSlots;
+      wait_free(&B.dempty[ds], tt / kDSlots);
+      RowDesc& R = rd[ds];
+      for (int r = lane; r < kBM; r += 32) {
+        const float *p0 = nullptr, *p1 = nullptr;
+        if (r < rows) {
+          const int64_t i = i0 + r;
+          const int64_t hrow = a.hdst_idx ? (int64_t)a.hdst_idx[i] : i;
+          if (kFfn) {
+            p0 = a.rbuf + i * kQLd;                    // [r_i ; h_i]  (eq 7)
+            p1 = a.hdst + hrow * a.ld_hdst;
+          } else {
+            p0 = a.hdst + hrow * a.ld_hdst;            // [h_i ; Phi(0)] (eq 4)
+          }
+        }
+        R.p0[r] = p0;
+        R.p1[r] = p1;
+        R.dt[r] = 0.f;
+        R.trow[r] = (!kFfn && a.table != nullptr) ? 0 : -1;   // precomputed_zeros = row 0
+        R.rdst[r] = r < rows ? r : -1;
       }
-      rd.p0[r] = p0;
-      rd.p1[r] = nullptr;
-      rd.dt[r] = 0.0f;                          // Phi(0): eq 4 / L2.27
-      rd.trow[r] = a.table != nullptr ? 0 : -1;  // precomputed_zeros == table row 0
+      warp_arrive(&B.dfull[ds]);
     }
-    __syncthreads();
-    mainloop<kNPq, kNPq>(a.sq, a.split, pipe, a.wq, w_bar, mma_bar, tmem, it, rd, rows, s_omega,
-                         s_phi, a.table);
-    // epilogue: thread (quarter q4, lane) = row, half selects columns [cb, cb+HC)
-    const int row = q4 * 32 + lane;
-    const int cb = half * HC;
-    float v[64];
-    const uint32_t ta = tmem + ((uint32_t)(q4 * 32) << 16) + cb;
-    tmem_ld32(ta, &v[0]);
-    tmem_ld32(ta + 32, &v[32]);
-    tmem_wait_ld();
-    if (row < rows) {
-      float* q = a.qbuf + (i0 + row) * kQLd;
+  } else if (warp == kWWarp) {                       // ---------------- weight loader
+    uint32_t wit = 0;
+    if (lane == 0)
+      while (sched.next(i0, rows)) wload_tile<kNPq>(sg, pipe, B, wpack, wit);
+    __syncwarp();
+  } else if (warp >= kProdWarp0) {                   // ---------------- producers
+    uint32_t ait = 0;
+    for (; sched.next(i0, rows); ++tt) {
+      const uint32_t ds = tt % kDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kDSlots) & 1u);
+      produce_tile<kNPq>(sg, split, pipe, B, ait, rd[ds], s_omega, s_phi, a.table);
+      warp_arrive(&B.dempty[ds]);
+    }
+  } else if (warp == kMmaWarp) {                     // ---------------- MMA issuer
+    uint32_t ait = 0, wit = 0;
+    if (lane == 0)
+      for (; sched.next(i0, rows); ++tt)
+        mma_tile<kNPq, kNPq>(sg, split, pipe, B, tmem + (tt & 1u) * kCols, ait, wit, tt);
+    __syncwarp();
+  } else {                                           // ---------------- epilogue
+    const int row = warp * 32 + lane;
+    const int D = P.d_model;
+    for (; sched.next(i0, rows); ++tt) {
+      const uint32_t ab = tt & 1u, ds = tt % kDSlots;
+      mbar_wait(&B.tfull[ab], (tt >> 1) & 1u);
+      tc_fence_after();
+      warp_arrive(&B.dempty[ds]);                     // descriptors not needed here
+      (void)ds;
+      const uint32_t ta = tmem + ab * kCols + ((uint32_t)(warp * 32) << 16);
+      float v[32];
+      if (!kFfn) {
+        float* q = a.qbuf + (i0 + row) * kQLd;
+#pragma unroll 1
+        for (int cq = 0; cq < 4; ++cq) {
+          tmem_ld32(ta + cq * 32, v);
+          tmem_wait_ld();
+          if (row < rows) {
 #pragma unroll
-      for (int j = 0; j < 64; ++j)
-        if (j < HC && cb + j < dm) q[cb + j] = v[j] + P.bq[cb + j];
+            for (int j = 0; j < 32; j += 4) {
+              const int col = cq * 32 + j;
+              if (col < D) {
+                float4 o = make_float4(v[j] + P.bq[col], v[j + 1] + P.bq[col + 1],
+                                       v[j + 2] + P.bq[col + 2], v[j + 3] + P.bq[col + 3]);
+                *reinterpret_cast<float4*>(q + col) = o;   // D % 4 == 0 (D == 100)
+              }
+            }
+          }
+        }
+      } else {
+        // out = LayerNorm(ReLU(acc + bo)): three passes over TMEM (sum, squares, write)
+        float s = 0.f;
+#pragma unroll 1
+        for (int cq = 0; cq < 4; ++cq) {
+          tmem_ld32(ta + cq * 32, v);
+          tmem_wait_ld();
+#pragma unroll
+          for (int j = 0; j < 32; ++j) {
+            const int col = cq * 32 + j;
+            if (col < D) s += fmaxf(v[j] + P.bo[col], 0.f);
+          }
+        }
+        const float mean = s / (float)D;
+        float q2 = 0.f;
+#pragma unroll 1
+        for (int cq = 0; cq < 4; ++cq) {
+          tmem_ld32(ta + cq * 32, v);
+          tmem_wait_ld();
+#pragma unroll
+          for (int j = 0; j < 32; ++j) {
+            const int col = cq * 32 + j;
+            if (col < D) {
+              const float d = fmaxf(v[j] + P.bo[col], 0.f) - mean;
+              q2 += d * d;
+            }
+          }
+        }
+        const float inv = rsqrtf(q2 / (float)D + P.ln_eps);
+        float* o = a.out + (i0 + row) * D;
+#pragma unroll 1
+        for (int cq = 0; cq < 4; ++cq) {
+          tmem_ld32(ta + cq * 32, v);
+          tmem_wait_ld();
+          if (row < rows) {
+#pragma unroll
+            for (int j = 0; j < 32; j += 4) {
+              const int col = cq * 32 + j;
+              if (col < D) {
+                float r4[4];
+#pragma unroll
+                for (int e = 0; e < 4; ++e)
+                  r4[e] = (fmaxf(v[j + e] + P.bo[col + e], 0.f) - mean) * inv * P.ln_gamma[col + e] +
+                          P.ln_beta[col + e];
+                *reinterpret_cast<float4*>(o + col) = make_float4(r4[0], r4[1], r4[2], r4[3]);
+              }
+            }
+          }
+        }
+      }
+      tc_fence_before();
+      warp_arrive(&B.tempty[ab]);
     }
-    tc_fence_before();
-    __syncthreads();
   }
-  epilogue_teardown<128>(tmem);
+  ws_teardown(tmem, 2 * kCols);
 }
 
-// ------------------------------------------------------------------ S13: FFN
-__global__ void __launch_bounds__(kThreads, 1) ffn_kernel(Args a) {
+// ------------------------------------------------------------------ S6,S7,S9-S12 (edge rows)
+constexpr int kNPkv = 200;   // [Wk ; Wv] rows (2 * d_model)
+constexpr int kKvEpiBytes = (2 * kMaxDpb * kMaxModel + kBM * 33) * 4;   // s_q, s_r, s_pv
+
+__global__ void __launch_bounds__(kWsThreads, 1) kv_kernel(Args a) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* pipe = align1024(smem_raw);
-  __shared__ uint64_t w_bar[2], mma_bar[2];
+  __shared__ Bars B;
   __shared__ uint32_t s_tmem;
-  __shared__ RowDesc rd;
-  __shared__ float s_part[2][kBM];
-  const tgl_attn_params& P = a.P;
-  const int64_t n = dev_count(a.n_dst_dev, a.n_dst_max);
-  const int64_t tiles = (n + kBM - 1) / kBM;
-  const uint32_t tmem = prologue<128>(w_bar, mma_bar, &s_tmem);
-  uint32_t it = 0;
-  const int D = P.d_out;
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int q4 = warp & 3, half = warp >> 2;
-  const int HC = (D + 1) / 2;
-  for (int64_t tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
-    const int64_t i0 = tile * kBM;
-    const int rows = (int)((n - i0) < kBM ? (n - i0) : kBM);
-    if (threadIdx.x < kBM) {
-      const int r = threadIdx.x;
-      const float *p0 = nullptr, *p1 = nullptr;
-      if (r < rows) {
-        const int64_t i = i0 + r;
-        const int64_t row = a.hdst_idx ? (int64_t)a.hdst_idx[i] : i;
-        p0 = a.rbuf + i * kQLd;                 // [r_i ; h_i], eq 7
-        p1 = a.hdst + row * a.ld_hdst;
-      }
-      rd.p0[r] = p0;
-      rd.p1[r] = p1;
-      rd.dt[r] = 0.f;
-      rd.trow[r] = -1;
-    }
-    __syncthreads();
-    mainloop<kNPq, kNPq>(a.so, a.split, pipe, a.wo, w_bar, mma_bar, tmem, it, rd, rows, nullptr,
-                         nullptr, nullptr);
-    const int row = q4 * 32 + lane;
-    const int cb = half * HC;
-    const int ce = cb + HC < D ? cb + HC : D;
-    float v[64];
-    const uint32_t ta = tmem + ((uint32_t)(q4 * 32) << 16) + cb;
-    tmem_ld32(ta, &v[0]);
-    tmem_ld32(ta + 32, &v[32]);
-    tmem_wait_ld();
-    float s = 0.f;
-#pragma unroll
-    for (int j = 0; j < 64; ++j) {
-      const int col = cb + j;
-      const float o = col < ce ? fmaxf(v[j] + P.bo[col], 0.f) : 0.f;   // ReLU
-      v[j] = o;
-      s += o;
-    }
-    s_part[half][row] = s;
-    __syncthreads();
-    const float mean = (s_part[0][row] + s_part[1][row]) / (float)D;
-    float q = 0.f;
-#pragma unroll
-    for (int j = 0; j < 64; ++j) {
-      const float d = cb + j < ce ? v[j] - mean : 0.f;
-      q += d * d;
-    }
-    __syncthreads();
-    s_part[half][row] = q;
-    __syncthreads();
-    const float var = (s_part[0][row] + s_part[1][row]) / (float)D;
-    const float inv = rsqrtf(var + P.ln_eps);
-    if (row < rows) {
-      float* o = a.out + (i0 + row) * D;
-#pragma unroll
-      for (int j = 0; j < 64; ++j) {
-        const int col = cb + j;
-        if (col < ce) o[col] = (v[j] - mean) * inv * P.ln_gamma[col] + P.ln_beta[col];
-      }
-    }
-    tc_fence_before();
-    __syncthreads();
-  }
-  epilogue_teardown<128>(tmem);
-}
-
-// ------------------------------------------------------------------ S6,S7,S9-S12
-constexpr int kNPkv = 200;   // 2 * d_model rows of [Wk ; Wv] (d_model = 100)
-
-__global__ void __launch_bounds__(kThreads, 1) kv_kernel(Args a) {
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* pipe = align1024(smem_raw);
-  __shared__ uint64_t w_bar[2], mma_bar[2];
-  __shared__ uint32_t s_tmem;
-  __shared__ RowDesc rd;
+  __shared__ RowDesc rd[kDSlots];
   __shared__ float s_omega[256], s_phi[256];
   __shared__ float s_bias[2 * kMaxModel];
-  __shared__ float s_q[kMaxDpb][kMaxModel];
-  __shared__ float s_r[kMaxDpb][kMaxModel];
-  __shared__ float s_lpart[2][kBM][2];
+  // epilogue state (one destination group at a time); big arrays live after the pipe
+  float (*s_q)[kMaxModel] = reinterpret_cast<float (*)[kMaxModel]>(pipe + Pipe<200>::kBytes);
+  float (*s_r)[kMaxModel] = s_q + kMaxDpb;
+  float (*s_pv)[33] = reinterpret_cast<float (*)[33]>(s_r + kMaxDpb);
   __shared__ float s_logit[kBM][2];
   __shared__ float s_p[kBM][2];
   __shared__ float s_m[kMaxDpb][2], s_l[kMaxDpb][2], s_sc[kMaxDpb][2];
   __shared__ int64_t s_seg[kMaxDpb + 1];
-  __shared__ float s_tdst[kMaxDpb];
+  constexpr uint32_t kCols = 256;
   const tgl_attn_params& P = a.P;
   const int64_t n = dev_count(a.n_dst_dev, a.n_dst_max);
-  const int64_t groups = (n + a.dpb - 1) / a.dpb;
-  const uint32_t tmem = prologue<256>(w_bar, mma_bar, &s_tmem);
+  const bool split = a.split != 0;
   const int dm = P.d_model, H = P.n_heads, dh = dm / H;
-  const int tid = threadIdx.x;
-  for (int j = tid; j < P.d_t; j += blockDim.x) {
+  for (int j = threadIdx.x; j < P.d_t; j += blockDim.x) {
     s_omega[j] = P.omega[j];
     s_phi[j] = P.phi[j];
   }
-  for (int j = tid; j < 2 * dm; j += blockDim.x) s_bias[j] = j < dm ? P.bk[j] : P.bv[j - dm];
-  const int64_t hoff = a.hsrc_off_dev ? *a.hsrc_off_dev : 0;
-  const int warp = tid >> 5, lane = tid & 31;
-  const int q4 = warp & 3, half = warp >> 2;
-  const int HC = (dm + 1) / 2;
-  const int cb = half * HC, ce = cb + HC < dm ? cb + HC : dm;
-  float* s_pv = reinterpret_cast<float*>(pipe);   // [kBM][dm+1] scratch, reuses stage memory
-  const int pv_ld = dm + 1;
-  uint32_t it = 0;
-
-  for (int64_t g = blockIdx.x; g < groups; g += gridDim.x) {
-    const int64_t d0 = g * a.dpb;
-    const int nd = (int)((n - d0) < a.dpb ? (n - d0) : a.dpb);
-    for (int x = tid; x < kMaxDpb * kMaxModel; x += blockDim.x) {
-      const int d = x / kMaxModel, c = x % kMaxModel;
-      s_q[d][c] = (d < nd && c < dm) ? a.qbuf[(d0 + d) * kQLd + c] : 0.f;
-      s_r[d][c] = 0.f;
+  for (int j = threadIdx.x; j < 2 * dm; j += blockDim.x) s_bias[j] = j < dm ? P.bk[j] : P.bv[j - dm];
+  ws_init(B, &s_tmem, 2 * kCols);
+  const uint32_t tmem = s_tmem;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  GroupSched sched(a.seg_ptr, n, a.dpb);
+  int64_t t0;
+  int rows;
+  uint32_t tt = 0;
+  if (warp == kDescWarp) {                           // ---------------- row descriptors
+    const int64_t hoff = a.hsrc_off_dev ? *a.hsrc_off_dev : 0;
+    while (sched.next_group()) {
+      // this group's segment offsets, kept in registers (lane d holds seg_ptr[d0+d])
+      const int64_t segl = lane <= sched.nd ? a.seg_ptr[sched.d0 + lane] : INT64_MAX;
+      const float tdl = lane < sched.nd ? a.dst_t[sched.d0 + lane] : 0.f;
+      for (; sched.next_tile(t0, rows); ++tt) {
+        const uint32_t ds = tt % kDSlots;
+        wait_free(&B.dempty[ds], tt / kDSlots);
+        RowDesc& R = rd[ds];
+#pragma unroll 1
+        for (int r = lane; r < kBM; r += 32) {
+          const int64_t e = t0 + r;
+          // local destination = #{1 <= d < nd : seg[d] <= e}  (offsets broadcast by shuffle)
+          int ld = 0;
+          for (int dd = 1; dd < sched.nd; ++dd)
+            ld += (__shfl_sync(0xffffffffu, segl, dd) <= e) ? 1 : 0;
+          const float td = __shfl_sync(0xffffffffu, tdl, ld & 31);
+          const float *p0 = nullptr, *p1 = nullptr;
+          float dt = 0.f;
+          int trow = -1, rr = -1;
+          if (r < rows) {
+            rr = ld;
+            const int64_t hr = a.hsrc_idx ? (int64_t)a.hsrc_idx[hoff + e] : hoff + e;
+            p0 = a.hsrc + hr * a.ld_hsrc;
+            if (P.d_e > 0) p1 = a.efeat + (int64_t)a.eid[e] * a.ld_e;
+            dt = td - a.edge_t[e];                       // fp32 delta (R18)
+            trow = (int)tenc_table_row(dt, a.table, a.window);
+          }
+          R.p0[r] = p0;
+          R.p1[r] = p1;
+          R.dt[r] = dt;
+          R.trow[r] = trow;
+          R.rdst[r] = rr;
+        }
+        warp_arrive(&B.dfull[ds]);
+      }
     }
-    if (tid < kMaxDpb * 2) {
-      s_m[tid >> 1][tid & 1] = -INFINITY;
-      s_l[tid >> 1][tid & 1] = 0.f;
+  } else if (warp == kWWarp) {                       // ---------------- weight loader
+    uint32_t wit = 0;
+    if (lane == 0)
+      while (sched.next(t0, rows)) wload_tile<kNPkv>(a.skv, pipe, B, a.wkv, wit);
+    __syncwarp();
+  } else if (warp >= kProdWarp0) {                   // ---------------- producers
+    uint32_t ait = 0;
+    for (; sched.next(t0, rows); ++tt) {
+      const uint32_t ds = tt % kDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kDSlots) & 1u);
+      produce_tile<kNPkv>(a.skv, split, pipe, B, ait, rd[ds], s_omega, s_phi, a.table);
+      warp_arrive(&B.dempty[ds]);
     }
-    if (tid <= nd) s_seg[tid] = a.seg_ptr[d0 + tid];
-    if (tid < nd) s_tdst[tid] = a.dst_t[d0 + tid];
-    __syncthreads();
-    const int64_t e_begin = s_seg[0], e_end = s_seg[nd];
-    for (int64_t c0 = e_begin; c0 < e_end; c0 += kBM) {
-      const int rows = (int)((e_end - c0) < kBM ? (e_end - c0) : kBM);
-      if (tid < kBM) {
-        const int r = tid;
-        int ld = -1;
-        const float *p0 = nullptr, *p1 = nullptr;
-        float dt = 0.f;
-        int trow = -1;
-        if (r < rows) {
-          const int64_t e = c0 + r;
-          int lo = 0, hi = nd;
-          while (hi - lo > 1) {
-            const int mid = (lo + hi) >> 1;
-            if (s_seg[mid] <= e) lo = mid; else hi = mid;
-          }
-          ld = lo;
-          const int64_t hr = a.hsrc_idx ? (int64_t)a.hsrc_idx[hoff + e] : hoff + e;
-          p0 = a.hsrc + hr * a.ld_hsrc;
-          if (P.d_e > 0) p1 = a.efeat + (int64_t)a.eid[e] * a.ld_e;
-          dt = s_tdst[ld] - a.edge_t[e];          // fp32 delta (R18)
-          trow = (int)tenc_table_row(dt, a.table, a.window);
-        }
-        rd.p0[r] = p0;
-        rd.p1[r] = p1;
-        rd.dt[r] = dt;
-        rd.trow[r] = trow;
-        rd.rdst[r] = ld;
+  } else if (warp == kMmaWarp) {                     // ---------------- MMA issuer
+    uint32_t ait = 0, wit = 0;
+    if (lane == 0)
+      for (; sched.next(t0, rows); ++tt)
+        mma_tile<kNPkv, kNPkv>(a.skv, split, pipe, B, tmem + (tt & 1u) * kCols, ait, wit, tt);
+    __syncwarp();
+  } else {                                           // ---------------- epilogue (128 threads)
+    const int tid = threadIdx.x;                      // 0..127
+    const int row = tid;
+    while (sched.next_group()) {
+      const int64_t d0 = sched.d0;
+      const int nd = sched.nd;
+      for (int x = tid; x < kMaxDpb * kMaxModel; x += kBM) {
+        const int d = x / kMaxModel, c = x % kMaxModel;
+        s_q[d][c] = (d < nd && c < dm) ? a.qbuf[(d0 + d) * kQLd + c] : 0.f;
+        s_r[d][c] = 0.f;
       }
-      __syncthreads();
-      mainloop<kNPkv, kNPkv>(a.skv, a.split, pipe, a.wkv, w_bar, mma_bar, tmem, it, rd, rows,
-                             s_omega, s_phi, a.table);
-      // ---- epilogue: TMEM lane = row; warp half selects columns [cb, ce)
-      const int row = q4 * 32 + lane;
-      const int d = row < rows ? rd.rdst[row] : -1;
-      const uint32_t ta = tmem + ((uint32_t)(q4 * 32) << 16);
-      float v[64];
-      tmem_ld32(ta + cb, &v[0]);        // K columns
-      tmem_ld32(ta + cb + 32, &v[32]);
-      tmem_wait_ld();
-      float p0 = 0.f, p1 = 0.f;
-      if (d >= 0) {
+      if (tid < kMaxDpb * 2) {
+        s_m[tid >> 1][tid & 1] = -INFINITY;
+        s_l[tid >> 1][tid & 1] = 0.f;
+      }
+      if (tid <= nd) s_seg[tid] = a.seg_ptr[d0 + tid];
+      named_bar(kBarEpi, kBM);
+      for (; sched.next_tile(t0, rows); ++tt) {
+        const int64_t c0 = t0;
+        const uint32_t ab = tt & 1u, ds = tt % kDSlots;
+        mbar_wait(&B.dfull[ds], (tt / kDSlots) & 1u);
+        mbar_wait(&B.tfull[ab], (tt >> 1) & 1u);
+        tc_fence_after();
+        const int d = rd[ds].rdst[row];
+        warp_arrive(&B.dempty[ds]);
+        const uint32_t ta = tmem + ab * kCols + ((uint32_t)(warp * 32) << 16);
+        float v[32];
+        // S10: logits per head from the K columns [0, dm)
+        float p0 = 0.f, p1 = 0.f;
+#pragma unroll 1
+        for (int cq = 0; cq < 4; ++cq) {
+          tmem_ld32(ta + cq * 32, v);
+          tmem_wait_ld();
+          if (d >= 0) {
 #pragma unroll
-        for (int j = 0; j < 64; ++j) {
-          const int col = cb + j;
-          if (col < ce) {
-            const float pr = s_q[d][col] * (v[j] + s_bias[col]);
-            if (col / dh == 0) p0 += pr; else p1 += pr;
+            for (int j = 0; j < 32; ++j) {
+              const int col = cq * 32 + j;
+              if (col < dm) {
+                const float pr = s_q[d][col] * (v[j] + s_bias[col]);
+                if (col < dh) p0 += pr; else p1 += pr;
+              }
+            }
           }
         }
-      }
-      s_lpart[half][row][0] = p0;
-      s_lpart[half][row][1] = p1;
-      __syncthreads();
-      if (tid < kBM && tid < rows) {   // S10: logits + LeakyReLU
-        float s0 = (s_lpart[0][tid][0] + s_lpart[1][tid][0]) * P.logit_scale;
-        float s1 = (s_lpart[0][tid][1] + s_lpart[1][tid][1]) * P.logit_scale;
-        if (P.leaky_slope >= 0.f) {
-          s0 = s0 < 0.f ? s0 * P.leaky_slope : s0;
-          s1 = s1 < 0.f ? s1 * P.leaky_slope : s1;
-        }
-        s_logit[tid][0] = s0;
-        s_logit[tid][1] = s1;
-      }
-      __syncthreads();
-      if (tid < nd * H) {               // S11: online segmented softmax statistics
-        const int dd = tid / H, h = tid % H;
-        const int64_t a0 = s_seg[dd] > c0 ? s_seg[dd] : c0;
-        const int64_t a1 = s_seg[dd + 1] < c0 + rows ? s_seg[dd + 1] : c0 + rows;
-        float sc = 1.f;
-        if (a0 < a1) {
-          float mc = -INFINITY;
-          for (int64_t e = a0; e < a1; ++e) mc = fmaxf(mc, s_logit[e - c0][h]);
-          const float mo = s_m[dd][h];
-          const float mn = fmaxf(mo, mc);
-          sc = (mo == -INFINITY) ? 0.f : expf(mo - mn);
-          float l = s_l[dd][h] * sc;
-          for (int64_t e = a0; e < a1; ++e) {
-            const float pe = expf(s_logit[e - c0][h] - mn);
-            s_p[e - c0][h] = pe;
-            l += pe;
+        if (d >= 0) {
+          float s0 = p0 * P.logit_scale, s1 = p1 * P.logit_scale;
+          if (P.leaky_slope >= 0.f) {
+            s0 = s0 < 0.f ? s0 * P.leaky_slope : s0;
+            s1 = s1 < 0.f ? s1 * P.leaky_slope : s1;
           }
-          s_m[dd][h] = mn;
-          s_l[dd][h] = l;
+          s_logit[row][0] = s0;
+          s_logit[row][1] = s1;
         }
-        s_sc[dd][h] = sc;
-      }
-      __syncthreads();
-      tmem_ld32(ta + dm + cb, &v[0]);    // V columns
-      tmem_ld32(ta + dm + cb + 32, &v[32]);
-      tmem_wait_ld();
-      if (row < rows) {
+        named_bar(kBarEpi, kBM);
+        // S11: online segmented softmax statistics, one thread per (dst, head)
+        if (tid < nd * H) {
+          const int dd = tid / H, h = tid % H;
+          const int64_t a0 = s_seg[dd] > c0 ? s_seg[dd] : c0;
+          const int64_t a1 = s_seg[dd + 1] < c0 + rows ? s_seg[dd + 1] : c0 + rows;
+          float sc = 1.f;
+          if (a0 < a1) {
+            float mc = -INFINITY;
+            for (int64_t e = a0; e < a1; ++e) mc = fmaxf(mc, s_logit[e - c0][h]);
+            const float mo = s_m[dd][h];
+            const float mn = fmaxf(mo, mc);
+            sc = (mo == -INFINITY) ? 0.f : expf(mo - mn);
+            float l = s_l[dd][h] * sc;
+            for (int64_t e = a0; e < a1; ++e) {
+              const float pe = expf(s_logit[e - c0][h] - mn);
+              s_p[e - c0][h] = pe;
+              l += pe;
+            }
+            s_m[dd][h] = mn;
+            s_l[dd][h] = l;
+          }
+          s_sc[dd][h] = sc;
+        }
+        named_bar(kBarEpi, kBM);
+        // S12: r = r * sc + sum_rows p * v, 32 V columns at a time (fixed order)
+#pragma unroll 1
+        for (int cq = 0; cq < 4; ++cq) {
+          tmem_ld32(ta + dm + cq * 32, v);
+          tmem_wait_ld();
+          if (d >= 0) {
 #pragma unroll
-        for (int j = 0; j < 64; ++j) {
-          const int col = cb + j;
-          if (col < ce) s_pv[row * pv_ld + col] = s_p[row][col / dh] * (v[j] + s_bias[dm + col]);
+            for (int j = 0; j < 32; ++j) {
+              const int col = cq * 32 + j;
+              s_pv[row][j] = col < dm ? s_p[row][col < dh ? 0 : 1] * (v[j] + s_bias[dm + col]) : 0.f;
+            }
+          }
+          named_bar(kBarEpi, kBM);
+          for (int x = tid; x < nd * 32; x += kBM) {
+            const int dd = x >> 5, j = x & 31, col = cq * 32 + j;
+            if (col >= dm) continue;
+            const int64_t a0 = s_seg[dd] > c0 ? s_seg[dd] : c0;
+            const int64_t a1 = s_seg[dd + 1] < c0 + rows ? s_seg[dd + 1] : c0 + rows;
+            if (a0 >= a1) continue;
+            float acc = s_r[dd][col] * s_sc[dd][col < dh ? 0 : 1];
+            for (int64_t e = a0; e < a1; ++e) acc += s_pv[e - c0][j];
+            s_r[dd][col] = acc;
+          }
+          named_bar(kBarEpi, kBM);
         }
+        tc_fence_before();
+        warp_arrive(&B.tempty[ab]);
       }
-      __syncthreads();
-      // S12: r = r * sc + sum over this chunk's rows (fixed order -> deterministic)
-      for (int x = tid; x < nd * dm; x += blockDim.x) {
+      // normalise; empty segment -> 0 (R19)
+      for (int x = tid; x < nd * dm; x += kBM) {
         const int dd = x / dm, col = x % dm;
-        const int64_t a0 = s_seg[dd] > c0 ? s_seg[dd] : c0;
-        const int64_t a1 = s_seg[dd + 1] < c0 + rows ? s_seg[dd + 1] : c0 + rows;
-        if (a0 >= a1) continue;
-        float acc = s_r[dd][col] * s_sc[dd][col / dh];
-        for (int64_t e = a0; e < a1; ++e) acc += s_pv[(e - c0) * pv_ld + col];
-        s_r[dd][col] = acc;
+        const float l = s_l[dd][col < dh ? 0 : 1];
+        a.rbuf[(d0 + dd) * kQLd + col] = l > 0.f ? s_r[dd][col] / l : 0.f;
       }
-      fence_proxy_async_smem();   // generic s_pv accesses before the next async-proxy writes
-      tc_fence_before();
-      __syncthreads();
+      named_bar(kBarEpi, kBM);
     }
-    // normalise (empty segment -> 0, R19)
-    for (int x = tid; x < nd * dm; x += blockDim.x) {
-      const int dd = x / dm, col = x % dm;
-      const float l = s_l[dd][col / dh];
-      a.rbuf[(d0 + dd) * kQLd + col] = l > 0.f ? s_r[dd][col] / l : 0.f;
-    }
-    __syncthreads();
   }
-  epilogue_teardown<256>(tmem);
+  ws_teardown(tmem, 2 * kCols);
+}
+
+}  // namespace tca
+
+// ------------------------------------------------------------------ host side
+namespace tca {
+
+struct PackedLayout {
+  size_t oq, okv, oo, total;
+};
+
+static PackedLayout packed_layout(const tgl_attn_params* P) {
+  PackedLayout L;
+  WsLayout W;
+  const Seg3 sq = make_seg3(P->d_hdst, 0, P->d_t);
+  const Seg3 skv = make_seg3(P->d_hsrc, P->d_e, P->d_t);
+  const Seg3 so = make_seg3(P->d_model, P->d_hdst, 0);
+  L.oq = W.take((size_t)sq.nchunks * 2 * kNPq * 128);
+  L.okv = W.take((size_t)skv.nchunks * 2 * kNPkv * 128);
+  L.oo = W.take((size_t)so.nchunks * 2 * kNPq * 128);
+  L.total = W.off;
+  return L;
+}
+
+static tgl_status launch_pack(const tgl_attn_params* P, uint8_t* base, cudaStream_t s) {
+  const PackedLayout L = packed_layout(P);
+  const Seg3 sq = make_seg3(P->d_hdst, 0, P->d_t);
+  const Seg3 skv = make_seg3(P->d_hsrc, P->d_e, P->d_t);
+  const Seg3 so = make_seg3(P->d_model, P->d_hdst, 0);
+  PackJob jq{P->Wq, nullptr, P->d_model, P->d_model, kNPq, P->d_hdst + P->d_t, sq, base + L.oq};
+  PackJob jkv{P->Wk, P->Wv, P->d_model, 2 * P->d_model, kNPkv, P->d_hsrc + P->d_e + P->d_t, skv,
+              base + L.okv};
+  PackJob jo{P->Wo, nullptr, P->d_out, P->d_out, kNPq, P->d_model + P->d_hdst, so, base + L.oo};
+  pack_weights_kernel<<<dim3(64, 3), 256, 0, s>>>(jq, jkv, jo);
+  return launch_check("pack_weights");
 }
 
 }  // namespace tca
 
 // host entry used by tgl_tblock_attn (attn.cu) for TGL_FP32 / TGL_BF16
 size_t tc_attn_ws_bytes(const tgl_attn_params* P, int64_t n_dst_max, size_t* o_q, size_t* o_r,
-                        size_t* o_wq, size_t* o_wkv, size_t* o_wo) {
+                        size_t* o_pack) {
   using namespace tca;
   WsLayout L;
   const int64_t nrows = n_dst_max > 0 ? n_dst_max : 1;
   *o_q = L.take(sizeof(float) * kQLd * nrows);
   *o_r = L.take(sizeof(float) * kQLd * nrows);
-  const Seg3 sq = make_seg3(P->d_hdst, 0, P->d_t);
-  const Seg3 skv = make_seg3(P->d_hsrc, P->d_e, P->d_t);
-  const Seg3 so = make_seg3(P->d_model, P->d_hdst, 0);
-  *o_wq = L.take((size_t)sq.nchunks * 2 * kNPq * 128);
-  *o_wkv = L.take((size_t)skv.nchunks * 2 * kNPkv * 128);
-  *o_wo = L.take((size_t)so.nchunks * 2 * kNPq * 128);
+  *o_pack = L.take(P->packed ? 0 : packed_layout(P).total);
   return L.off;
 }
 
 bool tc_attn_supported(const tgl_attn_params* P) {
   return P->d_model == 100 && P->d_out == 100 && P->n_heads >= 1 && P->n_heads <= 2 &&
-         P->d_t <= 256;
+         P->d_t <= 256 && P->d_hdst >= 0 && P->d_hsrc >= 0 && P->d_e >= 0;
 }
 
 tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int64_t* n_dst_dev,
@@ -633,9 +831,13 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
                           const float* edge_t, const float* table, int64_t window,
                           int32_t max_seg, float* out, void* ws, cudaStream_t s) {
   using namespace tca;
-  size_t o_q, o_r, o_wq, o_wkv, o_wo;
-  tc_attn_ws_bytes(P, n_dst_max, &o_q, &o_r, &o_wq, &o_wkv, &o_wo);
+  size_t o_q, o_r, o_pack;
+  tc_attn_ws_bytes(P, n_dst_max, &o_q, &o_r, &o_pack);
   char* w = static_cast<char*>(ws);
+  uint8_t* pk = P->packed ? const_cast<uint8_t*>(static_cast<const uint8_t*>(P->packed))
+                          : reinterpret_cast<uint8_t*>(w + o_pack);
+  if (!P->packed) TGL_TRY(launch_pack(P, pk, s));   // otherwise packed once by tgl_attn_pack
+  const PackedLayout PL = packed_layout(P);
   Args a;
   a.P = *P;
   a.n_dst_max = n_dst_max;
@@ -658,9 +860,9 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
   a.out = out;
   a.qbuf = reinterpret_cast<float*>(w + o_q);
   a.rbuf = reinterpret_cast<float*>(w + o_r);
-  a.wq = reinterpret_cast<const uint8_t*>(w + o_wq);
-  a.wkv = reinterpret_cast<const uint8_t*>(w + o_wkv);
-  a.wo = reinterpret_cast<const uint8_t*>(w + o_wo);
+  a.wq = pk + PL.oq;
+  a.wkv = pk + PL.okv;
+  a.wo = pk + PL.oo;
   a.sq = make_seg3(P->d_hdst, 0, P->d_t);
   a.skv = make_seg3(P->d_hsrc, P->d_e, P->d_t);
   a.so = make_seg3(P->d_model, P->d_hdst, 0);
@@ -672,23 +874,14 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
   a.dpb = dpb < 1 ? 1 : (dpb > kMaxDpb ? kMaxDpb : dpb);
   a.split = P->precision == TGL_FP32 ? 1 : 0;
 
-  // 1. pack weights (bf16 hi/lo, padded K, pre-swizzled)
-  PackJob jq{P->Wq, nullptr, P->d_model, P->d_model, kNPq, P->d_hdst + P->d_t, a.sq,
-             reinterpret_cast<uint8_t*>(w + o_wq)};
-  PackJob jkv{P->Wk, P->Wv, P->d_model, 2 * P->d_model, kNPkv, P->d_hsrc + P->d_e + P->d_t,
-              a.skv, reinterpret_cast<uint8_t*>(w + o_wkv)};
-  PackJob jo{P->Wo, nullptr, P->d_out, P->d_out, kNPq, P->d_model + P->d_hdst, a.so,
-             reinterpret_cast<uint8_t*>(w + o_wo)};
-  pack_weights_kernel<<<dim3(64, 3), 256, 0, s>>>(jq, jkv, jo);
-  TGL_TRY(launch_check("pack_weights"));
-
-  const int smem_q = Smem<kNPq>::kPipe + 1024;
-  const int smem_kv = Smem<kNPkv>::kPipe + 1024;
+  const int smem_q = Pipe<kNPq>::kBytes + 1024;
+  const int smem_kv = Pipe<kNPkv>::kBytes + 1024 + kKvEpiBytes;
   static bool attr_done = false;   // cached cudaFuncSetAttribute (idempotent)
   if (!attr_done) {
-    TGL_TRY(cuda_check(cudaFuncSetAttribute(q_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                            smem_q), "attr q"));
-    TGL_TRY(cuda_check(cudaFuncSetAttribute(ffn_kernel,
+    TGL_TRY(cuda_check(cudaFuncSetAttribute(dense_kernel<false>,
+                                            cudaFuncAttributeMaxDynamicSharedMemorySize, smem_q),
+                       "attr q"));
+    TGL_TRY(cuda_check(cudaFuncSetAttribute(dense_kernel<true>,
                                             cudaFuncAttributeMaxDynamicSharedMemorySize, smem_q),
                        "attr ffn"));
     TGL_TRY(cuda_check(cudaFuncSetAttribute(kv_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -697,14 +890,37 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
   }
   const int64_t tiles = ceil_div(n_dst_max, kBM);
   const unsigned gq = (unsigned)(tiles < kNumSMs ? tiles : kNumSMs);
-  q_kernel<<<gq, kThreads, smem_q, s>>>(a);
-  TGL_TRY(launch_check("tc q_kernel"));
+  dense_kernel<false><<<gq, kWsThreads, smem_q, s>>>(a);
+  TGL_TRY(launch_check("tc q kernel"));
   const int64_t groups = ceil_div(n_dst_max, a.dpb);
   const unsigned gkv = (unsigned)(groups < kNumSMs ? groups : kNumSMs);
-  kv_kernel<<<gkv, kThreads, smem_kv, s>>>(a);
-  TGL_TRY(launch_check("tc kv_kernel"));
-  ffn_kernel<<<gq, kThreads, smem_q, s>>>(a);
-  return launch_check("tc ffn_kernel");
+  kv_kernel<<<gkv, kWsThreads, smem_kv, s>>>(a);
+  TGL_TRY(launch_check("tc kv kernel"));
+  dense_kernel<true><<<gq, kWsThreads, smem_q, s>>>(a);
+  return launch_check("tc ffn kernel");
 }
 
 }  // namespace tgl
+
+using namespace tgl;
+
+extern "C" size_t tgl_attn_packed_bytes(const tgl_attn_params* P) {
+  if (P == nullptr || !tc_attn_supported(P)) return 0;
+  return tca::packed_layout(P).total;
+}
+
+extern "C" tgl_status tgl_attn_pack(const tgl_attn_params* P, void* packed, size_t bytes,
+                                    void* stream) {
+  TGL_REQUIRE(P != nullptr && packed != nullptr, "null pointer");
+  if (!tc_attn_supported(P)) {
+    set_error("tensor-core path needs d_model == d_out == 100, n_heads <= 2, d_t <= 256");
+    return TGL_EUNSUPPORTED;
+  }
+  TGL_REQUIRE(P->Wq && P->Wk && P->Wv && P->Wo, "null weight");
+  if (bytes < tca::packed_layout(P).total) {
+    set_error("packed buffer too small: %zu < %zu", bytes, tca::packed_layout(P).total);
+    return TGL_EWORKSPACE;
+  }
+  TGL_REQUIRE((reinterpret_cast<uintptr_t>(packed) & 255) == 0, "packed must be 256-aligned");
+  return tca::launch_pack(P, static_cast<uint8_t*>(packed), as_stream(stream));
+}

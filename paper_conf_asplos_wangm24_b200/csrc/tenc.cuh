@@ -1,7 +1,8 @@
 // tenc.cuh -- the time encoder Phi_j(dt) = cos(omega_j * dt + phi_j), eq (8) P:126,
 // evaluated like the paper's fp32 code `torch.cos(ts * w + b)` (reading R10):
 // round-to-nearest fp32 multiply, round-to-nearest fp32 add (no FMA contraction),
-// accurate cosf of that argument (this file must not be built with fast-math).
+// then an accurate cosine of that fp32 argument (this file must not be built with
+// fast-math).
 #pragma once
 #include "common.cuh"
 

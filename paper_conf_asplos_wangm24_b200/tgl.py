@@ -24,7 +24,8 @@ PRECISION = {"fp32": FP32, "bf16": BF16, "fp32_simt": FP32_SIMT}
 
 SYMBOLS = ["tgl_version", "tgl_status_string", "tgl_last_error", "tgl_build_tcsr",
            "tgl_batch_roots", "tgl_dedup", "tgl_sample", "tgl_next_block",
-           "tgl_time_precompute", "tgl_time_encode", "tgl_tblock_attn", "tgl_gather_rows"]
+           "tgl_time_precompute", "tgl_time_encode", "tgl_tblock_attn", "tgl_gather_rows",
+           "tgl_attn_packed_bytes", "tgl_attn_pack"]
 
 
 class TGLError(RuntimeError):
@@ -53,11 +54,14 @@ def _load():
         "tgl_tblock_attn": [vp, i64, vp, vp, vp, vp, vp, i64, vp, vp, vp, i64, vp, vp, i64, vp,
                             vp, i64, i32, vp, vp, sz, vp],
         "tgl_gather_rows": [i64, vp, vp, vp, i64, i32, vp, i64, vp],
+        "tgl_attn_pack": [vp, vp, C.c_size_t, vp],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
         f.argtypes = args
         f.restype = i32
+    lib.tgl_attn_packed_bytes.argtypes = [vp]
+    lib.tgl_attn_packed_bytes.restype = C.c_size_t
     return lib
 
 
@@ -235,16 +239,19 @@ class AttnParamsC(C.Structure):
                 ("ln_beta", C.c_void_p), ("ln_eps", C.c_float),
                 ("omega", C.c_void_p), ("phi", C.c_void_p),
                 ("leaky_slope", C.c_float), ("logit_scale", C.c_float),
-                ("precision", C.c_int32)]
+                ("precision", C.c_int32), ("packed", C.c_void_p)]
 
 
 _WEIGHTS = ("Wq", "bq", "Wk", "bk", "Wv", "bv", "Wo", "bo", "ln_gamma", "ln_beta", "omega", "phi")
 
 
 class AttnParams:
-    """Device copies of one layer's weights + the host struct of the ABI."""
+    """Device copies of one layer's weights + the host struct of the ABI.
 
-    def __init__(self, p: dict, device=None, precision="fp32"):
+    pack=True runs tgl_attn_pack once (tensor-core weight layout) so that every
+    tgl_tblock_attn call streams the packed weights instead of re-packing them."""
+
+    def __init__(self, p: dict, device=None, precision="fp32", pack: bool = False):
         device = device or torch.device("cuda")
         self.host = p
         self.t = {k: torch.as_tensor(p[k], dtype=torch.float32).contiguous().to(device)
@@ -258,7 +265,14 @@ class AttnParams:
                                   *[_p(self.t[k]) for k in _WEIGHTS[:10]], float(p["ln_eps"]),
                                   _p(self.t["omega"]), _p(self.t["phi"]),
                                   float(p["leaky_slope"]), float(p["logit_scale"]),
-                                  self.precision)
+                                  self.precision, None)
+        self.packed = None
+        if pack and self.precision != FP32_SIMT:
+            nb = _lib.tgl_attn_packed_bytes(C.byref(self.struct))
+            self.packed = torch.empty(max(nb, 256), dtype=torch.uint8, device=device)
+            _check(_lib.tgl_attn_pack(C.byref(self.struct), _p(self.packed), nb, _s()),
+                   "tgl_attn_pack")
+            self.struct.packed = _p(self.packed)
 
 
 def tblock_attn(P: AttnParams, seg_ptr, dst_t, hdst, hdst_idx, hsrc, hsrc_idx, efeat, eid,

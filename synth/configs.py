@@ -65,8 +65,10 @@ CONFIGS = {
     "WIKI": Config("WIKI", 8227, 1000, 157_474, 2_700_000, 172, 172, 600, 1, 10,
                    "recent", False, False, 0.8, 1.0, 0.5, True, seeds=_seeds(0)),
     # configs[1]: REDDIT-shaped, 2-layer, uniform 10, dedup + time-precompute on
+    # precompute window 2^22 covers every integer dt <= max(t) = 2.7e6 (reading R11)
     "REDDIT": Config("REDDIT", 10_000, 984, 672_447, 2_700_000, 172, 172, 600, 2, 10,
-                     "uniform", True, True, 0.8, 1.0, 0.5, True, seeds=_seeds(1)),
+                     "uniform", True, True, 0.8, 1.0, 0.5, True, window=1 << 22,
+                     seeds=_seeds(1)),
     # configs[2]: LastFM-shaped, heavy skew, 2-layer, recent 20, batch 2000
     "LASTFM": Config("LASTFM", 980, 1000, 1_293_103, 140_000_000, 128, 128, 2000, 2, 20,
                      "recent", False, False, 1.0, 1.3, 0.5, True, seeds=_seeds(2)),

@@ -206,7 +206,7 @@ def test_attention_vs_oracle(T, precision, n_dst, kmax, d_h, d_e, long_every):
     p, seg, dst_t, nfeat, dn, sn, ef, eid, et = attn_case(rng, n_dst, kmax, d_h, d_e,
                                                           long_every=long_every)
     exp = oracle.tblock_attn(p, seg, dst_t, nfeat, dn, nfeat, sn, ef, eid, et)
-    P = T.AttnParams(p, precision=precision)
+    P = T.AttnParams(p, precision=precision, pack=(n_dst % 2 == 1))
     tab = T.time_precompute(65536, P.t["omega"], P.t["phi"])
     for table in (None, tab):
         got = T.tblock_attn(P, cu(seg), cu(dst_t), cu(nfeat), cu(dn), cu(nfeat), cu(sn),
