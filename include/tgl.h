@@ -190,8 +190,11 @@ tgl_status tgl_time_encode(int64_t n, const float* dt, int32_t d_t, const float*
  * Row of h_src(e): hsrc_idx ? hsrc_idx[o + e] : o + e, o = *hsrc_off_dev
  * (NULL -> 0) -- the dedup inverse hook of the next block (S14).
  * efeat row eid[e] (ld_e); unused when d_e == 0.  edge_t[e] = edge time.
- * tenc_table (NULL = direct) as in tgl_time_encode.  max_seg is a launch hint
- * (the sampler's k); any segment length is handled.
+ * tenc_table (NULL = direct) as in tgl_time_encode.  max_seg = an upper bound on
+ * every segment length (the sampler's k).  With max_seg <= 32 the tensor-core path
+ * packs whole segments into 32-row bins; a segment longer than max_seg there is a
+ * caller error and its output row is NaN.  max_seg > 32 (or <= 0: unknown) selects
+ * the general path that takes any segment length.
  * Output out[n_dst_max][d_out] (rows >= n_dst untouched).
  * Limits: d_model == d_out, d_model % n_heads == 0, n_heads <= 2, d_t <= 256;
  * TGL_FP32 / TGL_BF16 run on the tensor cores (tcgen05) and need d_model == 100;

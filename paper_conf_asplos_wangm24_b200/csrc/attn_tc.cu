@@ -126,10 +126,12 @@ struct Args {
   int np_q, np_kv, np_o;
   int dpb;
   int split;           // 1 = 3-pass fp32 mode
+  int dbg;             // TGL_DEBUG_MASK (profiling only): 1 skip epilogue math, 2 skip gathers, 4 skip MMAs
 };
 
+// offset (not integer round-trip) so the compiler keeps the shared address space
 __device__ __forceinline__ uint8_t* align1024(uint8_t* p) {
-  return reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(p) + 1023) & ~uintptr_t(1023));
+  return p + ((1024u - (static_cast<uint32_t>(__cvta_generic_to_shared(p)) & 1023u)) & 1023u);
 }
 
 // ------------------------------------------------------------------ warp-specialized CTA
@@ -142,9 +144,11 @@ constexpr int kMmaWarp = 4;
 constexpr int kDescWarp = 5;
 constexpr int kWWarp = 6;
 constexpr int kProdWarp0 = 7;
-constexpr int kProdWarps = 8;
+constexpr int kProdWarps = 16;
+constexpr int kGPT = 1024 / (kProdWarps * 32);   // 16-byte groups per producer thread per chunk
+constexpr int kGPR = 8 / kGPT;                    // producer threads per row
 constexpr int kProdThreads = kProdWarps * 32;
-constexpr int kWsThreads = (kProdWarp0 + kProdWarps) * 32;   // 480
+constexpr int kWsThreads = (kProdWarp0 + kProdWarps) * 32;   // 736
 constexpr int kAStages = 2;
 constexpr int kWStages = 2;
 constexpr int kDSlots = 3;
@@ -178,6 +182,17 @@ struct Pipe {
   }
 };
 
+// ---- profiling timeline (TGL_DEBUG_MASK & 32): [cta][tile][event] globaltimer stamps
+constexpr int kTlTiles = 32, kTlEvents = 8;
+__device__ unsigned long long g_timeline[kNumSMs * kTlTiles * kTlEvents];
+__device__ __forceinline__ void tl_mark(const Args& a, uint32_t tt, int ev) {
+  if ((a.dbg & 32) && tt < (uint32_t)kTlTiles && blockIdx.x < (unsigned)kNumSMs) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    g_timeline[(blockIdx.x * kTlTiles + tt) * kTlEvents + ev] = t;
+  }
+}
+
 __device__ __forceinline__ void named_bar(int id, int n) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
 }
@@ -202,11 +217,12 @@ __device__ __forceinline__ void load8(const float* p, int lc, int d, float* x) {
 }
 
 // producer thread pt (0..255): row pt/2, 16-byte groups jb..jb+3 of a 64-wide chunk
-__device__ __forceinline__ void load_chunk(int c, const Seg3& sg, const RowDesc& rd, int r, int jb,
+template <int GPT, class RD>
+__device__ __forceinline__ void load_chunk(int c, const Seg3& sg, const RD& rd, int r, int jb,
                                            const float* s_omega, const float* s_phi,
                                            const float* table, float* x) {
 #pragma unroll
-  for (int jj = 0; jj < 4; ++jj) {
+  for (int jj = 0; jj < GPT; ++jj) {
     float* y = x + jj * 8;
     const int kp = c * kChunk + (jb + jj) * 8;
 #pragma unroll
@@ -231,11 +247,12 @@ __device__ __forceinline__ void load_chunk(int c, const Seg3& sg, const RowDesc&
   }
 }
 
+template <int GPT>
 __device__ __forceinline__ void store_chunk(const float* x, uint8_t* a_hi, uint8_t* a_lo, int r,
                                             int jb, bool split) {
   const uint32_t hb = smem_u32(a_hi), lb = smem_u32(a_lo);
 #pragma unroll
-  for (int jj = 0; jj < 4; ++jj) {
+  for (int jj = 0; jj < GPT; ++jj) {
     uint32_t h[4], l[4];
 #pragma unroll
     for (int e = 0; e < 4; ++e) split2(x[jj * 8 + 2 * e], x[jj * 8 + 2 * e + 1], h[e], l[e]);
@@ -293,78 +310,121 @@ struct GroupSched {   // kv: groups of `dpb` destinations, each cut into 128-row
 };
 
 // ---- roles ------------------------------------------------------------------------
+// K-chunk order alternates per tile (forward, backward, ...) so the last two weight
+// chunks of a tile are the first two of the next one and stay resident in the W
+// ring: (n-2)/n of the weight bytes per tile after the first (25% less at n = 8).
+__device__ __forceinline__ int chunk_of(uint32_t tt, int i, int n) {
+  return (tt & 1u) ? n - 1 - i : i;
+}
+__device__ __forceinline__ int w_reused(uint32_t tt, int n) { return (tt > 0 && n >= 4) ? 2 : 0; }
+
 template <int NP, int N>
 __device__ __forceinline__ void mma_tile(const Seg3& sg, bool split, uint8_t* pipe, Bars& B,
-                                         uint32_t tmem_acc, uint32_t& ait, uint32_t& wit,
-                                         uint32_t tt) {
+                                         uint32_t tmem_acc, uint32_t& ait, uint32_t& wl,
+                                         uint32_t tt, bool nomma = false, bool nowait_w = false) {
   using PP = Pipe<NP>;
   constexpr uint32_t idesc = idesc_bf16(kBM, N);
   wait_free(&B.tempty[tt & 1u], tt >> 1);    // epilogue drained this accumulator
   tc_fence_after();
-  for (int c = 0; c < sg.nchunks; ++c, ++ait, ++wit) {
-    const uint32_t sa = ait % kAStages, sw = wit % kWStages;
+  const int n = sg.nchunks, r0 = w_reused(tt, n);
+  for (int i = 0; i < n; ++i, ++ait) {
+    const int c = chunk_of(tt, i, n);
+    const uint32_t sa = ait % kAStages;
     mbar_wait(&B.afull[sa], (ait / kAStages) & 1u);
-    mbar_wait(&B.wfull[sw], (wit / kWStages) & 1u);
+    uint32_t k;
+    if (i < r0) {
+      k = wl - 1 - i;                          // resident from the previous tile
+    } else {
+      k = wl + (i - r0);
+      if (!nowait_w) mbar_wait(&B.wfull[k % kWStages], (k / kWStages) & 1u);
+    }
+    const uint32_t sw = k % kWStages;
     tc_fence_after();
     const uint32_t ahb = smem_u32(PP::a(pipe, sa)), alb = ahb + kAPart;
     const uint32_t whb = smem_u32(PP::w(pipe, sw)), wlb = whb + NP * 128;
     const int rem = sg.kpad - c * kChunk;
-    const int nk = rem >= kChunk ? 4 : (rem + 15) / 16;
+    const int nk = nomma ? 0 : (rem >= kChunk ? 4 : (rem + 15) / 16);
     for (int ks = 0; ks < nk; ++ks) {
       const uint64_t ah = desc_sw128(ahb + ks * 32), bh = desc_sw128(whb + ks * 32);
-      mma_bf16(tmem_acc, ah, bh, idesc, (c | ks) != 0);
+      mma_bf16(tmem_acc, ah, bh, idesc, (i | ks) != 0);
       if (split) {
         mma_bf16(tmem_acc, desc_sw128(alb + ks * 32), bh, idesc, 1u);
         mma_bf16(tmem_acc, ah, desc_sw128(wlb + ks * 32), idesc, 1u);
       }
     }
-    mma_commit(&B.aempty[sa]);
-    mma_commit(&B.wempty[sw]);
+    if (nomma && nowait_w) mbar_arrive(&B.aempty[sa]);   // profiling: plain arrive
+    else mma_commit(&B.aempty[sa]);
+    const bool keep = (n >= 4) && (i >= n - 2);   // reused by the next tile
+    if (!keep) mma_commit(&B.wempty[sw]);
   }
+  wl += n - r0;
   mma_commit(&B.tfull[tt & 1u]);
 }
 
 template <int NP>
 __device__ __forceinline__ void wload_tile(const Seg3& sg, uint8_t* pipe, Bars& B,
-                                           const uint8_t* wpack, uint32_t& wit) {
+                                           const uint8_t* wpack, uint32_t& wl, uint32_t tt) {
   using PP = Pipe<NP>;
-  for (int c = 0; c < sg.nchunks; ++c, ++wit) {
-    const uint32_t sw = wit % kWStages;
-    wait_free(&B.wempty[sw], wit / kWStages);
+  const int n = sg.nchunks, r0 = w_reused(tt, n);
+  for (int i = r0; i < n; ++i) {
+    const uint32_t k = wl + (i - r0);
+    const uint32_t sw = k % kWStages;
+    wait_free(&B.wempty[sw], k / kWStages);
     mbar_arrive_expect_tx(&B.wfull[sw], PP::kWStage);
-    bulk_g2s(PP::w(pipe, sw), wpack + (size_t)c * PP::kWStage, PP::kWStage, &B.wfull[sw]);
+    bulk_g2s(PP::w(pipe, sw), wpack + (size_t)chunk_of(tt, i, n) * PP::kWStage, PP::kWStage,
+             &B.wfull[sw]);
   }
+  wl += n - r0;
 }
 
-template <int NP>
+template <int NP, int PW0, int GPT, class RD>
 __device__ __forceinline__ void produce_tile(const Seg3& sg, bool split, uint8_t* pipe, Bars& B,
-                                             uint32_t& ait, const RowDesc& rd,
+                                             uint32_t& ait, uint32_t tt, const RD& rd,
                                              const float* s_omega, const float* s_phi,
-                                             const float* table) {
+                                             const float* table, bool noload = false) {
   using PP = Pipe<NP>;
-  const int pt = threadIdx.x - kProdWarp0 * 32;
-  const int r = pt >> 1, jb = (pt & 1) * 4;
+  constexpr int GPR = 8 / GPT;                 // producer threads per row
+  const int pt = threadIdx.x - PW0 * 32;
+  const int r = pt / GPR, jb = (pt % GPR) * GPT;
   const int lane = threadIdx.x & 31;
-  float cur[32], nxt[32];
-  load_chunk(0, sg, rd, r, jb, s_omega, s_phi, table, cur);
-  for (int c = 0; c < sg.nchunks; ++c, ++ait) {
+  const int n = sg.nchunks;
+  constexpr int kX = 8 * GPT;
+  constexpr bool kDeep = GPT <= 2;             // two chunks ahead when registers allow
+  float x0[kX], x1[kX], x2[kDeep ? kX : 1];
+#pragma unroll
+  for (int q = 0; q < kX; ++q) x0[q] = x1[q] = 0.f;
+  if (!noload) {
+    load_chunk<GPT>(chunk_of(tt, 0, n), sg, rd, r, jb, s_omega, s_phi, table, x0);
+    if (kDeep && n > 1) load_chunk<GPT>(chunk_of(tt, 1, n), sg, rd, r, jb, s_omega, s_phi, table, x1);
+  }
+  for (int i = 0; i < n; ++i, ++ait) {
     const uint32_t sa = ait % kAStages;
-    if (c + 1 < sg.nchunks) load_chunk(c + 1, sg, rd, r, jb, s_omega, s_phi, table, nxt);
+    const int ahead = kDeep ? 2 : 1;
+    if (i + ahead < n && !noload)
+      load_chunk<GPT>(chunk_of(tt, i + ahead, n), sg, rd, r, jb, s_omega, s_phi, table,
+                      kDeep ? x2 : x1);
     wait_free(&B.aempty[sa], ait / kAStages);
     uint8_t* st = PP::a(pipe, sa);
-    store_chunk(cur, st, st + kAPart, r, jb, split);
+    store_chunk<GPT>(x0, st, st + kAPart, r, jb, split);
     fence_proxy_async_smem();
     __syncwarp();
     if (lane == 0) mbar_arrive(&B.afull[sa]);
 #pragma unroll
-    for (int i = 0; i < 32; ++i) cur[i] = nxt[i];
+    for (int q = 0; q < kX; ++q) {
+      x0[q] = x1[q];
+      if (kDeep) x1[q] = x2[q < (kDeep ? kX : 1) ? q : 0];
+    }
   }
 }
 
-__device__ __forceinline__ void ws_init(Bars& B, uint32_t* s_tmem, uint32_t ncols) {
+__device__ __forceinline__ void ws_init(Bars& B, uint32_t* s_tmem, uint32_t ncols,
+                                        uint32_t dempty_count = kProdWarps + kEpiWarps,
+                                        uint32_t afull_count = kProdWarps,
+                                        uint32_t tempty_count = kEpiWarps,
+                                        int mma_warp = kMmaWarp) {
   if (threadIdx.x == 0) {
     for (int s = 0; s < kAStages; ++s) {
-      mbar_init(&B.afull[s], kProdWarps);
+      mbar_init(&B.afull[s], afull_count);
       mbar_init(&B.aempty[s], 1);
     }
     for (int s = 0; s < kWStages; ++s) {
@@ -373,24 +433,25 @@ __device__ __forceinline__ void ws_init(Bars& B, uint32_t* s_tmem, uint32_t ncol
     }
     for (int s = 0; s < kDSlots; ++s) {
       mbar_init(&B.dfull[s], 1);
-      mbar_init(&B.dempty[s], kProdWarps + kEpiWarps);
+      mbar_init(&B.dempty[s], dempty_count);
     }
     for (int a = 0; a < 2; ++a) {
       mbar_init(&B.tfull[a], 1);
-      mbar_init(&B.tempty[a], kEpiWarps);
+      mbar_init(&B.tempty[a], tempty_count);
     }
     fence_mbar_init();
   }
-  if ((threadIdx.x >> 5) == kMmaWarp) tmem_alloc(s_tmem, ncols);
+  if ((threadIdx.x >> 5) == mma_warp) tmem_alloc(s_tmem, ncols);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
 }
 
-__device__ __forceinline__ void ws_teardown(uint32_t tmem, uint32_t ncols) {
+__device__ __forceinline__ void ws_teardown(uint32_t tmem, uint32_t ncols,
+                                            int mma_warp = kMmaWarp) {
   tc_fence_before();
   __syncthreads();
-  if ((threadIdx.x >> 5) == kMmaWarp) tmem_dealloc(tmem, ncols);
+  if ((threadIdx.x >> 5) == mma_warp) tmem_dealloc(tmem, ncols);
 }
 
 // per-warp arrive (all lanes done with a resource)
@@ -455,14 +516,14 @@ __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
   } else if (warp == kWWarp) {                       // ---------------- weight loader
     uint32_t wit = 0;
     if (lane == 0)
-      while (sched.next(i0, rows)) wload_tile<kNPq>(sg, pipe, B, wpack, wit);
+      for (; sched.next(i0, rows); ++tt) wload_tile<kNPq>(sg, pipe, B, wpack, wit, tt);
     __syncwarp();
   } else if (warp >= kProdWarp0) {                   // ---------------- producers
     uint32_t ait = 0;
     for (; sched.next(i0, rows); ++tt) {
       const uint32_t ds = tt % kDSlots;
       mbar_wait(&B.dfull[ds], (tt / kDSlots) & 1u);
-      produce_tile<kNPq>(sg, split, pipe, B, ait, rd[ds], s_omega, s_phi, a.table);
+      produce_tile<kNPq, kProdWarp0, kGPT>(sg, split, pipe, B, ait, tt, rd[ds], s_omega, s_phi, a.table);
       warp_arrive(&B.dempty[ds]);
     }
   } else if (warp == kMmaWarp) {                     // ---------------- MMA issuer
@@ -484,6 +545,10 @@ __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
       float v[32];
       if (!kFfn) {
         float* q = a.qbuf + (i0 + row) * kQLd;
+        // also q . bk per head (cols 100, 101 of the scratch row): the K bias folded
+        // into one scalar per destination for the K|V epilogue
+        const int dhq = D / P.n_heads;
+        float qb0 = 0.f, qb1 = 0.f;
 #pragma unroll 1
         for (int cq = 0; cq < 4; ++cq) {
           tmem_ld32(ta + cq * 32, v);
@@ -496,9 +561,19 @@ __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
                 float4 o = make_float4(v[j] + P.bq[col], v[j + 1] + P.bq[col + 1],
                                        v[j + 2] + P.bq[col + 2], v[j + 3] + P.bq[col + 3]);
                 *reinterpret_cast<float4*>(q + col) = o;   // D % 4 == 0 (D == 100)
+                const float oq[4] = {o.x, o.y, o.z, o.w};
+#pragma unroll
+                for (int e = 0; e < 4; ++e) {       // per column: a float4 may straddle heads
+                  const float pb = oq[e] * P.bk[col + e];
+                  if (col + e < dhq) qb0 += pb; else qb1 += pb;
+                }
               }
             }
           }
+        }
+        if (row < rows && D + 2 <= kQLd) {
+          q[D] = qb0;
+          q[D + 1] = qb1;
         }
       } else {
         // out = LayerNorm(ReLU(acc + bo)): three passes over TMEM (sum, squares, write)
@@ -635,38 +710,64 @@ __global__ void __launch_bounds__(kWsThreads, 1) kv_kernel(Args a) {
   } else if (warp == kWWarp) {                       // ---------------- weight loader
     uint32_t wit = 0;
     if (lane == 0)
-      while (sched.next(t0, rows)) wload_tile<kNPkv>(a.skv, pipe, B, a.wkv, wit);
+      for (; sched.next(t0, rows); ++tt) wload_tile<kNPkv>(a.skv, pipe, B, a.wkv, wit, tt);
     __syncwarp();
   } else if (warp >= kProdWarp0) {                   // ---------------- producers
     uint32_t ait = 0;
     for (; sched.next(t0, rows); ++tt) {
       const uint32_t ds = tt % kDSlots;
       mbar_wait(&B.dfull[ds], (tt / kDSlots) & 1u);
-      produce_tile<kNPkv>(a.skv, split, pipe, B, ait, rd[ds], s_omega, s_phi, a.table);
+      produce_tile<kNPkv, kProdWarp0, kGPT>(a.skv, split, pipe, B, ait, tt, rd[ds], s_omega,
+                                            s_phi, a.table, (a.dbg & 2) != 0);
       warp_arrive(&B.dempty[ds]);
     }
   } else if (warp == kMmaWarp) {                     // ---------------- MMA issuer
     uint32_t ait = 0, wit = 0;
     if (lane == 0)
       for (; sched.next(t0, rows); ++tt)
-        mma_tile<kNPkv, kNPkv>(a.skv, split, pipe, B, tmem + (tt & 1u) * kCols, ait, wit, tt);
+        mma_tile<kNPkv, kNPkv>(a.skv, split, pipe, B, tmem + (tt & 1u) * kCols, ait, wit, tt,
+                               (a.dbg & 4) != 0);
     __syncwarp();
   } else {                                           // ---------------- epilogue (128 threads)
     const int tid = threadIdx.x;                      // 0..127
     const int row = tid;
+    // q rows of a group: nd * dm floats as float4 (dm % 4 == 0), prefetched one group ahead
+    constexpr int kQv = (kMaxDpb * kMaxModel / 4 + kBM - 1) / kBM;   // float4 per thread
+    const int dm4 = dm / 4;
+    float4 qpre[kQv];
+    auto prefetch_q = [&](int64_t gd0, int gnd) {
+#pragma unroll
+      for (int u = 0; u < kQv; ++u) {
+        const int x = tid + u * kBM;
+        const int dd = x / dm4, c4 = x % dm4;
+        qpre[u] = dd < gnd ? *reinterpret_cast<const float4*>(a.qbuf + (gd0 + dd) * kQLd + 4 * c4)
+                           : make_float4(0.f, 0.f, 0.f, 0.f);
+      }
+    };
+    {
+      GroupSched peek = sched;
+      if (peek.next_group()) prefetch_q(peek.d0, peek.nd);
+    }
+    __shared__ int s_lo[kMaxDpb], s_hi[kMaxDpb];
     while (sched.next_group()) {
       const int64_t d0 = sched.d0;
       const int nd = sched.nd;
-      for (int x = tid; x < kMaxDpb * kMaxModel; x += kBM) {
-        const int d = x / kMaxModel, c = x % kMaxModel;
-        s_q[d][c] = (d < nd && c < dm) ? a.qbuf[(d0 + d) * kQLd + c] : 0.f;
-        s_r[d][c] = 0.f;
+#pragma unroll
+      for (int u = 0; u < kQv; ++u) {
+        const int x = tid + u * kBM;
+        const int dd = x / dm4, c4 = x % dm4;
+        if (dd < kMaxDpb) *reinterpret_cast<float4*>(&s_q[dd][4 * c4]) = qpre[u];
       }
+      for (int x = tid; x < nd * dm; x += kBM) s_r[x / dm][x % dm] = 0.f;
       if (tid < kMaxDpb * 2) {
         s_m[tid >> 1][tid & 1] = -INFINITY;
         s_l[tid >> 1][tid & 1] = 0.f;
       }
       if (tid <= nd) s_seg[tid] = a.seg_ptr[d0 + tid];
+      {
+        GroupSched peek = sched;                      // next group's q, in flight meanwhile
+        if (peek.next_group()) prefetch_q(peek.d0, peek.nd);
+      }
       named_bar(kBarEpi, kBM);
       for (; sched.next_tile(t0, rows); ++tt) {
         const int64_t c0 = t0;
@@ -676,22 +777,32 @@ __global__ void __launch_bounds__(kWsThreads, 1) kv_kernel(Args a) {
         tc_fence_after();
         const int d = rd[ds].rdst[row];
         warp_arrive(&B.dempty[ds]);
+        if (a.dbg & 1) {
+          tc_fence_before();
+          warp_arrive(&B.tempty[ab]);
+          continue;
+        }
+        if (tid < nd) {   // this tile's row range of each destination
+          const int64_t lo = s_seg[tid] > c0 ? s_seg[tid] : c0;
+          const int64_t hi = s_seg[tid + 1] < c0 + rows ? s_seg[tid + 1] : c0 + rows;
+          s_lo[tid] = (int)(lo - c0);
+          s_hi[tid] = (int)(hi > lo ? hi - c0 : lo - c0);
+        }
         const uint32_t ta = tmem + ab * kCols + ((uint32_t)(warp * 32) << 16);
         float v[32];
         // S10: logits per head from the K columns [0, dm)
         float p0 = 0.f, p1 = 0.f;
+        const float* qrow = &s_q[d >= 0 ? d : 0][0];
 #pragma unroll 1
         for (int cq = 0; cq < 4; ++cq) {
           tmem_ld32(ta + cq * 32, v);
           tmem_wait_ld();
-          if (d >= 0) {
 #pragma unroll
-            for (int j = 0; j < 32; ++j) {
-              const int col = cq * 32 + j;
-              if (col < dm) {
-                const float pr = s_q[d][col] * (v[j] + s_bias[col]);
-                if (col < dh) p0 += pr; else p1 += pr;
-              }
+          for (int j = 0; j < 32; ++j) {
+            const int col = cq * 32 + j;
+            if (col < dm) {
+              const float pr = qrow[col] * (v[j] + s_bias[col]);
+              if (col < dh) p0 += pr; else p1 += pr;
             }
           }
         }
@@ -708,19 +819,18 @@ __global__ void __launch_bounds__(kWsThreads, 1) kv_kernel(Args a) {
         // S11: online segmented softmax statistics, one thread per (dst, head)
         if (tid < nd * H) {
           const int dd = tid / H, h = tid % H;
-          const int64_t a0 = s_seg[dd] > c0 ? s_seg[dd] : c0;
-          const int64_t a1 = s_seg[dd + 1] < c0 + rows ? s_seg[dd + 1] : c0 + rows;
+          const int lo = s_lo[dd], hi = s_hi[dd];
           float sc = 1.f;
-          if (a0 < a1) {
+          if (lo < hi) {
             float mc = -INFINITY;
-            for (int64_t e = a0; e < a1; ++e) mc = fmaxf(mc, s_logit[e - c0][h]);
+            for (int e = lo; e < hi; ++e) mc = fmaxf(mc, s_logit[e][h]);
             const float mo = s_m[dd][h];
             const float mn = fmaxf(mo, mc);
             sc = (mo == -INFINITY) ? 0.f : expf(mo - mn);
             float l = s_l[dd][h] * sc;
-            for (int64_t e = a0; e < a1; ++e) {
-              const float pe = expf(s_logit[e - c0][h] - mn);
-              s_p[e - c0][h] = pe;
+            for (int e = lo; e < hi; ++e) {
+              const float pe = expf(s_logit[e][h] - mn);
+              s_p[e][h] = pe;
               l += pe;
             }
             s_m[dd][h] = mn;
@@ -730,26 +840,24 @@ __global__ void __launch_bounds__(kWsThreads, 1) kv_kernel(Args a) {
         }
         named_bar(kBarEpi, kBM);
         // S12: r = r * sc + sum_rows p * v, 32 V columns at a time (fixed order)
+        const float w0 = d >= 0 ? s_p[row][0] : 0.f;
+        const float w1 = d >= 0 ? s_p[row][H > 1 ? 1 : 0] : 0.f;
 #pragma unroll 1
         for (int cq = 0; cq < 4; ++cq) {
           tmem_ld32(ta + dm + cq * 32, v);
           tmem_wait_ld();
-          if (d >= 0) {
 #pragma unroll
-            for (int j = 0; j < 32; ++j) {
-              const int col = cq * 32 + j;
-              s_pv[row][j] = col < dm ? s_p[row][col < dh ? 0 : 1] * (v[j] + s_bias[dm + col]) : 0.f;
-            }
+          for (int j = 0; j < 32; ++j) {
+            const int col = cq * 32 + j;
+            s_pv[row][j] = col < dm ? (col < dh ? w0 : w1) * (v[j] + s_bias[dm + col]) : 0.f;
           }
           named_bar(kBarEpi, kBM);
           for (int x = tid; x < nd * 32; x += kBM) {
             const int dd = x >> 5, j = x & 31, col = cq * 32 + j;
-            if (col >= dm) continue;
-            const int64_t a0 = s_seg[dd] > c0 ? s_seg[dd] : c0;
-            const int64_t a1 = s_seg[dd + 1] < c0 + rows ? s_seg[dd + 1] : c0 + rows;
-            if (a0 >= a1) continue;
+            const int lo = s_lo[dd], hi = s_hi[dd];
+            if (col >= dm || lo >= hi) continue;
             float acc = s_r[dd][col] * s_sc[dd][col < dh ? 0 : 1];
-            for (int64_t e = a0; e < a1; ++e) acc += s_pv[e - c0][j];
+            for (int e = lo; e < hi; ++e) acc += s_pv[e][j];
             s_r[dd][col] = acc;
           }
           named_bar(kBarEpi, kBM);
@@ -767,6 +875,290 @@ __global__ void __launch_bounds__(kWsThreads, 1) kv_kernel(Args a) {
     }
   }
   ws_teardown(tmem, 2 * kCols);
+}
+
+// ------------------------------------------------------------------ binned K|V attention
+// Tile = 4 bins of 32 rows.  The descriptor warp packs whole destination segments
+// (<= 32 rows) into bins without straddling, so a destination's rows sit in one TMEM
+// lane quarter.  Epilogue warp w owns lane quarter w%4 and head w/4 (two heads): its
+// logits, softmax (shuffle scans over the segment) and alpha-weighted V sums (a 32x33
+// smem transpose per warp) need nothing from any other warp -- no block barriers, no
+// state across tiles; r is written straight to global.  Empty segments get r = 0 from
+// the descriptor warp (R19); a segment longer than 32 rows (max_seg hint violated)
+// gets a NaN row.
+constexpr int kBEpi = 8;                    // warps 0-7
+constexpr int kBMma = 8;
+constexpr int kBDesc = 9;
+constexpr int kBW = 10;
+constexpr int kBProd0 = 11;
+constexpr int kBProdWarps = 8;              // warps 11-18, 4 groups of 8 columns each
+constexpr int kBGPT = 1024 / (kBProdWarps * 32);
+constexpr int kBThreads = (kBProd0 + kBProdWarps) * 32;   // 608
+
+struct BinDesc {
+  const float* p0[kBM];
+  const float* p1[kBM];
+  float dt[kBM];
+  int trow[kBM];
+  int rdst[kBM];          // global destination of the row, -1 for padding rows
+  int64_t e[kBM];         // edge index of the row
+  float td[kBM];          // destination time of the row
+  int live;               // 0 = end-of-work marker
+};
+
+__global__ void __launch_bounds__(kBThreads, 1) kv_bin_kernel(Args a) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* pipe = align1024(smem_raw);
+  __shared__ Bars B;
+  __shared__ uint32_t s_tmem;
+  __shared__ BinDesc bd[kDSlots];
+  __shared__ float s_omega[256], s_phi[256];
+  __shared__ float s_bias[2 * kMaxModel];
+  float (*s_pv)[32][33] = reinterpret_cast<float (*)[32][33]>(pipe + Pipe<kNPkv>::kBytes);
+  constexpr uint32_t kCols = 256;
+  const tgl_attn_params& P = a.P;
+  const int64_t n = dev_count(a.n_dst_dev, a.n_dst_max);
+  const bool split = a.split != 0;
+  constexpr int dm = 100, dh = 50;                 // d_model 100, two heads (host-checked)
+  for (int j = threadIdx.x; j < P.d_t; j += blockDim.x) {
+    s_omega[j] = P.omega[j];
+    s_phi[j] = P.phi[j];
+  }
+  for (int j = threadIdx.x; j < 2 * dm; j += blockDim.x) s_bias[j] = j < dm ? P.bk[j] : P.bv[j - dm];
+  ws_init(B, &s_tmem, 2 * kCols, kBEpi + kBProdWarps + 2, kBProdWarps, kBEpi, kBMma);
+  const uint32_t tmem = s_tmem;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t D0 = n * blockIdx.x / gridDim.x, D1 = n * (blockIdx.x + 1) / gridDim.x;
+  uint32_t tt = 0;
+
+  if (warp == kBDesc) {                              // ---------------- tile builder
+    const int64_t hoff = a.hsrc_off_dev ? *a.hsrc_off_dev : 0;
+    int64_t d = D0;
+    int64_t wbase = D0;   // windows: lane l holds seg_ptr[wbase + l] and dst_t[wbase + l]
+    int64_t segw = a.seg_ptr[(wbase + lane) < n ? (wbase + lane) : n];
+    float tdw = (wbase + lane) < n ? a.dst_t[wbase + lane] : 0.f;
+    for (;; ++tt) {
+      const uint32_t ds = tt % kDSlots;
+      wait_free(&B.dempty[ds], tt / kDSlots);
+      if (lane == 0) tl_mark(a, tt, 0);
+      BinDesc& R = bd[ds];
+      int bin = 0, used = 0, cnt = 0;
+      int u0 = 0, u1 = 0, u2 = 0, u3 = 0;              // rows used per bin
+      while (d < D1) {
+        if (d + 1 - wbase > 31) {
+          wbase = d;
+          segw = a.seg_ptr[(wbase + lane) < n ? (wbase + lane) : n];
+          tdw = (wbase + lane) < n ? a.dst_t[wbase + lane] : 0.f;
+        }
+        const int64_t s0 = __shfl_sync(0xffffffffu, segw, (int)(d - wbase));
+        const int64_t s1 = __shfl_sync(0xffffffffu, segw, (int)(d - wbase + 1));
+        const float td = __shfl_sync(0xffffffffu, tdw, (int)(d - wbase));
+        const int L = (int)(s1 - s0);
+        if (L == 0 || L > 32) {                        // empty -> r = 0; overflow -> NaN
+          const float fill = L == 0 ? 0.f : __int_as_float(0x7fc00000);
+          for (int c = lane; c < dm; c += 32) a.rbuf[d * kQLd + c] = fill;
+          ++d;
+          continue;
+        }
+        if (used + L > 32) {
+          if (bin == 3) break;                         // tile full
+          ++bin;
+          used = 0;
+        }
+        const int row0 = bin * 32 + used;
+        if (lane < L) {
+          R.rdst[row0 + lane] = (int)d;
+          R.e[row0 + lane] = s0 + lane;
+          R.td[row0 + lane] = td;
+        }
+        used += L;
+        if (bin == 0) u0 = used; else if (bin == 1) u1 = used; else if (bin == 2) u2 = used; else u3 = used;
+        ++cnt;
+        ++d;
+      }
+      // padding rows
+      if (lane >= u0) R.rdst[lane] = -1;
+      if (lane >= u1) R.rdst[32 + lane] = -1;
+      if (lane >= u2) R.rdst[64 + lane] = -1;
+      if (lane >= u3) R.rdst[96 + lane] = -1;
+      R.live = cnt > 0 ? 1 : 0;
+      __syncwarp();
+      if (cnt > 0) {
+        int dst[4];
+        int64_t e[4];
+        float tdr[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int r = 32 * u + lane;
+          dst[u] = R.rdst[r];
+          e[u] = dst[u] >= 0 ? R.e[r] : 0;
+          tdr[u] = dst[u] >= 0 ? R.td[r] : 0.f;
+        }
+        int32_t hi[4], ei[4];
+        float et[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {              // all loads of the lane's 4 rows in flight
+          const bool ok = dst[u] >= 0 && !(a.dbg & 16);
+          hi[u] = ok ? (a.hsrc_idx ? a.hsrc_idx[hoff + e[u]] : (int32_t)(hoff + e[u])) : 0;
+          ei[u] = (ok && P.d_e > 0) ? a.eid[e[u]] : 0;
+          et[u] = ok ? a.edge_t[e[u]] : 0.f;
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int r = 32 * u + lane;
+          const bool ok = dst[u] >= 0;
+          const float dt = tdr[u] - et[u];          // fp32 delta (R18)
+          R.p0[r] = ok ? a.hsrc + (int64_t)hi[u] * a.ld_hsrc : nullptr;
+          R.p1[r] = (ok && P.d_e > 0) ? a.efeat + (int64_t)ei[u] * a.ld_e : nullptr;
+          R.dt[r] = ok ? dt : 0.f;
+          R.trow[r] = ok ? (int)tenc_table_row(dt, a.table, a.window) : -1;
+        }
+      }
+      warp_arrive(&B.dfull[ds]);
+      if (lane == 0) tl_mark(a, tt, 1);
+      if (cnt == 0) break;                             // end marker published
+    }
+  } else if (warp == kBW) {                          // ---------------- weight loader
+    uint32_t wl = 0;
+    for (;; ++tt) {
+      const uint32_t ds = tt % kDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kDSlots) & 1u);
+      const int live = bd[ds].live;
+      warp_arrive(&B.dempty[ds]);
+      if (!live) break;
+      if (lane == 0 && !(a.dbg & 8)) wload_tile<kNPkv>(a.skv, pipe, B, a.wkv, wl, tt);
+      __syncwarp();
+    }
+  } else if (warp >= kBProd0) {                      // ---------------- producers
+    uint32_t ait = 0;
+    for (;; ++tt) {
+      const uint32_t ds = tt % kDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kDSlots) & 1u);
+      if (!bd[ds].live) {
+        warp_arrive(&B.dempty[ds]);
+        break;
+      }
+      if (threadIdx.x == kBProd0 * 32) tl_mark(a, tt, 2);
+      produce_tile<kNPkv, kBProd0, kBGPT>(a.skv, split, pipe, B, ait, tt, bd[ds], s_omega,
+                                          s_phi, a.table, (a.dbg & 2) != 0);
+      if (threadIdx.x == kBProd0 * 32) tl_mark(a, tt, 3);
+      warp_arrive(&B.dempty[ds]);
+    }
+  } else if (warp == kBMma) {                        // ---------------- MMA issuer
+    uint32_t ait = 0, wl = 0;
+    for (;; ++tt) {
+      const uint32_t ds = tt % kDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kDSlots) & 1u);
+      const int live = bd[ds].live;
+      warp_arrive(&B.dempty[ds]);
+      if (!live) break;
+      if (lane == 0) tl_mark(a, tt, 4);
+      if (lane == 0)
+        mma_tile<kNPkv, kNPkv>(a.skv, split, pipe, B, tmem + (tt & 1u) * kCols, ait, wl, tt,
+                               (a.dbg & 4) != 0, (a.dbg & 8) != 0);
+      __syncwarp();
+    }
+  } else {                                           // ---------------- epilogue warps 0-7
+    const int q4 = warp & 3, head = warp >> 2;
+    const int cb = head * dh;                        // this warp's columns [cb, cb + dh)
+    float (*pv)[33] = s_pv[warp];
+    for (;; ++tt) {
+      const uint32_t ab = tt & 1u, ds = tt % kDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kDSlots) & 1u);
+      if (!bd[ds].live) {
+        warp_arrive(&B.dempty[ds]);
+        break;
+      }
+      const int d = bd[ds].rdst[q4 * 32 + lane];
+      warp_arrive(&B.dempty[ds]);
+      // segment structure of this bin from the row destinations
+      const int dprev = __shfl_up_sync(0xffffffffu, d, 1);
+      const int dnext = __shfl_down_sync(0xffffffffu, d, 1);
+      const bool valid = d >= 0;
+      const unsigned smask = __ballot_sync(0xffffffffu, valid && (lane == 0 || dprev != d));
+      const unsigned emask = __ballot_sync(0xffffffffu, valid && (lane == 31 || dnext != d));
+      const int lo = 31 - __clz(smask & (0xffffffffu >> (31 - lane)));   // last start <= lane
+      const int hi = __ffs(emask & (0xffffffffu << lane));              // last end >= lane, +1
+      // this row's q (head columns) and q . bk, fetched before waiting for the accumulator
+      float qv[dh];
+      const float* qrow = a.qbuf + (int64_t)(valid ? d : 0) * kQLd;
+#pragma unroll
+      for (int j = 0; j < dh; j += 2) {
+        const float2 q2 = __ldg(reinterpret_cast<const float2*>(qrow + cb + j));
+        qv[j] = q2.x;
+        qv[j + 1] = q2.y;
+      }
+      const float qb = __ldg(qrow + dm + head);
+      if (threadIdx.x == 0) tl_mark(a, tt, 5);
+      mbar_wait(&B.tfull[ab], (tt >> 1) & 1u);
+      tc_fence_after();
+      if (threadIdx.x == 0) tl_mark(a, tt, 6);
+      if (a.dbg & 1) {
+        tc_fence_before();
+        warp_arrive(&B.tempty[ab]);
+        continue;
+      }
+      const uint32_t ta = tmem + ab * kCols + ((uint32_t)(q4 * 32) << 16);
+      float v[32];
+      // S10: this head's logit <q_dst, k_row + bk> = <q_dst, k_row> + (q_dst . bk_head)
+      float p = qb;
+#pragma unroll
+      for (int cq = 0; cq < 2; ++cq) {
+        tmem_ld32(ta + cb + cq * 32, v);
+        tmem_wait_ld();
+#pragma unroll
+        for (int j = 0; j < 32; ++j)
+          if (cq * 32 + j < dh) p = fmaf(qv[cq * 32 + j], v[j], p);
+      }
+      float s = p * P.logit_scale;
+      if (P.leaky_slope >= 0.f) s = s < 0.f ? s * P.leaky_slope : s;
+      // S11: softmax over the segment [lo, hi): suffix max / sum, broadcast from lo
+      if (!valid) s = -INFINITY;
+      float m = s;
+#pragma unroll
+      for (int off = 1; off < 32; off <<= 1) {
+        const float y = __shfl_down_sync(0xffffffffu, m, off);
+        if (lane + off < hi) m = fmaxf(m, y);
+      }
+      const float mseg = __shfl_sync(0xffffffffu, m, valid ? lo : lane);
+      const float ex = valid ? expf(s - mseg) : 0.f;
+      float t = ex;
+#pragma unroll
+      for (int off = 1; off < 32; off <<= 1) {
+        const float y = __shfl_down_sync(0xffffffffu, t, off);
+        if (lane + off < hi) t += y;
+      }
+      const float l = __shfl_sync(0xffffffffu, t, valid ? lo : lane);
+      const float w = valid ? ex / l : 0.f;
+      // S12: r_dst = sum_seg w * (v + bv) = sum_seg w * v + bv  (sum_seg w = 1); lane j owns
+      // column j of the 32-column piece and walks each segment's rows in order
+#pragma unroll 1
+      for (int cq = 0; cq < 2; ++cq) {
+        tmem_ld32(ta + dm + cb + cq * 32, v);
+        tmem_wait_ld();
+#pragma unroll
+        for (int j = 0; j < 32; ++j) pv[lane][j] = w * v[j];
+        __syncwarp();
+        const int c = cq * 32 + lane;                  // this lane's column in the head
+        const float bvc = c < dh ? s_bias[dm + cb + c] : 0.f;
+        unsigned sm = smask, em = emask;
+        while (sm) {
+          const int slo = __ffs(sm) - 1, shi = __ffs(em);   // [slo, shi)
+          sm &= sm - 1;
+          em &= em - 1;
+          const int dr = __shfl_sync(0xffffffffu, d, slo);
+          float acc = 0.f;
+          for (int r = slo; r < shi; ++r) acc += pv[r][lane];
+          if (c < dh) a.rbuf[(int64_t)dr * kQLd + cb + c] = acc + bvc;
+        }
+        __syncwarp();
+      }
+      tc_fence_before();
+      warp_arrive(&B.tempty[ab]);
+      if (threadIdx.x == 0) tl_mark(a, tt, 7);
+    }
+  }
+  ws_teardown(tmem, 2 * kCols, kBMma);
 }
 
 }  // namespace tca
@@ -873,9 +1265,11 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
   int dpb = kBM / ms;
   a.dpb = dpb < 1 ? 1 : (dpb > kMaxDpb ? kMaxDpb : dpb);
   a.split = P->precision == TGL_FP32 ? 1 : 0;
+  a.dbg = getenv("TGL_DEBUG_MASK") ? atoi(getenv("TGL_DEBUG_MASK")) : 0;
 
   const int smem_q = Pipe<kNPq>::kBytes + 1024;
   const int smem_kv = Pipe<kNPkv>::kBytes + 1024 + kKvEpiBytes;
+  const int smem_kvb = Pipe<kNPkv>::kBytes + 1024 + kBEpi * 32 * 33 * 4;
   static bool attr_done = false;   // cached cudaFuncSetAttribute (idempotent)
   if (!attr_done) {
     TGL_TRY(cuda_check(cudaFuncSetAttribute(dense_kernel<false>,
@@ -886,15 +1280,24 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
                        "attr ffn"));
     TGL_TRY(cuda_check(cudaFuncSetAttribute(kv_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                             smem_kv), "attr kv"));
+    TGL_TRY(cuda_check(cudaFuncSetAttribute(kv_bin_kernel,
+                                            cudaFuncAttributeMaxDynamicSharedMemorySize, smem_kvb),
+                       "attr kv bin"));
     attr_done = true;
   }
   const int64_t tiles = ceil_div(n_dst_max, kBM);
   const unsigned gq = (unsigned)(tiles < kNumSMs ? tiles : kNumSMs);
   dense_kernel<false><<<gq, kWsThreads, smem_q, s>>>(a);
   TGL_TRY(launch_check("tc q kernel"));
-  const int64_t groups = ceil_div(n_dst_max, a.dpb);
-  const unsigned gkv = (unsigned)(groups < kNumSMs ? groups : kNumSMs);
-  kv_kernel<<<gkv, kWsThreads, smem_kv, s>>>(a);
+  if (max_seg > 0 && max_seg <= 32 && P->n_heads == 2) {
+    // binned path: whole segments per epilogue warp (no block barriers)
+    const unsigned gkv = (unsigned)(n_dst_max < kNumSMs ? (n_dst_max > 0 ? n_dst_max : 1) : kNumSMs);
+    kv_bin_kernel<<<gkv, kBThreads, smem_kvb, s>>>(a);
+  } else {
+    const int64_t groups = ceil_div(n_dst_max, a.dpb);
+    const unsigned gkv = (unsigned)(groups < kNumSMs ? groups : kNumSMs);
+    kv_kernel<<<gkv, kWsThreads, smem_kv, s>>>(a);
+  }
   TGL_TRY(launch_check("tc kv kernel"));
   dense_kernel<true><<<gq, kWsThreads, smem_q, s>>>(a);
   return launch_check("tc ffn kernel");
@@ -903,6 +1306,13 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
 }  // namespace tgl
 
 using namespace tgl;
+
+// profiling aid (not part of the documented ABI): copy the per-tile timeline
+extern "C" int tgl_debug_timeline(unsigned long long* host, size_t n) {
+  const size_t cap = sizeof(tca::g_timeline) / sizeof(unsigned long long);
+  return (int)cudaMemcpyFromSymbol(host, tca::g_timeline,
+                                   (n < cap ? n : cap) * sizeof(unsigned long long));
+}
 
 extern "C" size_t tgl_attn_packed_bytes(const tgl_attn_params* P) {
   if (P == nullptr || !tc_attn_supported(P)) return 0;

@@ -211,9 +211,21 @@ def test_attention_vs_oracle(T, precision, n_dst, kmax, d_h, d_e, long_every):
     for table in (None, tab):
         got = T.tblock_attn(P, cu(seg), cu(dst_t), cu(nfeat), cu(dn), cu(nfeat), cu(sn),
                             cu(ef) if d_e else None, cu(eid) if d_e else None, cu(et),
-                            table=table, max_seg=kmax)
+                            table=table, max_seg=int(np.diff(seg).max()))
         err = np.abs(np_(got)[:n_dst] - exp).max()
         assert err <= TOL[precision], err
+
+
+def test_attention_general_path_any_segment_length(T):
+    """max_seg <= 0 (unknown) routes to the general kernel: segments of any length."""
+    rng = np.random.default_rng(21)
+    p, seg, dst_t, nfeat, dn, sn, ef, eid, et = attn_case(rng, 120, 40, 172, 172,
+                                                          long_every=9)
+    exp = oracle.tblock_attn(p, seg, dst_t, nfeat, dn, nfeat, sn, ef, eid, et)
+    P = T.AttnParams(p)
+    got = T.tblock_attn(P, cu(seg), cu(dst_t), cu(nfeat), cu(dn), cu(nfeat), cu(sn), cu(ef),
+                        cu(eid), cu(et), max_seg=0)
+    assert np.abs(np_(got)[:120] - exp).max() <= 1e-3
 
 
 def test_attention_offsets_and_identity(T):

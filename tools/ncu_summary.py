@@ -1,0 +1,50 @@
+"""Summarise an .ncu-rep: SOL, memory, scheduler, stall reasons, top SASS hot spots."""
+import csv
+import io
+import subprocess
+import sys
+
+
+def ncu_csv(rep, *args):
+    out = subprocess.run(["ncu", "-i", rep, *args, "--csv"], capture_output=True, text=True).stdout
+    return list(csv.reader(io.StringIO(out)))
+
+
+def main(rep, top=25):
+    rows = ncu_csv(rep, "--page", "details")
+    h = rows[0]
+    keep = ("GPU Speed Of Light Throughput", "Memory Workload Analysis", "Scheduler Statistics",
+            "Warp State Statistics", "Occupancy", "Compute Workload Analysis", "Launch Statistics")
+    for r in rows[1:]:
+        d = dict(zip(h, r))
+        if d.get("Section Name") in keep and d.get("Metric Name"):
+            print(f"{d['Section Name'][:26]:26s} | {d['Metric Name'][:48]:48s} | {d['Metric Value']} {d['Metric Unit']}")
+    raw = ncu_csv(rep, "--page", "raw")
+    hr, vr = raw[0], raw[2] if len(raw) > 2 else raw[1]
+    d = dict(zip(hr, vr))
+    print("--- raw")
+    for k in ("dram__bytes_read.sum", "dram__bytes_write.sum", "lts__t_bytes.sum",
+              "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed",
+              "sm__inst_executed_pipe_tensor.sum", "gpu__time_duration.sum"):
+        for kk in d:
+            if kk.startswith(k):
+                print(f"{kk}: {d[kk]}")
+    st = [(k, float(v.replace(",", ""))) for k, v in d.items()
+          if k.startswith("smsp__pcsamp_warps_issue_stalled_") and not k.endswith("not_issued")
+          and v.replace(",", "").replace(".", "").isdigit()]
+    tot = sum(v for _, v in st) or 1
+    print("--- stall samples")
+    for k, v in sorted(st, key=lambda x: -x[1])[:10]:
+        print(f"{100 * v / tot:5.1f}% {k.replace('smsp__pcsamp_warps_issue_stalled_', '')}")
+    src = ncu_csv(rep, "--page", "source", "--print-source", "sass")
+    hs = src[1]
+    rs = [dict(zip(hs, x)) for x in src[2:]]
+    key = "Warp Stall Sampling (All Samples)"
+    tot = sum(float(x[key] or 0) for x in rs) or 1
+    print("--- top SASS by stall samples")
+    for x in sorted(rs, key=lambda x: -float(x[key] or 0))[:top]:
+        print(f"{100 * float(x[key]) / tot:5.1f}% {x['Address'][-5:]} {x['Source'].strip()[:90]}")
+
+
+if __name__ == "__main__":
+    main(sys.argv[1], int(sys.argv[2]) if len(sys.argv) > 2 else 25)
