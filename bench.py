@@ -289,7 +289,7 @@ def run_ours(args):
     edges_per_s = int(e_tot.item()) / (total_ms / 1e3)
 
     # ---- dominant call: tgl_tblock_attn on the tail block, timed eagerly with events
-    rec_ms, rec_shape = [], None
+    rec_ms, rec_shape, brk = [], None, {}
     for i in range(max(3, min(args.steps, 20))):
         flush.zero_()
         pipe.start_dev.fill_(batch_of(args.warmup + i) * cfg.batch)
@@ -298,6 +298,9 @@ def run_ours(args):
         torch.cuda.synchronize()
         tail = pipe.L - 1
         rec_ms.append(rec[tail][0].elapsed_time(rec[tail][1]))
+        mk = rec["_marks"]
+        for (n0_, e0_), (n1_, e1_) in zip(mk[:-1], mk[1:]):
+            brk.setdefault(n1_, []).append(e0_.elapsed_time(e1_))
         bt = pipe.blocks[tail]
         U = int(bt.u_dev.item())
         E = int(bt.seg_ptr[U].item())
@@ -387,7 +390,8 @@ def run_ours(args):
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
                 "gpu_launches": pipe.launches_per_forward * args.steps,
                 "gpu_launches_per_step": pipe.launches_per_forward,
-                "step_ms_p50": statistics.median(step_ms)}
+                "step_ms_p50": statistics.median(step_ms),
+                "breakdown_ms_eager": {k_: statistics.median(v_) for k_, v_ in brk.items()}}
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()

@@ -59,6 +59,10 @@ def lib():
         L.or_sample.argtypes = [C.c_int64, i64p, i32p, i32p, f32p, C.c_int64, i32p, f32p,
                                 C.c_int32, C.c_int32, C.c_uint64, C.c_uint32, i64p, i32p,
                                 i32p, f32p]
+        L.or_sample_keyed.restype = C.c_int
+        L.or_sample_keyed.argtypes = [C.c_int64, i64p, i32p, i32p, f32p, C.c_int64, i32p, i32p,
+                                      f32p, C.c_int32, C.c_int32, C.c_uint64, C.c_uint32, i64p,
+                                      i32p, i32p, f32p]
         L.or_dedup.restype = C.c_int64
         L.or_dedup.argtypes = [C.c_int64, i32p, f32p, i32p, f32p, i32p]
         L.or_time_encode.argtypes = [C.c_int64, f32p, C.c_int32, f32p, f32p, f32p]
@@ -125,6 +129,26 @@ def sample(tcsr, qnode, qtime, k: int, strategy: int, seed: int = 0, layer: int 
     rc = lib().or_sample(indptr.shape[0] - 1, indptr, nbr, eid, ts, nq, qnode, qtime, k,
                          strategy, C.c_uint64(seed & 0xFFFFFFFFFFFFFFFF), layer, seg_ptr,
                          o_nbr, o_eid, o_ts)
+    if rc != 0:
+        raise ValueError("bad sample arguments")
+    m = int(seg_ptr[-1])
+    return seg_ptr, o_nbr[:m].copy(), o_eid[:m].copy(), o_ts[:m].copy()
+
+
+def sample_keyed(tcsr, qnode, qkey, qtime, k: int, strategy: int, seed: int = 0,
+                 layer: int = 0):
+    """`sample` on a CSR whose owners are renumbered: qkey = original node ids (R6 key)."""
+    indptr, nbr, eid, ts = tcsr
+    qnode, qkey, qtime = _c(qnode, np.int32), _c(qkey, np.int32), _c(qtime, np.float32)
+    nq = qnode.shape[0]
+    seg_ptr = np.zeros(nq + 1, np.int64)
+    cap = max(nq * k, 1)
+    o_nbr = np.zeros(cap, np.int32)
+    o_eid = np.zeros(cap, np.int32)
+    o_ts = np.zeros(cap, np.float32)
+    rc = lib().or_sample_keyed(indptr.shape[0] - 1, indptr, nbr, eid, ts, nq, qnode, qkey,
+                               qtime, k, strategy, seed & 0xFFFFFFFFFFFFFFFF, layer, seg_ptr,
+                               o_nbr, o_eid, o_ts)
     if rc != 0:
         raise ValueError("bad sample arguments")
     m = int(seg_ptr[-1])

@@ -174,12 +174,15 @@ static int64_t sample_count(const int64_t* indptr, const float* ts, int32_t v, f
   return n < k ? n : k;
 }
 
-/* returns 0, or -1 on a query node out of range / bad k / bad strategy */
-int or_sample(int64_t num_nodes, const int64_t* indptr, const int32_t* nbr,
-              const int32_t* eid, const float* ts, int64_t nq, const int32_t* qnode,
-              const float* qtime, int32_t k, int32_t strategy, uint64_t seed,
-              uint32_t layer, int64_t* seg_ptr, int32_t* out_nbr, int32_t* out_eid,
-              float* out_ts) {
+/* qkey[q] is the node id that keys the Philox counter (R6); it equals qnode[q]
+ * except when the CSR is a sub-graph with locally renumbered owners (the large-config
+ * checks build one per queried node).  returns 0, or -1 on a query node out of
+ * range / bad k / bad strategy */
+int or_sample_keyed(int64_t num_nodes, const int64_t* indptr, const int32_t* nbr,
+                    const int32_t* eid, const float* ts, int64_t nq, const int32_t* qnode,
+                    const int32_t* qkey, const float* qtime, int32_t k, int32_t strategy,
+                    uint64_t seed, uint32_t layer, int64_t* seg_ptr, int32_t* out_nbr,
+                    int32_t* out_eid, float* out_ts) {
   if (k <= 0 || (strategy != 0 && strategy != 1)) return -1;
   for (int64_t q = 0; q < nq; ++q)
     if (qnode[q] < 0 || qnode[q] >= num_nodes) return -1;
@@ -200,7 +203,7 @@ int or_sample(int64_t num_nodes, const int64_t* indptr, const int32_t* nbr,
       if (strategy == 0 || n <= k) {
         j = start + (n - m) + s;
       } else {
-        uint32_t ctr[4] = {(uint32_t)qnode[q], time_key_bits(qtime[q]), layer,
+        uint32_t ctr[4] = {(uint32_t)qkey[q], time_key_bits(qtime[q]), layer,
                            (uint32_t)(s >> 2)};
         uint32_t key[2] = {(uint32_t)(seed & 0xFFFFFFFFu), (uint32_t)(seed >> 32)};
         uint32_t r[4];
@@ -213,6 +216,15 @@ int or_sample(int64_t num_nodes, const int64_t* indptr, const int32_t* nbr,
     }
   }
   return 0;
+}
+
+int or_sample(int64_t num_nodes, const int64_t* indptr, const int32_t* nbr,
+              const int32_t* eid, const float* ts, int64_t nq, const int32_t* qnode,
+              const float* qtime, int32_t k, int32_t strategy, uint64_t seed,
+              uint32_t layer, int64_t* seg_ptr, int32_t* out_nbr, int32_t* out_eid,
+              float* out_ts) {
+  return or_sample_keyed(num_nodes, indptr, nbr, eid, ts, nq, qnode, qnode, qtime, k, strategy,
+                         seed, layer, seg_ptr, out_nbr, out_eid, out_ts);
 }
 
 /* ---------------------------------------------------------------------- */

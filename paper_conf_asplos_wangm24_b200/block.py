@@ -119,6 +119,15 @@ class TGATPipeline:
         tgl_tblock_attn call are stored as record[layer] = (start, end)."""
         g, k, s = self.g, self.sampler.k, stream
         b0 = self.blocks[0]
+        marks = None if record is None else record.setdefault("_marks", [])
+
+        def mark(name):
+            if marks is not None:
+                ev = torch.cuda.Event(enable_timing=True)
+                ev.record(s if s is not None else torch.cuda.current_stream())
+                marks.append((name, ev))
+
+        mark("start")
         if self.staging:
             st = self.stage
             tgl.batch_roots(self.batch, self.stage_n, None, st["src"], st["dst"], st["t"],
@@ -126,16 +135,19 @@ class TGATPipeline:
         else:
             tgl.batch_roots(self.batch, self.E, self.start_dev, g["src"], g["dst"], g["t"],
                             g["neg"], b0.dst_node, b0.dst_t, b0.n_dev, stream=s)
+        mark("roots")
         for l, b in enumerate(self.blocks):
             if l > 0:  # S5 next_block (R14): [dst after dedup ; sampled src]
                 p = self.blocks[l - 1]
                 tgl.next_block(p.n_max, p.u_dev, p.uniq_node, p.uniq_t, p.n_max * k, p.seg_ptr,
                                p.nbr, p.ts, b.dst_node, b.dst_t, b.n_dev, stream=s)
+                mark(f"next_block{l}")
             if self.use_dedup:  # S3
                 _call_ws(tgl.lib().tgl_dedup,
                          [b.n_max, tgl._p(b.n_dev), tgl._p(b.dst_node), tgl._p(b.dst_t),
                           tgl._p(b.uniq_node), tgl._p(b.uniq_t), tgl._p(b.u_dev),
                           tgl._p(b.inv)], b.ws["dedup"], s, "tgl_dedup")
+                mark(f"dedup{l}")
             # S4 sample
             _call_ws(tgl.lib().tgl_sample,
                      [tgl.C.byref(self.tcsr.struct), b.n_max, tgl._p(b.u_dev),
@@ -143,6 +155,7 @@ class TGATPipeline:
                       tgl.STRATEGY[self.sampler.strategy], self.sampler.seed, l,
                       tgl._p(b.seg_ptr), tgl._p(b.nbr), tgl._p(b.eid), tgl._p(b.ts)],
                      b.ws["sample"], s, "tgl_sample")
+            mark(f"sample{l}")
         # S15 aggregate: tail -> head
         for l in range(self.L - 1, -1, -1):
             b = self.blocks[l]
@@ -173,8 +186,10 @@ class TGATPipeline:
             if record is not None:
                 ev[1].record(s if s is not None else torch.cuda.current_stream())
                 record[l] = ev
+            mark(f"attn{l}")
         if self.use_dedup:  # S14 at the roots
             tgl.gather_rows(b0.inv, b0.out, n_dev=b0.n_dev, n_max=b0.n_max, out=self.emb, stream=s)
+            mark("gather")
             return self.emb
         return b0.out[:3 * self.batch]
 
