@@ -22,13 +22,19 @@ from . import UNIFORM, RECENT, sample_keyed, tblock_attn
 STRATEGY = {"recent": RECENT, "uniform": UNIFORM}
 
 
-def node_segments(src: np.ndarray, dst: np.ndarray, t: np.ndarray, nodes) -> dict:
+def node_segments(src: np.ndarray, dst: np.ndarray, t: np.ndarray, nodes,
+                  num_nodes: int | None = None) -> dict:
+    """{v: (nbr int32, eid int32, ts float32)} for each v in `nodes` (undirected T-CSR)."""
     nodes = np.unique(np.asarray(nodes, dtype=np.int64))
     out = {}
     if nodes.size == 0:
         return out
-    fwd = np.nonzero(np.isin(src, nodes))[0]
-    rev = np.nonzero(np.isin(dst, nodes))[0]
+    if num_nodes is None:
+        num_nodes = int(max(src.max(initial=0), dst.max(initial=0), nodes.max())) + 1
+    mark = np.zeros(num_nodes, dtype=bool)
+    mark[nodes] = True
+    fwd = np.flatnonzero(mark[src])
+    rev = np.flatnonzero(mark[dst])
     owner = np.concatenate([src[fwd], dst[rev]]).astype(np.int64)
     nbr = np.concatenate([dst[fwd], src[rev]]).astype(np.int32)
     eid = np.concatenate([fwd, rev]).astype(np.int64)
@@ -63,18 +69,25 @@ def sample_nodes(segs: dict, qnode, qtime, k, strategy, seed, layer):
                         STRATEGY.get(strategy, strategy), seed, layer)
 
 
-def embed_recursive(src, dst, t, cfg, params, roots_node, roots_t, seed: int):
-    """Root embeddings (fp64) by Listing 1's recursion over the oracle primitives."""
+def embed_recursive(src, dst, t, cfg, params, roots_node, roots_t, seed: int,
+                    segs: dict | None = None):
+    """Root embeddings (fp64) by Listing 1's recursion over the oracle primitives.
+
+    Features are `synth.feature_rows(feat seed, rows, dim)` (node) and
+    `feature_rows(feat seed + 7919, eids, d_e)` (edge), the tables `make_graph` and
+    `synth.gpu.device_feature_table` materialise."""
     import synth
     L = len(params)
     k = cfg.k
     nseed, eseed = cfg.seeds["feat"], cfg.seeds["feat"] + 7919
-    segs = node_segments(src, dst, t, roots_node)
+    segs = {} if segs is None else segs
 
     def ensure(nodes):
         need = [int(v) for v in np.unique(nodes) if int(v) not in segs]
         if need:
-            segs.update(node_segments(src, dst, t, need))
+            segs.update(node_segments(src, dst, t, need, cfg.n_nodes))
+
+    ensure(roots_node)
 
     def embed(v, tq, depth):
         if depth == L:

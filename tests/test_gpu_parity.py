@@ -200,6 +200,8 @@ def attn_case(rng, n_dst, kmax, d_h, d_e, empty=True, long_every=0):
                                                           (777, 10, 172, 172, 0),
                                                           (300, 20, 128, 128, 0),
                                                           (200, 10, 100, 0, 0),
+                                                          (333, 10, 413, 186, 0),
+                                                          (517, 10, 128, 0, 0),
                                                           (150, 10, 24, 12, 7)])
 def test_attention_vs_oracle(T, precision, n_dst, kmax, d_h, d_e, long_every):
     rng = np.random.default_rng(n_dst + kmax)
