@@ -171,15 +171,15 @@ class TGATPipeline:
                 else:
                     hdst_idx = hsrc_idx = None
             ef = g["efeat"]
-            ld_e = ef.shape[1] if ef.dim() == 2 else 0
+            ld_e = ef.stride(0) if (ef.dim() == 2 and ef.shape[1] > 0) else 0
             if record is not None:
                 ev = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
                 ev[0].record(s if s is not None else torch.cuda.current_stream())
             _call_ws(tgl.lib().tgl_tblock_attn,
                      [tgl.C.byref(a.struct), b.n_max, tgl._p(b.u_dev), tgl._p(b.seg_ptr),
-                      tgl._p(b.uniq_t), tgl._p(hdst), tgl._p(hdst_idx), hdst.shape[1],
-                      tgl._p(hsrc), tgl._p(hsrc_idx), tgl._p(off), hsrc.shape[1],
-                      tgl._p(ef) if ld_e else None, tgl._p(b.eid) if ld_e else None, ld_e,
+                      tgl._p(b.uniq_t), tgl._prow(hdst), tgl._p(hdst_idx), hdst.stride(0),
+                      tgl._prow(hsrc), tgl._p(hsrc_idx), tgl._p(off), hsrc.stride(0),
+                      tgl._prow(ef) if ld_e else None, tgl._p(b.eid) if ld_e else None, ld_e,
                       tgl._p(b.ts), tgl._p(self.tables[l]),
                       0 if self.tables[l] is None else self.tables[l].shape[0], k,
                       tgl._p(b.out)], b.ws["attn"], s, "tgl_tblock_attn")

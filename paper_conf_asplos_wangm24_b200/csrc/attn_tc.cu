@@ -18,7 +18,11 @@
 // Precision: TGL_FP32 = 3 bf16 passes (hi*hi + lo*hi + hi*lo, fp32 accumulate;
 // operand error ~2^-16, inside the 1e-3 contract); TGL_BF16 = 1 pass.
 // Pipeline: 2 smem stages; the gather of chunk c+1 overlaps the MMAs of chunk c.
+#include <cuda.h>
 #include <cuda_bf16.h>
+#include <cudaTypedefs.h>
+#include <stdlib.h>
+#include <string.h>
 
 #include "common.cuh"
 #include "tc.cuh"
@@ -241,7 +245,7 @@ __device__ __forceinline__ void load_chunk(int c, const Seg3& sg, const RD& rd, 
         const float dt = rd.dt[r];
 #pragma unroll
         for (int e = 0; e < 8; ++e)
-          if (j0 + e < sg.d2) y[e] = tenc_direct(dt, s_omega[j0 + e], s_phi[j0 + e]);
+          if (j0 + e < sg.d2) y[e] = tenc_fast(dt, s_omega[j0 + e], s_phi[j0 + e]);
       }
     }
   }
@@ -906,6 +910,118 @@ struct BinDesc {
   int live;               // 0 = end-of-work marker
 };
 
+// Epilogue of the binned K|V kernels (warps 0-7): S10-S12 for one tile per trip.
+// Warp w owns TMEM lane quarter w%4 and head w/4; see kv_bin_kernel.
+template <int NS, class D>
+__device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uint64_t* dempty,
+                                             uint64_t* tfull, uint64_t* tempty, const D* bd,
+                                             uint32_t tmem, float (*s_pv)[32][33],
+                                             const float* s_bias) {
+  constexpr uint32_t kCols = 256;
+  constexpr int dm = 100, dh = 50;
+  const tgl_attn_params& P = a.P;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  uint32_t tt = 0;
+  const int q4 = warp & 3, head = warp >> 2;
+  const int cb = head * dh;                        // this warp's columns [cb, cb + dh)
+  float (*pv)[33] = s_pv[warp];
+  for (;; ++tt) {
+    const uint32_t ab = tt & 1u, ds = tt % NS;
+    mbar_wait(&dfull[ds], (tt / NS) & 1u);
+    if (!bd[ds].live) {
+      warp_arrive(&dempty[ds]);
+      break;
+    }
+    const int d = bd[ds].rdst[q4 * 32 + lane];
+    warp_arrive(&dempty[ds]);
+    // segment structure of this bin from the row destinations
+    const int dprev = __shfl_up_sync(0xffffffffu, d, 1);
+    const int dnext = __shfl_down_sync(0xffffffffu, d, 1);
+    const bool valid = d >= 0;
+    const unsigned smask = __ballot_sync(0xffffffffu, valid && (lane == 0 || dprev != d));
+    const unsigned emask = __ballot_sync(0xffffffffu, valid && (lane == 31 || dnext != d));
+    const int lo = 31 - __clz(smask & (0xffffffffu >> (31 - lane)));   // last start <= lane
+    const int hi = __ffs(emask & (0xffffffffu << lane));              // last end >= lane, +1
+    // this row's q (head columns) and q . bk, fetched before waiting for the accumulator
+    float qv[dh];
+    const float* qrow = a.qbuf + (int64_t)(valid ? d : 0) * kQLd;
+#pragma unroll
+    for (int j = 0; j < dh; j += 2) {
+      const float2 q2 = __ldg(reinterpret_cast<const float2*>(qrow + cb + j));
+      qv[j] = q2.x;
+      qv[j + 1] = q2.y;
+    }
+    const float qb = __ldg(qrow + dm + head);
+    if (threadIdx.x == 0) tl_mark(a, tt, 5);
+    mbar_wait(&tfull[ab], (tt >> 1) & 1u);
+    tc_fence_after();
+    if (threadIdx.x == 0) tl_mark(a, tt, 6);
+    if (a.dbg & 1) {
+      tc_fence_before();
+      warp_arrive(&tempty[ab]);
+      continue;
+    }
+    const uint32_t ta = tmem + ab * kCols + ((uint32_t)(q4 * 32) << 16);
+    float v[32];
+    // S10: this head's logit <q_dst, k_row + bk> = <q_dst, k_row> + (q_dst . bk_head)
+    float p = qb;
+#pragma unroll
+    for (int cq = 0; cq < 2; ++cq) {
+      tmem_ld32(ta + cb + cq * 32, v);
+      tmem_wait_ld();
+#pragma unroll
+      for (int j = 0; j < 32; ++j)
+        if (cq * 32 + j < dh) p = fmaf(qv[cq * 32 + j], v[j], p);
+    }
+    float s = p * P.logit_scale;
+    if (P.leaky_slope >= 0.f) s = s < 0.f ? s * P.leaky_slope : s;
+    // S11: softmax over the segment [lo, hi): suffix max / sum, broadcast from lo
+    if (!valid) s = -INFINITY;
+    float m = s;
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+      const float y = __shfl_down_sync(0xffffffffu, m, off);
+      if (lane + off < hi) m = fmaxf(m, y);
+    }
+    const float mseg = __shfl_sync(0xffffffffu, m, valid ? lo : lane);
+    const float ex = valid ? expf(s - mseg) : 0.f;
+    float t = ex;
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+      const float y = __shfl_down_sync(0xffffffffu, t, off);
+      if (lane + off < hi) t += y;
+    }
+    const float l = __shfl_sync(0xffffffffu, t, valid ? lo : lane);
+    const float w = valid ? ex / l : 0.f;
+    // S12: r_dst = sum_seg w * (v + bv) = sum_seg w * v + bv  (sum_seg w = 1); lane j owns
+    // column j of the 32-column piece and walks each segment's rows in order
+#pragma unroll 1
+    for (int cq = 0; cq < 2; ++cq) {
+      tmem_ld32(ta + dm + cb + cq * 32, v);
+      tmem_wait_ld();
+#pragma unroll
+      for (int j = 0; j < 32; ++j) pv[lane][j] = w * v[j];
+      __syncwarp();
+      const int c = cq * 32 + lane;                  // this lane's column in the head
+      const float bvc = c < dh ? s_bias[dm + cb + c] : 0.f;
+      unsigned sm = smask, em = emask;
+      while (sm) {
+        const int slo = __ffs(sm) - 1, shi = __ffs(em);   // [slo, shi)
+        sm &= sm - 1;
+        em &= em - 1;
+        const int dr = __shfl_sync(0xffffffffu, d, slo);
+        float acc = 0.f;
+        for (int r = slo; r < shi; ++r) acc += pv[r][lane];
+        if (c < dh) a.rbuf[(int64_t)dr * kQLd + cb + c] = acc + bvc;
+      }
+      __syncwarp();
+    }
+    tc_fence_before();
+    warp_arrive(&tempty[ab]);
+    if (threadIdx.x == 0) tl_mark(a, tt, 7);
+  }
+}
+
 __global__ void __launch_bounds__(kBThreads, 1) kv_bin_kernel(Args a) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* pipe = align1024(smem_raw);
@@ -1001,6 +1117,8 @@ __global__ void __launch_bounds__(kBThreads, 1) kv_bin_kernel(Args a) {
           const bool ok = dst[u] >= 0 && !(a.dbg & 16);
           hi[u] = ok ? (a.hsrc_idx ? a.hsrc_idx[hoff + e[u]] : (int32_t)(hoff + e[u])) : 0;
           ei[u] = (ok && P.d_e > 0) ? a.eid[e[u]] : 0;
+          if (a.dbg & 128) ei[u] &= 0x3FF;            // profiling: edge rows in 700 KB
+          if (a.dbg & 256) hi[u] &= 0x3FF;
           et[u] = ok ? a.edge_t[e[u]] : 0.f;
         }
 #pragma unroll
@@ -1059,106 +1177,466 @@ __global__ void __launch_bounds__(kBThreads, 1) kv_bin_kernel(Args a) {
       __syncwarp();
     }
   } else {                                           // ---------------- epilogue warps 0-7
-    const int q4 = warp & 3, head = warp >> 2;
-    const int cb = head * dh;                        // this warp's columns [cb, cb + dh)
-    float (*pv)[33] = s_pv[warp];
-    for (;; ++tt) {
-      const uint32_t ab = tt & 1u, ds = tt % kDSlots;
-      mbar_wait(&B.dfull[ds], (tt / kDSlots) & 1u);
-      if (!bd[ds].live) {
-        warp_arrive(&B.dempty[ds]);
-        break;
-      }
-      const int d = bd[ds].rdst[q4 * 32 + lane];
-      warp_arrive(&B.dempty[ds]);
-      // segment structure of this bin from the row destinations
-      const int dprev = __shfl_up_sync(0xffffffffu, d, 1);
-      const int dnext = __shfl_down_sync(0xffffffffu, d, 1);
-      const bool valid = d >= 0;
-      const unsigned smask = __ballot_sync(0xffffffffu, valid && (lane == 0 || dprev != d));
-      const unsigned emask = __ballot_sync(0xffffffffu, valid && (lane == 31 || dnext != d));
-      const int lo = 31 - __clz(smask & (0xffffffffu >> (31 - lane)));   // last start <= lane
-      const int hi = __ffs(emask & (0xffffffffu << lane));              // last end >= lane, +1
-      // this row's q (head columns) and q . bk, fetched before waiting for the accumulator
-      float qv[dh];
-      const float* qrow = a.qbuf + (int64_t)(valid ? d : 0) * kQLd;
-#pragma unroll
-      for (int j = 0; j < dh; j += 2) {
-        const float2 q2 = __ldg(reinterpret_cast<const float2*>(qrow + cb + j));
-        qv[j] = q2.x;
-        qv[j + 1] = q2.y;
-      }
-      const float qb = __ldg(qrow + dm + head);
-      if (threadIdx.x == 0) tl_mark(a, tt, 5);
-      mbar_wait(&B.tfull[ab], (tt >> 1) & 1u);
-      tc_fence_after();
-      if (threadIdx.x == 0) tl_mark(a, tt, 6);
-      if (a.dbg & 1) {
-        tc_fence_before();
-        warp_arrive(&B.tempty[ab]);
-        continue;
-      }
-      const uint32_t ta = tmem + ab * kCols + ((uint32_t)(q4 * 32) << 16);
-      float v[32];
-      // S10: this head's logit <q_dst, k_row + bk> = <q_dst, k_row> + (q_dst . bk_head)
-      float p = qb;
-#pragma unroll
-      for (int cq = 0; cq < 2; ++cq) {
-        tmem_ld32(ta + cb + cq * 32, v);
-        tmem_wait_ld();
-#pragma unroll
-        for (int j = 0; j < 32; ++j)
-          if (cq * 32 + j < dh) p = fmaf(qv[cq * 32 + j], v[j], p);
-      }
-      float s = p * P.logit_scale;
-      if (P.leaky_slope >= 0.f) s = s < 0.f ? s * P.leaky_slope : s;
-      // S11: softmax over the segment [lo, hi): suffix max / sum, broadcast from lo
-      if (!valid) s = -INFINITY;
-      float m = s;
-#pragma unroll
-      for (int off = 1; off < 32; off <<= 1) {
-        const float y = __shfl_down_sync(0xffffffffu, m, off);
-        if (lane + off < hi) m = fmaxf(m, y);
-      }
-      const float mseg = __shfl_sync(0xffffffffu, m, valid ? lo : lane);
-      const float ex = valid ? expf(s - mseg) : 0.f;
-      float t = ex;
-#pragma unroll
-      for (int off = 1; off < 32; off <<= 1) {
-        const float y = __shfl_down_sync(0xffffffffu, t, off);
-        if (lane + off < hi) t += y;
-      }
-      const float l = __shfl_sync(0xffffffffu, t, valid ? lo : lane);
-      const float w = valid ? ex / l : 0.f;
-      // S12: r_dst = sum_seg w * (v + bv) = sum_seg w * v + bv  (sum_seg w = 1); lane j owns
-      // column j of the 32-column piece and walks each segment's rows in order
-#pragma unroll 1
-      for (int cq = 0; cq < 2; ++cq) {
-        tmem_ld32(ta + dm + cb + cq * 32, v);
-        tmem_wait_ld();
-#pragma unroll
-        for (int j = 0; j < 32; ++j) pv[lane][j] = w * v[j];
-        __syncwarp();
-        const int c = cq * 32 + lane;                  // this lane's column in the head
-        const float bvc = c < dh ? s_bias[dm + cb + c] : 0.f;
-        unsigned sm = smask, em = emask;
-        while (sm) {
-          const int slo = __ffs(sm) - 1, shi = __ffs(em);   // [slo, shi)
-          sm &= sm - 1;
-          em &= em - 1;
-          const int dr = __shfl_sync(0xffffffffu, d, slo);
-          float acc = 0.f;
-          for (int r = slo; r < shi; ++r) acc += pv[r][lane];
-          if (c < dh) a.rbuf[(int64_t)dr * kQLd + cb + c] = acc + bvc;
-        }
-        __syncwarp();
-      }
-      tc_fence_before();
-      warp_arrive(&B.tempty[ab]);
-      if (threadIdx.x == 0) tl_mark(a, tt, 7);
-    }
+    bin_epilogue<kDSlots>(a, B.dfull, B.dempty, B.tfull, B.tempty, bd, tmem, s_pv, s_bias);
   }
   ws_teardown(tmem, 2 * kCols, kBMma);
+}
+
+// ------------------------------------------------------------------ TMA-gathered K|V attention
+// kv_tma_kernel: the binned K|V attention of kv_bin_kernel with the A operand moved by
+// the TMA engine instead of producer threads.  K is cut into 32-column fp32 chunks
+// per concat segment ([h_src | e | Phi], each padded to 32; the padding K step is
+// skipped when a chunk holds <= 16 real columns).  Per chunk and tile:
+//   TMA warp   : 32 lanes each issue one cp.async.bulk.tensor tile::gather4 (4 rows x
+//                128 B) -> a 16 KB fp32 image of 128 gathered rows (h_src rows by
+//                hsrc_idx, edge-feature rows by eid, precompute-table rows by Delta t),
+//                zero-filled past the segment width, completion on an mbarrier (tx bytes);
+//   converters : 8 warps rewrite the image IN PLACE, 8-row group by 8-row group, as
+//                bf16 hi | lo (512 B each) in the SW64 K-major UMMA layout, computing
+//                Phi(Delta t) = cos(w Delta t + phi) for rows the table does not cover;
+//   MMA warp   : tcgen05.mma M=128 N=200 K=16 from the converted image and a SW64
+//                weight chunk (hi|lo, one bulk copy), 3 passes in fp32 mode.
+// No thread ever waits on a global load in the steady state: up to kTAStages chunks
+// (96 KB) of gathers are in flight per SM.
+constexpr int kTC = 32;                       // fp32 columns per K chunk
+constexpr int kTAStage = kBM * kTC * 4;       // 16 KB
+constexpr int kTAStages = 6;
+constexpr int kTWStages = 3;
+constexpr int kTWHalf = kNPkv * 64;           // one of W_hi / W_lo of a chunk (12.8 KB)
+constexpr int kTWStage = 2 * kTWHalf;
+constexpr int kTMma = 8, kTW = 9, kTTma = 10, kTDesc0 = 11, kTDescWarps = 2, kTConv0 = 13,
+              kTConvWarps = 7;
+constexpr int kTThreads = (kTConv0 + kTConvWarps) * 32;   // 640 (96 registers per thread)
+constexpr int kTDSlots = 4;
+constexpr int kTPipeBytes = kTAStages * kTAStage + kTWStages * kTWStage;
+constexpr int kTSmem = 1024 + kTPipeBytes + kBEpi * 32 * 33 * 4;
+
+struct KvPlan {       // 32-column chunks of the three K segments
+  int d[3];           // widths (h_src, e, time)
+  int c[3];           // chunks per segment
+  int n;              // total chunks
+};
+static KvPlan make_plan(int d0, int d1, int d2) {
+  KvPlan p;
+  p.d[0] = d0; p.d[1] = d1; p.d[2] = d2;
+  for (int s = 0; s < 3; ++s) p.c[s] = (p.d[s] + kTC - 1) / kTC;
+  p.n = p.c[0] + p.c[1] + p.c[2];
+  return p;
+}
+__host__ __device__ __forceinline__ void plan_chunk(const KvPlan& p, int c, int& seg, int& col) {
+  seg = c < p.c[0] ? 0 : (c < p.c[0] + p.c[1] ? 1 : 2);
+  col = (c - (seg > 0 ? p.c[0] : 0) - (seg > 1 ? p.c[1] : 0)) * kTC;
+}
+__device__ __forceinline__ int plan_ksteps(const KvPlan& p, int c) {
+  int seg, col;
+  plan_chunk(p, c, seg, col);
+  return p.d[seg] - col > 16 ? 2 : 1;
+}
+
+struct TmaMaps {
+  CUtensorMap m[3];   // h_src, edge features, precompute table (fp32, box 32 x 1)
+};
+
+struct TBars {
+  uint64_t afull[kTAStages], aready[kTAStages], aempty[kTAStages];
+  uint64_t wfull[kTWStages], wempty[kTWStages];
+  uint64_t dfull[kTDSlots], dempty[kTDSlots];
+  uint64_t tfull[2], tempty[2];
+};
+
+struct TDesc {
+  int hrow[kBM];      // gather row of h_src
+  int erow[kBM];      // gather row of the edge features
+  int trow[kBM];      // precompute-table row, -1 = evaluate eq 8 directly
+  float dt[kBM];
+  int rdst[kBM];      // destination of the row, -1 = padding
+  int live;
+};
+
+__device__ __forceinline__ void tma_gather4(uint32_t dst, const CUtensorMap* map, int col,
+                                            int r0, int r1, int r2, int r3, uint32_t bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(dst),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(col), "r"(r0), "r"(r1), "r"(r2), "r"(r3),
+      "r"(bar)
+      : "memory");
+}
+
+// K-major SW64 descriptor: rows of 64 B (32 bf16), 8-row groups `sbo` bytes apart.
+__device__ __forceinline__ uint64_t desc_sw64(uint32_t saddr, uint32_t sbo) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr >> 4) & 0x3FFFu);
+  d |= (uint64_t)1u << 16;
+  d |= (uint64_t)((sbo >> 4) & 0x3FFFu) << 32;
+  d |= (uint64_t)1u << 46;
+  d |= (uint64_t)4u << 61;
+  return d;
+}
+// byte offset of bf16 column c (0..31) of row r in an SW64 K-major 8-row atom
+__device__ __forceinline__ uint32_t sw64_off(int r, int c) {
+  return (uint32_t)((r & 7) * 64 + ((((c >> 3) ^ ((r >> 1) & 3)) & 3) << 4) + (c & 7) * 2);
+}
+
+__global__ void pack_kv64_kernel(const float* Wk, const float* Wv, int dm, int ksrc, KvPlan p,
+                                 uint8_t* out) {
+  const int kw = p.n * kTC;
+  const int64_t total = (int64_t)kNPkv * kw;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const int n = (int)(x / kw), kp = (int)(x % kw);
+    const int c = kp / kTC, cc = kp % kTC;
+    int seg, col;
+    plan_chunk(p, c, seg, col);
+    float v = 0.f;
+    if (n < 2 * dm && col + cc < p.d[seg]) {
+      const int src = (seg > 0 ? p.d[0] : 0) + (seg > 1 ? p.d[1] : 0) + col + cc;
+      v = n < dm ? Wk[(int64_t)n * ksrc + src] : Wv[(int64_t)(n - dm) * ksrc + src];
+    }
+    const __nv_bfloat16 hi = __float2bfloat16_rn(v);
+    const __nv_bfloat16 lo = __float2bfloat16_rn(v - __bfloat162float(hi));
+    const int64_t off = (int64_t)c * kTWStage + (n >> 3) * 512 + sw64_off(n, cc);
+    *reinterpret_cast<__nv_bfloat16*>(out + off) = hi;
+    *reinterpret_cast<__nv_bfloat16*>(out + off + kTWHalf) = lo;
+  }
+}
+
+__global__ void __launch_bounds__(kTThreads, 1)
+    kv_tma_kernel(const Args a, const KvPlan plan, const __grid_constant__ TmaMaps maps,
+                  const uint8_t* __restrict__ wkv, const int bdst) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* pipe = align1024(smem_raw);
+  __shared__ TBars B;
+  __shared__ uint32_t s_tmem;
+  __shared__ TDesc bd[kTDSlots];
+  __shared__ float s_omega[256], s_phi[256];
+  __shared__ float s_bias[2 * kMaxModel];
+  __shared__ int64_t s_seg[kTDescWarps][4 * 32 + 1];   // descriptor warps' tile scratch
+  __shared__ float s_td[kTDescWarps][4 * 32];
+  float (*s_pv)[32][33] = reinterpret_cast<float (*)[32][33]>(pipe + kTPipeBytes);
+  constexpr uint32_t kCols = 256;
+  const tgl_attn_params& P = a.P;
+  const int64_t n = dev_count(a.n_dst_dev, a.n_dst_max);
+  const bool split = a.split != 0;
+  constexpr int dm = 100;
+  for (int j = threadIdx.x; j < P.d_t; j += blockDim.x) {
+    s_omega[j] = P.omega[j];
+    s_phi[j] = P.phi[j];
+  }
+  for (int j = threadIdx.x; j < 2 * dm; j += blockDim.x) s_bias[j] = j < dm ? P.bk[j] : P.bv[j - dm];
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < kTAStages; ++s) {
+      mbar_init(&B.afull[s], 1);
+      mbar_init(&B.aready[s], kTConvWarps);
+      mbar_init(&B.aempty[s], 1);
+    }
+    for (int s = 0; s < kTWStages; ++s) {
+      mbar_init(&B.wfull[s], 1);
+      mbar_init(&B.wempty[s], 1);
+    }
+    for (int s = 0; s < kTDSlots; ++s) {
+      mbar_init(&B.dfull[s], 1);
+      mbar_init(&B.dempty[s], kBEpi + kTConvWarps + 3);   // epi, conv, mma, w, tma
+    }
+    for (int s = 0; s < 2; ++s) {
+      mbar_init(&B.tfull[s], 1);
+      mbar_init(&B.tempty[s], kBEpi);
+    }
+    fence_mbar_init();
+  }
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (warp == kTMma) tmem_alloc(&s_tmem, 2 * kCols);
+  if (warp == kTTma && lane == 0)
+    for (int s = 0; s < 3; ++s)
+      asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&maps.m[s]))
+                   : "memory");
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = s_tmem;
+  const int64_t D0 = n * blockIdx.x / gridDim.x, D1 = n * (blockIdx.x + 1) / gridDim.x;
+  const int nch = plan.n;
+  uint32_t tt = 0;
+
+  if (warp >= kTDesc0 && warp < kTDesc0 + kTDescWarps) {   // ------- tile builders
+    // Fixed packing: tile T holds destinations [T*dpt, (T+1)*dpt), dpt = 4*bdst, bin u
+    // the bdst destinations [u*bdst, (u+1)*bdst) of the tile, their segments
+    // concatenated (<= 32 rows when every segment has <= max_seg = 32/bdst rows), so a
+    // destination's rows sit in one TMEM lane quarter.  Tiles go round-robin over the
+    // CTAs; descriptor warp w builds the CTA's tiles tt = w, w+2, ... into slot tt % 4.
+    const int dw = warp - kTDesc0;
+    const int64_t hoff = a.hsrc_off_dev ? *a.hsrc_off_dev : 0;
+    const int dpt = 4 * bdst;
+    const int64_t ntiles = (n + dpt - 1) / dpt;
+    int64_t* sg = s_seg[dw];
+    float* stdv = s_td[dw];
+    for (tt = dw;; tt += kTDescWarps) {
+      const uint32_t ds = tt % kTDSlots;
+      wait_free(&B.dempty[ds], tt / kTDSlots);
+      if (lane == 0) tl_mark(a, tt, 0);
+      TDesc& R = bd[ds];
+      const int64_t T = blockIdx.x + (int64_t)tt * gridDim.x;
+      if (T >= ntiles) {                             // end marker
+        if (lane == 0) R.live = 0;
+        warp_arrive(&B.dfull[ds]);
+        break;
+      }
+      const int64_t d0 = T * dpt;
+      const int nd = (int)((n - d0) < dpt ? (n - d0) : dpt);
+      for (int j = lane; j <= nd; j += 32) sg[j] = a.seg_ptr[d0 + j];
+      for (int j = lane; j < nd; j += 32) stdv[j] = a.dst_t[d0 + j];
+      __syncwarp();
+      int64_t er[4] = {0, 0, 0, 0};
+      float tr[4] = {0.f, 0.f, 0.f, 0.f};
+      int dr[4] = {-1, -1, -1, -1};
+      unsigned zero_bins = 0;                        // bins whose rows overflow 32
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int j0 = u * bdst;
+        if (j0 >= nd) continue;
+        const int j1 = (j0 + bdst) < nd ? j0 + bdst : nd;
+        const int64_t e0 = sg[j0], e1 = sg[j1];
+        if (e1 - e0 > 32) {                          // max_seg violated: NaN rows
+          zero_bins |= 1u << u;
+          continue;
+        }
+        const int64_t e = e0 + lane;
+        if (e < e1) {
+          int j = j0;
+          while (sg[j + 1] <= e) ++j;
+          dr[u] = (int)(d0 + j);
+          er[u] = e;
+          tr[u] = stdv[j];
+        }
+      }
+      // empty segments -> r = 0 (R19); overflowing bins -> NaN
+      for (int j = 0; j < nd; ++j) {
+        const bool ovf = (zero_bins >> (j / bdst)) & 1u;
+        if (sg[j + 1] == sg[j] || ovf) {
+          const float fill = ovf ? __int_as_float(0x7fc00000) : 0.f;
+          for (int c = lane; c < dm; c += 32) a.rbuf[(d0 + j) * kQLd + c] = fill;
+        }
+      }
+      R.live = 1;
+      int32_t hi[4], ei[4];
+      float et[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {                   // all loads of the lane's 4 rows in flight
+        const bool ok = dr[u] >= 0 && !(a.dbg & 16);
+        hi[u] = ok ? (a.hsrc_idx ? a.hsrc_idx[hoff + er[u]] : (int32_t)(hoff + er[u])) : 0;
+        ei[u] = (ok && P.d_e > 0) ? a.eid[er[u]] : 0;
+        et[u] = ok ? a.edge_t[er[u]] : 0.f;
+        if (a.dbg & 128) ei[u] &= 0x3FF;              // profiling: edge rows in 700 KB
+        if (a.dbg & 256) hi[u] &= 0x3FF;
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int r = 32 * u + lane;
+        const bool ok = dr[u] >= 0;
+        const float dt = tr[u] - et[u];               // fp32 delta (R18)
+        R.hrow[r] = hi[u];
+        R.erow[r] = ei[u];
+        R.dt[r] = ok ? dt : 0.f;
+        R.trow[r] = ok ? (int)tenc_table_row(dt, a.table, a.window) : (a.table ? 0 : -1);
+        R.rdst[r] = dr[u];
+      }
+      warp_arrive(&B.dfull[ds]);
+      if (lane == 0) tl_mark(a, tt, 1);
+    }
+  } else if (warp == kTW) {                          // ---------------- weight loader
+    uint32_t wl = 0;
+    const uint32_t wbytes = split ? kTWStage : kTWHalf;
+    for (;; ++tt) {
+      const uint32_t ds = tt % kTDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kTDSlots) & 1u);
+      const int live = bd[ds].live;
+      warp_arrive(&B.dempty[ds]);
+      if (!live) break;
+      if (lane == 0) {
+        const int r0 = (tt > 0 && nch >= 4) ? 2 : 0;
+        for (int i = r0; i < nch; ++i) {
+          const uint32_t k = wl + (i - r0);
+          const uint32_t sw = k % kTWStages;
+          wait_free(&B.wempty[sw], k / kTWStages);
+          if (a.dbg & 8) {
+            mbar_arrive(&B.wfull[sw]);
+            continue;
+          }
+          mbar_arrive_expect_tx(&B.wfull[sw], wbytes);
+          bulk_g2s(pipe + kTAStages * kTAStage + sw * kTWStage,
+                   wkv + (size_t)chunk_of(tt, i, nch) * kTWStage, wbytes, &B.wfull[sw]);
+        }
+        wl += nch - r0;
+      }
+      __syncwarp();
+    }
+  } else if (warp == kTTma) {                        // ---------------- TMA gathers
+    uint32_t ait = 0;
+    for (;; ++tt) {
+      const uint32_t ds = tt % kTDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kTDSlots) & 1u);
+      const TDesc& R = bd[ds];
+      const int live = R.live;
+      int rows[3][4];
+      bool thit = false;                   // some row of the tile reads the table
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        rows[0][u] = R.hrow[4 * lane + u];
+        rows[1][u] = R.erow[4 * lane + u];
+        const int t = R.trow[4 * lane + u];
+        rows[2][u] = t > 0 ? t : 0;
+        thit |= t >= 0;
+      }
+      warp_arrive(&B.dempty[ds]);
+      if (!live) break;
+      thit = __any_sync(0xffffffffu, thit) && a.table != nullptr;
+      if (lane == 0) tl_mark(a, tt, 2);
+      for (int i = 0; i < nch; ++i, ++ait) {
+        const int c = chunk_of(tt, i, nch);
+        int seg, col;
+        plan_chunk(plan, c, seg, col);
+        const uint32_t s = ait % kTAStages;
+        wait_free(&B.aempty[s], ait / kTAStages);
+        const bool tma = (seg < 2 || thit) && !(a.dbg & 2);
+        if (lane == 0) {
+          if (tma) mbar_arrive_expect_tx(&B.afull[s], kTAStage);
+          else mbar_arrive(&B.afull[s]);
+        }
+        __syncwarp();
+        if (tma) {
+          int r[4];
+#pragma unroll
+          for (int u = 0; u < 4; ++u) r[u] = seg == 0 ? rows[0][u] : (seg == 1 ? rows[1][u] : rows[2][u]);
+          const CUtensorMap* m = seg == 0 ? &maps.m[0] : (seg == 1 ? &maps.m[1] : &maps.m[2]);
+          tma_gather4(smem_u32(pipe + s * kTAStage + lane * 512), m, col, r[0], r[1], r[2], r[3],
+                      smem_u32(&B.afull[s]));
+        }
+      }
+    }
+  } else if (warp >= kTConv0) {                      // ---------------- converters
+    // warp cw converts the 8-row groups g = cw, cw + 7, cw + 14 (< 16) of each chunk;
+    // lane: row rr (and rr + 4) of the group, 16-byte column chunk j
+    const int cw = warp - kTConv0;
+    const int rr = lane >> 3, j = lane & 7;
+    uint32_t ait = 0;
+    for (;; ++tt) {
+      const uint32_t ds = tt % kTDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kTDSlots) & 1u);
+      const TDesc& R = bd[ds];
+      const int live = R.live;
+      float dt[6];
+      int tr[6];
+#pragma unroll
+      for (int u = 0; u < 6; ++u) {                  // rows (g, rr + 4(u&1)), g = cw + 7(u>>1)
+        const int g = cw + kTConvWarps * (u >> 1);
+        const int r = g * 8 + rr + 4 * (u & 1);
+        dt[u] = g < 16 ? R.dt[r] : 0.f;
+        tr[u] = g < 16 ? R.trow[r] : 0;
+      }
+      warp_arrive(&B.dempty[ds]);
+      if (!live) break;
+      for (int i = 0; i < nch; ++i, ++ait) {
+        const int c = chunk_of(tt, i, nch);
+        int seg, col;
+        plan_chunk(plan, c, seg, col);
+        const uint32_t s = ait % kTAStages;
+        mbar_wait(&B.afull[s], (ait / kTAStages) & 1u);
+        const uint32_t sb = smem_u32(pipe + s * kTAStage);
+        if (a.dbg & 64) {
+          warp_arrive(&B.aready[s]);
+          continue;
+        }
+#pragma unroll
+        for (int gg = 0; gg < 3; ++gg) {
+          const int g = cw + kTConvWarps * gg;
+          if (g >= 16) break;
+          float4 x[2];
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int u = 2 * gg + h, r = rr + 4 * h;
+            if (seg < 2 || tr[u] >= 0) {
+              x[h] = ld_shared_f4(sb + g * 1024 + r * 128 + j * 16);
+            } else {
+              float y[4];
+#pragma unroll
+              for (int e = 0; e < 4; ++e) {
+                const int cc = col + 4 * j + e;
+                y[e] = cc < P.d_t ? tenc_fast(dt[u], s_omega[cc], s_phi[cc]) : 0.f;
+              }
+              x[h] = make_float4(y[0], y[1], y[2], y[3]);
+            }
+          }
+          __syncwarp();
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int r = rr + 4 * h;
+            uint32_t h0, h1, l0, l1;
+            split2(x[h].x, x[h].y, h0, l0);
+            split2(x[h].z, x[h].w, h1, l1);
+            const uint32_t off = sb + g * 1024 + sw64_off(r, 4 * j);
+            asm volatile("st.shared.v2.b32 [%0], {%1, %2};" ::"r"(off), "r"(h0), "r"(h1) : "memory");
+            if (split)
+              asm volatile("st.shared.v2.b32 [%0], {%1, %2};" ::"r"(off + 512), "r"(l0), "r"(l1)
+                           : "memory");
+          }
+        }
+        fence_proxy_async_smem();
+        warp_arrive(&B.aready[s]);
+      }
+      if (threadIdx.x == kTConv0 * 32) tl_mark(a, tt, 3);
+    }
+  } else if (warp == kTMma) {                        // ---------------- MMA issuer
+    uint32_t ait = 0, wl = 0;
+    constexpr uint32_t idesc = idesc_bf16(kBM, kNPkv);
+    for (;; ++tt) {
+      const uint32_t ds = tt % kTDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kTDSlots) & 1u);
+      const int live = bd[ds].live;
+      warp_arrive(&B.dempty[ds]);
+      if (!live) break;
+      if (lane == 0) {
+        const uint32_t acc = tmem + (tt & 1u) * kCols;
+        wait_free(&B.tempty[tt & 1u], tt >> 1);
+        tc_fence_after();
+        tl_mark(a, tt, 4);
+        const int r0 = (tt > 0 && nch >= 4) ? 2 : 0;
+        for (int i = 0; i < nch; ++i, ++ait) {
+          const int c = chunk_of(tt, i, nch);
+          const uint32_t s = ait % kTAStages;
+          mbar_wait(&B.aready[s], (ait / kTAStages) & 1u);
+          uint32_t k;
+          if (i < r0) {
+            k = wl - 1 - i;
+          } else {
+            k = wl + (i - r0);
+            mbar_wait(&B.wfull[k % kTWStages], (k / kTWStages) & 1u);
+          }
+          const uint32_t sw = k % kTWStages;
+          tc_fence_after();
+          const uint32_t ab = smem_u32(pipe + s * kTAStage);
+          const uint32_t wb = smem_u32(pipe + kTAStages * kTAStage + sw * kTWStage);
+          const int nk = (a.dbg & 4) ? 0 : plan_ksteps(plan, c);
+          for (int ks = 0; ks < nk; ++ks) {
+            const uint64_t ah = desc_sw64(ab + ks * 32, 1024), bh = desc_sw64(wb + ks * 32, 512);
+            mma_bf16(acc, ah, bh, idesc, (i | ks) != 0);
+            if (split) {
+              mma_bf16(acc, desc_sw64(ab + 512 + ks * 32, 1024), bh, idesc, 1u);
+              mma_bf16(acc, ah, desc_sw64(wb + kTWHalf + ks * 32, 512), idesc, 1u);
+            }
+          }
+          mma_commit(&B.aempty[s]);
+          const bool keep = (nch >= 4) && (i >= nch - 2);
+          if (!keep) mma_commit(&B.wempty[sw]);
+        }
+        wl += nch - r0;
+        mma_commit(&B.tfull[tt & 1u]);
+      }
+      __syncwarp();
+    }
+  } else {                                           // ---------------- epilogue warps 0-7
+    bin_epilogue<kTDSlots>(a, B.dfull, B.dempty, B.tfull, B.tempty, bd, tmem, s_pv, s_bias);
+  }
+  ws_teardown(tmem, 2 * kCols, kTMma);
 }
 
 }  // namespace tca
@@ -1167,7 +1645,7 @@ __global__ void __launch_bounds__(kBThreads, 1) kv_bin_kernel(Args a) {
 namespace tca {
 
 struct PackedLayout {
-  size_t oq, okv, oo, total;
+  size_t oq, okv, oo, okv64, total;
 };
 
 static PackedLayout packed_layout(const tgl_attn_params* P) {
@@ -1179,6 +1657,7 @@ static PackedLayout packed_layout(const tgl_attn_params* P) {
   L.oq = W.take((size_t)sq.nchunks * 2 * kNPq * 128);
   L.okv = W.take((size_t)skv.nchunks * 2 * kNPkv * 128);
   L.oo = W.take((size_t)so.nchunks * 2 * kNPq * 128);
+  L.okv64 = W.take((size_t)make_plan(P->d_hsrc, P->d_e, P->d_t).n * kTWStage);
   L.total = W.off;
   return L;
 }
@@ -1193,7 +1672,48 @@ static tgl_status launch_pack(const tgl_attn_params* P, uint8_t* base, cudaStrea
               base + L.okv};
   PackJob jo{P->Wo, nullptr, P->d_out, P->d_out, kNPq, P->d_model + P->d_hdst, so, base + L.oo};
   pack_weights_kernel<<<dim3(64, 3), 256, 0, s>>>(jq, jkv, jo);
-  return launch_check("pack_weights");
+  TGL_TRY(launch_check("pack_weights"));
+  pack_kv64_kernel<<<64, 256, 0, s>>>(P->Wk, P->Wv, P->d_model, P->d_hsrc + P->d_e + P->d_t,
+                                      make_plan(P->d_hsrc, P->d_e, P->d_t), base + L.okv64);
+  return launch_check("pack_kv64");
+}
+
+}  // namespace tca
+
+namespace tca {
+
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no -lcuda)
+static PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  if (fn == nullptr) {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) ==
+            cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(f);
+  }
+  return fn;
+}
+
+// Row table [rows][ld] fp32 as a 2-D tensor map with a 32-column x 1-row box (the
+// gather4 unit).  Columns >= width read as zero (OOB fill).  False when TMA cannot
+// address the table (base not 16-B aligned or a row pitch that is not a multiple of
+// 16 B) -- the caller then takes the register-gather kernel.
+static bool encode_rows(CUtensorMap* m, const float* base, int width, int64_t ld, int64_t rows) {
+  memset(m, 0, sizeof(*m));
+  if (width <= 0) return true;                       // segment absent: map unused
+  if (base == nullptr || (reinterpret_cast<uintptr_t>(base) & 15) || ((ld * 4) & 15)) return false;
+  PFN_cuTensorMapEncodeTiled_v12000 enc = tensor_map_encoder();
+  if (enc == nullptr) return false;
+  cuuint64_t dims[2] = {(cuuint64_t)width, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)ld * 4};
+  cuuint32_t box[2] = {(cuuint32_t)kTC, 1};
+  cuuint32_t es[2] = {1, 1};
+  return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box,
+             es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+             CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
 }  // namespace tca
@@ -1270,6 +1790,8 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
   const int smem_q = Pipe<kNPq>::kBytes + 1024;
   const int smem_kv = Pipe<kNPkv>::kBytes + 1024 + kKvEpiBytes;
   const int smem_kvb = Pipe<kNPkv>::kBytes + 1024 + kBEpi * 32 * 33 * 4;
+  // TGL_KV = "bin" forces the register-gather kernel, "tma" requires the TMA one
+  const char* kvsel = getenv("TGL_KV");
   static bool attr_done = false;   // cached cudaFuncSetAttribute (idempotent)
   if (!attr_done) {
     TGL_TRY(cuda_check(cudaFuncSetAttribute(dense_kernel<false>,
@@ -1283,13 +1805,34 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
     TGL_TRY(cuda_check(cudaFuncSetAttribute(kv_bin_kernel,
                                             cudaFuncAttributeMaxDynamicSharedMemorySize, smem_kvb),
                        "attr kv bin"));
+    TGL_TRY(cuda_check(cudaFuncSetAttribute(kv_tma_kernel,
+                                            cudaFuncAttributeMaxDynamicSharedMemorySize, kTSmem),
+                       "attr kv tma"));
     attr_done = true;
   }
   const int64_t tiles = ceil_div(n_dst_max, kBM);
   const unsigned gq = (unsigned)(tiles < kNumSMs ? tiles : kNumSMs);
   dense_kernel<false><<<gq, kWsThreads, smem_q, s>>>(a);
   TGL_TRY(launch_check("tc q kernel"));
-  if (max_seg > 0 && max_seg <= 32 && P->n_heads == 2) {
+  const bool binned = max_seg > 0 && max_seg <= 32 && P->n_heads == 2;
+  TmaMaps maps;
+  const bool tma = binned && !(kvsel && strcmp(kvsel, "bin") == 0) &&
+                   encode_rows(&maps.m[0], hsrc, P->d_hsrc, ld_hsrc, 0x7fffffffLL) &&
+                   encode_rows(&maps.m[1], efeat, P->d_e, ld_e, 0x7fffffffLL) &&
+                   encode_rows(&maps.m[2], table, table ? P->d_t : 0, P->d_t,
+                               window > 0 ? window : 1);
+  if (kvsel && strcmp(kvsel, "tma") == 0 && !tma) {
+    set_error("TGL_KV=tma: the TMA gather path cannot take this call (alignment / max_seg)");
+    return TGL_EUNSUPPORTED;
+  }
+  if (tma) {
+    const unsigned gkv = (unsigned)(n_dst_max < kNumSMs ? (n_dst_max > 0 ? n_dst_max : 1) : kNumSMs);
+    const int bdst = 32 / max_seg;                 // destinations per 32-row bin
+    const int64_t ttiles = ceil_div(n_dst_max, 4 * bdst);
+    const unsigned gt = (unsigned)(ttiles < kNumSMs ? (ttiles > 0 ? ttiles : 1) : kNumSMs);
+    kv_tma_kernel<<<gt, kTThreads, kTSmem, s>>>(a, make_plan(P->d_hsrc, P->d_e, P->d_t), maps,
+                                                pk + PL.okv64, bdst);
+  } else if (binned) {
     // binned path: whole segments per epilogue warp (no block barriers)
     const unsigned gkv = (unsigned)(n_dst_max < kNumSMs ? (n_dst_max > 0 ? n_dst_max : 1) : kNumSMs);
     kv_bin_kernel<<<gkv, kBThreads, smem_kvb, s>>>(a);

@@ -91,6 +91,16 @@ def _p(t):
     return t.data_ptr()
 
 
+def _prow(t):
+    """Pointer of a row table: contiguous, or a row-padded 2-D view (unit column
+    stride, pitch = stride(0)) such as the 16-byte pitches the TMA gathers need."""
+    if t is None:
+        return None
+    assert t.is_cuda and (t.is_contiguous() or (t.dim() == 2 and t.stride(1) == 1)), \
+        "expected a CUDA row table with unit column stride"
+    return t.data_ptr()
+
+
 def _s(stream=None):
     s = stream if stream is not None else torch.cuda.current_stream()
     return s.cuda_stream
@@ -283,11 +293,15 @@ def tblock_attn(P: AttnParams, seg_ptr, dst_t, hdst, hdst_idx, hsrc, hsrc_idx, e
         out = torch.empty(max(n_dst_max, 1), P.d_out, dtype=torch.float32,
                           device=seg_ptr.device)
     window = 0 if table is None else table.shape[0]
-    ld_e = efeat.shape[1] if (efeat is not None and efeat.dim() == 2) else 0
+    # row pitches from the strides: row-padded views (16-byte pitches) are passed as is
+    for t in (hdst, hsrc, efeat):
+        if t is not None and t.dim() == 2 and t.shape[1] > 0 and t.stride(1) != 1:
+            raise ValueError("feature tables need unit column stride")
+    ld_e = efeat.stride(0) if (efeat is not None and efeat.dim() == 2 and efeat.shape[1]) else 0
     _ws_call(_lib.tgl_tblock_attn,
-             [C.byref(P.struct), n_dst_max, _p(n_dst_dev), _p(seg_ptr), _p(dst_t), _p(hdst),
-              _p(hdst_idx), hdst.shape[1], _p(hsrc), _p(hsrc_idx), _p(hsrc_off_dev),
-              hsrc.shape[1], _p(efeat) if ld_e else None, _p(eid) if ld_e else None, ld_e,
+             [C.byref(P.struct), n_dst_max, _p(n_dst_dev), _p(seg_ptr), _p(dst_t), _prow(hdst),
+              _p(hdst_idx), hdst.stride(0), _prow(hsrc), _p(hsrc_idx), _p(hsrc_off_dev),
+              hsrc.stride(0), _prow(efeat) if ld_e else None, _p(eid) if ld_e else None, ld_e,
               _p(edge_t), _p(table), window, max_seg, _p(out)], ws, _s(stream),
              "tgl_tblock_attn")
     return out

@@ -195,7 +195,18 @@ def attn_case(rng, n_dst, kmax, d_h, d_e, empty=True, long_every=0):
     return p, seg, dst_t, nfeat, dst_node, src_node, efeat, eid, edge_t
 
 
-@pytest.mark.parametrize("precision", ["fp32", "bf16", "fp32_simt"])
+def cu_pad(a, mult=4):
+    """Device copy whose rows are padded to a multiple of `mult` columns (16-B pitch
+    for fp32), returned as a view of the true width -- the layout TMA gathers need."""
+    n, d = a.shape
+    dp = max(mult, (d + mult - 1) // mult * mult)
+    t = torch.zeros(n, dp, dtype=torch.float32, device="cuda")
+    t[:, :d] = cu(a)
+    return t[:, :d]
+
+
+@pytest.mark.parametrize("precision,kv", [("fp32", "tma"), ("bf16", "tma"), ("fp32", "bin"),
+                                          ("bf16", "bin"), ("fp32_simt", None)])
 @pytest.mark.parametrize("n_dst,kmax,d_h,d_e,long_every", [(1, 10, 172, 172, 0),
                                                           (777, 10, 172, 172, 0),
                                                           (300, 20, 128, 128, 0),
@@ -203,19 +214,41 @@ def attn_case(rng, n_dst, kmax, d_h, d_e, empty=True, long_every=0):
                                                           (333, 10, 413, 186, 0),
                                                           (517, 10, 128, 0, 0),
                                                           (150, 10, 24, 12, 7)])
-def test_attention_vs_oracle(T, precision, n_dst, kmax, d_h, d_e, long_every):
+def test_attention_vs_oracle(T, monkeypatch, precision, kv, n_dst, kmax, d_h, d_e, long_every):
+    """TGL_KV selects the K|V kernel: "tma" (TMA gather4, needs 16-B row pitches: the
+    odd GDELT widths 413/186 go in row-padded views) or "bin" (register gathers)."""
     rng = np.random.default_rng(n_dst + kmax)
     p, seg, dst_t, nfeat, dn, sn, ef, eid, et = attn_case(rng, n_dst, kmax, d_h, d_e,
                                                           long_every=long_every)
+    if kv and np.diff(seg).max() <= 32:      # longer segments take the general kernel
+        monkeypatch.setenv("TGL_KV", kv)
     exp = oracle.tblock_attn(p, seg, dst_t, nfeat, dn, nfeat, sn, ef, eid, et)
     P = T.AttnParams(p, precision=precision, pack=(n_dst % 2 == 1))
     tab = T.time_precompute(65536, P.t["omega"], P.t["phi"])
+    put = cu_pad if kv == "tma" else cu
+    nf = put(nfeat)
     for table in (None, tab):
-        got = T.tblock_attn(P, cu(seg), cu(dst_t), cu(nfeat), cu(dn), cu(nfeat), cu(sn),
-                            cu(ef) if d_e else None, cu(eid) if d_e else None, cu(et),
+        got = T.tblock_attn(P, cu(seg), cu(dst_t), nf, cu(dn), nf, cu(sn),
+                            put(ef) if d_e else None, cu(eid) if d_e else None, cu(et),
                             table=table, max_seg=int(np.diff(seg).max()))
         err = np.abs(np_(got)[:n_dst] - exp).max()
         assert err <= TOL[precision], err
+
+
+def test_attention_tma_rejects_unaligned_pitch(T, monkeypatch):
+    """TGL_KV=tma on a 413-float row pitch (1652 B, not a multiple of 16): EUNSUPPORTED,
+    while the default dispatch falls back to the register-gather kernel."""
+    rng = np.random.default_rng(5)
+    p, seg, dst_t, nfeat, dn, sn, ef, eid, et = attn_case(rng, 64, 10, 413, 186)
+    exp = oracle.tblock_attn(p, seg, dst_t, nfeat, dn, nfeat, sn, ef, eid, et)
+    P = T.AttnParams(p)
+    args = (P, cu(seg), cu(dst_t), cu(nfeat), cu(dn), cu(nfeat), cu(sn), cu(ef), cu(eid), cu(et))
+    monkeypatch.setenv("TGL_KV", "tma")
+    with pytest.raises(T.TGLError):
+        T.tblock_attn(*args, max_seg=10)
+    monkeypatch.delenv("TGL_KV")
+    got = T.tblock_attn(*args, max_seg=10)
+    assert np.abs(np_(got)[:64] - exp).max() <= 1e-3
 
 
 def test_attention_general_path_any_segment_length(T):

@@ -1,0 +1,85 @@
+"""Time the REDDIT tail-block tgl_tblock_attn call per K|V kernel and debug mask.
+
+    python tools/kv_probe.py [precision]
+
+TGL_DEBUG_MASK bits (profiling only): 1 skip epilogue math, 2 skip A gathers,
+4 skip MMAs, 8 skip weight copies, 16 skip descriptor index loads, 64 skip the
+converters (kv_tma), 32 per-tile timeline.
+"""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np
+import torch
+
+import synth
+from paper_conf_asplos_wangm24_b200 import TGATPipeline, TSampler, tgl
+from paper_conf_asplos_wangm24_b200.block import _call_ws
+
+prec = sys.argv[1] if len(sys.argv) > 1 else "fp32"
+cfg = synth.get_config(os.environ.get("CFG", "REDDIT"))
+g = synth.make_graph(cfg)
+neg = synth.make_negatives(cfg)
+params = synth.gen.model_params(cfg)
+cu = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+dev = {"src": cu(g.src), "dst": cu(g.dst), "t": cu(g.t), "neg": cu(neg), "nfeat": cu(g.nfeat),
+       "efeat": cu(g.efeat)}
+tc = tgl.build_tcsr(cfg.n_nodes, dev["src"], dev["dst"], dev["t"], True, True)
+pipe = TGATPipeline(dev, tc, params, cfg.batch, TSampler(cfg.k, cfg.strategy, cfg.seeds["sampler"]),
+                    cfg.dedup, cfg.precompute, cfg.window, prec)
+b0 = int(0.7 * cfg.n_batches)
+pipe.start_dev.fill_(b0 * cfg.batch)
+pipe.forward()
+torch.cuda.synchronize()
+L = len(pipe.blocks) - 1
+b = pipe.blocks[L]
+a = pipe.attn[L]
+lib = tgl.lib()
+nf, ef = dev["nfeat"], dev["efeat"]
+tab = pipe.tables[L] if pipe.tables[L] is not None else None
+if os.environ.get("PROBE_WINDOW"):          # 0 = direct evaluation, else a smaller table
+    w = int(os.environ["PROBE_WINDOW"])
+    tab = tgl.time_precompute(w, a.t["omega"], a.t["phi"]) if w > 0 else None
+
+
+def call():
+    _call_ws(lib.tgl_tblock_attn,
+             [tgl.C.byref(a.struct), b.n_max, tgl._p(b.u_dev), tgl._p(b.seg_ptr), tgl._p(b.uniq_t),
+              tgl._prow(nf), tgl._p(b.uniq_node), nf.stride(0), tgl._prow(nf), tgl._p(b.nbr), None,
+              nf.stride(0), tgl._prow(ef), tgl._p(b.eid), ef.stride(0), tgl._p(b.ts),
+              tgl._p(tab), 0 if tab is None else tab.shape[0], cfg.k, tgl._p(b.out)],
+             b.ws["attn"], None, "tail attn")
+
+
+flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+nd = int(b.u_dev.item())
+ne = int(b.seg_ptr[nd].item())
+print(f"tail block: {nd} dst, {ne} edges, precision {prec}")
+ref = None
+KVS = os.environ.get("PROBE_KV", "bin,tma").split(",")
+MASKS = [int(m) for m in os.environ.get("PROBE_MASKS", "0,1,2,4,8,64,6,95").split(",")]
+for kv in KVS:
+    for mask in MASKS:
+        if kv == "bin" and mask & 64:
+            continue
+        os.environ["TGL_KV"] = kv
+        os.environ["TGL_DEBUG_MASK"] = str(mask)
+        ts = []
+        for it in range(8):
+            flush.zero_()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            call()
+            e1.record()
+            torch.cuda.synchronize()
+            ts.append(e0.elapsed_time(e1))
+        out = b.out[:nd].clone()
+        if mask == 0:
+            if ref is None:
+                ref = out
+            err = (out - ref).abs().max().item()
+        else:
+            err = float("nan")
+        print(f"{kv:4s} mask {mask:3d}: {np.median(ts[2:]) * 1e3:8.1f} us  (vs bin: {err:.2e})")
+os.environ["TGL_DEBUG_MASK"] = "0"
