@@ -18,9 +18,7 @@
 // Precision: TGL_FP32 = 3 bf16 passes (hi*hi + lo*hi + hi*lo, fp32 accumulate;
 // operand error ~2^-16, inside the 1e-3 contract); TGL_BF16 = 1 pass.
 // Pipeline: 2 smem stages; the gather of chunk c+1 overlaps the MMAs of chunk c.
-#include <cuda.h>
 #include <cuda_bf16.h>
-#include <cudaTypedefs.h>
 #include <stdlib.h>
 #include <string.h>
 
@@ -189,6 +187,28 @@ struct Pipe {
 // ---- profiling timeline (TGL_DEBUG_MASK & 32): [cta][tile][event] globaltimer stamps
 constexpr int kTlTiles = 32, kTlEvents = 8;
 __device__ unsigned long long g_timeline[kNumSMs * kTlTiles * kTlEvents];
+__device__ unsigned long long g_trace[8192];         // (TGL_DEBUG_MASK & 4096) CTA-0 event trace
+__device__ unsigned int g_trace_n;
+// per-warp slices of 512 events; the per-warp count lives in shared memory
+__shared__ unsigned s_trace_n[32];
+__device__ __forceinline__ void trace(const Args& a, int ev, uint32_t k) {
+  if ((a.dbg & 4096) && blockIdx.x == 0 && (threadIdx.x & 31) == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    const int w = (threadIdx.x >> 5) & 15;
+    const unsigned n = s_trace_n[w];
+    if (n < 511) {
+      g_trace[w * 512 + n] = (t << 16) | ((unsigned long long)(ev & 0xff) << 8) | (k & 0xff);
+      g_trace[w * 512 + 511] = n + 1;
+      s_trace_n[w] = n + 1;
+    }
+  }
+}
+__device__ unsigned long long g_prof[kNumSMs * 16];   // (TGL_DEBUG_MASK & 512) cycle counters
+__device__ __forceinline__ void prof_add(const Args& a, int slot, long long dt) {
+  if ((a.dbg & 512) && (threadIdx.x & 31) == 0 && blockIdx.x < (unsigned)kNumSMs)
+    atomicAdd(&g_prof[blockIdx.x * 16 + slot], (unsigned long long)dt);
+}
 __device__ __forceinline__ void tl_mark(const Args& a, uint32_t tt, int ev) {
   if ((a.dbg & 32) && tt < (uint32_t)kTlTiles && blockIdx.x < (unsigned)kNumSMs) {
     unsigned long long t;
@@ -206,6 +226,9 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 // wait for the (u-1)-th completion of a ring slot (no wait on first use)
 __device__ __forceinline__ void wait_free(uint64_t* bar, uint32_t u) {
   if (u >= 1) mbar_wait(bar, (u - 1) & 1u);
+}
+__device__ __forceinline__ void wait_free_sleep(uint64_t* bar, uint32_t u, uint32_t ns) {
+  if (u >= 1) mbar_wait_sleep(bar, (u - 1) & 1u, ns);
 }
 
 __device__ __forceinline__ void load8(const float* p, int lc, int d, float* x) {
@@ -385,7 +408,8 @@ template <int NP, int PW0, int GPT, class RD>
 __device__ __forceinline__ void produce_tile(const Seg3& sg, bool split, uint8_t* pipe, Bars& B,
                                              uint32_t& ait, uint32_t tt, const RD& rd,
                                              const float* s_omega, const float* s_phi,
-                                             const float* table, bool noload = false) {
+                                             const float* table, bool noload = false,
+                                             int dbg = 0) {
   using PP = Pipe<NP>;
   constexpr int GPR = 8 / GPT;                 // producer threads per row
   const int pt = threadIdx.x - PW0 * 32;
@@ -410,7 +434,7 @@ __device__ __forceinline__ void produce_tile(const Seg3& sg, bool split, uint8_t
     wait_free(&B.aempty[sa], ait / kAStages);
     uint8_t* st = PP::a(pipe, sa);
     store_chunk<GPT>(x0, st, st + kAPart, r, jb, split);
-    fence_proxy_async_smem();
+    if (!(dbg & 2048)) fence_proxy_async_smem();
     __syncwarp();
     if (lane == 0) mbar_arrive(&B.afull[sa]);
 #pragma unroll
@@ -891,6 +915,7 @@ __global__ void __launch_bounds__(kWsThreads, 1) kv_kernel(Args a) {
 // the descriptor warp (R19); a segment longer than 32 rows (max_seg hint violated)
 // gets a NaN row.
 constexpr int kBEpi = 8;                    // warps 0-7
+constexpr int kBarBinEpi = 1;               // named barrier of the 8 epilogue warps
 constexpr int kBMma = 8;
 constexpr int kBDesc = 9;
 constexpr int kBW = 10;
@@ -927,7 +952,9 @@ __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uin
   float (*pv)[33] = s_pv[warp];
   for (;; ++tt) {
     const uint32_t ab = tt & 1u, ds = tt % NS;
-    mbar_wait(&dfull[ds], (tt / NS) & 1u);
+    // one warp polls, the other seven block in bar.sync (no issue slots spent waiting)
+    if (warp == 0) mbar_wait(&dfull[ds], (tt / NS) & 1u);
+    named_bar(kBarBinEpi, kBEpi * 32);
     if (!bd[ds].live) {
       warp_arrive(&dempty[ds]);
       break;
@@ -953,7 +980,12 @@ __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uin
     }
     const float qb = __ldg(qrow + dm + head);
     if (threadIdx.x == 0) tl_mark(a, tt, 5);
-    mbar_wait(&tfull[ab], (tt >> 1) & 1u);
+    const long long e0c = clock64();
+    if (warp == 0) mbar_wait(&tfull[ab], (tt >> 1) & 1u);
+    named_bar(kBarBinEpi, kBEpi * 32);
+    const long long e1c = clock64();
+    if (warp == 0) trace(a, 9, tt);
+    if (warp == 0) prof_add(a, 11, e1c - e0c);      // epilogue: wait for the accumulator
     tc_fence_after();
     if (threadIdx.x == 0) tl_mark(a, tt, 6);
     if (a.dbg & 1) {
@@ -1017,6 +1049,8 @@ __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uin
       __syncwarp();
     }
     tc_fence_before();
+    if (warp == 0) trace(a, 10, tt);
+    if (warp == 0) prof_add(a, 12, clock64() - e1c);   // epilogue: tile work
     warp_arrive(&tempty[ab]);
     if (threadIdx.x == 0) tl_mark(a, tt, 7);
   }
@@ -1158,7 +1192,7 @@ __global__ void __launch_bounds__(kBThreads, 1) kv_bin_kernel(Args a) {
       }
       if (threadIdx.x == kBProd0 * 32) tl_mark(a, tt, 2);
       produce_tile<kNPkv, kBProd0, kBGPT>(a.skv, split, pipe, B, ait, tt, bd[ds], s_omega,
-                                          s_phi, a.table, (a.dbg & 2) != 0);
+                                          s_phi, a.table, (a.dbg & 2) != 0, a.dbg);
       if (threadIdx.x == kBProd0 * 32) tl_mark(a, tt, 3);
       warp_arrive(&B.dempty[ds]);
     }
@@ -1182,31 +1216,33 @@ __global__ void __launch_bounds__(kBThreads, 1) kv_bin_kernel(Args a) {
   ws_teardown(tmem, 2 * kCols, kBMma);
 }
 
-// ------------------------------------------------------------------ TMA-gathered K|V attention
-// kv_tma_kernel: the binned K|V attention of kv_bin_kernel with the A operand moved by
-// the TMA engine instead of producer threads.  K is cut into 32-column fp32 chunks
-// per concat segment ([h_src | e | Phi], each padded to 32; the padding K step is
-// skipped when a chunk holds <= 16 real columns).  Per chunk and tile:
-//   TMA warp   : 32 lanes each issue one cp.async.bulk.tensor tile::gather4 (4 rows x
-//                128 B) -> a 16 KB fp32 image of 128 gathered rows (h_src rows by
-//                hsrc_idx, edge-feature rows by eid, precompute-table rows by Delta t),
-//                zero-filled past the segment width, completion on an mbarrier (tx bytes);
-//   converters : 8 warps rewrite the image IN PLACE, 8-row group by 8-row group, as
-//                bf16 hi | lo (512 B each) in the SW64 K-major UMMA layout, computing
-//                Phi(Delta t) = cos(w Delta t + phi) for rows the table does not cover;
+// ------------------------------------------------------------------ async-gathered K|V attention
+// kv_async_kernel: the binned K|V attention with the A operand gathered by LDGSTS
+// (cp.async, 16 B per lane, no register staging) so that ~80 KB of row gathers are in
+// flight per SM.  K is cut into 32-column fp32 chunks per concat segment ([h_src | e |
+// Phi], each padded to 32; the padding K step is skipped when a chunk holds <= 16 real
+// columns).  Per chunk and tile:
+//   producers  : 8 warps; warp w owns the 8-row groups w and w + 8 of the 128-row tile.
+//                It issues the cp.async of a 2-chunk unit kAheadU units before
+//                converting it;
+//                the 16 KB fp32 image (row r at r*128 B) is rewritten IN PLACE, group by
+//                group, as bf16 hi | lo (512 B each) in the SW64 K-major UMMA layout;
+//                Phi(Delta t) = cos(w Delta t + phi) is evaluated for rows the
+//                precompute table does not cover (their time chunks are not loaded);
 //   MMA warp   : tcgen05.mma M=128 N=200 K=16 from the converted image and a SW64
-//                weight chunk (hi|lo, one bulk copy), 3 passes in fp32 mode.
-// No thread ever waits on a global load in the steady state: up to kTAStages chunks
-// (96 KB) of gathers are in flight per SM.
+//                weight chunk (hi|lo, one bulk copy), 3 passes in fp32 mode;
+//   epilogue   : logits, segment softmax and alpha-weighted V sums from TMEM (bin_epilogue).
+// (A TMA tile::gather4 variant of the producers was measured at ~5 B/clk/SM on B200 --
+// 128-byte row boxes -- and dropped.)
 constexpr int kTC = 32;                       // fp32 columns per K chunk
 constexpr int kTAStage = kBM * kTC * 4;       // 16 KB
 constexpr int kTAStages = 6;
+constexpr int kAheadU = kTAStages / 2 - 1;    // 2-chunk units of gathers in flight per producer
 constexpr int kTWStages = 3;
 constexpr int kTWHalf = kNPkv * 64;           // one of W_hi / W_lo of a chunk (12.8 KB)
 constexpr int kTWStage = 2 * kTWHalf;
-constexpr int kTMma = 8, kTW = 9, kTTma = 10, kTDesc0 = 11, kTDescWarps = 2, kTConv0 = 13,
-              kTConvWarps = 7;
-constexpr int kTThreads = (kTConv0 + kTConvWarps) * 32;   // 640 (96 registers per thread)
+constexpr int kTMma = 8, kTW = 9, kTDesc0 = 10, kTDescWarps = 2, kTProd0 = 12, kTProdWarps = 8;
+constexpr int kTThreads = (kTProd0 + kTProdWarps) * 32;   // 640 (96 registers per thread)
 constexpr int kTDSlots = 4;
 constexpr int kTPipeBytes = kTAStages * kTAStage + kTWStages * kTWStage;
 constexpr int kTSmem = 1024 + kTPipeBytes + kBEpi * 32 * 33 * 4;
@@ -1227,40 +1263,46 @@ __host__ __device__ __forceinline__ void plan_chunk(const KvPlan& p, int c, int&
   seg = c < p.c[0] ? 0 : (c < p.c[0] + p.c[1] ? 1 : 2);
   col = (c - (seg > 0 ? p.c[0] : 0) - (seg > 1 ? p.c[1] : 0)) * kTC;
 }
+__device__ __forceinline__ int col_of_time(const KvPlan& p, int c) {
+  return (c - p.c[0] - p.c[1]) * kTC;
+}
 __device__ __forceinline__ int plan_ksteps(const KvPlan& p, int c) {
   int seg, col;
   plan_chunk(p, c, seg, col);
   return p.d[seg] - col > 16 ? 2 : 1;
 }
 
-struct TmaMaps {
-  CUtensorMap m[3];   // h_src, edge features, precompute table (fp32, box 32 x 1)
-};
-
 struct TBars {
-  uint64_t afull[kTAStages], aready[kTAStages], aempty[kTAStages];
+  uint64_t aready[kTAStages], aempty[kTAStages];
   uint64_t wfull[kTWStages], wempty[kTWStages];
   uint64_t dfull[kTDSlots], dempty[kTDSlots];
   uint64_t tfull[2], tempty[2];
 };
 
 struct TDesc {
-  int hrow[kBM];      // gather row of h_src
-  int erow[kBM];      // gather row of the edge features
+  int hrow[kBM];      // row of h_src
+  int erow[kBM];      // row of the edge features
   int trow[kBM];      // precompute-table row, -1 = evaluate eq 8 directly
   float dt[kBM];
   int rdst[kBM];      // destination of the row, -1 = padding
   int live;
 };
 
-__device__ __forceinline__ void tma_gather4(uint32_t dst, const CUtensorMap* map, int col,
-                                            int r0, int r1, int r2, int r3, uint32_t bar) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes"
-      " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(dst),
-      "l"(reinterpret_cast<uint64_t>(map)), "r"(col), "r"(r0), "r"(r1), "r"(r2), "r"(r3),
-      "r"(bar)
-      : "memory");
+// 16-byte LDGSTS with zero fill past src_bytes (0..16)
+__device__ __forceinline__ void cp_async16_zfill(uint32_t dst, const void* src, uint32_t src_bytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src),
+               "r"(src_bytes)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_dyn(int pending) {   // <= pending groups left
+  switch (pending) {
+    case 0: cp_async_wait<0>(); break;
+    case 1: cp_async_wait<1>(); break;
+    case 2: cp_async_wait<2>(); break;
+    case 3: cp_async_wait<3>(); break;
+    case 4: cp_async_wait<4>(); break;
+    default: cp_async_wait<5>(); break;
+  }
 }
 
 // K-major SW64 descriptor: rows of 64 B (32 bf16), 8-row groups `sbo` bytes apart.
@@ -1301,9 +1343,21 @@ __global__ void pack_kv64_kernel(const float* Wk, const float* Wv, int dm, int k
   }
 }
 
+// 16 bytes of row `row` (columns cb..cb+3, zero past `width`; row < 0 -> zeros)
+__device__ __forceinline__ float4 ld_row4(const float* base, int row, int64_t ld, int cb,
+                                          int width) {
+  if (row < 0 || cb >= width) return make_float4(0.f, 0.f, 0.f, 0.f);
+  const float* p = base + (int64_t)row * ld + cb;
+  if (cb + 4 <= width) return __ldg(reinterpret_cast<const float4*>(p));
+  float4 v = make_float4(__ldg(p), 0.f, 0.f, 0.f);
+  if (cb + 1 < width) v.y = __ldg(p + 1);
+  if (cb + 2 < width) v.z = __ldg(p + 2);
+  return v;
+}
+
 __global__ void __launch_bounds__(kTThreads, 1)
-    kv_tma_kernel(const Args a, const KvPlan plan, const __grid_constant__ TmaMaps maps,
-                  const uint8_t* __restrict__ wkv, const int bdst) {
+    kv_async_kernel(const Args a, const KvPlan plan, const uint8_t* __restrict__ wkv,
+                    const int bdst) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* pipe = align1024(smem_raw);
   __shared__ TBars B;
@@ -1326,8 +1380,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
   for (int j = threadIdx.x; j < 2 * dm; j += blockDim.x) s_bias[j] = j < dm ? P.bk[j] : P.bv[j - dm];
   if (threadIdx.x == 0) {
     for (int s = 0; s < kTAStages; ++s) {
-      mbar_init(&B.afull[s], 1);
-      mbar_init(&B.aready[s], kTConvWarps);
+      mbar_init(&B.aready[s], kTProdWarps);
       mbar_init(&B.aempty[s], 1);
     }
     for (int s = 0; s < kTWStages; ++s) {
@@ -1336,7 +1389,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
     }
     for (int s = 0; s < kTDSlots; ++s) {
       mbar_init(&B.dfull[s], 1);
-      mbar_init(&B.dempty[s], kBEpi + kTConvWarps + 3);   // epi, conv, mma, w, tma
+      mbar_init(&B.dempty[s], kBEpi + kTProdWarps + 2);   // epilogue, producers, mma, w
     }
     for (int s = 0; s < 2; ++s) {
       mbar_init(&B.tfull[s], 1);
@@ -1344,17 +1397,13 @@ __global__ void __launch_bounds__(kTThreads, 1)
     }
     fence_mbar_init();
   }
+  if (threadIdx.x < 32) s_trace_n[threadIdx.x] = 0;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (warp == kTMma) tmem_alloc(&s_tmem, 2 * kCols);
-  if (warp == kTTma && lane == 0)
-    for (int s = 0; s < 3; ++s)
-      asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&maps.m[s]))
-                   : "memory");
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = s_tmem;
-  const int64_t D0 = n * blockIdx.x / gridDim.x, D1 = n * (blockIdx.x + 1) / gridDim.x;
   const int nch = plan.n;
   uint32_t tt = 0;
 
@@ -1372,7 +1421,10 @@ __global__ void __launch_bounds__(kTThreads, 1)
     float* stdv = s_td[dw];
     for (tt = dw;; tt += kTDescWarps) {
       const uint32_t ds = tt % kTDSlots;
-      wait_free(&B.dempty[ds], tt / kTDSlots);
+      const long long d0c = clock64();
+      wait_free_sleep(&B.dempty[ds], tt / kTDSlots, 1000);
+      const long long d1c = clock64();
+      if (dw == 0) prof_add(a, 9, d1c - d0c);        // desc: wait for a slot
       if (lane == 0) tl_mark(a, tt, 0);
       TDesc& R = bd[ds];
       const int64_t T = blockIdx.x + (int64_t)tt * gridDim.x;
@@ -1389,7 +1441,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
       int64_t er[4] = {0, 0, 0, 0};
       float tr[4] = {0.f, 0.f, 0.f, 0.f};
       int dr[4] = {-1, -1, -1, -1};
-      unsigned zero_bins = 0;                        // bins whose rows overflow 32
+      unsigned ovf_bins = 0;                         // bins whose rows overflow 32
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
         const int j0 = u * bdst;
@@ -1397,7 +1449,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
         const int j1 = (j0 + bdst) < nd ? j0 + bdst : nd;
         const int64_t e0 = sg[j0], e1 = sg[j1];
         if (e1 - e0 > 32) {                          // max_seg violated: NaN rows
-          zero_bins |= 1u << u;
+          ovf_bins |= 1u << u;
           continue;
         }
         const int64_t e = e0 + lane;
@@ -1409,9 +1461,9 @@ __global__ void __launch_bounds__(kTThreads, 1)
           tr[u] = stdv[j];
         }
       }
-      // empty segments -> r = 0 (R19); overflowing bins -> NaN
+      // empty segments -> r = 0 (R19); destinations of an overflowing bin -> NaN
       for (int j = 0; j < nd; ++j) {
-        const bool ovf = (zero_bins >> (j / bdst)) & 1u;
+        const bool ovf = (ovf_bins >> (j / bdst)) & 1u;
         if (sg[j + 1] == sg[j] || ovf) {
           const float fill = ovf ? __int_as_float(0x7fc00000) : 0.f;
           for (int c = lane; c < dm; c += 32) a.rbuf[(d0 + j) * kQLd + c] = fill;
@@ -1434,13 +1486,14 @@ __global__ void __launch_bounds__(kTThreads, 1)
         const int r = 32 * u + lane;
         const bool ok = dr[u] >= 0;
         const float dt = tr[u] - et[u];               // fp32 delta (R18)
-        R.hrow[r] = hi[u];
-        R.erow[r] = ei[u];
+        R.hrow[r] = ok ? hi[u] : -1;
+        R.erow[r] = ok ? ei[u] : -1;
         R.dt[r] = ok ? dt : 0.f;
-        R.trow[r] = ok ? (int)tenc_table_row(dt, a.table, a.window) : (a.table ? 0 : -1);
+        R.trow[r] = ok ? (int)tenc_table_row(dt, a.table, a.window) : -1;
         R.rdst[r] = dr[u];
       }
       warp_arrive(&B.dfull[ds]);
+      if (dw == 0) prof_add(a, 10, clock64() - d1c); // desc: build
       if (lane == 0) tl_mark(a, tt, 1);
     }
   } else if (warp == kTW) {                          // ---------------- weight loader
@@ -1448,7 +1501,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
     const uint32_t wbytes = split ? kTWStage : kTWHalf;
     for (;; ++tt) {
       const uint32_t ds = tt % kTDSlots;
-      mbar_wait(&B.dfull[ds], (tt / kTDSlots) & 1u);
+      mbar_wait_sleep(&B.dfull[ds], (tt / kTDSlots) & 1u, 1000);
       const int live = bd[ds].live;
       warp_arrive(&B.dempty[ds]);
       if (!live) break;
@@ -1457,7 +1510,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
         for (int i = r0; i < nch; ++i) {
           const uint32_t k = wl + (i - r0);
           const uint32_t sw = k % kTWStages;
-          wait_free(&B.wempty[sw], k / kTWStages);
+          wait_free_sleep(&B.wempty[sw], k / kTWStages, 500);
           if (a.dbg & 8) {
             mbar_arrive(&B.wfull[sw]);
             continue;
@@ -1470,168 +1523,234 @@ __global__ void __launch_bounds__(kTThreads, 1)
       }
       __syncwarp();
     }
-  } else if (warp == kTTma) {                        // ---------------- TMA gathers
-    uint32_t ait = 0;
-    for (;; ++tt) {
-      const uint32_t ds = tt % kTDSlots;
-      mbar_wait(&B.dfull[ds], (tt / kTDSlots) & 1u);
-      const TDesc& R = bd[ds];
-      const int live = R.live;
-      int rows[3][4];
-      bool thit = false;                   // some row of the tile reads the table
-#pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        rows[0][u] = R.hrow[4 * lane + u];
-        rows[1][u] = R.erow[4 * lane + u];
-        const int t = R.trow[4 * lane + u];
-        rows[2][u] = t > 0 ? t : 0;
-        thit |= t >= 0;
-      }
-      warp_arrive(&B.dempty[ds]);
-      if (!live) break;
-      thit = __any_sync(0xffffffffu, thit) && a.table != nullptr;
-      if (lane == 0) tl_mark(a, tt, 2);
-      for (int i = 0; i < nch; ++i, ++ait) {
-        const int c = chunk_of(tt, i, nch);
-        int seg, col;
-        plan_chunk(plan, c, seg, col);
-        const uint32_t s = ait % kTAStages;
-        wait_free(&B.aempty[s], ait / kTAStages);
-        const bool tma = (seg < 2 || thit) && !(a.dbg & 2);
-        if (lane == 0) {
-          if (tma) mbar_arrive_expect_tx(&B.afull[s], kTAStage);
-          else mbar_arrive(&B.afull[s]);
-        }
-        __syncwarp();
-        if (tma) {
-          int r[4];
-#pragma unroll
-          for (int u = 0; u < 4; ++u) r[u] = seg == 0 ? rows[0][u] : (seg == 1 ? rows[1][u] : rows[2][u]);
-          const CUtensorMap* m = seg == 0 ? &maps.m[0] : (seg == 1 ? &maps.m[1] : &maps.m[2]);
-          tma_gather4(smem_u32(pipe + s * kTAStage + lane * 512), m, col, r[0], r[1], r[2], r[3],
-                      smem_u32(&B.afull[s]));
-        }
-      }
-    }
-  } else if (warp >= kTConv0) {                      // ---------------- converters
-    // warp cw converts the 8-row groups g = cw, cw + 7, cw + 14 (< 16) of each chunk;
-    // lane: row rr (and rr + 4) of the group, 16-byte column chunk j
-    const int cw = warp - kTConv0;
+  } else if (warp >= kTProd0) {                      // ---------------- producers
+    // Work unit = two consecutive chunks of a tile (one cp.async group, one fence):
+    // loads run kAheadU units ahead of the conversion.  Lane: rows rr and rr + 4 of
+    // groups pw and pw + 8 (rows u = 0..3 -> rw0..rw3), 16-byte column piece j.
+    const int pw = warp - kTProd0;
     const int rr = lane >> 3, j = lane & 7;
-    uint32_t ait = 0;
-    for (;; ++tt) {
-      const uint32_t ds = tt % kTDSlots;
-      mbar_wait(&B.dfull[ds], (tt / kTDSlots) & 1u);
-      const TDesc& R = bd[ds];
-      const int live = R.live;
-      float dt[6];
-      int tr[6];
+    const int rw0 = pw * 8 + rr, rw1 = rw0 + 4, rw2 = rw0 + 64, rw3 = rw0 + 68;
+    const int npair = (nch + 1) >> 1;
+    const uint32_t pipe_s = smem_u32(pipe);
+    uint32_t lt = 0, ct = 0, al = 0, ac = 0, ul = 0, uc = 0;
+    int lp = 0, cp = 0;
+    bool lend = false;
+    int hr0, hr1, hr2, hr3, er0, er1, er2, er3, tr0, tr1, tr2, tr3;
+    float cdt0 = 0.f, cdt1 = 0.f, cdt2 = 0.f, cdt3 = 0.f;
+    int ctr0 = -1, ctr1 = -1, ctr2 = -1, ctr3 = -1;
+#define TGL_ENTER_LOAD_TILE()                                                          \
+  do {                                                                                 \
+    const uint32_t ds_ = lt % kTDSlots;                                                \
+    mbar_wait_sleep(&B.dfull[ds_], (lt / kTDSlots) & 1u, 500);                         \
+    const TDesc& R_ = bd[ds_];                                                         \
+    if (!R_.live) {                                                                    \
+      lend = true;                                                                     \
+      break;                                                                           \
+    }                                                                                  \
+    hr0 = R_.hrow[rw0]; hr1 = R_.hrow[rw1]; hr2 = R_.hrow[rw2]; hr3 = R_.hrow[rw3];    \
+    er0 = R_.erow[rw0]; er1 = R_.erow[rw1]; er2 = R_.erow[rw2]; er3 = R_.erow[rw3];    \
+    tr0 = R_.trow[rw0]; tr1 = R_.trow[rw1]; tr2 = R_.trow[rw2]; tr3 = R_.trow[rw3];    \
+  } while (0)
+    TGL_ENTER_LOAD_TILE();
+    for (;;) {
+      // ---- keep kAheadU units of gathers in flight
+      while (!lend && ul < uc + kAheadU && lt < ct + kTDSlots - 1) {
+        const int i0 = 2 * lp, cnt = (nch - i0) < 2 ? (nch - i0) : 2;
 #pragma unroll
-      for (int u = 0; u < 6; ++u) {                  // rows (g, rr + 4(u&1)), g = cw + 7(u>>1)
-        const int g = cw + kTConvWarps * (u >> 1);
-        const int r = g * 8 + rr + 4 * (u & 1);
-        dt[u] = g < 16 ? R.dt[r] : 0.f;
-        tr[u] = g < 16 ? R.trow[r] : 0;
-      }
-      warp_arrive(&B.dempty[ds]);
-      if (!live) break;
-      for (int i = 0; i < nch; ++i, ++ait) {
-        const int c = chunk_of(tt, i, nch);
-        int seg, col;
-        plan_chunk(plan, c, seg, col);
-        const uint32_t s = ait % kTAStages;
-        mbar_wait(&B.afull[s], (ait / kTAStages) & 1u);
-        const uint32_t sb = smem_u32(pipe + s * kTAStage);
-        if (a.dbg & 64) {
-          warp_arrive(&B.aready[s]);
-          continue;
-        }
-#pragma unroll
-        for (int gg = 0; gg < 3; ++gg) {
-          const int g = cw + kTConvWarps * gg;
-          if (g >= 16) break;
-          float4 x[2];
-#pragma unroll
-          for (int h = 0; h < 2; ++h) {
-            const int u = 2 * gg + h, r = rr + 4 * h;
-            if (seg < 2 || tr[u] >= 0) {
-              x[h] = ld_shared_f4(sb + g * 1024 + r * 128 + j * 16);
-            } else {
-              float y[4];
-#pragma unroll
-              for (int e = 0; e < 4; ++e) {
-                const int cc = col + 4 * j + e;
-                y[e] = cc < P.d_t ? tenc_fast(dt[u], s_omega[cc], s_phi[cc]) : 0.f;
-              }
-              x[h] = make_float4(y[0], y[1], y[2], y[3]);
-            }
-          }
-          __syncwarp();
-#pragma unroll
-          for (int h = 0; h < 2; ++h) {
-            const int r = rr + 4 * h;
-            uint32_t h0, h1, l0, l1;
-            split2(x[h].x, x[h].y, h0, l0);
-            split2(x[h].z, x[h].w, h1, l1);
-            const uint32_t off = sb + g * 1024 + sw64_off(r, 4 * j);
-            asm volatile("st.shared.v2.b32 [%0], {%1, %2};" ::"r"(off), "r"(h0), "r"(h1) : "memory");
-            if (split)
-              asm volatile("st.shared.v2.b32 [%0], {%1, %2};" ::"r"(off + 512), "r"(l0), "r"(l1)
-                           : "memory");
+        for (int q = 0; q < 2; ++q) {
+          if (q >= cnt) break;
+          const int c = chunk_of(lt, i0 + q, nch);
+          const int seg = c < plan.c[0] ? 0 : (c < plan.c[0] + plan.c[1] ? 1 : 2);
+          const int col = (c - (seg > 0 ? plan.c[0] : 0) - (seg > 1 ? plan.c[1] : 0)) * kTC;
+          const int width = seg == 0 ? plan.d[0] : (seg == 1 ? plan.d[1] : plan.d[2]);
+          const uint32_t s = (al + q) % kTAStages;
+          wait_free(&B.aempty[s], (al + q) / kTAStages);
+          const uint32_t sb = pipe_s + s * kTAStage + rw0 * 128 + j * 16;
+          const int cb = col + 4 * j;                // first fp32 column of this lane
+          const uint32_t nb = cb >= width ? 0u : (uint32_t)min(16, (width - cb) * 4);
+          if (!(a.dbg & 2)) {
+            const float* base = seg == 0 ? a.hsrc : (seg == 1 ? a.efeat : a.table);
+            const int64_t ld = seg == 0 ? a.ld_hsrc : (seg == 1 ? a.ld_e : (int64_t)P.d_t);
+            const int x0 = seg == 0 ? hr0 : (seg == 1 ? er0 : tr0);
+            const int x1 = seg == 0 ? hr1 : (seg == 1 ? er1 : tr1);
+            const int x2 = seg == 0 ? hr2 : (seg == 1 ? er2 : tr2);
+            const int x3 = seg == 0 ? hr3 : (seg == 1 ? er3 : tr3);
+            // padding rows and rows the table misses (time chunks) load nothing
+            const float* b = base + cb;
+            if (x0 >= 0) cp_async16_zfill(sb, b + (int64_t)x0 * ld, nb);
+            if (x1 >= 0) cp_async16_zfill(sb + 512, b + (int64_t)x1 * ld, nb);
+            if (x2 >= 0) cp_async16_zfill(sb + 8192, b + (int64_t)x2 * ld, nb);
+            if (x3 >= 0) cp_async16_zfill(sb + 8192 + 512, b + (int64_t)x3 * ld, nb);
           }
         }
-        fence_proxy_async_smem();
-        warp_arrive(&B.aready[s]);
+        cp_async_commit();
+        al += cnt;
+        ++ul;
+        if (++lp == npair) {
+          lp = 0;
+          ++lt;
+          TGL_ENTER_LOAD_TILE();
+        }
       }
-      if (threadIdx.x == kTConv0 * 32) tl_mark(a, tt, 3);
+      if (uc == ul) break;                           // everything loaded has been converted
+      // ---- convert unit uc (loaded kAheadU units ago)
+      if (cp == 0) {                                 // entering tile ct: per-row time inputs
+        const uint32_t ds = ct % kTDSlots;
+        const TDesc& R = bd[ds];
+        cdt0 = R.dt[rw0]; cdt1 = R.dt[rw1]; cdt2 = R.dt[rw2]; cdt3 = R.dt[rw3];
+        ctr0 = R.trow[rw0]; ctr1 = R.trow[rw1]; ctr2 = R.trow[rw2]; ctr3 = R.trow[rw3];
+        warp_arrive(&B.dempty[ds]);                  // last read of this slot by the warp
+        if (threadIdx.x == kTProd0 * 32) tl_mark(a, ct, 2);
+      }
+      const int i0 = 2 * cp, cnt = (nch - i0) < 2 ? (nch - i0) : 2;
+      cp_async_wait_dyn((int)(ul - uc - 1));
+      __syncwarp();
+      float4 x[2][4];
+      uint32_t gb[2];
+#pragma unroll
+      for (int q = 0; q < 2; ++q) {                  // all shared loads of the unit first
+        gb[q] = pipe_s + ((ac + q) % kTAStages) * kTAStage + pw * 1024;
+        if (q < cnt) {
+          x[q][0] = ld_shared_f4(gb[q] + rr * 128 + j * 16);
+          x[q][1] = ld_shared_f4(gb[q] + (rr + 4) * 128 + j * 16);
+          x[q][2] = ld_shared_f4(gb[q] + 8192 + rr * 128 + j * 16);
+          x[q][3] = ld_shared_f4(gb[q] + 8192 + (rr + 4) * 128 + j * 16);
+        }
+      }
+#pragma unroll
+      for (int q = 0; q < 2; ++q) {
+        if (q >= cnt) break;
+        const int c = chunk_of(ct, i0 + q, nch);
+        if (c >= plan.c[0] + plan.c[1] && !(a.dbg & 1024)) {   // time chunk: Phi where the table misses
+          const int cc = col_of_time(plan, c) + 4 * j;
+          float w[4], f[4];
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            const bool ok = cc + e < P.d_t;
+            w[e] = ok ? s_omega[cc + e] : 0.f;
+            f[e] = ok ? s_phi[cc + e] : 0.f;
+          }
+#define TGL_PHI4(X, DT, TR)                                                              \
+  if (TR < 0) {                                                                          \
+    X.x = (cc < P.d_t) ? tenc_fast(DT, w[0], f[0]) : 0.f;                                \
+    X.y = (cc + 1 < P.d_t) ? tenc_fast(DT, w[1], f[1]) : 0.f;                            \
+    X.z = (cc + 2 < P.d_t) ? tenc_fast(DT, w[2], f[2]) : 0.f;                            \
+    X.w = (cc + 3 < P.d_t) ? tenc_fast(DT, w[3], f[3]) : 0.f;                            \
+  }
+          TGL_PHI4(x[q][0], cdt0, ctr0)
+          TGL_PHI4(x[q][1], cdt1, ctr1)
+          TGL_PHI4(x[q][2], cdt2, ctr2)
+          TGL_PHI4(x[q][3], cdt3, ctr3)
+#undef TGL_PHI4
+        }
+      }
+      __syncwarp();
+      if (!(a.dbg & 64)) {
+        const uint32_t o0 = sw64_off(rr, 4 * j), o1 = sw64_off(rr + 4, 4 * j);
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+          if (q >= cnt) break;
+          uint32_t h0, h1, l0, l1;
+#define TGL_SPLIT_STORE(X, ADDR)                                                         \
+  split2(X.x, X.y, h0, l0);                                                              \
+  split2(X.z, X.w, h1, l1);                                                              \
+  asm volatile("st.shared.v2.b32 [%0], {%1, %2};" ::"r"(ADDR), "r"(h0), "r"(h1) : "memory"); \
+  if (split)                                                                             \
+    asm volatile("st.shared.v2.b32 [%0], {%1, %2};" ::"r"((ADDR) + 512), "r"(l0), "r"(l1)   \
+                 : "memory");
+          TGL_SPLIT_STORE(x[q][0], gb[q] + o0)
+          TGL_SPLIT_STORE(x[q][1], gb[q] + o1)
+          TGL_SPLIT_STORE(x[q][2], gb[q] + 8192 + o0)
+          TGL_SPLIT_STORE(x[q][3], gb[q] + 8192 + o1)
+#undef TGL_SPLIT_STORE
+        }
+      }
+      if (!(a.dbg & 2048)) fence_proxy_async_smem();   // 2048: profiling only (unsafe)
+      __syncwarp();
+      if (lane == 0) {
+        mbar_arrive(&B.aready[ac % kTAStages]);
+        if (cnt == 2) mbar_arrive(&B.aready[(ac + 1) % kTAStages]);
+      }
+      ac += cnt;
+      ++uc;
+      if (++cp == npair) {
+        cp = 0;
+        if (threadIdx.x == kTProd0 * 32) tl_mark(a, ct, 3);
+        ++ct;
+      }
     }
+#undef TGL_ENTER_LOAD_TILE
   } else if (warp == kTMma) {                        // ---------------- MMA issuer
+    // The whole warp walks the loop (uniform control flow; one elected lane issues),
+    // two K chunks per trip to halve the per-chunk handshake cost.
     uint32_t ait = 0, wl = 0;
     constexpr uint32_t idesc = idesc_bf16(kBM, kNPkv);
+    const uint32_t pipe_s = smem_u32(pipe);
+    const uint32_t w_s = pipe_s + kTAStages * kTAStage;
     for (;; ++tt) {
       const uint32_t ds = tt % kTDSlots;
       mbar_wait(&B.dfull[ds], (tt / kTDSlots) & 1u);
       const int live = bd[ds].live;
       warp_arrive(&B.dempty[ds]);
       if (!live) break;
-      if (lane == 0) {
-        const uint32_t acc = tmem + (tt & 1u) * kCols;
-        wait_free(&B.tempty[tt & 1u], tt >> 1);
-        tc_fence_after();
-        tl_mark(a, tt, 4);
-        const int r0 = (tt > 0 && nch >= 4) ? 2 : 0;
-        for (int i = 0; i < nch; ++i, ++ait) {
-          const int c = chunk_of(tt, i, nch);
-          const uint32_t s = ait % kTAStages;
-          mbar_wait(&B.aready[s], (ait / kTAStages) & 1u);
-          uint32_t k;
-          if (i < r0) {
-            k = wl - 1 - i;
+      const uint32_t acc = tmem + (tt & 1u) * kCols;
+      const long long m2 = clock64();
+      wait_free_sleep(&B.tempty[tt & 1u], tt >> 1, 200);
+      prof_add(a, 7, clock64() - m2);                  // MMA: wait for the accumulator
+      tc_fence_after();
+      trace(a, 7, tt);
+      if (lane == 0) tl_mark(a, tt, 4);
+      const int r0 = (tt > 0 && nch >= 4) ? 2 : 0;
+      for (int i = 0; i < nch; i += 2, ait += 2) {
+        const int cnt = (nch - i) < 2 ? (nch - i) : 2;
+        uint32_t st[2], kw[2];
+        int cc[2];
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+          if (q >= cnt) break;
+          const uint32_t a_ = ait + q;
+          st[q] = a_ % kTAStages;
+          cc[q] = chunk_of(tt, i + q, nch);
+          mbar_wait(&B.aready[st[q]], (a_ / kTAStages) & 1u);
+          if (i + q < r0) {
+            kw[q] = wl - 1 - (i + q);                  // resident from the previous tile
           } else {
-            k = wl + (i - r0);
-            mbar_wait(&B.wfull[k % kTWStages], (k / kTWStages) & 1u);
+            kw[q] = wl + (i + q - r0);
+            mbar_wait(&B.wfull[kw[q] % kTWStages], (kw[q] / kTWStages) & 1u);
           }
-          const uint32_t sw = k % kTWStages;
-          tc_fence_after();
-          const uint32_t ab = smem_u32(pipe + s * kTAStage);
-          const uint32_t wb = smem_u32(pipe + kTAStages * kTAStage + sw * kTWStage);
-          const int nk = (a.dbg & 4) ? 0 : plan_ksteps(plan, c);
-          for (int ks = 0; ks < nk; ++ks) {
-            const uint64_t ah = desc_sw64(ab + ks * 32, 1024), bh = desc_sw64(wb + ks * 32, 512);
-            mma_bf16(acc, ah, bh, idesc, (i | ks) != 0);
-            if (split) {
-              mma_bf16(acc, desc_sw64(ab + 512 + ks * 32, 1024), bh, idesc, 1u);
-              mma_bf16(acc, ah, desc_sw64(wb + kTWHalf + ks * 32, 512), idesc, 1u);
+        }
+        tc_fence_after();
+        if (elect_one()) {
+#pragma unroll
+          for (int q = 0; q < 2; ++q) {
+            if (q >= cnt) break;
+            const uint32_t ab = pipe_s + st[q] * kTAStage;
+            const uint32_t wb = w_s + (kw[q] % kTWStages) * kTWStage;
+            const int nk = (a.dbg & 4) ? 0 : plan_ksteps(plan, cc[q]);
+            for (int ks = 0; ks < nk; ++ks) {
+              const uint64_t ah = desc_sw64(ab + ks * 32, 1024), bh = desc_sw64(wb + ks * 32, 512);
+              mma_bf16(acc, ah, bh, idesc, ((i + q) | ks) != 0);
+              if (split) {
+                mma_bf16(acc, desc_sw64(ab + 512 + ks * 32, 1024), bh, idesc, 1u);
+                mma_bf16(acc, ah, desc_sw64(wb + kTWHalf + ks * 32, 512), idesc, 1u);
+              }
             }
           }
-          mma_commit(&B.aempty[s]);
-          const bool keep = (nch >= 4) && (i >= nch - 2);
-          if (!keep) mma_commit(&B.wempty[sw]);
+#pragma unroll
+          for (int q = 0; q < 2; ++q) {
+            if (q >= cnt) break;
+            mma_commit(&B.aempty[st[q]]);
+            const bool keep = (nch >= 4) && (i + q >= nch - 2);   // reused by the next tile
+            if (!keep) mma_commit(&B.wempty[kw[q] % kTWStages]);
+          }
         }
-        wl += nch - r0;
-        mma_commit(&B.tfull[tt & 1u]);
+        __syncwarp();
       }
+      ait -= (uint32_t)((nch & 1) ? 1 : 0);            // the last trip may hold one chunk
+      wl += nch - r0;
+      if (elect_one()) mma_commit(&B.tfull[tt & 1u]);
       __syncwarp();
+      prof_add(a, 8, clock64() - m2);                  // MMA: whole tile
     }
   } else {                                           // ---------------- epilogue warps 0-7
     bin_epilogue<kTDSlots>(a, B.dfull, B.dempty, B.tfull, B.tempty, bd, tmem, s_pv, s_bias);
@@ -1682,38 +1801,11 @@ static tgl_status launch_pack(const tgl_attn_params* P, uint8_t* base, cudaStrea
 
 namespace tca {
 
-// cuTensorMapEncodeTiled through the runtime's driver entry point (no -lcuda)
-static PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
-  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
-  if (fn == nullptr) {
-    void* f = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) ==
-            cudaSuccess &&
-        q == cudaDriverEntryPointSuccess)
-      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(f);
-  }
-  return fn;
-}
-
-// Row table [rows][ld] fp32 as a 2-D tensor map with a 32-column x 1-row box (the
-// gather4 unit).  Columns >= width read as zero (OOB fill).  False when TMA cannot
-// address the table (base not 16-B aligned or a row pitch that is not a multiple of
-// 16 B) -- the caller then takes the register-gather kernel.
-static bool encode_rows(CUtensorMap* m, const float* base, int width, int64_t ld, int64_t rows) {
-  memset(m, 0, sizeof(*m));
-  if (width <= 0) return true;                       // segment absent: map unused
-  if (base == nullptr || (reinterpret_cast<uintptr_t>(base) & 15) || ((ld * 4) & 15)) return false;
-  PFN_cuTensorMapEncodeTiled_v12000 enc = tensor_map_encoder();
-  if (enc == nullptr) return false;
-  cuuint64_t dims[2] = {(cuuint64_t)width, (cuuint64_t)rows};
-  cuuint64_t strides[1] = {(cuuint64_t)ld * 4};
-  cuuint32_t box[2] = {(cuuint32_t)kTC, 1};
-  cuuint32_t es[2] = {1, 1};
-  return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box,
-             es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-             CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
-             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+// The async gathers move 16-byte pieces of feature rows: a row table qualifies when
+// its base is 16-byte aligned and its row pitch a multiple of 16 bytes.
+static bool rows_16b(const float* base, int width, int64_t ld) {
+  if (width <= 0) return true;                       // segment absent
+  return base != nullptr && !(reinterpret_cast<uintptr_t>(base) & 15) && !((ld * 4) & 15);
 }
 
 }  // namespace tca
@@ -1790,7 +1882,7 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
   const int smem_q = Pipe<kNPq>::kBytes + 1024;
   const int smem_kv = Pipe<kNPkv>::kBytes + 1024 + kKvEpiBytes;
   const int smem_kvb = Pipe<kNPkv>::kBytes + 1024 + kBEpi * 32 * 33 * 4;
-  // TGL_KV = "bin" forces the register-gather kernel, "tma" requires the TMA one
+  // TGL_KV = "bin" forces the register-gather kernel, "async" requires the LDGSTS one
   const char* kvsel = getenv("TGL_KV");
   static bool attr_done = false;   // cached cudaFuncSetAttribute (idempotent)
   if (!attr_done) {
@@ -1805,9 +1897,9 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
     TGL_TRY(cuda_check(cudaFuncSetAttribute(kv_bin_kernel,
                                             cudaFuncAttributeMaxDynamicSharedMemorySize, smem_kvb),
                        "attr kv bin"));
-    TGL_TRY(cuda_check(cudaFuncSetAttribute(kv_tma_kernel,
+    TGL_TRY(cuda_check(cudaFuncSetAttribute(kv_async_kernel,
                                             cudaFuncAttributeMaxDynamicSharedMemorySize, kTSmem),
-                       "attr kv tma"));
+                       "attr kv async"));
     attr_done = true;
   }
   const int64_t tiles = ceil_div(n_dst_max, kBM);
@@ -1815,23 +1907,20 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
   dense_kernel<false><<<gq, kWsThreads, smem_q, s>>>(a);
   TGL_TRY(launch_check("tc q kernel"));
   const bool binned = max_seg > 0 && max_seg <= 32 && P->n_heads == 2;
-  TmaMaps maps;
-  const bool tma = binned && !(kvsel && strcmp(kvsel, "bin") == 0) &&
-                   encode_rows(&maps.m[0], hsrc, P->d_hsrc, ld_hsrc, 0x7fffffffLL) &&
-                   encode_rows(&maps.m[1], efeat, P->d_e, ld_e, 0x7fffffffLL) &&
-                   encode_rows(&maps.m[2], table, table ? P->d_t : 0, P->d_t,
-                               window > 0 ? window : 1);
-  if (kvsel && strcmp(kvsel, "tma") == 0 && !tma) {
-    set_error("TGL_KV=tma: the TMA gather path cannot take this call (alignment / max_seg)");
+  const bool async = binned && !(kvsel && strcmp(kvsel, "bin") == 0) &&
+                     rows_16b(hsrc, P->d_hsrc, ld_hsrc) && rows_16b(efeat, P->d_e, ld_e) &&
+                     rows_16b(table, table ? P->d_t : 0, P->d_t);
+  if (kvsel && strcmp(kvsel, "async") == 0 && !async) {
+    set_error("TGL_KV=async: the async-gather path cannot take this call (16-B row pitch / "
+              "max_seg <= 32 / 2 heads)");
     return TGL_EUNSUPPORTED;
   }
-  if (tma) {
-    const unsigned gkv = (unsigned)(n_dst_max < kNumSMs ? (n_dst_max > 0 ? n_dst_max : 1) : kNumSMs);
+  if (async) {
     const int bdst = 32 / max_seg;                 // destinations per 32-row bin
     const int64_t ttiles = ceil_div(n_dst_max, 4 * bdst);
     const unsigned gt = (unsigned)(ttiles < kNumSMs ? (ttiles > 0 ? ttiles : 1) : kNumSMs);
-    kv_tma_kernel<<<gt, kTThreads, kTSmem, s>>>(a, make_plan(P->d_hsrc, P->d_e, P->d_t), maps,
-                                                pk + PL.okv64, bdst);
+    kv_async_kernel<<<gt, kTThreads, kTSmem, s>>>(a, make_plan(P->d_hsrc, P->d_e, P->d_t),
+                                                  pk + PL.okv64, bdst);
   } else if (binned) {
     // binned path: whole segments per epilogue warp (no block barriers)
     const unsigned gkv = (unsigned)(n_dst_max < kNumSMs ? (n_dst_max > 0 ? n_dst_max : 1) : kNumSMs);
@@ -1876,4 +1965,20 @@ extern "C" tgl_status tgl_attn_pack(const tgl_attn_params* P, void* packed, size
   }
   TGL_REQUIRE((reinterpret_cast<uintptr_t>(packed) & 255) == 0, "packed must be 256-aligned");
   return tca::launch_pack(P, static_cast<uint8_t*>(packed), as_stream(stream));
+}
+
+extern "C" int tgl_debug_prof(unsigned long long* host, int reset) {
+  if (reset) {
+    static unsigned long long z[tgl::kNumSMs * 16];
+    return (int)cudaMemcpyToSymbol(tgl::tca::g_prof, z, sizeof(z));
+  }
+  return (int)cudaMemcpyFromSymbol(host, tgl::tca::g_prof, sizeof(unsigned long long) * tgl::kNumSMs * 16);
+}
+
+extern "C" int tgl_debug_trace(unsigned long long* host, int reset) {
+  if (reset) {
+    static unsigned long long z[8192];
+    return (int)cudaMemcpyToSymbol(tgl::tca::g_trace, z, sizeof(z));
+  }
+  return (int)cudaMemcpyFromSymbol(host, tgl::tca::g_trace, sizeof(unsigned long long) * 8192);
 }

@@ -21,8 +21,12 @@ __device__ __forceinline__ float tenc_direct(float dt, float omega, float phi) {
 // take the accurate cosf.  Accurate cosf falls back to Payne-Hanek reduction for
 // |b| > 105615 (REDDIT/LASTFM Delta t reach 1e6-1e8 with omega_0 = 1), which costs
 // hundreds of instructions and local memory per element.
+static __device__ __noinline__ float tenc_cos_slow(float b) { return cosf(b); }
+
 __device__ __forceinline__ float tenc_cos_fast(float b) {
-  if (!(fabsf(b) < 1e9f)) return cosf(b);
+  // out of line: an inlined cosf would drag its Payne-Hanek path (local-memory table
+  // walk) into every call site, predicated on in the steady state
+  if (!(fabsf(b) < 1e9f)) return tenc_cos_slow(b);
   const float k = rintf(b * 0.159154943091895336f);
   float r = fmaf(-k, 6.28318548202514648f, b);
   r = fmaf(-k, -1.74845560007449713e-7f, r);

@@ -205,7 +205,7 @@ def cu_pad(a, mult=4):
     return t[:, :d]
 
 
-@pytest.mark.parametrize("precision,kv", [("fp32", "tma"), ("bf16", "tma"), ("fp32", "bin"),
+@pytest.mark.parametrize("precision,kv", [("fp32", "async"), ("bf16", "async"), ("fp32", "bin"),
                                           ("bf16", "bin"), ("fp32_simt", None)])
 @pytest.mark.parametrize("n_dst,kmax,d_h,d_e,long_every", [(1, 10, 172, 172, 0),
                                                           (777, 10, 172, 172, 0),
@@ -215,8 +215,8 @@ def cu_pad(a, mult=4):
                                                           (517, 10, 128, 0, 0),
                                                           (150, 10, 24, 12, 7)])
 def test_attention_vs_oracle(T, monkeypatch, precision, kv, n_dst, kmax, d_h, d_e, long_every):
-    """TGL_KV selects the K|V kernel: "tma" (TMA gather4, needs 16-B row pitches: the
-    odd GDELT widths 413/186 go in row-padded views) or "bin" (register gathers)."""
+    """TGL_KV selects the K|V kernel: "async" (cp.async gathers, needs 16-B row pitches:
+    the odd GDELT widths 413/186 go in row-padded views) or "bin" (register gathers)."""
     rng = np.random.default_rng(n_dst + kmax)
     p, seg, dst_t, nfeat, dn, sn, ef, eid, et = attn_case(rng, n_dst, kmax, d_h, d_e,
                                                           long_every=long_every)
@@ -225,7 +225,7 @@ def test_attention_vs_oracle(T, monkeypatch, precision, kv, n_dst, kmax, d_h, d_
     exp = oracle.tblock_attn(p, seg, dst_t, nfeat, dn, nfeat, sn, ef, eid, et)
     P = T.AttnParams(p, precision=precision, pack=(n_dst % 2 == 1))
     tab = T.time_precompute(65536, P.t["omega"], P.t["phi"])
-    put = cu_pad if kv == "tma" else cu
+    put = cu_pad if kv == "async" else cu
     nf = put(nfeat)
     for table in (None, tab):
         got = T.tblock_attn(P, cu(seg), cu(dst_t), nf, cu(dn), nf, cu(sn),
@@ -235,15 +235,15 @@ def test_attention_vs_oracle(T, monkeypatch, precision, kv, n_dst, kmax, d_h, d_
         assert err <= TOL[precision], err
 
 
-def test_attention_tma_rejects_unaligned_pitch(T, monkeypatch):
-    """TGL_KV=tma on a 413-float row pitch (1652 B, not a multiple of 16): EUNSUPPORTED,
+def test_attention_async_rejects_unaligned_pitch(T, monkeypatch):
+    """TGL_KV=async on a 413-float row pitch (1652 B, not a multiple of 16): EUNSUPPORTED,
     while the default dispatch falls back to the register-gather kernel."""
     rng = np.random.default_rng(5)
     p, seg, dst_t, nfeat, dn, sn, ef, eid, et = attn_case(rng, 64, 10, 413, 186)
     exp = oracle.tblock_attn(p, seg, dst_t, nfeat, dn, nfeat, sn, ef, eid, et)
     P = T.AttnParams(p)
     args = (P, cu(seg), cu(dst_t), cu(nfeat), cu(dn), cu(nfeat), cu(sn), cu(ef), cu(eid), cu(et))
-    monkeypatch.setenv("TGL_KV", "tma")
+    monkeypatch.setenv("TGL_KV", "async")
     with pytest.raises(T.TGLError):
         T.tblock_attn(*args, max_seg=10)
     monkeypatch.delenv("TGL_KV")

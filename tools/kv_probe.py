@@ -4,7 +4,7 @@
 
 TGL_DEBUG_MASK bits (profiling only): 1 skip epilogue math, 2 skip A gathers,
 4 skip MMAs, 8 skip weight copies, 16 skip descriptor index loads, 64 skip the
-converters (kv_tma), 32 per-tile timeline.
+converters (kv_async), 32 per-tile timeline.
 """
 import os
 import sys
@@ -57,7 +57,7 @@ nd = int(b.u_dev.item())
 ne = int(b.seg_ptr[nd].item())
 print(f"tail block: {nd} dst, {ne} edges, precision {prec}")
 ref = None
-KVS = os.environ.get("PROBE_KV", "bin,tma").split(",")
+KVS = os.environ.get("PROBE_KV", "bin,async").split(",")
 MASKS = [int(m) for m in os.environ.get("PROBE_MASKS", "0,1,2,4,8,64,6,95").split(",")]
 for kv in KVS:
     for mask in MASKS:
@@ -83,3 +83,45 @@ for kv in KVS:
             err = float("nan")
         print(f"{kv:4s} mask {mask:3d}: {np.median(ts[2:]) * 1e3:8.1f} us  (vs bin: {err:.2e})")
 os.environ["TGL_DEBUG_MASK"] = "0"
+
+if os.environ.get("PROBE_PROF"):
+    import ctypes as C
+    lib.tgl_debug_prof.argtypes = [C.c_void_p, C.c_int]
+    host = (C.c_ulonglong * (148 * 16))()
+    for kv in ("async",):
+        os.environ["TGL_KV"] = kv
+        os.environ["TGL_DEBUG_MASK"] = str(512 | int(os.environ.get("PROBE_PROF_MASK", "0")))
+        call(); torch.cuda.synchronize()
+        lib.tgl_debug_prof(None, 1)
+        call(); torch.cuda.synchronize()
+        lib.tgl_debug_prof(host, 0)
+        v = np.frombuffer(host, dtype=np.uint64).reshape(148, 16).astype(np.float64)
+        names = ["P:stage-free", "P:issue", "P:data-wait", "P:convert", "P:fence+arrive",
+                 "MMA:A-wait", "MMA:W-wait", "MMA:acc-wait", "MMA:tile", "D:slot-wait",
+                 "D:build", "E:acc-wait", "E:work"]
+        med = np.median(v[:, :13], axis=0)
+        print(kv, "cycles per CTA (median):", "  ".join(f"{n} {m:.0f}" for n, m in zip(names, med)))
+    os.environ["TGL_DEBUG_MASK"] = "0"
+
+if os.environ.get("PROBE_TRACE"):
+    import ctypes as C
+    lib.tgl_debug_trace.argtypes = [C.c_void_p, C.c_int]
+    host = (C.c_ulonglong * 8192)()
+    os.environ["TGL_KV"] = "async"
+    os.environ["TGL_DEBUG_MASK"] = str(4096 | int(os.environ.get("PROBE_TRACE_MASK", "0")))
+    call(); torch.cuda.synchronize()
+    lib.tgl_debug_trace(None, 1)
+    call(); torch.cuda.synchronize()
+    lib.tgl_debug_trace(host, 0)
+    v = np.frombuffer(host, dtype=np.uint64).reshape(16, 512)
+    v = np.concatenate([r[:int(r[511] & 0x1ff)] for r in v])
+    t = (v >> 16).astype(np.int64)
+    ev = ((v >> 8) & 0xff).astype(int)
+    k = (v & 0xff).astype(int)
+    o = np.argsort(t, kind="stable")
+    t0 = t[o[0]]
+    names = {1: "P.stage-free", 3: "P.data-ready", 4: "P.converted", 5: "M.A-ready", 6: "M.issued",
+             7: "M.tile-start", 9: "E.acc-ready", 10: "E.done", 11: "W.slot-free", 12: "M.W-ready"}
+    for x in o[:400]:
+        print(f"{(t[x] - t0) / 1000:8.2f} us  {names.get(ev[x], ev[x]):14s} {k[x]}")
+    os.environ["TGL_DEBUG_MASK"] = "0"

@@ -1,9 +1,9 @@
 """Per-tile role timeline of the REDDIT tail K|V kernel (TGL_DEBUG_MASK=32).
 
-    TGL_KV=tma|bin python tools/kv_timeline.py [precision]
+    TGL_KV=async|bin python tools/kv_timeline.py [precision]
 
 Events (globaltimer, us from the CTA's first descriptor): 0 desc start, 1 desc done,
-2 A loads start (tma) / producer start (bin), 3 conversion/producer done, 4 MMA start,
+2 producer start, 3 conversion/producer done, 4 MMA start,
 5 epilogue ready (q fetched), 6 accumulator ready, 7 epilogue done.
 """
 import ctypes as C
