@@ -196,6 +196,30 @@ def algorithmic_attn(cfg, n_dst: int, n_edges: int, d_hdst: int, d_hsrc: int):
     return flops, bytes_
 
 
+def algorithmic_kv(cfg, n_dst: float, n_edges: float, d_hsrc: int):
+    """Per launch of the K|V attention kernel (S6, S7, S9-S12):
+    FLOPs = E * (2 * 2*d_model * K) for [K;V] = W [h ; e ; Phi] (K = d_hs + d_e + d_t)
+            + E * 4 * d_model for the logits and the alpha-weighted sum;
+    bytes = E * (4 (d_hs + d_e) + 12)  (gathered rows + nbr/eid/ts; Phi computed or
+            table-read, counted 0 as in SURVEY §8(d))
+            + n_dst * (8 + 4 + 4 (d_model + 2) + 4 d_model)  (seg_ptr, t, q row, r row)."""
+    dm = cfg.d_model
+    k = d_hsrc + cfg.d_e + cfg.d_t
+    flops = n_edges * (2 * 2 * dm * k + 4 * dm)
+    bytes_ = n_edges * (4 * (d_hsrc + cfg.d_e) + 12) + n_dst * (12 + 4 * (dm + 2) + 4 * dm)
+    return flops, bytes_
+
+
+def ncu_traffic(precision: str):
+    """dram__bytes_read.sum + dram__bytes_write.sum per launch of the K|V kernel from the
+    committed `ncu --set full` capture (profiles/), or None."""
+    try:
+        d = json.load(open(os.path.join(ROOT, "profiles", "r01_kv_split_traffic.json")))
+        return d[precision]
+    except Exception:
+        return None
+
+
 def run_ours(args):
     import numpy as np
     import torch
@@ -289,13 +313,17 @@ def run_ours(args):
     edges_per_s = int(e_tot.item()) / (total_ms / 1e3)
 
     # ---- dominant call: tgl_tblock_attn on the tail block, timed eagerly with events
-    rec_ms, rec_shape, brk = [], None, {}
+    rec_ms, rec_shape, brk, kv_ms = [], None, {}, []
+    lib = tgl.lib()
     for i in range(max(3, min(args.steps, 20))):
         flush.zero_()
         pipe.start_dev.fill_(batch_of(args.warmup + i) * cfg.batch)
         rec = {}
+        lib.tgl_kv_timing(1)          # CUDA events around each K|V kernel, on its stream
         pipe.forward(record=rec)
         torch.cuda.synchronize()
+        kv_ms.append(lib.tgl_kv_timing_ms(0))   # the tail block runs first
+        lib.tgl_kv_timing(0)
         tail = pipe.L - 1
         rec_ms.append(rec[tail][0].elapsed_time(rec[tail][1]))
         mk = rec["_marks"]
@@ -309,29 +337,43 @@ def run_ours(args):
     E_avg = sum(e for _, e in rec_shape) / len(rec_shape)
     fl, by = algorithmic_attn(cfg, U_avg, E_avg, cfg.d_v, cfg.d_v)
     attn_ms = sum(rec_ms) / len(rec_ms)
+    kv_fl, kv_by = algorithmic_kv(cfg, U_avg, E_avg, cfg.d_v)
+    kv_ok = [m for m in kv_ms if m > 0]
+    kv_avg = sum(kv_ok) / len(kv_ok) if kv_ok else float("nan")
     peaks = {}
     try:
         peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
     except Exception:
         pass
     sm_max = clocks.get("sm_max_mhz") or peaks.get("sm_max_mhz", 1965.0)
-    achieved_tf = fl / (attn_ms / 1e3) / 1e12
+    hbm_peak = peaks.get("hbm_gbs", 6545.9)
+    bf16_peak = peaks.get("bf16_tflops", 1613.6)
+    kv_tf = kv_fl / (kv_avg / 1e3) / 1e12
+    kv_gbs = kv_by / (kv_avg / 1e3) / 1e9
     if args.precision == "fp32_simt":
         peak = 148 * 128 * 2 * sm_max * 1e6 / 1e12     # TFLOP/s, FFMA on all SMs
-        bound, note = "alu", "FP32 FFMA peak = 148 SM x 128 lanes x 2 x clocks.max.sm (derived)"
+        bound, unit, ach = "alu", "TFLOP/s", kv_tf
+        note = "FP32 FFMA peak = 148 SM x 128 lanes x 2 x clocks.max.sm (derived)"
+    elif args.precision == "fp32":
+        # fp32 = 3 bf16 MMA passes per algorithmic FLOP: the tensor roofline for fp32
+        # operands is the measured bf16 burst peak / 3; it binds before HBM
+        peak, bound, unit, ach = bf16_peak / 3, "tensor", "TFLOP/s", kv_tf
+        note = "measured cuBLAS bf16 burst peak (MEASURED_PEAKS.json) / 3 passes"
     else:
-        peak = peaks.get("bf16_tflops", 1613.6)
-        bound = "tensor"
-        note = ("measured cuBLAS bf16 burst peak (MEASURED_PEAKS.json); fp32 mode issues 3 bf16 "
-                "MMA passes per algorithmic FLOP, so frac <= 1/3 by construction"
-                if args.precision == "fp32" else "measured cuBLAS bf16 burst peak")
-    roofline = {"kernel": "tgl_tblock_attn on the tail block (q + K|V-attention + ffn kernels)",
-                "bound": bound, "achieved": achieved_tf, "peak": peak, "unit": "TFLOP/s",
-                "frac": achieved_tf / peak, "traffic": None,
-                "hbm_achieved_gbs": by / (attn_ms / 1e3) / 1e9,
-                "hbm_peak_gbs": peaks.get("hbm_gbs", 6545.9),
-                "per_launch_ms": attn_ms, "algorithmic_flops": fl, "algorithmic_bytes": by,
-                "n_dst_avg": U_avg, "n_edges_avg": E_avg, "peak_note": note}
+        peak, bound, unit, ach = hbm_peak, "hbm", "GB/s", kv_gbs
+        note = "measured HBM copy bandwidth (MEASURED_PEAKS.json); bf16 MMA time < HBM time"
+    tr = ncu_traffic(args.precision)
+    roofline = {"kernel": "kv_split_kernel (K|V attention of the tail block: S6,S7,S9-S12)",
+                "bound": bound, "achieved": ach, "peak": peak, "unit": unit,
+                "frac": ach / peak,
+                "traffic": tr["dram_bytes_per_launch"] if tr else None,
+                "traffic_note": (f"ncu --set full, {tr['source']}" if tr else None),
+                "per_launch_ms": kv_avg, "launches_timed": len(kv_ok),
+                "algorithmic_flops": kv_fl, "algorithmic_bytes": kv_by,
+                "tensor_tflops": kv_tf, "tensor_frac_bf16_peak": kv_tf / bf16_peak,
+                "hbm_gbs": kv_gbs, "hbm_frac": kv_gbs / hbm_peak,
+                "n_dst_avg": U_avg, "n_edges_avg": E_avg, "peak_note": note,
+                "attn_call_ms": attn_ms, "attn_call_tflops": fl / (attn_ms / 1e3) / 1e12}
 
     # ---- e2e through the public API: pinned host batch -> device -> host embeddings
     e2e = None

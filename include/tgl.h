@@ -235,6 +235,15 @@ tgl_status tgl_tblock_attn(const tgl_attn_params* P, int64_t n_dst_max, const in
                            int32_t max_seg, float* out, void* ws, size_t* ws_bytes,
                            void* stream);
 
+/* Measurement hook (bench.py): while armed (arm = 1; arming resets the count),
+ * the first 8 tensor-core tgl_tblock_attn calls each record a pair of CUDA events
+ * on their stream around their K|V attention kernel (S6, S7, S9-S12; the dominant
+ * kernel).  tgl_kv_timing_ms(i) synchronises on the i-th stop event and returns
+ * that kernel's duration in ms (negative if call i was not recorded).  Host-side
+ * state, not thread-safe; measurement only (never armed during graph capture). */
+int tgl_kv_timing(int arm);
+float tgl_kv_timing_ms(int i);
+
 /* ---------------------------------------------------------------------------
  * S14  Dedup inverse applied to rows (the hook of P:279 / TGOpt dedup_invert
  * P:179): out[j][:] = table[idx[j]][:] for j < n, n = *n_dev (NULL -> n_max).

@@ -22,6 +22,8 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 # no --use_fast_math: the time encoder needs the accurate cosf (reading R10)
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2", "--expt-relaxed-constexpr",
          "-I", os.path.join(ROOT, "include")]
+# profiling experiments only (e.g. "-DTGL_KV_ASTAGES=8"); unset for every product build
+FLAGS += os.environ.get("TGL_NVCC_EXTRA", "").split()
 
 
 def _deps():

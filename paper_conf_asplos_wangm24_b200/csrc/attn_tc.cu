@@ -193,13 +193,13 @@ __device__ unsigned int g_trace_n;
 __shared__ unsigned s_trace_n[32];
 __device__ __forceinline__ void trace(const Args& a, int ev, uint32_t k) {
   if ((a.dbg & 4096) && blockIdx.x == 0 && (threadIdx.x & 31) == 0) {
-    unsigned long long t;
-    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-    const int w = (threadIdx.x >> 5) & 15;
+    // SM cycle counter (cheap, consistent within the CTA); the probe converts at 1965 MHz
+    const unsigned long long t = (unsigned long long)clock64();
+    const int w = (threadIdx.x >> 5) & 31;           // 32 slices of 256 events
     const unsigned n = s_trace_n[w];
-    if (n < 511) {
-      g_trace[w * 512 + n] = (t << 16) | ((unsigned long long)(ev & 0xff) << 8) | (k & 0xff);
-      g_trace[w * 512 + 511] = n + 1;
+    if (n < 255) {
+      g_trace[w * 256 + n] = (t << 16) | ((unsigned long long)(ev & 0xff) << 8) | (k & 0xff);
+      g_trace[w * 256 + 255] = n + 1;
       s_trace_n[w] = n + 1;
     }
   }
@@ -914,6 +914,9 @@ __global__ void __launch_bounds__(kWsThreads, 1) kv_kernel(Args a) {
 // state across tiles; r is written straight to global.  Empty segments get r = 0 from
 // the descriptor warp (R19); a segment longer than 32 rows (max_seg hint violated)
 // gets a NaN row.
+#ifndef TGL_SLEEP_EPI
+#define TGL_SLEEP_EPI 128
+#endif
 constexpr int kBEpi = 8;                    // warps 0-7
 constexpr int kBarBinEpi = 1;               // named barrier of the 8 epilogue warps
 constexpr int kBMma = 8;
@@ -953,7 +956,7 @@ __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uin
   for (;; ++tt) {
     const uint32_t ab = tt & 1u, ds = tt % NS;
     // one warp polls, the other seven block in bar.sync (no issue slots spent waiting)
-    if (warp == 0) mbar_wait(&dfull[ds], (tt / NS) & 1u);
+    if (warp == 0) mbar_wait_sleep(&dfull[ds], (tt / NS) & 1u, TGL_SLEEP_EPI);
     named_bar(kBarBinEpi, kBEpi * 32);
     if (!bd[ds].live) {
       warp_arrive(&dempty[ds]);
@@ -981,7 +984,7 @@ __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uin
     const float qb = __ldg(qrow + dm + head);
     if (threadIdx.x == 0) tl_mark(a, tt, 5);
     const long long e0c = clock64();
-    if (warp == 0) mbar_wait(&tfull[ab], (tt >> 1) & 1u);
+    if (warp == 0) mbar_wait_sleep(&tfull[ab], (tt >> 1) & 1u, TGL_SLEEP_EPI);
     named_bar(kBarBinEpi, kBEpi * 32);
     const long long e1c = clock64();
     if (warp == 0) trace(a, 9, tt);
@@ -1236,14 +1239,26 @@ __global__ void __launch_bounds__(kBThreads, 1) kv_bin_kernel(Args a) {
 // 128-byte row boxes -- and dropped.)
 constexpr int kTC = 32;                       // fp32 columns per K chunk
 constexpr int kTAStage = kBM * kTC * 4;       // 16 KB
-constexpr int kTAStages = 6;
-constexpr int kAheadU = kTAStages / 2 - 1;    // 2-chunk units of gathers in flight per producer
-constexpr int kTWStages = 3;
+#ifndef TGL_KV_ASTAGES
+#define TGL_KV_ASTAGES 6
+#endif
+#ifndef TGL_KV_AHEAD
+#define TGL_KV_AHEAD (TGL_KV_ASTAGES / 2 - 1)
+#endif
+#ifndef TGL_KV_WSTAGES
+#define TGL_KV_WSTAGES 3
+#endif
+#ifndef TGL_KV_DSLOTS
+#define TGL_KV_DSLOTS 4
+#endif
+constexpr int kTAStages = TGL_KV_ASTAGES;
+constexpr int kAheadU = TGL_KV_AHEAD;         // 2-chunk units of gathers in flight per producer
+constexpr int kTWStages = TGL_KV_WSTAGES;
 constexpr int kTWHalf = kNPkv * 64;           // one of W_hi / W_lo of a chunk (12.8 KB)
 constexpr int kTWStage = 2 * kTWHalf;
 constexpr int kTMma = 8, kTW = 9, kTDesc0 = 10, kTDescWarps = 2, kTProd0 = 12, kTProdWarps = 8;
 constexpr int kTThreads = (kTProd0 + kTProdWarps) * 32;   // 640 (96 registers per thread)
-constexpr int kTDSlots = 4;
+constexpr int kTDSlots = TGL_KV_DSLOTS;
 constexpr int kTPipeBytes = kTAStages * kTAStage + kTWStages * kTWStage;
 constexpr int kTSmem = 1024 + kTPipeBytes + kBEpi * 32 * 33 * 4;
 
@@ -1425,6 +1440,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
       wait_free_sleep(&B.dempty[ds], tt / kTDSlots, 1000);
       const long long d1c = clock64();
       if (dw == 0) prof_add(a, 9, d1c - d0c);        // desc: wait for a slot
+      trace(a, 20, tt);
       if (lane == 0) tl_mark(a, tt, 0);
       TDesc& R = bd[ds];
       const int64_t T = blockIdx.x + (int64_t)tt * gridDim.x;
@@ -1494,6 +1510,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
       }
       warp_arrive(&B.dfull[ds]);
       if (dw == 0) prof_add(a, 10, clock64() - d1c); // desc: build
+      trace(a, 21, tt);
       if (lane == 0) tl_mark(a, tt, 1);
     }
   } else if (warp == kTW) {                          // ---------------- weight loader
@@ -1584,6 +1601,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
           }
         }
         cp_async_commit();
+        if (pw == 0) trace(a, 1, ul);
         al += cnt;
         ++ul;
         if (++lp == npair) {
@@ -1605,6 +1623,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
       const int i0 = 2 * cp, cnt = (nch - i0) < 2 ? (nch - i0) : 2;
       cp_async_wait_dyn((int)(ul - uc - 1));
       __syncwarp();
+      if (pw == 0) trace(a, 3, uc);
       float4 x[2][4];
       uint32_t gb[2];
 #pragma unroll
@@ -1667,6 +1686,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
       }
       if (!(a.dbg & 2048)) fence_proxy_async_smem();   // 2048: profiling only (unsafe)
       __syncwarp();
+      if (pw == 0) trace(a, 4, uc);
       if (lane == 0) {
         mbar_arrive(&B.aready[ac % kTAStages]);
         if (cnt == 2) mbar_arrive(&B.aready[(ac + 1) % kTAStages]);
@@ -1720,6 +1740,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
           }
         }
         tc_fence_after();
+        trace(a, 5, ait);
         if (elect_one()) {
 #pragma unroll
           for (int q = 0; q < 2; ++q) {
@@ -1753,6 +1774,491 @@ __global__ void __launch_bounds__(kTThreads, 1)
       prof_add(a, 8, clock64() - m2);                  // MMA: whole tile
     }
   } else {                                           // ---------------- epilogue warps 0-7
+    bin_epilogue<kTDSlots>(a, B.dfull, B.dempty, B.tfull, B.tempty, bd, tmem, s_pv, s_bias);
+  }
+  ws_teardown(tmem, 2 * kCols, kTMma);
+}
+
+// ------------------------------------------------------------------ split-role K|V attention
+// kv_split_kernel: the binned K|V attention of kv_async_kernel with the gather and the
+// bf16 conversion in DIFFERENT warps, so that neither waits on the other's latency:
+//   loaders    (4 warps): per 32-column chunk, 8 LDGSTS of 16 B per lane into an fp32
+//                         row image (row r at r*128 B); completion is tracked by the
+//                         stage's mbarrier (cp.async.mbarrier.arrive.noinc), so a loader
+//                         never waits for its own copies -- only for a free stage, and it
+//                         runs up to kSF chunks (64 KB) ahead;
+//   converters (4 warps): fp32 image -> bf16 hi | lo in the SW64 K-major UMMA layout of a
+//                         separate bf16 ring (Phi(dt) evaluated for rows the precompute
+//                         table does not cover), then release the fp32 stage;
+//   MMA warp, weight warp, descriptor warps and the 8 epilogue warps as in kv_async.
+// Per-chunk bookkeeping (segment, column, width, K steps) comes from a shared table, so
+// the steady-state loops are straight-line code.
+#ifndef TGL_KV_FSTAGES
+#define TGL_KV_FSTAGES 3
+#endif
+#ifndef TGL_KV_BSTAGES
+#define TGL_KV_BSTAGES 4
+#endif
+// poll back-off (ns) of the roles that usually wait long: polling warps take issue
+// slots and sync-unit bandwidth from the converters (measured: ~1/3 of all executed
+// instructions were try_wait re-polls before back-off)
+#ifndef TGL_SLEEP_DESC
+#define TGL_SLEEP_DESC 256
+#endif
+#ifndef TGL_SLEEP_W
+#define TGL_SLEEP_W 64
+#endif
+#ifndef TGL_SLEEP_LOAD
+#define TGL_SLEEP_LOAD 64
+#endif
+#ifndef TGL_KV_LAG
+#define TGL_KV_LAG 0
+#endif
+// per-role cycle counters of kv_split_kernel (profiling builds: -DTGL_KV_PROF)
+#ifdef TGL_KV_PROF
+#define TGL_PROF_CLK(v) const long long v = clock64()
+#else
+#define TGL_PROF_CLK(v) (void)0
+#endif
+#ifndef TGL_KV_SPLIT_WSTAGES
+#define TGL_KV_SPLIT_WSTAGES 2
+#endif
+constexpr int kSW = TGL_KV_SPLIT_WSTAGES;           // weight stages (25.6 KB each)
+constexpr int kSF = TGL_KV_FSTAGES;            // fp32 image stages (16 KB each)
+constexpr int kSB = TGL_KV_BSTAGES;            // bf16 hi|lo stages (16 KB each)
+constexpr int kSStage = kBM * kTC * 4;         // 16 KB
+constexpr int kSLoad0 = kTProd0, kSLoadWarps = 4;
+#ifndef TGL_KV_CONV_WARPS
+#define TGL_KV_CONV_WARPS 8
+#endif
+constexpr int kSConv0 = kTProd0 + kSLoadWarps, kSConvWarps = TGL_KV_CONV_WARPS;
+constexpr int kSRowsPerConv = kBM / kSConvWarps;     // 16 (8 warps) or 32 (4 warps)
+constexpr int kSKc = kSRowsPerConv / 4;              // rows per converter lane
+constexpr int kSThreads = (kSConv0 + kSConvWarps) * 32;   // 768 with 8 converter warps
+constexpr int kSPipeBytes = (kSF + kSB) * kSStage + kSW * kTWStage;
+constexpr int kSSmem = 1024 + kSPipeBytes + kBEpi * 32 * 33 * 4;
+constexpr int kSMaxChunks = 48;
+
+struct SBars {
+  uint64_t ffull[kSF], fempty[kSF];
+  uint64_t bfull[kSB], bempty[kSB];
+  uint64_t wfull[kSW], wempty[kSW];
+  uint64_t dfull[kTDSlots], dempty[kTDSlots];
+  uint64_t tfull[2], tempty[2];
+};
+
+// arrive on `bar` once every cp.async this thread issued so far has landed
+__device__ __forceinline__ void cp_async_mbar_arrive_noinc(uint64_t* bar) {
+  asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(bar))
+               : "memory");
+}
+
+__global__ void __launch_bounds__(kSThreads, 1)
+    kv_split_kernel(const Args a, const KvPlan plan, const uint8_t* __restrict__ wkv,
+                    const int bdst) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* pipe = align1024(smem_raw);
+  __shared__ SBars B;
+  __shared__ uint32_t s_tmem;
+  __shared__ TDesc bd[kTDSlots];
+  __shared__ float s_omega[256], s_phi[256];
+  __shared__ float s_bias[2 * kMaxModel];
+  __shared__ int64_t s_seg[kTDescWarps][4 * 32 + 1];
+  __shared__ float s_td[kTDescWarps][4 * 32];
+  __shared__ int4 s_chunk[kSMaxChunks];          // {segment, first column, width, K steps}
+  float (*s_pv)[32][33] = reinterpret_cast<float (*)[32][33]>(pipe + kSPipeBytes);
+  constexpr uint32_t kCols = 256;
+  const tgl_attn_params& P = a.P;
+  const int64_t n = dev_count(a.n_dst_dev, a.n_dst_max);
+  const bool split = a.split != 0;
+  constexpr int dm = 100;
+  const int nch = plan.n;
+  for (int j = threadIdx.x; j < P.d_t; j += blockDim.x) {
+    s_omega[j] = P.omega[j];
+    s_phi[j] = P.phi[j];
+  }
+  for (int j = threadIdx.x; j < 2 * dm; j += blockDim.x) s_bias[j] = j < dm ? P.bk[j] : P.bv[j - dm];
+  for (int c = threadIdx.x; c < nch; c += blockDim.x) {
+    int seg, col;
+    plan_chunk(plan, c, seg, col);
+    const int width = seg == 0 ? plan.d[0] : (seg == 1 ? plan.d[1] : plan.d[2]);
+    s_chunk[c] = make_int4(seg, col, width, width - col > 16 ? 2 : 1);
+  }
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < kSF; ++s) {
+      mbar_init(&B.ffull[s], TGL_KV_LAG > 0 ? kSLoadWarps : kSLoadWarps * 32);
+      mbar_init(&B.fempty[s], kSConvWarps);
+    }
+    for (int s = 0; s < kSB; ++s) {
+      mbar_init(&B.bfull[s], kSConvWarps);
+      mbar_init(&B.bempty[s], 1);
+    }
+    for (int s = 0; s < kSW; ++s) {
+      mbar_init(&B.wfull[s], 1);
+      mbar_init(&B.wempty[s], 1);
+    }
+    for (int s = 0; s < kTDSlots; ++s) {
+      mbar_init(&B.dfull[s], 1);
+      mbar_init(&B.dempty[s], kBEpi + kSLoadWarps + kSConvWarps + 2);
+    }
+    for (int s = 0; s < 2; ++s) {
+      mbar_init(&B.tfull[s], 1);
+      mbar_init(&B.tempty[s], kBEpi);
+    }
+    fence_mbar_init();
+  }
+  if (threadIdx.x < 32) s_trace_n[threadIdx.x] = 0;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (warp == kTMma) tmem_alloc(&s_tmem, 2 * kCols);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = s_tmem;
+  const uint32_t pipe_s = smem_u32(pipe);
+  const uint32_t f_s = pipe_s;                                  // fp32 ring
+  const uint32_t b_s = pipe_s + kSF * kSStage;                  // bf16 ring
+  const uint32_t w_s = pipe_s + (kSF + kSB) * kSStage;          // weight ring
+  uint32_t tt = 0;
+
+  if (warp >= kTDesc0 && warp < kTDesc0 + kTDescWarps) {   // ------- tile builders
+    // identical to kv_async_kernel (fixed packing of bdst destinations per 32-row bin)
+    const int dw = warp - kTDesc0;
+    const int64_t hoff = a.hsrc_off_dev ? *a.hsrc_off_dev : 0;
+    const int dpt = 4 * bdst;
+    const int64_t ntiles = (n + dpt - 1) / dpt;
+    int64_t* sg = s_seg[dw];
+    float* stdv = s_td[dw];
+    for (tt = dw;; tt += kTDescWarps) {
+      const uint32_t ds = tt % kTDSlots;
+      wait_free_sleep(&B.dempty[ds], tt / kTDSlots, TGL_SLEEP_DESC);
+      trace(a, 20, tt);
+      TDesc& R = bd[ds];
+      const int64_t T = blockIdx.x + (int64_t)tt * gridDim.x;
+      if (T >= ntiles) {
+        if (lane == 0) R.live = 0;
+        warp_arrive(&B.dfull[ds]);
+        break;
+      }
+      const int64_t d0 = T * dpt;
+      const int nd = (int)((n - d0) < dpt ? (n - d0) : dpt);
+      for (int j = lane; j <= nd; j += 32) sg[j] = a.seg_ptr[d0 + j];
+      for (int j = lane; j < nd; j += 32) stdv[j] = a.dst_t[d0 + j];
+      __syncwarp();
+      int64_t er[4] = {0, 0, 0, 0};
+      float tr[4] = {0.f, 0.f, 0.f, 0.f};
+      int dr[4] = {-1, -1, -1, -1};
+      unsigned ovf_bins = 0;
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int j0 = u * bdst;
+        if (j0 >= nd) continue;
+        const int j1 = (j0 + bdst) < nd ? j0 + bdst : nd;
+        const int64_t e0 = sg[j0], e1 = sg[j1];
+        if (e1 - e0 > 32) {
+          ovf_bins |= 1u << u;
+          continue;
+        }
+        const int64_t e = e0 + lane;
+        if (e < e1) {
+          int j = j0;
+          while (sg[j + 1] <= e) ++j;
+          dr[u] = (int)(d0 + j);
+          er[u] = e;
+          tr[u] = stdv[j];
+        }
+      }
+      for (int j = 0; j < nd; ++j) {
+        const bool ovf = (ovf_bins >> (j / bdst)) & 1u;
+        if (sg[j + 1] == sg[j] || ovf) {
+          const float fill = ovf ? __int_as_float(0x7fc00000) : 0.f;
+          for (int c = lane; c < dm; c += 32) a.rbuf[(d0 + j) * kQLd + c] = fill;
+        }
+      }
+      R.live = 1;
+      int32_t hi[4], ei[4];
+      float et[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const bool ok = dr[u] >= 0;
+        hi[u] = ok ? (a.hsrc_idx ? a.hsrc_idx[hoff + er[u]] : (int32_t)(hoff + er[u])) : 0;
+        ei[u] = (ok && P.d_e > 0) ? a.eid[er[u]] : 0;
+        et[u] = ok ? a.edge_t[er[u]] : 0.f;
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int r = 32 * u + lane;
+        const bool ok = dr[u] >= 0;
+        const float dt = tr[u] - et[u];               // fp32 delta (R18)
+        R.hrow[r] = ok ? hi[u] : -1;
+        R.erow[r] = ok ? ei[u] : -1;
+        R.dt[r] = ok ? dt : 0.f;
+        R.trow[r] = ok ? (int)tenc_table_row(dt, a.table, a.window) : -1;
+        R.rdst[r] = dr[u];
+      }
+      warp_arrive(&B.dfull[ds]);
+      trace(a, 21, tt);
+    }
+  } else if (warp == kTW) {                          // ---------------- weight loader
+    uint32_t wl = 0;
+    const uint32_t wbytes = split ? kTWStage : kTWHalf;
+    for (;; ++tt) {
+      const uint32_t ds = tt % kTDSlots;
+      mbar_wait_sleep(&B.dfull[ds], (tt / kTDSlots) & 1u, TGL_SLEEP_W);
+      const int live = bd[ds].live;
+      warp_arrive(&B.dempty[ds]);
+      if (!live) break;
+      if (lane == 0) {
+        const int r0 = (tt > 0 && nch >= 4) ? 2 : 0;
+        for (int i = r0; i < nch; ++i) {
+          const uint32_t k = wl + (i - r0);
+          const uint32_t sw = k % kSW;
+          wait_free_sleep(&B.wempty[sw], k / kSW, TGL_SLEEP_W);
+          trace(a, 11, k);
+          if (a.dbg & 8) {                           // profiling: no weight bytes
+            mbar_arrive(&B.wfull[sw]);
+            continue;
+          }
+          mbar_arrive_expect_tx(&B.wfull[sw], wbytes);
+          bulk_g2s(pipe + (kSF + kSB) * kSStage + sw * kTWStage,
+                   wkv + (size_t)chunk_of(tt, i, nch) * kTWStage, wbytes, &B.wfull[sw]);
+        }
+        wl += nch - r0;
+      }
+      __syncwarp();
+    }
+  } else if (warp >= kSLoad0 && warp < kSLoad0 + kSLoadWarps) {   // ---------- loaders
+    // lane: rows lw*32 + (lane>>3) + 4k (k = 0..7), 16-byte piece (lane & 7) of the chunk
+    const int lw = warp - kSLoad0;
+    const int r0 = lw * 32 + (lane >> 3), pc = lane & 7;
+    const uint32_t lofs = (uint32_t)r0 * 128 + pc * 16;
+    uint32_t g = 0;
+    for (;; ++tt) {
+      const uint32_t ds = tt % kTDSlots;
+      mbar_wait_sleep(&B.dfull[ds], (tt / kTDSlots) & 1u, TGL_SLEEP_LOAD);
+      const TDesc& R = bd[ds];
+      if (!R.live) {
+#if TGL_KV_LAG > 0
+        cp_async_wait<0>();                          // the last LAG chunks
+        __syncwarp();
+        if (lane == 0)
+          for (uint32_t j = g >= TGL_KV_LAG ? g - TGL_KV_LAG : 0; j < g; ++j)
+            mbar_arrive(&B.ffull[j % kSF]);
+#endif
+        warp_arrive(&B.dempty[ds]);
+        break;
+      }
+      for (int i = 0; i < nch; ++i, ++g) {
+        const int c = chunk_of(tt, i, nch);
+        const int4 ch = s_chunk[c];
+        const int seg = ch.x;
+        const float* base = seg == 0 ? a.hsrc : (seg == 1 ? a.efeat : a.table);
+        const int64_t ld = seg == 0 ? a.ld_hsrc : (seg == 1 ? a.ld_e : (int64_t)P.d_t);
+        const int* ridx = seg == 0 ? R.hrow : (seg == 1 ? R.erow : R.trow);
+        const int cb = ch.y + 4 * pc;
+        const uint32_t nb = cb >= ch.z ? 0u : (uint32_t)min(16, (ch.z - cb) * 4);
+        const float* b = base + (nb ? cb : 0);
+        int x[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) x[k] = ridx[r0 + 4 * k];
+        const uint32_t sf = g % kSF;
+        TGL_PROF_CLK(l0);
+        wait_free_sleep(&B.fempty[sf], g / kSF, TGL_SLEEP_LOAD);
+        TGL_PROF_CLK(l1);
+        const uint32_t dst = f_s + sf * kSStage + lofs;
+#pragma unroll
+        if (!(a.dbg & 2))                            // profiling: no gathers
+#pragma unroll
+          for (int k = 0; k < 8; ++k)
+            if (x[k] >= 0) cp_async16_zfill(dst + k * 512, b + (int64_t)x[k] * ld, nb);
+#if TGL_KV_LAG > 0
+        // one arrive per warp: chunk g - LAG is complete once at most LAG newer groups
+        // are pending (far fewer mbarrier operations than one noinc arrive per thread)
+        cp_async_commit();
+        if (g >= TGL_KV_LAG) {
+          cp_async_wait<TGL_KV_LAG>();
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&B.ffull[(g - TGL_KV_LAG) % kSF]);
+        }
+#else
+        cp_async_mbar_arrive_noinc(&B.ffull[sf]);
+#endif
+#ifdef TGL_KV_PROF
+        if (lw == 0) {
+          prof_add(a, 5, l1 - l0);
+          prof_add(a, 6, clock64() - l1);
+        }
+#endif
+        if (lw == 0) trace(a, 1, g);
+      }
+      __syncwarp();
+      warp_arrive(&B.dempty[ds]);
+    }
+  } else if (warp >= kSConv0 && warp < kSConv0 + kSConvWarps) {   // -------- converters
+    // lane: rows cw*32 + (lane>>3) + 4k; row r lands in 8-row group r>>3 of the bf16
+    // stage ([hi 512 B | lo 512 B] per group, SW64 K-major)
+    const int cw = warp - kSConv0;
+    const int r0 = cw * kSRowsPerConv + (lane >> 3), pc = lane & 7;
+    const uint32_t lofs = (uint32_t)r0 * 128 + pc * 16;
+    const uint32_t o_even = sw64_off(lane >> 3, 4 * pc), o_odd = sw64_off((lane >> 3) + 4, 4 * pc);
+    uint32_t g = 0;
+    for (;; ++tt) {
+      const uint32_t ds = tt % kTDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kTDSlots) & 1u);
+      const TDesc& R = bd[ds];
+      if (!R.live) {
+        warp_arrive(&B.dempty[ds]);
+        break;
+      }
+      float dtk[kSKc];
+      int trk[kSKc];
+#pragma unroll
+      for (int k = 0; k < kSKc; ++k) {
+        dtk[k] = R.dt[r0 + 4 * k];
+        trk[k] = R.rdst[r0 + 4 * k] >= 0 ? R.trow[r0 + 4 * k] : 0;   // padding: no Phi
+      }
+      __syncwarp();
+      warp_arrive(&B.dempty[ds]);
+      for (int i = 0; i < nch; ++i, ++g) {
+        const int c = chunk_of(tt, i, nch);
+        const int4 ch = s_chunk[c];
+        const uint32_t sf = g % kSF, sb = g % kSB;
+        TGL_PROF_CLK(c0);
+        mbar_wait(&B.ffull[sf], (g / kSF) & 1u);
+        TGL_PROF_CLK(c1);
+        if (cw == 0) trace(a, 3, g);
+        float4 x[kSKc];
+        const uint32_t src = f_s + sf * kSStage + lofs;
+        if (a.dbg & 64) {                            // profiling: no conversion work
+          wait_free(&B.bempty[sb], g / kSB);
+          __syncwarp();
+          if (lane == 0) {
+            mbar_arrive(&B.fempty[sf]);
+            mbar_arrive(&B.bfull[sb]);
+          }
+          continue;
+        }
+#pragma unroll
+        for (int k = 0; k < kSKc; ++k) x[k] = ld_shared_f4(src + k * 512);
+        if (ch.x == 2) {                             // time chunk: Phi where the table misses
+          const int cc = ch.y + 4 * pc;
+          float w[4], f[4];
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            const bool ok = cc + e < P.d_t;
+            w[e] = ok ? s_omega[cc + e] : 0.f;
+            f[e] = ok ? s_phi[cc + e] : 0.f;
+          }
+#pragma unroll
+          for (int k = 0; k < kSKc; ++k) {
+            if (trk[k] < 0) {
+              x[k].x = (cc < P.d_t) ? tenc_fast(dtk[k], w[0], f[0]) : 0.f;
+              x[k].y = (cc + 1 < P.d_t) ? tenc_fast(dtk[k], w[1], f[1]) : 0.f;
+              x[k].z = (cc + 2 < P.d_t) ? tenc_fast(dtk[k], w[2], f[2]) : 0.f;
+              x[k].w = (cc + 3 < P.d_t) ? tenc_fast(dtk[k], w[3], f[3]) : 0.f;
+            }
+          }
+        }
+        TGL_PROF_CLK(c2a);
+        wait_free(&B.bempty[sb], g / kSB);
+        TGL_PROF_CLK(c2);
+        const uint32_t dst = b_s + sb * kSStage + (uint32_t)cw * (kSRowsPerConv / 8) * 1024;
+#pragma unroll
+        for (int k = 0; k < kSKc; ++k) {
+          // row r0 + 4k: group cw*(rows/8) + k/2, row-in-group (lane>>3) + 4*(k&1)
+          const uint32_t ad = dst + (k >> 1) * 1024 + ((k & 1) ? o_odd : o_even);
+          uint32_t h0, h1, l0, l1;
+          split2(x[k].x, x[k].y, h0, l0);
+          split2(x[k].z, x[k].w, h1, l1);
+          asm volatile("st.shared.v2.b32 [%0], {%1, %2};" ::"r"(ad), "r"(h0), "r"(h1) : "memory");
+          if (split)
+            asm volatile("st.shared.v2.b32 [%0], {%1, %2};" ::"r"(ad + 512), "r"(l0), "r"(l1)
+                         : "memory");
+        }
+        TGL_PROF_CLK(c3);
+        fence_proxy_async_smem();
+        __syncwarp();
+#ifdef TGL_KV_PROF
+        const long long c4 = clock64();
+        if (cw == 0) {
+          prof_add(a, 0, c1 - c0);
+          prof_add(a, 1, c2a - c1);
+          prof_add(a, 2, c2 - c2a);
+          prof_add(a, 3, c3 - c2);
+          prof_add(a, 4, c4 - c3);
+        }
+#endif
+        if (cw == 0) trace(a, 4, g);
+        if (lane == 0) {
+          mbar_arrive(&B.fempty[sf]);
+          mbar_arrive(&B.bfull[sb]);
+        }
+      }
+    }
+  } else if (warp == kTMma) {                        // ---------------- MMA issuer
+    uint32_t g = 0, wl = 0;
+    constexpr uint32_t idesc = idesc_bf16(kBM, kNPkv);
+    for (;; ++tt) {
+      const uint32_t ds = tt % kTDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kTDSlots) & 1u);
+      const int live = bd[ds].live;
+      warp_arrive(&B.dempty[ds]);
+      if (!live) break;
+      const uint32_t acc = tmem + (tt & 1u) * kCols;
+      wait_free(&B.tempty[tt & 1u], tt >> 1);
+      tc_fence_after();
+      trace(a, 7, tt);
+      const int r0 = (tt > 0 && nch >= 4) ? 2 : 0;
+      for (int i = 0; i < nch; ++i, ++g) {
+        const int c = chunk_of(tt, i, nch);
+        const int nk = s_chunk[c].w;
+        const uint32_t sb = g % kSB;
+        TGL_PROF_CLK(m0);
+        mbar_wait(&B.bfull[sb], (g / kSB) & 1u);
+        TGL_PROF_CLK(m1);
+#ifdef TGL_KV_PROF
+        prof_add(a, 7, m1 - m0);
+#endif
+        trace(a, 12, g);
+        uint32_t kw;
+        if (i < r0) {
+          kw = wl - 1 - i;                           // resident from the previous tile
+        } else {
+          kw = wl + (i - r0);
+          mbar_wait(&B.wfull[kw % kSW], (kw / kSW) & 1u);
+        }
+        tc_fence_after();
+#ifdef TGL_KV_PROF
+        prof_add(a, 8, clock64() - m1);
+#endif
+        trace(a, 5, g);
+        if (elect_one()) {
+          const uint32_t ab = b_s + sb * kSStage;
+          const uint32_t wb = w_s + (kw % kSW) * kTWStage;
+          for (int ks = 0; ks < nk; ++ks) {
+            const uint64_t ah = desc_sw64(ab + ks * 32, 1024), bh = desc_sw64(wb + ks * 32, 512);
+            if (a.dbg & 4) break;                    // profiling: no MMAs
+            mma_bf16(acc, ah, bh, idesc, (i | ks) != 0);
+            if (split) {
+              mma_bf16(acc, desc_sw64(ab + 512 + ks * 32, 1024), bh, idesc, 1u);
+              mma_bf16(acc, ah, desc_sw64(wb + kTWHalf + ks * 32, 512), idesc, 1u);
+            }
+          }
+          const bool keep = (nch >= 4) && (i >= nch - 2);   // reused by the next tile
+          if (a.dbg & 8192) {                        // profiling: plain arrives, no commit
+            mbar_arrive(&B.bempty[sb]);
+            if (!keep) mbar_arrive(&B.wempty[kw % kSW]);
+          } else {
+            mma_commit(&B.bempty[sb]);
+            if (!keep) mma_commit(&B.wempty[kw % kSW]);
+          }
+        }
+        __syncwarp();
+      }
+      wl += nch - r0;
+      if (elect_one()) mma_commit(&B.tfull[tt & 1u]);
+      __syncwarp();
+    }
+  } else if (warp < kBEpi) {                         // ---------------- epilogue warps 0-7
     bin_epilogue<kTDSlots>(a, B.dfull, B.dempty, B.tfull, B.tempty, bd, tmem, s_pv, s_bias);
   }
   ws_teardown(tmem, 2 * kCols, kTMma);
@@ -1811,6 +2317,12 @@ static bool rows_16b(const float* base, int width, int64_t ld) {
 }  // namespace tca
 
 // host entry used by tgl_tblock_attn (attn.cu) for TGL_FP32 / TGL_BF16
+// measurement hook state (tgl_kv_timing): host-side only, armed by bench.py
+constexpr int kKvEvMax = 8;
+static bool g_kv_armed = false;
+static int g_kv_n = 0;                               // K|V launches recorded since arming
+static cudaEvent_t g_kv_ev[kKvEvMax][2] = {};
+
 size_t tc_attn_ws_bytes(const tgl_attn_params* P, int64_t n_dst_max, size_t* o_q, size_t* o_r,
                         size_t* o_pack) {
   using namespace tca;
@@ -1900,6 +2412,9 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
     TGL_TRY(cuda_check(cudaFuncSetAttribute(kv_async_kernel,
                                             cudaFuncAttributeMaxDynamicSharedMemorySize, kTSmem),
                        "attr kv async"));
+    TGL_TRY(cuda_check(cudaFuncSetAttribute(kv_split_kernel,
+                                            cudaFuncAttributeMaxDynamicSharedMemorySize, kSSmem),
+                       "attr kv split"));
     attr_done = true;
   }
   const int64_t tiles = ceil_div(n_dst_max, kBM);
@@ -1910,12 +2425,31 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
   const bool async = binned && !(kvsel && strcmp(kvsel, "bin") == 0) &&
                      rows_16b(hsrc, P->d_hsrc, ld_hsrc) && rows_16b(efeat, P->d_e, ld_e) &&
                      rows_16b(table, table ? P->d_t : 0, P->d_t);
-  if (kvsel && strcmp(kvsel, "async") == 0 && !async) {
+  // default: the split-role kernel; TGL_KV=async keeps the single-role LDGSTS producers
+  const bool use_split = async && !(kvsel && strcmp(kvsel, "async") == 0);
+  if (kvsel && (strcmp(kvsel, "async") == 0 || strcmp(kvsel, "split") == 0) && !async) {
     set_error("TGL_KV=async: the async-gather path cannot take this call (16-B row pitch / "
               "max_seg <= 32 / 2 heads)");
     return TGL_EUNSUPPORTED;
   }
-  if (async) {
+  const bool kv_rec = g_kv_armed && g_kv_n < kKvEvMax;
+  if (kv_rec) {
+    for (int e = 0; e < 2; ++e)
+      if (g_kv_ev[g_kv_n][e] == nullptr)
+        TGL_TRY(cuda_check(cudaEventCreate(&g_kv_ev[g_kv_n][e]), "event"));
+    TGL_TRY(cuda_check(cudaEventRecord(g_kv_ev[g_kv_n][0], s), "event record"));
+  }
+  if (use_split) {
+    const int bdst = 32 / max_seg;                 // destinations per 32-row bin
+    const int64_t ttiles = ceil_div(n_dst_max, 4 * bdst);
+    const unsigned gt = (unsigned)(ttiles < kNumSMs ? (ttiles > 0 ? ttiles : 1) : kNumSMs);
+    const KvPlan plan = make_plan(P->d_hsrc, P->d_e, P->d_t);
+    if (plan.n > kSMaxChunks) {
+      set_error("K|V attention: %d K chunks > %d", plan.n, kSMaxChunks);
+      return TGL_EUNSUPPORTED;
+    }
+    kv_split_kernel<<<gt, kSThreads, kSSmem, s>>>(a, plan, pk + PL.okv64, bdst);
+  } else if (async) {
     const int bdst = 32 / max_seg;                 // destinations per 32-row bin
     const int64_t ttiles = ceil_div(n_dst_max, 4 * bdst);
     const unsigned gt = (unsigned)(ttiles < kNumSMs ? (ttiles > 0 ? ttiles : 1) : kNumSMs);
@@ -1931,6 +2465,10 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
     kv_kernel<<<gkv, kWsThreads, smem_kv, s>>>(a);
   }
   TGL_TRY(launch_check("tc kv kernel"));
+  if (kv_rec) {
+    TGL_TRY(cuda_check(cudaEventRecord(g_kv_ev[g_kv_n][1], s), "event record"));
+    ++g_kv_n;
+  }
   dense_kernel<true><<<gq, kWsThreads, smem_q, s>>>(a);
   return launch_check("tc ffn kernel");
 }
@@ -1944,6 +2482,21 @@ extern "C" int tgl_debug_timeline(unsigned long long* host, size_t n) {
   const size_t cap = sizeof(tca::g_timeline) / sizeof(unsigned long long);
   return (int)cudaMemcpyFromSymbol(host, tca::g_timeline,
                                    (n < cap ? n : cap) * sizeof(unsigned long long));
+}
+
+extern "C" int tgl_kv_timing(int arm) {
+  tgl::g_kv_armed = arm != 0;
+  tgl::g_kv_n = 0;
+  return 0;
+}
+
+extern "C" float tgl_kv_timing_ms(int i) {
+  if (i < 0 || i >= tgl::g_kv_n) return -1.f;
+  float ms = -1.f;
+  if (cudaEventSynchronize(tgl::g_kv_ev[i][1]) != cudaSuccess) return -1.f;
+  if (cudaEventElapsedTime(&ms, tgl::g_kv_ev[i][0], tgl::g_kv_ev[i][1]) != cudaSuccess)
+    return -1.f;
+  return ms;
 }
 
 extern "C" size_t tgl_attn_packed_bytes(const tgl_attn_params* P) {

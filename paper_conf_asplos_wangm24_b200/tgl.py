@@ -25,7 +25,7 @@ PRECISION = {"fp32": FP32, "bf16": BF16, "fp32_simt": FP32_SIMT}
 SYMBOLS = ["tgl_version", "tgl_status_string", "tgl_last_error", "tgl_build_tcsr",
            "tgl_batch_roots", "tgl_dedup", "tgl_sample", "tgl_next_block",
            "tgl_time_precompute", "tgl_time_encode", "tgl_tblock_attn", "tgl_gather_rows",
-           "tgl_attn_packed_bytes", "tgl_attn_pack"]
+           "tgl_attn_packed_bytes", "tgl_attn_pack", "tgl_kv_timing", "tgl_kv_timing_ms"]
 
 
 class TGLError(RuntimeError):
@@ -62,6 +62,10 @@ def _load():
         f.restype = i32
     lib.tgl_attn_packed_bytes.argtypes = [vp]
     lib.tgl_attn_packed_bytes.restype = C.c_size_t
+    lib.tgl_kv_timing.argtypes = [C.c_int]
+    lib.tgl_kv_timing.restype = C.c_int
+    lib.tgl_kv_timing_ms.argtypes = [C.c_int]
+    lib.tgl_kv_timing_ms.restype = C.c_float
     return lib
 
 

@@ -88,7 +88,7 @@ if os.environ.get("PROBE_PROF"):
     import ctypes as C
     lib.tgl_debug_prof.argtypes = [C.c_void_p, C.c_int]
     host = (C.c_ulonglong * (148 * 16))()
-    for kv in ("async",):
+    for kv in (os.environ.get("PROBE_PROF_KV", "split"),):
         os.environ["TGL_KV"] = kv
         os.environ["TGL_DEBUG_MASK"] = str(512 | int(os.environ.get("PROBE_PROF_MASK", "0")))
         call(); torch.cuda.synchronize()
@@ -96,9 +96,12 @@ if os.environ.get("PROBE_PROF"):
         call(); torch.cuda.synchronize()
         lib.tgl_debug_prof(host, 0)
         v = np.frombuffer(host, dtype=np.uint64).reshape(148, 16).astype(np.float64)
-        names = ["P:stage-free", "P:issue", "P:data-wait", "P:convert", "P:fence+arrive",
+        names = (["C:ffull-wait", "C:lds+phi", "C:bempty-wait", "C:cvt+sts", "C:fence",
+                  "L:fempty-wait", "L:issue", "M:bfull-wait", "M:wfull-wait", "9", "10",
+                  "E:acc-wait", "E:work"] if kv == "split" else
+                 ["P:stage-free", "P:issue", "P:data-wait", "P:convert", "P:fence+arrive",
                  "MMA:A-wait", "MMA:W-wait", "MMA:acc-wait", "MMA:tile", "D:slot-wait",
-                 "D:build", "E:acc-wait", "E:work"]
+                 "D:build", "E:acc-wait", "E:work"])
         med = np.median(v[:, :13], axis=0)
         print(kv, "cycles per CTA (median):", "  ".join(f"{n} {m:.0f}" for n, m in zip(names, med)))
     os.environ["TGL_DEBUG_MASK"] = "0"
@@ -107,21 +110,21 @@ if os.environ.get("PROBE_TRACE"):
     import ctypes as C
     lib.tgl_debug_trace.argtypes = [C.c_void_p, C.c_int]
     host = (C.c_ulonglong * 8192)()
-    os.environ["TGL_KV"] = "async"
+    os.environ["TGL_KV"] = os.environ.get("PROBE_TRACE_KV", "split")
     os.environ["TGL_DEBUG_MASK"] = str(4096 | int(os.environ.get("PROBE_TRACE_MASK", "0")))
     call(); torch.cuda.synchronize()
     lib.tgl_debug_trace(None, 1)
     call(); torch.cuda.synchronize()
     lib.tgl_debug_trace(host, 0)
-    v = np.frombuffer(host, dtype=np.uint64).reshape(16, 512)
-    v = np.concatenate([r[:int(r[511] & 0x1ff)] for r in v])
+    v = np.frombuffer(host, dtype=np.uint64).reshape(32, 256)
+    v = np.concatenate([r[:int(r[255] & 0xff)] for r in v])
     t = (v >> 16).astype(np.int64)
     ev = ((v >> 8) & 0xff).astype(int)
     k = (v & 0xff).astype(int)
     o = np.argsort(t, kind="stable")
     t0 = t[o[0]]
-    names = {1: "P.stage-free", 3: "P.data-ready", 4: "P.converted", 5: "M.A-ready", 6: "M.issued",
-             7: "M.tile-start", 9: "E.acc-ready", 10: "E.done", 11: "W.slot-free", 12: "M.W-ready"}
-    for x in o[:400]:
-        print(f"{(t[x] - t0) / 1000:8.2f} us  {names.get(ev[x], ev[x]):14s} {k[x]}")
+    names = {20: "D.build-start", 21: "D.built", 1: "P.load-issued", 3: "P.data-ready", 4: "P.converted", 5: "M.A-ready", 6: "M.issued",
+             7: "M.tile-start", 9: "E.acc-ready", 10: "E.done", 11: "W.issue", 12: "M.B-full"}
+    for x in o[:int(os.environ.get('PROBE_TRACE_N', '400'))]:
+        print(f"{(t[x] - t0) / 1965:8.2f} us  {names.get(ev[x], ev[x]):14s} {k[x]}")
     os.environ["TGL_DEBUG_MASK"] = "0"
