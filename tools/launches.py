@@ -1,10 +1,18 @@
-"""Summarise an ncu launch list (gpu__time_duration.sum per launch): last `frac` of launches."""
+"""Summarise an ncu launch list (gpu__time_duration.sum per launch) per pipeline step.
+
+A step is the launch sequence from one `batch_roots_kernel` to the next; one-off setup
+launches (T-CSR build, time-precompute table, weight packing) fall outside every step.
+Prints the per-kernel share of the median step (cold-cache, serialised ncu timings).
+
+    python tools/launches.py launches.csv
+"""
 import csv
+import statistics
 import sys
 from collections import defaultdict
 
 
-def main(path, nsteps=3):
+def main(path):
     rows = list(csv.reader(open(path)))
     hdr, data = None, []
     for r in rows:
@@ -12,19 +20,32 @@ def main(path, nsteps=3):
             hdr = r
             continue
         if hdr and len(r) == len(hdr):
-            data.append(dict(zip(hdr, r)))
-    tot, cnt = defaultdict(float), defaultdict(int)
-    part = data[-len(data) // nsteps:]
-    for d in part:
-        n = d["Kernel Name"].split("(")[0][:50]
-        tot[n] += float(d["Metric Value"].replace(",", ""))
+            d = dict(zip(hdr, r))
+            data.append((d["Kernel Name"].split("(")[0][:50], float(d["Metric Value"].replace(",", ""))))
+    steps, cur = [], None
+    for name, v in data:
+        if "batch_roots_kernel" in name:
+            if cur:
+                steps.append(cur)
+            cur = []
+        if cur is not None and "Fill" not in name:
+            cur.append((name, v))
+    if cur and any("gather_rows" in n for n, _ in cur):
+        steps.append(cur)
+    steps = [s for s in steps if any("gather_rows" in n for n, _ in s)]
+    tot = [sum(v for _, v in s) for s in steps]
+    med = sorted(range(len(steps)), key=lambda i: tot[i])[len(steps) // 2]
+    s = steps[med]
+    agg, cnt = defaultdict(float), defaultdict(int)
+    for n, v in s:
+        agg[n] += v
         cnt[n] += 1
-    s = sum(tot.values())
-    unit = data[0]["Metric Unit"]
-    print(f"launches={len(data)} last-step launches={len(part)} total={s:.0f} {unit}")
-    for n, v in sorted(tot.items(), key=lambda x: -x[1]):
-        print(f"{v:10.0f} {unit} {100 * v / s:5.1f}% x{cnt[n]:<3d} {n}")
+    T = sum(agg.values())
+    print(f"launches={len(data)} steps={len(steps)} median step: {len(s)} launches, {T / 1e3:.1f} us "
+          f"(ncu: serialised, cold cache)")
+    for n, v in sorted(agg.items(), key=lambda x: -x[1]):
+        print(f"{v / 1e3:9.1f} us {100 * v / T:5.1f}% x{cnt[n]:<3d} {n}")
 
 
 if __name__ == "__main__":
-    main(sys.argv[1], int(sys.argv[2]) if len(sys.argv) > 2 else 3)
+    main(sys.argv[1])
