@@ -505,9 +505,22 @@ __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
   const Seg3& sg = kFfn ? a.so : a.sq;
   const uint8_t* wpack = kFfn ? a.wo : a.wq;
   const bool split = a.split != 0;
+  // epilogue vectors staged once in shared memory: read inside the TMEM loops, a global
+  // load there is a dependent L2/HBM round trip per 32-column piece
+  __shared__ float s_v0[kMaxModel], s_v1[kMaxModel], s_v2[kMaxModel];
   for (int j = threadIdx.x; j < P.d_t; j += blockDim.x) {
     s_omega[j] = P.omega[j];
     s_phi[j] = P.phi[j];
+  }
+  for (int j = threadIdx.x; j < P.d_model; j += blockDim.x) {
+    if (kFfn) {
+      s_v0[j] = P.bo[j];
+      s_v1[j] = P.ln_gamma[j];
+      s_v2[j] = P.ln_beta[j];
+    } else {
+      s_v0[j] = P.bq[j];
+      s_v1[j] = P.bk[j];
+    }
   }
   ws_init(B, &s_tmem, 2 * kCols);
   const uint32_t tmem = s_tmem;
@@ -586,13 +599,13 @@ __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
             for (int j = 0; j < 32; j += 4) {
               const int col = cq * 32 + j;
               if (col < D) {
-                float4 o = make_float4(v[j] + P.bq[col], v[j + 1] + P.bq[col + 1],
-                                       v[j + 2] + P.bq[col + 2], v[j + 3] + P.bq[col + 3]);
+                float4 o = make_float4(v[j] + s_v0[col], v[j + 1] + s_v0[col + 1],
+                                       v[j + 2] + s_v0[col + 2], v[j + 3] + s_v0[col + 3]);
                 *reinterpret_cast<float4*>(q + col) = o;   // D % 4 == 0 (D == 100)
                 const float oq[4] = {o.x, o.y, o.z, o.w};
 #pragma unroll
                 for (int e = 0; e < 4; ++e) {       // per column: a float4 may straddle heads
-                  const float pb = oq[e] * P.bk[col + e];
+                  const float pb = oq[e] * s_v1[col + e];
                   if (col + e < dhq) qb0 += pb; else qb1 += pb;
                 }
               }
@@ -613,7 +626,7 @@ __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
 #pragma unroll
           for (int j = 0; j < 32; ++j) {
             const int col = cq * 32 + j;
-            if (col < D) s += fmaxf(v[j] + P.bo[col], 0.f);
+            if (col < D) s += fmaxf(v[j] + s_v0[col], 0.f);
           }
         }
         const float mean = s / (float)D;
@@ -626,7 +639,7 @@ __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
           for (int j = 0; j < 32; ++j) {
             const int col = cq * 32 + j;
             if (col < D) {
-              const float d = fmaxf(v[j] + P.bo[col], 0.f) - mean;
+              const float d = fmaxf(v[j] + s_v0[col], 0.f) - mean;
               q2 += d * d;
             }
           }
@@ -645,8 +658,8 @@ __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
                 float r4[4];
 #pragma unroll
                 for (int e = 0; e < 4; ++e)
-                  r4[e] = (fmaxf(v[j + e] + P.bo[col + e], 0.f) - mean) * inv * P.ln_gamma[col + e] +
-                          P.ln_beta[col + e];
+                  r4[e] = (fmaxf(v[j + e] + s_v0[col + e], 0.f) - mean) * inv * s_v1[col + e] +
+                          s_v2[col + e];
                 *reinterpret_cast<float4*>(o + col) = make_float4(r4[0], r4[1], r4[2], r4[3]);
               }
             }

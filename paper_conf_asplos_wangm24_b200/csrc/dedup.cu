@@ -12,7 +12,7 @@
 namespace tgl {
 
 constexpr int kDedupThreads = 256;
-constexpr int kDedupItems = 8;
+constexpr int kDedupItems = 2;   // 512-pair tiles: many CTAs in flight for the ~2k-20k pairs of a batch
 constexpr int kDedupTile = kDedupThreads * kDedupItems;
 
 __device__ __forceinline__ unsigned long long pair_key(int32_t node, float t) {

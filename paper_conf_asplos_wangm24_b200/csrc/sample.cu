@@ -1,6 +1,7 @@
 // sample.cu -- S4 temporal neighbourhood sampling (readings R1, R4-R7).
 //
-// One CTA = one tile of 32 queries (8 warps x 4 queries), tiles taken from an
+// One CTA = one tile of 32 queries (32 warps x 1 query: every search of the tile is
+// in flight at once -- the probes are dependent loads), tiles taken from an
 // atomic ticket.  Per query a warp runs a 32-ary search for the first segment
 // entry with !(ts < t) (monotone predicate, so NaN t -> 0 candidates), then the
 // tile's counts are prefix-summed with a decoupled look-back so `seg_ptr` and
@@ -13,8 +14,8 @@
 
 namespace tgl {
 
-constexpr int kSampleWarps = 8;
-constexpr int kQueriesPerWarp = 4;
+constexpr int kSampleWarps = 32;
+constexpr int kQueriesPerWarp = 1;
 constexpr int kSampleTile = kSampleWarps * kQueriesPerWarp;  // 32
 
 __device__ __forceinline__ int64_t warp_lower_time(const float* __restrict__ ts, int64_t lo,
