@@ -2245,15 +2245,21 @@ __global__ void __launch_bounds__(kSThreads, 1)
 #endif
         trace(a, 5, g);
         if (elect_one()) {
-          const uint32_t ab = b_s + sb * kSStage;
-          const uint32_t wb = w_s + (kw % kSW) * kTWStage;
-          for (int ks = 0; ks < nk; ++ks) {
-            const uint64_t ah = desc_sw64(ab + ks * 32, 1024), bh = desc_sw64(wb + ks * 32, 512);
-            if (a.dbg & 4) break;                    // profiling: no MMAs
-            mma_bf16(acc, ah, bh, idesc, (i | ks) != 0);
-            if (split) {
-              mma_bf16(acc, desc_sw64(ab + 512 + ks * 32, 1024), bh, idesc, 1u);
-              mma_bf16(acc, ah, desc_sw64(wb + kTWHalf + ks * 32, 512), idesc, 1u);
+          // descriptors built once per chunk; a K step (32 B) / the lo half advance the
+          // 14-bit start-address field (addr >> 4) by plain adds (no carry: smem < 256 KB)
+          const uint64_t a0 = desc_sw64(b_s + sb * kSStage, 1024);
+          const uint64_t w0 = desc_sw64(w_s + (kw % kSW) * kTWStage, 512);
+          if (!(a.dbg & 4)) {                        // profiling: no MMAs
+#pragma unroll
+            for (int ks = 0; ks < 2; ++ks) {
+              if (ks < nk) {
+                const uint64_t ah = a0 + 2 * ks, bh = w0 + 2 * ks;
+                mma_bf16(acc, ah, bh, idesc, (i | ks) != 0);
+                if (split) {
+                  mma_bf16(acc, ah + (512 >> 4), bh, idesc, 1u);
+                  mma_bf16(acc, ah, bh + (kTWHalf >> 4), idesc, 1u);
+                }
+              }
             }
           }
           const bool keep = (nch >= 4) && (i >= nch - 2);   // reused by the next tile

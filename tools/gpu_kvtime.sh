@@ -13,10 +13,11 @@ for r in rows:
         d = dict(zip(hdr, r))
         if "kv_" in d["Kernel Name"]: kv.append(float(d["Metric Value"]) / 1000)
 masks = os.environ.get("MASKS", "0,79").split(",")
-per = len(kv) // (len(masks) + 1) if kv else 0
+kv = kv[2:]                      # the pipeline's own forward: tail + head K|V launches
+per = 8                          # kv_probe.py times 8 calls per mask
 out = []
 for i, m in enumerate(masks):
-    seg = kv[(i + 1) * per + 2:(i + 2) * per] if per else []
+    seg = kv[i * per + 2:(i + 1) * per]
     out.append(f"mask {m}: {sorted(seg)[len(seg)//2] if seg else float('nan'):.1f} us")
 print(f"== {sys.argv[1] or 'default'}: " + "  ".join(out))
 PY
