@@ -1279,12 +1279,23 @@ struct KvPlan {       // 32-column chunks of the three K segments
   int d[3];           // widths (h_src, e, time)
   int c[3];           // chunks per segment
   int n;              // total chunks
+  int contig;         // 1: chunks cut the concatenation [h | e | Phi] without per-segment
+                      //    padding (segment widths multiples of 4: a 16-byte piece never
+                      //    straddles two segments); 0: each segment padded to 32
 };
 static KvPlan make_plan(int d0, int d1, int d2) {
   KvPlan p;
   p.d[0] = d0; p.d[1] = d1; p.d[2] = d2;
   for (int s = 0; s < 3; ++s) p.c[s] = (p.d[s] + kTC - 1) / kTC;
   p.n = p.c[0] + p.c[1] + p.c[2];
+  p.contig = 0;
+  return p;
+}
+static bool contig_ok(int d0, int d1) { return d0 % 4 == 0 && d1 % 4 == 0; }
+static KvPlan make_plan_contig(int d0, int d1, int d2) {
+  KvPlan p = make_plan(d0, d1, d2);
+  p.n = (d0 + d1 + d2 + kTC - 1) / kTC;
+  p.contig = 1;
   return p;
 }
 __host__ __device__ __forceinline__ void plan_chunk(const KvPlan& p, int c, int& seg, int& col) {
@@ -1356,12 +1367,17 @@ __global__ void pack_kv64_kernel(const float* Wk, const float* Wv, int dm, int k
        x += (int64_t)gridDim.x * blockDim.x) {
     const int n = (int)(x / kw), kp = (int)(x % kw);
     const int c = kp / kTC, cc = kp % kTC;
-    int seg, col;
-    plan_chunk(p, c, seg, col);
     float v = 0.f;
-    if (n < 2 * dm && col + cc < p.d[seg]) {
-      const int src = (seg > 0 ? p.d[0] : 0) + (seg > 1 ? p.d[1] : 0) + col + cc;
-      v = n < dm ? Wk[(int64_t)n * ksrc + src] : Wv[(int64_t)(n - dm) * ksrc + src];
+    if (p.contig) {                                // K column kp of [h | e | Phi]
+      if (n < 2 * dm && kp < ksrc)
+        v = n < dm ? Wk[(int64_t)n * ksrc + kp] : Wv[(int64_t)(n - dm) * ksrc + kp];
+    } else {
+      int seg, col;
+      plan_chunk(p, c, seg, col);
+      if (n < 2 * dm && col + cc < p.d[seg]) {
+        const int src = (seg > 0 ? p.d[0] : 0) + (seg > 1 ? p.d[1] : 0) + col + cc;
+        v = n < dm ? Wk[(int64_t)n * ksrc + src] : Wv[(int64_t)(n - dm) * ksrc + src];
+      }
     }
     const __nv_bfloat16 hi = __float2bfloat16_rn(v);
     const __nv_bfloat16 lo = __float2bfloat16_rn(v - __bfloat162float(hi));
@@ -1891,11 +1907,17 @@ __global__ void __launch_bounds__(kSThreads, 1)
     s_phi[j] = P.phi[j];
   }
   for (int j = threadIdx.x; j < 2 * dm; j += blockDim.x) s_bias[j] = j < dm ? P.bk[j] : P.bv[j - dm];
+  const int ktot = plan.d[0] + plan.d[1] + plan.d[2];
+  const int e0 = plan.d[0], e1 = plan.d[0] + plan.d[1];   // segment starts in [h | e | Phi]
   for (int c = threadIdx.x; c < nch; c += blockDim.x) {
-    int seg, col;
-    plan_chunk(plan, c, seg, col);
-    const int width = seg == 0 ? plan.d[0] : (seg == 1 ? plan.d[1] : plan.d[2]);
-    s_chunk[c] = make_int4(seg, col, width, width - col > 16 ? 2 : 1);
+    if (plan.contig) {                               // seg -1: resolved per 16-byte piece
+      s_chunk[c] = make_int4(-1, c * kTC, ktot, ktot - c * kTC > 16 ? 2 : 1);
+    } else {
+      int seg, col;
+      plan_chunk(plan, c, seg, col);
+      const int width = seg == 0 ? plan.d[0] : (seg == 1 ? plan.d[1] : plan.d[2]);
+      s_chunk[c] = make_int4(seg, col, width, width - col > 16 ? 2 : 1);
+    }
   }
   if (threadIdx.x == 0) {
     for (int s = 0; s < kSF; ++s) {
@@ -2063,12 +2085,19 @@ __global__ void __launch_bounds__(kSThreads, 1)
       for (int i = 0; i < nch; ++i, ++g) {
         const int c = chunk_of(tt, i, nch);
         const int4 ch = s_chunk[c];
-        const int seg = ch.x;
+        int seg = ch.x, cb = ch.y + 4 * pc;
+        uint32_t nb;
+        if (seg < 0) {                               // contiguous plan: this lane's segment
+          const int g = cb;
+          seg = g < e0 ? 0 : (g < e1 ? 1 : 2);
+          cb = g - (seg == 0 ? 0 : (seg == 1 ? e0 : e1));
+          nb = g < ktot ? 16u : 0u;                  // widths are multiples of 4
+        } else {
+          nb = cb >= ch.z ? 0u : (uint32_t)min(16, (ch.z - cb) * 4);
+        }
         const float* base = seg == 0 ? a.hsrc : (seg == 1 ? a.efeat : a.table);
         const int64_t ld = seg == 0 ? a.ld_hsrc : (seg == 1 ? a.ld_e : (int64_t)P.d_t);
         const int* ridx = seg == 0 ? R.hrow : (seg == 1 ? R.erow : R.trow);
-        const int cb = ch.y + 4 * pc;
-        const uint32_t nb = cb >= ch.z ? 0u : (uint32_t)min(16, (ch.z - cb) * 4);
         const float* b = base + (nb ? cb : 0);
         int x[8];
 #pragma unroll
@@ -2152,8 +2181,14 @@ __global__ void __launch_bounds__(kSThreads, 1)
         }
 #pragma unroll
         for (int k = 0; k < kSKc; ++k) x[k] = ld_shared_f4(src + k * 512);
-        if (ch.x == 2) {                             // time chunk: Phi where the table misses
-          const int cc = ch.y + 4 * pc;
+        if (ch.x < 0 && ch.y + 4 * pc >= ktot) {     // K padding of the contiguous plan
+#pragma unroll
+          for (int k = 0; k < kSKc; ++k) x[k] = make_float4(0.f, 0.f, 0.f, 0.f);
+        }
+        // time columns of this lane's piece: Phi where the table misses
+        const bool tpiece = ch.x == 2 || (ch.x < 0 && ch.y + 4 * pc >= e1 && ch.y + 4 * pc < ktot);
+        if (tpiece) {
+          const int cc = ch.x < 0 ? ch.y + 4 * pc - e1 : ch.y + 4 * pc;
           float w[4], f[4];
 #pragma unroll
           for (int e = 0; e < 4; ++e) {
@@ -2289,7 +2324,7 @@ __global__ void __launch_bounds__(kSThreads, 1)
 namespace tca {
 
 struct PackedLayout {
-  size_t oq, okv, oo, okv64, total;
+  size_t oq, okv, oo, okv64, okvc, total;
 };
 
 static PackedLayout packed_layout(const tgl_attn_params* P) {
@@ -2302,6 +2337,7 @@ static PackedLayout packed_layout(const tgl_attn_params* P) {
   L.okv = W.take((size_t)skv.nchunks * 2 * kNPkv * 128);
   L.oo = W.take((size_t)so.nchunks * 2 * kNPq * 128);
   L.okv64 = W.take((size_t)make_plan(P->d_hsrc, P->d_e, P->d_t).n * kTWStage);
+  L.okvc = W.take((size_t)make_plan_contig(P->d_hsrc, P->d_e, P->d_t).n * kTWStage);
   L.total = W.off;
   return L;
 }
@@ -2319,7 +2355,11 @@ static tgl_status launch_pack(const tgl_attn_params* P, uint8_t* base, cudaStrea
   TGL_TRY(launch_check("pack_weights"));
   pack_kv64_kernel<<<64, 256, 0, s>>>(P->Wk, P->Wv, P->d_model, P->d_hsrc + P->d_e + P->d_t,
                                       make_plan(P->d_hsrc, P->d_e, P->d_t), base + L.okv64);
-  return launch_check("pack_kv64");
+  TGL_TRY(launch_check("pack_kv64"));
+  pack_kv64_kernel<<<64, 256, 0, s>>>(P->Wk, P->Wv, P->d_model, P->d_hsrc + P->d_e + P->d_t,
+                                      make_plan_contig(P->d_hsrc, P->d_e, P->d_t),
+                                      base + L.okvc);
+  return launch_check("pack_kv64 contiguous");
 }
 
 }  // namespace tca
@@ -2413,7 +2453,9 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
   const int smem_q = Pipe<kNPq>::kBytes + 1024;
   const int smem_kv = Pipe<kNPkv>::kBytes + 1024 + kKvEpiBytes;
   const int smem_kvb = Pipe<kNPkv>::kBytes + 1024 + kBEpi * 32 * 33 * 4;
-  // TGL_KV = "bin" forces the register-gather kernel, "async" requires the LDGSTS one
+  // TGL_KV (tests / probes only): "bin" forces the register-gather kernel, "async" the
+  // single-role LDGSTS kernel, "split" / "split_pad" the split-role kernel with the
+  // contiguous / per-segment-padded K plan (default: split, contiguous when possible)
   const char* kvsel = getenv("TGL_KV");
   static bool attr_done = false;   // cached cudaFuncSetAttribute (idempotent)
   if (!attr_done) {
@@ -2446,7 +2488,8 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
                      rows_16b(table, table ? P->d_t : 0, P->d_t);
   // default: the split-role kernel; TGL_KV=async keeps the single-role LDGSTS producers
   const bool use_split = async && !(kvsel && strcmp(kvsel, "async") == 0);
-  if (kvsel && (strcmp(kvsel, "async") == 0 || strcmp(kvsel, "split") == 0) && !async) {
+  if (kvsel && (strcmp(kvsel, "async") == 0 || strcmp(kvsel, "split") == 0 ||
+                strcmp(kvsel, "split_pad") == 0) && !async) {
     set_error("TGL_KV=async: the async-gather path cannot take this call (16-B row pitch / "
               "max_seg <= 32 / 2 heads)");
     return TGL_EUNSUPPORTED;
@@ -2462,12 +2505,15 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
     const int bdst = 32 / max_seg;                 // destinations per 32-row bin
     const int64_t ttiles = ceil_div(n_dst_max, 4 * bdst);
     const unsigned gt = (unsigned)(ttiles < kNumSMs ? (ttiles > 0 ? ttiles : 1) : kNumSMs);
-    const KvPlan plan = make_plan(P->d_hsrc, P->d_e, P->d_t);
+    const bool contig = contig_ok(P->d_hsrc, P->d_e) && !(kvsel && strcmp(kvsel, "split_pad") == 0);
+    const KvPlan plan = contig ? make_plan_contig(P->d_hsrc, P->d_e, P->d_t)
+                               : make_plan(P->d_hsrc, P->d_e, P->d_t);
     if (plan.n > kSMaxChunks) {
       set_error("K|V attention: %d K chunks > %d", plan.n, kSMaxChunks);
       return TGL_EUNSUPPORTED;
     }
-    kv_split_kernel<<<gt, kSThreads, kSSmem, s>>>(a, plan, pk + PL.okv64, bdst);
+    kv_split_kernel<<<gt, kSThreads, kSSmem, s>>>(a, plan, pk + (contig ? PL.okvc : PL.okv64),
+                                                  bdst);
   } else if (async) {
     const int bdst = 32 / max_seg;                 // destinations per 32-row bin
     const int64_t ttiles = ceil_div(n_dst_max, 4 * bdst);

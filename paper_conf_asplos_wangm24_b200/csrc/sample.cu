@@ -1,7 +1,7 @@
 // sample.cu -- S4 temporal neighbourhood sampling (readings R1, R4-R7).
 //
-// One CTA = one tile of 32 queries (32 warps x 1 query: every search of the tile is
-// in flight at once -- the probes are dependent loads), tiles taken from an
+// One CTA = one tile of 32 queries (8 warps x 4 queries searched in lockstep, so
+// each round of dependent probes has 4 independent loads per lane), tiles taken from an
 // atomic ticket.  Per query a warp runs a 32-ary search for the first segment
 // entry with !(ts < t) (monotone predicate, so NaN t -> 0 candidates), then the
 // tile's counts are prefix-summed with a decoupled look-back so `seg_ptr` and
@@ -14,8 +14,8 @@
 
 namespace tgl {
 
-constexpr int kSampleWarps = 32;
-constexpr int kQueriesPerWarp = 1;
+constexpr int kSampleWarps = 8;
+constexpr int kQueriesPerWarp = 4;
 constexpr int kSampleTile = kSampleWarps * kQueriesPerWarp;  // 32
 
 __device__ __forceinline__ int64_t warp_lower_time(const float* __restrict__ ts, int64_t lo,
@@ -61,21 +61,66 @@ sample_kernel(const int64_t* __restrict__ indptr, const int32_t* __restrict__ nb
     return;
   }
 
-  // phase 1: search
+  // phase 1: search -- the warp's 4 queries advance together (one 32-ary narrowing
+  // round per iteration, the 4 probes of a round independent), then the final window
+  int64_t lo[kQueriesPerWarp], hi[kQueriesPerWarp], st[kQueriesPerWarp];
+  float tq[kQueriesPerWarp];
 #pragma unroll
   for (int j = 0; j < kQueriesPerWarp; ++j) {
-    const int lq = warp * kQueriesPerWarp + j;
-    const int64_t q = q0 + lq;
-    int64_t start = 0, n = 0;
+    const int64_t q = q0 + warp * kQueriesPerWarp + j;
+    lo[j] = hi[j] = 0;
+    tq[j] = 0.f;
     if (q < nq) {
       const int32_t v = __ldg(qnode + q);
-      const float t = __ldg(qtime + q);
-      start = __ldg(indptr + v);
-      const int64_t end = __ldg(indptr + v + 1);
-      n = warp_lower_time(ts, start, end, t, lane) - start;
+      tq[j] = __ldg(qtime + q);
+      lo[j] = __ldg(indptr + v);
+      hi[j] = __ldg(indptr + v + 1);
     }
+    st[j] = lo[j];
+  }
+  while (true) {
+    bool any = false;
+    float pv[kQueriesPerWarp];
+    int64_t stepv[kQueriesPerWarp];
+#pragma unroll
+    for (int j = 0; j < kQueriesPerWarp; ++j) {      // issue this round's probes
+      stepv[j] = 0;
+      pv[j] = 0.f;
+      if (hi[j] - lo[j] > 32) {
+        any = true;
+        stepv[j] = (hi[j] - lo[j] + 31) >> 5;
+        const int64_t jj = lo[j] + (int64_t)lane * stepv[j];
+        if (jj < hi[j]) pv[j] = __ldg(ts + jj);
+      }
+    }
+    if (!any) break;
+#pragma unroll
+    for (int j = 0; j < kQueriesPerWarp; ++j) {
+      if (stepv[j] == 0) continue;
+      const int64_t jj = lo[j] + (int64_t)lane * stepv[j];
+      const bool p = (jj < hi[j]) && (pv[j] < tq[j]);
+      const int c = __popc(__ballot_sync(0xffffffffu, p));
+      if (c == 0) {
+        hi[j] = lo[j];                               // pos = lo
+        continue;
+      }
+      const int64_t next = lo[j] + (int64_t)c * stepv[j];
+      const int64_t new_lo = lo[j] + (int64_t)(c - 1) * stepv[j] + 1;
+      hi[j] = (c < 32 && next < hi[j]) ? next : hi[j];
+      lo[j] = new_lo;
+    }
+  }
+  float fv[kQueriesPerWarp];
+#pragma unroll
+  for (int j = 0; j < kQueriesPerWarp; ++j)          // final windows (<= 32 entries)
+    fv[j] = (lo[j] + lane < hi[j]) ? __ldg(ts + lo[j] + lane) : 0.f;
+#pragma unroll
+  for (int j = 0; j < kQueriesPerWarp; ++j) {
+    const bool p = (lo[j] + lane < hi[j]) && (fv[j] < tq[j]);
+    const int64_t n = lo[j] + __popc(__ballot_sync(0xffffffffu, p)) - st[j];
+    const int lq = warp * kQueriesPerWarp + j;
     if (lane == 0) {
-      s_start[lq] = start;
+      s_start[lq] = st[j];
       s_n[lq] = n;
       s_cnt[lq] = (int32_t)(n < k ? n : k);
     }

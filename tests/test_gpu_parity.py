@@ -205,7 +205,9 @@ def cu_pad(a, mult=4):
     return t[:, :d]
 
 
-@pytest.mark.parametrize("precision,kv", [("fp32", "async"), ("bf16", "async"), ("fp32", "bin"),
+@pytest.mark.parametrize("precision,kv", [("fp32", "split"), ("bf16", "split"),
+                                          ("fp32", "split_pad"), ("bf16", "split_pad"),
+                                          ("fp32", "async"), ("bf16", "async"), ("fp32", "bin"),
                                           ("bf16", "bin"), ("fp32_simt", None)])
 @pytest.mark.parametrize("n_dst,kmax,d_h,d_e,long_every", [(1, 10, 172, 172, 0),
                                                           (777, 10, 172, 172, 0),
@@ -215,8 +217,11 @@ def cu_pad(a, mult=4):
                                                           (517, 10, 128, 0, 0),
                                                           (150, 10, 24, 12, 7)])
 def test_attention_vs_oracle(T, monkeypatch, precision, kv, n_dst, kmax, d_h, d_e, long_every):
-    """TGL_KV selects the K|V kernel: "async" (cp.async gathers, needs 16-B row pitches:
-    the odd GDELT widths 413/186 go in row-padded views) or "bin" (register gathers)."""
+    """TGL_KV selects the K|V kernel: "split" (default: loader / converter warps, K chunks
+    cut contiguously over [h | e | Phi] when the widths are multiples of 4), "split_pad"
+    (the same kernel with every segment padded to 32 columns), "async" (single-role
+    cp.async producers) -- all three need 16-B row pitches: the odd GDELT widths 413/186
+    go in row-padded views -- or "bin" (register gathers)."""
     rng = np.random.default_rng(n_dst + kmax)
     p, seg, dst_t, nfeat, dn, sn, ef, eid, et = attn_case(rng, n_dst, kmax, d_h, d_e,
                                                           long_every=long_every)
@@ -225,7 +230,7 @@ def test_attention_vs_oracle(T, monkeypatch, precision, kv, n_dst, kmax, d_h, d_
     exp = oracle.tblock_attn(p, seg, dst_t, nfeat, dn, nfeat, sn, ef, eid, et)
     P = T.AttnParams(p, precision=precision, pack=(n_dst % 2 == 1))
     tab = T.time_precompute(65536, P.t["omega"], P.t["phi"])
-    put = cu_pad if kv == "async" else cu
+    put = cu_pad if kv in ("async", "split", "split_pad") else cu
     nf = put(nfeat)
     for table in (None, tab):
         got = T.tblock_attn(P, cu(seg), cu(dst_t), nf, cu(dn), nf, cu(sn),
