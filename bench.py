@@ -130,6 +130,62 @@ def oracle_rate(cfg, g, neg, params, batches, seconds: float):
         "cores": oracle.num_threads(), "tcsr_build_s": t_build}
 
 
+BIG = ("GDELT", "MAG")   # generated on the device (synth.gpu); host RAM holds only the COO
+
+
+class HostGraph:
+    """Host view of a device-generated graph: what batch slicing and the oracle need."""
+
+    def __init__(self, cfg, src, dst, t):
+        self.cfg, self.src, self.dst, self.t, self.num_edges = cfg, src, dst, t, cfg.n_edges
+
+
+def load_world_device(cfg_name: str):
+    """GDELT/MAG: COO, negatives and feature tables generated on cuda (synth.gpu, the
+    same counter-based values as synth.make_graph), host copies of the COO only."""
+    import synth
+    import torch
+    from synth import gpu as sg
+    cfg = synth.get_config(cfg_name)
+    d = torch.device("cuda")
+    src, dst, t = sg.device_graph(cfg, d)
+    neg = sg.device_negatives(cfg, d)
+    # 16-byte row pitch (GDELT's 413 / 186 floats padded to 416 / 188): the K|V kernel's
+    # cp.async gathers need it; the values are the same counter-based features
+    nfeat = sg.device_feature_table(cfg.seeds["feat"], cfg.n_nodes, cfg.d_v, d, pitch_mult=4)
+    efeat = (sg.device_feature_table(cfg.seeds["feat"] + 7919, cfg.n_edges, cfg.d_e, d,
+                                     pitch_mult=4)
+             if cfg.d_e else torch.zeros((0, 0), dtype=torch.float32, device=d))
+    g = HostGraph(cfg, src.cpu().numpy(), dst.cpu().numpy(), t.cpu().numpy())
+    neg_h = neg.cpu().numpy()
+    dev = {"src": src, "dst": dst, "t": t, "neg": neg, "nfeat": nfeat, "efeat": efeat}
+    return cfg, g, neg_h, synth.gen.model_params(cfg), dev
+
+
+def oracle_rate_big(cfg, g, neg, params, batches, seconds: float, frac: int = 0):
+    """Listing 1's recursion (oracle/big.py) root by root on whole-graph-free segments:
+    the whole-graph oracle cannot hold GDELT/MAG.  Bounded by `seconds` of CPU work."""
+    import oracle
+    from oracle import big
+    from oracle import pipeline as opipe
+    segs, done, t_run, nb = {}, 0, 0.0, 0
+    for b in batches:
+        nb += 1
+        qn, qt = opipe.roots(*synth_batch(g, neg, b))
+        for v, tq in zip(qn, qt):
+            t0 = time.perf_counter()
+            big.embed_recursive(g.src, g.dst, g.t, cfg, params, [v], [tq],
+                                cfg.seeds["sampler"], segs=segs)
+            t_run += time.perf_counter() - t0
+            done += 1
+            if t_run >= seconds:
+                break
+        if t_run >= seconds:
+            break
+    return {"emb_per_s": done / t_run, "batches": nb, "roots": done, "seconds": t_run,
+            "cores": oracle.num_threads(), "edges_per_s": float("nan")}
+
+
 def synth_batch(g, neg, b):
     import synth
     return synth.batch_roots_inputs(g, neg, b)
@@ -140,6 +196,8 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
+    if args.config.upper() in BIG:
+        return run_reference_big(args)
     cfg, g, neg, params = load_world(args.config)
     import oracle
     from oracle import pipeline as opipe
@@ -182,6 +240,58 @@ def run_reference(args):
     return 0
 
 
+def run_reference_big(args):
+    """--impl reference on GDELT/MAG: the oracle's recursion (oracle/big.py) on a few roots
+    per step; the COO comes from the same seeded generator as our arm (synth.gpu on a
+    GPU box -- input generation only -- else synth.make_graph)."""
+    import oracle
+    import synth
+    from oracle import big
+    from oracle import pipeline as opipe
+    import torch
+    cfg = synth.get_config(args.config.upper())
+    if torch.cuda.is_available():                   # the same COO our arm generates
+        from synth import gpu as sg
+        d = torch.device("cuda")
+        src, dst, t = sg.device_graph(cfg, d)
+        gg = HostGraph(cfg, src.cpu().numpy(), dst.cpu().numpy(), t.cpu().numpy())
+        neg = sg.device_negatives(cfg, d).cpu().numpy()
+        del src, dst, t
+    else:
+        gg = synth.make_graph(cfg, with_features=False)
+        neg = synth.make_negatives(cfg)
+    params = synth.gen.model_params(cfg)
+    b0 = int(0.7 * cfg.n_batches)
+    per_step = 2                                    # roots per step (bounded sample)
+    times, roots, segs = [], 0, {}
+    for i in range(args.warmup + args.steps):
+        qn, qt = opipe.roots(*synth_batch(gg, neg, b0 + i))
+        t0 = time.perf_counter()
+        big.embed_recursive(gg.src, gg.dst, gg.t, cfg, params, qn[:per_step], qt[:per_step],
+                            cfg.seeds["sampler"], segs=segs)
+        dt = time.perf_counter() - t0
+        if i >= args.warmup:
+            times.append(dt)
+            roots += per_step
+    T = sum(times)
+    val = roots / T
+    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "embeddings/s",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1e3 * T / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": cfg.name, "roots_per_step": per_step, "layers": cfg.n_layers,
+                       "k": cfg.k, "strategy": cfg.strategy, "dedup": cfg.dedup,
+                       "precompute": cfg.precompute},
+            "cpu_baseline": {"value": val, "unit": "embeddings/s",
+                             "cores": oracle.num_threads(), "kind": "oracle",
+                             "sample": f"first {per_step} roots of each batch from 70% of the "
+                                       f"stream, Listing 1's recursion (oracle/big.py)"},
+            "e2e": {"value": val, "unit": "embeddings/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
 # ---------------------------------------------------------------------- our arm
 def algorithmic_attn(cfg, n_dst: int, n_edges: int, d_hdst: int, d_hsrc: int):
     """Per tgl_tblock_attn call: FLOPs and bytes the method must do."""
@@ -210,14 +320,18 @@ def algorithmic_kv(cfg, n_dst: float, n_edges: float, d_hsrc: int):
     return flops, bytes_
 
 
-def ncu_traffic(precision: str):
+def ncu_traffic(config: str, precision: str):
     """dram__bytes_read.sum + dram__bytes_write.sum per launch of the K|V kernel from the
-    committed `ncu --set full` capture (profiles/), or None."""
+    committed `ncu --set full` capture of this config and precision (profiles/), or None."""
     try:
         d = json.load(open(os.path.join(ROOT, "profiles", "r01_kv_split_traffic.json")))
-        return d[precision]
+        return d[config][precision]
     except Exception:
         return None
+
+
+KV_KERNELS = {0: "kv_split_kernel (contiguous K plan)", 1: "kv_split_kernel (padded K plan)",
+              2: "kv_async_kernel", 3: "kv_bin_kernel", 4: "kv_kernel (general)"}
 
 
 def run_ours(args):
@@ -235,10 +349,13 @@ def run_ours(args):
     from paper_conf_asplos_wangm24_b200 import TGATPipeline, TSampler, tgl
     from paper_conf_asplos_wangm24_b200 import dist as pdist
 
-    cfg, g, neg, params = load_world(args.config)
     cu = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
-    dev = {"src": cu(g.src), "dst": cu(g.dst), "t": cu(g.t), "neg": cu(neg),
-           "nfeat": cu(g.nfeat), "efeat": cu(g.efeat)}
+    if args.config.upper() in BIG:
+        cfg, g, neg, params, dev = load_world_device(args.config.upper())
+    else:
+        cfg, g, neg, params = load_world(args.config)
+        dev = {"src": cu(g.src), "dst": cu(g.dst), "t": cu(g.t), "neg": cu(neg),
+               "nfeat": cu(g.nfeat), "efeat": cu(g.efeat)}
     torch.cuda.synchronize()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     ev0.record()
@@ -323,7 +440,6 @@ def run_ours(args):
         pipe.forward(record=rec)
         torch.cuda.synchronize()
         kv_ms.append(lib.tgl_kv_timing_ms(0))   # the tail block runs first
-        lib.tgl_kv_timing(0)
         tail = pipe.L - 1
         rec_ms.append(rec[tail][0].elapsed_time(rec[tail][1]))
         mk = rec["_marks"]
@@ -337,6 +453,7 @@ def run_ours(args):
     E_avg = sum(e for _, e in rec_shape) / len(rec_shape)
     fl, by = algorithmic_attn(cfg, U_avg, E_avg, cfg.d_v, cfg.d_v)
     attn_ms = sum(rec_ms) / len(rec_ms)
+    lib.tgl_kv_timing(0)
     kv_fl, kv_by = algorithmic_kv(cfg, U_avg, E_avg, cfg.d_v)
     kv_ok = [m for m in kv_ms if m > 0]
     kv_avg = sum(kv_ok) / len(kv_ok) if kv_ok else float("nan")
@@ -362,8 +479,9 @@ def run_ours(args):
     else:
         peak, bound, unit, ach = hbm_peak, "hbm", "GB/s", kv_gbs
         note = "measured HBM copy bandwidth (MEASURED_PEAKS.json); bf16 MMA time < HBM time"
-    tr = ncu_traffic(args.precision)
-    roofline = {"kernel": "kv_split_kernel (K|V attention of the tail block: S6,S7,S9-S12)",
+    tr = ncu_traffic(cfg.name, args.precision)
+    kname = KV_KERNELS.get(int(lib.tgl_kv_timing_kernel(0)), "?")
+    roofline = {"kernel": f"{kname}: K|V attention of the tail block (S6,S7,S9-S12)",
                 "bound": bound, "achieved": ach, "peak": peak, "unit": unit,
                 "frac": ach / peak,
                 "traffic": tr["dram_bytes_per_launch"] if tr else None,
@@ -408,11 +526,15 @@ def run_ours(args):
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        r = oracle_rate(cfg, g, neg, params, [batch_of(i) for i in range(200)], args.cpu_seconds)
+        rate = oracle_rate_big if cfg.name in BIG else oracle_rate
+        r = rate(cfg, g, neg, params, [batch_of(i) for i in range(200)], args.cpu_seconds)
+        smp = (f"{r['roots']} roots of {r['batches']} batch(es) from 70% of the stream, one "
+               f"at a time by Listing 1's recursion (oracle/big.py), {r['seconds']:.1f} s"
+               if cfg.name in BIG else
+               f"{r['batches']} whole batch(es) ({r['roots']} roots) from 70% of the stream, "
+               f"{r['seconds']:.1f} s")
         cpu = {"value": r["emb_per_s"], "unit": "embeddings/s", "cores": r["cores"],
-               "kind": "oracle", "sample": f"{r['batches']} whole batch(es) "
-               f"({r['roots']} roots) from 70% of the stream, {r['seconds']:.1f} s",
-               "sampled_edges_per_s": r["edges_per_s"]}
+               "kind": "oracle", "sample": smp, "sampled_edges_per_s": r["edges_per_s"]}
 
     if rank == 0:
         line = {"metric": METRIC, "value": emb_per_s, "unit": "embeddings/s",

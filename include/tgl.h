@@ -235,7 +235,7 @@ tgl_status tgl_tblock_attn(const tgl_attn_params* P, int64_t n_dst_max, const in
                            int32_t max_seg, float* out, void* ws, size_t* ws_bytes,
                            void* stream);
 
-/* Measurement hook (bench.py): while armed (arm = 1; arming resets the count),
+/* Measurement hook (bench.py): while armed (arm = 1; arming resets the records),
  * the first 8 tensor-core tgl_tblock_attn calls each record a pair of CUDA events
  * on their stream around their K|V attention kernel (S6, S7, S9-S12; the dominant
  * kernel).  tgl_kv_timing_ms(i) synchronises on the i-th stop event and returns
@@ -243,6 +243,10 @@ tgl_status tgl_tblock_attn(const tgl_attn_params* P, int64_t n_dst_max, const in
  * state, not thread-safe; measurement only (never armed during graph capture). */
 int tgl_kv_timing(int arm);
 float tgl_kv_timing_ms(int i);
+/* Which K|V kernel call i ran: 0 split-role (contiguous K chunks), 1 split-role (per-
+ * segment padded K chunks), 2 single-role cp.async, 3 register-gather (rows without a
+ * 16-byte pitch), 4 general (segments > 32 rows); -1 if call i was not recorded. */
+int tgl_kv_timing_kernel(int i);
 
 /* ---------------------------------------------------------------------------
  * S14  Dedup inverse applied to rows (the hook of P:279 / TGOpt dedup_invert

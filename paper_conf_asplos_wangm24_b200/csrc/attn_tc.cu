@@ -2381,6 +2381,8 @@ constexpr int kKvEvMax = 8;
 static bool g_kv_armed = false;
 static int g_kv_n = 0;                               // K|V launches recorded since arming
 static cudaEvent_t g_kv_ev[kKvEvMax][2] = {};
+static int g_kv_kind[kKvEvMax] = {};                 // 0 split/contig, 1 split/padded, 2 async,
+                                                     // 3 bin, 4 general
 
 size_t tc_attn_ws_bytes(const tgl_attn_params* P, int64_t n_dst_max, size_t* o_q, size_t* o_r,
                         size_t* o_pack) {
@@ -2495,6 +2497,7 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
     return TGL_EUNSUPPORTED;
   }
   const bool kv_rec = g_kv_armed && g_kv_n < kKvEvMax;
+  int kv_kind = 4;
   if (kv_rec) {
     for (int e = 0; e < 2; ++e)
       if (g_kv_ev[g_kv_n][e] == nullptr)
@@ -2514,16 +2517,19 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
     }
     kv_split_kernel<<<gt, kSThreads, kSSmem, s>>>(a, plan, pk + (contig ? PL.okvc : PL.okv64),
                                                   bdst);
+    kv_kind = contig ? 0 : 1;
   } else if (async) {
     const int bdst = 32 / max_seg;                 // destinations per 32-row bin
     const int64_t ttiles = ceil_div(n_dst_max, 4 * bdst);
     const unsigned gt = (unsigned)(ttiles < kNumSMs ? (ttiles > 0 ? ttiles : 1) : kNumSMs);
     kv_async_kernel<<<gt, kTThreads, kTSmem, s>>>(a, make_plan(P->d_hsrc, P->d_e, P->d_t),
                                                   pk + PL.okv64, bdst);
+    kv_kind = 2;
   } else if (binned) {
     // binned path: whole segments per epilogue warp (no block barriers)
     const unsigned gkv = (unsigned)(n_dst_max < kNumSMs ? (n_dst_max > 0 ? n_dst_max : 1) : kNumSMs);
     kv_bin_kernel<<<gkv, kBThreads, smem_kvb, s>>>(a);
+    kv_kind = 3;
   } else {
     const int64_t groups = ceil_div(n_dst_max, a.dpb);
     const unsigned gkv = (unsigned)(groups < kNumSMs ? groups : kNumSMs);
@@ -2532,6 +2538,7 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
   TGL_TRY(launch_check("tc kv kernel"));
   if (kv_rec) {
     TGL_TRY(cuda_check(cudaEventRecord(g_kv_ev[g_kv_n][1], s), "event record"));
+    g_kv_kind[g_kv_n] = kv_kind;
     ++g_kv_n;
   }
   dense_kernel<true><<<gq, kWsThreads, smem_q, s>>>(a);
@@ -2551,8 +2558,12 @@ extern "C" int tgl_debug_timeline(unsigned long long* host, size_t n) {
 
 extern "C" int tgl_kv_timing(int arm) {
   tgl::g_kv_armed = arm != 0;
-  tgl::g_kv_n = 0;
+  if (arm) tgl::g_kv_n = 0;                        // disarming keeps the records
   return 0;
+}
+
+extern "C" int tgl_kv_timing_kernel(int i) {
+  return (i < 0 || i >= tgl::g_kv_n) ? -1 : tgl::g_kv_kind[i];
 }
 
 extern "C" float tgl_kv_timing_ms(int i) {

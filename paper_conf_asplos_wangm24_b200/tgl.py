@@ -25,7 +25,8 @@ PRECISION = {"fp32": FP32, "bf16": BF16, "fp32_simt": FP32_SIMT}
 SYMBOLS = ["tgl_version", "tgl_status_string", "tgl_last_error", "tgl_build_tcsr",
            "tgl_batch_roots", "tgl_dedup", "tgl_sample", "tgl_next_block",
            "tgl_time_precompute", "tgl_time_encode", "tgl_tblock_attn", "tgl_gather_rows",
-           "tgl_attn_packed_bytes", "tgl_attn_pack", "tgl_kv_timing", "tgl_kv_timing_ms"]
+           "tgl_attn_packed_bytes", "tgl_attn_pack", "tgl_kv_timing", "tgl_kv_timing_ms",
+           "tgl_kv_timing_kernel"]
 
 
 class TGLError(RuntimeError):
@@ -66,6 +67,8 @@ def _load():
     lib.tgl_kv_timing.restype = C.c_int
     lib.tgl_kv_timing_ms.argtypes = [C.c_int]
     lib.tgl_kv_timing_ms.restype = C.c_float
+    lib.tgl_kv_timing_kernel.argtypes = [C.c_int]
+    lib.tgl_kv_timing_kernel.restype = C.c_int
     return lib
 
 

@@ -39,15 +39,23 @@ def feature_rows_torch(seed: int, rows: torch.Tensor, dim: int) -> torch.Tensor:
     return v.to(torch.float32) * (2.0 ** -23)
 
 
-def device_feature_table(seed: int, n_rows: int, dim: int, device, chunk_elems: int = 1 << 27):
-    out = torch.empty((n_rows, dim), dtype=torch.float32, device=device)
+def device_feature_table(seed: int, n_rows: int, dim: int, device, chunk_elems: int = 1 << 27,
+                         pitch_mult: int = 1):
+    """[n_rows, dim] feature table on `device`; with pitch_mult > 1 the rows are stored with
+    a pitch rounded up to a multiple of pitch_mult floats (e.g. 4: 16-byte row pitch, the
+    layout the cp.async gathers of the K|V kernel take) and a [:, :dim] view is returned.
+    The padding columns are zero and never read."""
+    pitch = max(pitch_mult, (dim + pitch_mult - 1) // pitch_mult * pitch_mult) if dim else 0
+    out = torch.empty((n_rows, pitch), dtype=torch.float32, device=device)
+    if pitch > dim:
+        out[:, dim:] = 0
     if dim == 0 or n_rows == 0:
-        return out
+        return out[:, :dim]
     rows_per = max(1, chunk_elems // dim)
     for r0 in range(0, n_rows, rows_per):
         r1 = min(n_rows, r0 + rows_per)
-        out[r0:r1] = feature_rows_torch(seed, torch.arange(r0, r1, device=device), dim)
-    return out
+        out[r0:r1, :dim] = feature_rows_torch(seed, torch.arange(r0, r1, device=device), dim)
+    return out[:, :dim]
 
 
 def _zipf_rank(u: torch.Tensor, n: int, a: float) -> torch.Tensor:

@@ -1,7 +1,7 @@
 # per-kernel ncu durations of the REDDIT tail K|V kernel for compile variants x masks
 mkdir -p gpurun_out
 for v in "$@"; do
-  TGL_NVCC_EXTRA="$v" python -c "from paper_conf_asplos_wangm24_b200 import build; build.build(force=True)" > gpurun_out/build_v.log 2>&1 || { echo "build failed: $v"; tail -20 gpurun_out/build_v.log; continue; }
+  TGL_NVCC_EXTRA="$v" python paper_conf_asplos_wangm24_b200/build.py -f > gpurun_out/build_v.log 2>&1 || { echo "build failed: $v"; tail -20 gpurun_out/build_v.log; continue; }
   PROBE_KV=${KV:-split} PROBE_MASKS=${MASKS:-0,79} timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/pl.csv python tools/kv_probe.py ${PREC:-fp32} > /dev/null 2>&1
   python - "$v" <<'PY'
 import csv, os, sys
@@ -22,4 +22,4 @@ for i, m in enumerate(masks):
 print(f"== {sys.argv[1] or 'default'}: " + "  ".join(out))
 PY
 done
-python -c "from paper_conf_asplos_wangm24_b200 import build; build.build(force=True)" > /dev/null 2>&1
+python paper_conf_asplos_wangm24_b200/build.py -f > /dev/null 2>&1

@@ -1,7 +1,7 @@
 # build K|V kernel variants (compile-time pipeline depths) and time the REDDIT tail call
 mkdir -p gpurun_out
 run() {
-  TGL_NVCC_EXTRA="$1" python -c "from paper_conf_asplos_wangm24_b200 import build; build.build(force=True)" > gpurun_out/build_v.log 2>&1 || { echo "build failed: $1"; cat gpurun_out/build_v.log; return; }
+  TGL_NVCC_EXTRA="$1" python paper_conf_asplos_wangm24_b200/build.py -f > gpurun_out/build_v.log 2>&1 || { echo "build failed: $1"; cat gpurun_out/build_v.log; return; }
   echo "== variant: $1"
   for w in ${WINDOWS:-default}; do
     if [ "$w" = default ]; then unset PROBE_WINDOW; else export PROBE_WINDOW=$w; fi
@@ -12,4 +12,4 @@ run() {
   unset PROBE_WINDOW
 }
 for v in "$@"; do run "$v"; done
-python -c "from paper_conf_asplos_wangm24_b200 import build; build.build(force=True)" > /dev/null 2>&1
+python paper_conf_asplos_wangm24_b200/build.py -f > /dev/null 2>&1
