@@ -953,10 +953,12 @@ struct BinDesc {
 
 // Epilogue of the binned K|V kernels (warps 0-7): S10-S12 for one tile per trip.
 // Warp w owns TMEM lane quarter w%4 and head w/4; see kv_bin_kernel.
-template <int NS, class D>
+// kPW: row pitch of the per-warp transpose buffer (33: 32 columns per pass; 17: 16
+// columns per pass, half the shared memory -- the split kernel spends it on stages)
+template <int NS, class D, int kPW = 33>
 __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uint64_t* dempty,
                                              uint64_t* tfull, uint64_t* tempty, const D* bd,
-                                             uint32_t tmem, float (*s_pv)[32][33],
+                                             uint32_t tmem, float* s_pvf,
                                              const float* s_bias) {
   constexpr uint32_t kCols = 256;
   constexpr int dm = 100, dh = 50;
@@ -965,7 +967,8 @@ __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uin
   uint32_t tt = 0;
   const int q4 = warp & 3, head = warp >> 2;
   const int cb = head * dh;                        // this warp's columns [cb, cb + dh)
-  float (*pv)[33] = s_pv[warp];
+  constexpr int kCW = kPW - 1;                     // columns per transpose pass
+  float* pvw = s_pvf + warp * 32 * kPW;
   for (;; ++tt) {
     const uint32_t ab = tt & 1u, ds = tt % NS;
     // one warp polls, the other seven block in bar.sync (no issue slots spent waiting)
@@ -1048,21 +1051,25 @@ __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uin
       tmem_ld32(ta + dm + cb + cq * 32, v);
       tmem_wait_ld();
 #pragma unroll
-      for (int j = 0; j < 32; ++j) pv[lane][j] = w * v[j];
-      __syncwarp();
-      const int c = cq * 32 + lane;                  // this lane's column in the head
-      const float bvc = c < dh ? s_bias[dm + cb + c] : 0.f;
-      unsigned sm = smask, em = emask;
-      while (sm) {
-        const int slo = __ffs(sm) - 1, shi = __ffs(em);   // [slo, shi)
-        sm &= sm - 1;
-        em &= em - 1;
-        const int dr = __shfl_sync(0xffffffffu, d, slo);
-        float acc = 0.f;
-        for (int r = slo; r < shi; ++r) acc += pv[r][lane];
-        if (c < dh) a.rbuf[(int64_t)dr * kQLd + cb + c] = acc + bvc;
+      for (int hh = 0; hh < 32 / kCW; ++hh) {
+#pragma unroll
+        for (int j = 0; j < kCW; ++j) pvw[lane * kPW + j] = w * v[hh * kCW + j];
+        __syncwarp();
+        const int c = cq * 32 + hh * kCW + lane;     // this lane's column in the head
+        const bool act = lane < kCW && c < dh;
+        const float bvc = act ? s_bias[dm + cb + c] : 0.f;
+        unsigned sm = smask, em = emask;
+        while (sm) {
+          const int slo = __ffs(sm) - 1, shi = __ffs(em);   // [slo, shi)
+          sm &= sm - 1;
+          em &= em - 1;
+          const int dr = __shfl_sync(0xffffffffu, d, slo);
+          float acc = 0.f;
+          for (int r = slo; r < shi; ++r) acc += pvw[r * kPW + (lane & (kCW - 1))];
+          if (act) a.rbuf[(int64_t)dr * kQLd + cb + c] = acc + bvc;
+        }
+        __syncwarp();
       }
-      __syncwarp();
     }
     tc_fence_before();
     if (warp == 0) trace(a, 10, tt);
@@ -1227,7 +1234,8 @@ __global__ void __launch_bounds__(kBThreads, 1) kv_bin_kernel(Args a) {
       __syncwarp();
     }
   } else {                                           // ---------------- epilogue warps 0-7
-    bin_epilogue<kDSlots>(a, B.dfull, B.dempty, B.tfull, B.tempty, bd, tmem, s_pv, s_bias);
+    bin_epilogue<kDSlots>(a, B.dfull, B.dempty, B.tfull, B.tempty, bd, tmem, &s_pv[0][0][0],
+                          s_bias);
   }
   ws_teardown(tmem, 2 * kCols, kBMma);
 }
@@ -1803,7 +1811,8 @@ __global__ void __launch_bounds__(kTThreads, 1)
       prof_add(a, 8, clock64() - m2);                  // MMA: whole tile
     }
   } else {                                           // ---------------- epilogue warps 0-7
-    bin_epilogue<kTDSlots>(a, B.dfull, B.dempty, B.tfull, B.tempty, bd, tmem, s_pv, s_bias);
+    bin_epilogue<kTDSlots>(a, B.dfull, B.dempty, B.tfull, B.tempty, bd, tmem, &s_pv[0][0][0],
+                           s_bias);
   }
   ws_teardown(tmem, 2 * kCols, kTMma);
 }
@@ -1865,14 +1874,19 @@ constexpr int kSRowsPerConv = kBM / kSConvWarps;     // 16 (8 warps) or 32 (4 wa
 constexpr int kSKc = kSRowsPerConv / 4;              // rows per converter lane
 constexpr int kSThreads = (kSConv0 + kSConvWarps) * 32;   // 768 with 8 converter warps
 constexpr int kSPipeBytes = (kSF + kSB) * kSStage + kSW * kTWStage;
-constexpr int kSSmem = 1024 + kSPipeBytes + kBEpi * 32 * 33 * 4;
+#ifndef TGL_KV_SPLIT_DSLOTS
+#define TGL_KV_SPLIT_DSLOTS 3
+#endif
+constexpr int kSDSlots = TGL_KV_SPLIT_DSLOTS;       // tile descriptor ring
+constexpr int kSPW = 17;                             // 16-column epilogue transposes
+constexpr int kSSmem = 1024 + kSPipeBytes + kBEpi * 32 * kSPW * 4;
 constexpr int kSMaxChunks = 48;
 
 struct SBars {
   uint64_t ffull[kSF], fempty[kSF];
   uint64_t bfull[kSB], bempty[kSB];
   uint64_t wfull[kSW], wempty[kSW];
-  uint64_t dfull[kTDSlots], dempty[kTDSlots];
+  uint64_t dfull[kSDSlots], dempty[kSDSlots];
   uint64_t tfull[2], tempty[2];
 };
 
@@ -1889,13 +1903,13 @@ __global__ void __launch_bounds__(kSThreads, 1)
   uint8_t* pipe = align1024(smem_raw);
   __shared__ SBars B;
   __shared__ uint32_t s_tmem;
-  __shared__ TDesc bd[kTDSlots];
+  __shared__ TDesc bd[kSDSlots];
   __shared__ float s_omega[256], s_phi[256];
   __shared__ float s_bias[2 * kMaxModel];
   __shared__ int64_t s_seg[kTDescWarps][4 * 32 + 1];
   __shared__ float s_td[kTDescWarps][4 * 32];
   __shared__ int4 s_chunk[kSMaxChunks];          // {segment, first column, width, K steps}
-  float (*s_pv)[32][33] = reinterpret_cast<float (*)[32][33]>(pipe + kSPipeBytes);
+  float* s_pvf = reinterpret_cast<float*>(pipe + kSPipeBytes);
   constexpr uint32_t kCols = 256;
   const tgl_attn_params& P = a.P;
   const int64_t n = dev_count(a.n_dst_dev, a.n_dst_max);
@@ -1932,7 +1946,7 @@ __global__ void __launch_bounds__(kSThreads, 1)
       mbar_init(&B.wfull[s], 1);
       mbar_init(&B.wempty[s], 1);
     }
-    for (int s = 0; s < kTDSlots; ++s) {
+    for (int s = 0; s < kSDSlots; ++s) {
       mbar_init(&B.dfull[s], 1);
       mbar_init(&B.dempty[s], kBEpi + kSLoadWarps + kSConvWarps + 2);
     }
@@ -1964,8 +1978,8 @@ __global__ void __launch_bounds__(kSThreads, 1)
     int64_t* sg = s_seg[dw];
     float* stdv = s_td[dw];
     for (tt = dw;; tt += kTDescWarps) {
-      const uint32_t ds = tt % kTDSlots;
-      wait_free_sleep(&B.dempty[ds], tt / kTDSlots, TGL_SLEEP_DESC);
+      const uint32_t ds = tt % kSDSlots;
+      wait_free_sleep(&B.dempty[ds], tt / kSDSlots, TGL_SLEEP_DESC);
       trace(a, 20, tt);
       TDesc& R = bd[ds];
       const int64_t T = blockIdx.x + (int64_t)tt * gridDim.x;
@@ -2037,8 +2051,8 @@ __global__ void __launch_bounds__(kSThreads, 1)
     uint32_t wl = 0;
     const uint32_t wbytes = split ? kTWStage : kTWHalf;
     for (;; ++tt) {
-      const uint32_t ds = tt % kTDSlots;
-      mbar_wait_sleep(&B.dfull[ds], (tt / kTDSlots) & 1u, TGL_SLEEP_W);
+      const uint32_t ds = tt % kSDSlots;
+      mbar_wait_sleep(&B.dfull[ds], (tt / kSDSlots) & 1u, TGL_SLEEP_W);
       const int live = bd[ds].live;
       warp_arrive(&B.dempty[ds]);
       if (!live) break;
@@ -2068,8 +2082,8 @@ __global__ void __launch_bounds__(kSThreads, 1)
     const uint32_t lofs = (uint32_t)r0 * 128 + pc * 16;
     uint32_t g = 0;
     for (;; ++tt) {
-      const uint32_t ds = tt % kTDSlots;
-      mbar_wait_sleep(&B.dfull[ds], (tt / kTDSlots) & 1u, TGL_SLEEP_LOAD);
+      const uint32_t ds = tt % kSDSlots;
+      mbar_wait_sleep(&B.dfull[ds], (tt / kSDSlots) & 1u, TGL_SLEEP_LOAD);
       const TDesc& R = bd[ds];
       if (!R.live) {
 #if TGL_KV_LAG > 0
@@ -2144,8 +2158,8 @@ __global__ void __launch_bounds__(kSThreads, 1)
     const uint32_t o_even = sw64_off(lane >> 3, 4 * pc), o_odd = sw64_off((lane >> 3) + 4, 4 * pc);
     uint32_t g = 0;
     for (;; ++tt) {
-      const uint32_t ds = tt % kTDSlots;
-      mbar_wait(&B.dfull[ds], (tt / kTDSlots) & 1u);
+      const uint32_t ds = tt % kSDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kSDSlots) & 1u);
       const TDesc& R = bd[ds];
       if (!R.live) {
         warp_arrive(&B.dempty[ds]);
@@ -2246,8 +2260,8 @@ __global__ void __launch_bounds__(kSThreads, 1)
     uint32_t g = 0, wl = 0;
     constexpr uint32_t idesc = idesc_bf16(kBM, kNPkv);
     for (;; ++tt) {
-      const uint32_t ds = tt % kTDSlots;
-      mbar_wait(&B.dfull[ds], (tt / kTDSlots) & 1u);
+      const uint32_t ds = tt % kSDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kSDSlots) & 1u);
       const int live = bd[ds].live;
       warp_arrive(&B.dempty[ds]);
       if (!live) break;
@@ -2313,7 +2327,8 @@ __global__ void __launch_bounds__(kSThreads, 1)
       __syncwarp();
     }
   } else if (warp < kBEpi) {                         // ---------------- epilogue warps 0-7
-    bin_epilogue<kTDSlots>(a, B.dfull, B.dempty, B.tfull, B.tempty, bd, tmem, s_pv, s_bias);
+    bin_epilogue<kSDSlots, TDesc, kSPW>(a, B.dfull, B.dempty, B.tfull, B.tempty, bd, tmem,
+                                        s_pvf, s_bias);
   }
   ws_teardown(tmem, 2 * kCols, kTMma);
 }
