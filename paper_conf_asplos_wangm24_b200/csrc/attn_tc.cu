@@ -2201,9 +2201,17 @@ __global__ void __launch_bounds__(kSThreads, 1)
         }
         // time columns of this lane's piece: Phi where the table misses
         const bool tpiece = ch.x == 2 || (ch.x < 0 && ch.y + 4 * pc >= e1 && ch.y + 4 * pc < ktot);
-        if (tpiece) {
-          const int cc = ch.x < 0 ? ch.y + 4 * pc - e1 : ch.y + 4 * pc;
-          float w[4], f[4];
+        // branch-free fast path for the 4 x kSKc elements of a time piece (w = 0 past d_t
+        // gives cos(0) there, zeroed below); the rare |b| >= 1e9 takes the accurate cosf
+        // after ONE warp vote, taken outside the per-lane condition (a chunk of the
+        // contiguous plan mixes time and edge-feature pieces)
+        const int cc = ch.x < 0 ? ch.y + 4 * pc - e1 : ch.y + 4 * pc;
+        float w[4], f[4], cv[kSKc][4];
+        bool bad = false;
+        bool need = false;                           // a row of this lane misses the table
+#pragma unroll
+        for (int k = 0; k < kSKc; ++k) need |= trk[k] < 0;
+        if (tpiece && need) {
 #pragma unroll
           for (int e = 0; e < 4; ++e) {
             const bool ok = cc + e < P.d_t;
@@ -2211,12 +2219,28 @@ __global__ void __launch_bounds__(kSThreads, 1)
             f[e] = ok ? s_phi[cc + e] : 0.f;
           }
 #pragma unroll
+          for (int k = 0; k < kSKc; ++k)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+              const float bb = __fadd_rn(__fmul_rn(w[e], dtk[k]), f[e]);   // R10 argument
+              bad |= !(fabsf(bb) < 1e9f) && trk[k] < 0;
+              cv[k][e] = tenc_cos_reduced(bb);
+            }
+        }
+        if (__any_sync(0xffffffffu, bad) && tpiece && need) {
+#pragma unroll
+          for (int k = 0; k < kSKc; ++k)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) cv[k][e] = tenc_fast(dtk[k], w[e], f[e]);
+        }
+        if (tpiece && need) {
+#pragma unroll
           for (int k = 0; k < kSKc; ++k) {
             if (trk[k] < 0) {
-              x[k].x = (cc < P.d_t) ? tenc_fast(dtk[k], w[0], f[0]) : 0.f;
-              x[k].y = (cc + 1 < P.d_t) ? tenc_fast(dtk[k], w[1], f[1]) : 0.f;
-              x[k].z = (cc + 2 < P.d_t) ? tenc_fast(dtk[k], w[2], f[2]) : 0.f;
-              x[k].w = (cc + 3 < P.d_t) ? tenc_fast(dtk[k], w[3], f[3]) : 0.f;
+              x[k].x = (cc < P.d_t) ? cv[k][0] : 0.f;
+              x[k].y = (cc + 1 < P.d_t) ? cv[k][1] : 0.f;
+              x[k].z = (cc + 2 < P.d_t) ? cv[k][2] : 0.f;
+              x[k].w = (cc + 3 < P.d_t) ? cv[k][3] : 0.f;
             }
           }
         }

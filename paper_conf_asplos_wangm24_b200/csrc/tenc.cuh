@@ -23,6 +23,14 @@ __device__ __forceinline__ float tenc_direct(float dt, float omega, float phi) {
 // hundreds of instructions and local memory per element.
 static __device__ __noinline__ float tenc_cos_slow(float b) { return cosf(b); }
 
+// the reduction + SFU cosine alone (valid for |b| < 1e9; callers check)
+__device__ __forceinline__ float tenc_cos_reduced(float b) {
+  const float k = rintf(b * 0.159154943091895336f);
+  float r = fmaf(-k, 6.28318548202514648f, b);
+  r = fmaf(-k, -1.74845560007449713e-7f, r);
+  return __cosf(r);
+}
+
 __device__ __forceinline__ float tenc_cos_fast(float b) {
   // out of line: an inlined cosf would drag its Payne-Hanek path (local-memory table
   // walk) into every call site, predicated on in the steady state

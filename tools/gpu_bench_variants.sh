@@ -3,7 +3,7 @@ mkdir -p gpurun_out
 for v in "$@"; do
   TGL_NVCC_EXTRA="$v" python paper_conf_asplos_wangm24_b200/build.py -f > gpurun_out/build_v.log 2>&1 || { echo "build failed: $v"; tail -20 gpurun_out/build_v.log; continue; }
   for c in ${CONFIGS:-REDDIT MAG}; do
-    timeout 900 python bench.py --config $c --steps 10 --warmup 3 --no-cpu-baseline > gpurun_out/bv.log 2>&1
+    timeout 400 python bench.py --config $c --steps 10 --warmup 3 --no-cpu-baseline > gpurun_out/bv.log 2>&1
     python -c "
 import json,sys
 d=json.loads(open('gpurun_out/bv.log').read().strip().splitlines()[-1]); r=d['roofline']
