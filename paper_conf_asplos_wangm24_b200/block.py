@@ -91,7 +91,9 @@ class TGATPipeline:
                           "neg": z(batch, i32)}
             self.stage_n = batch
         # kernels launched per forward (libtgl only; memsets excluded)
-        per_block = [(1 if l > 0 else 0) + (3 if use_dedup else 0) + 1 + 3 for l in range(self.L)]
+        # dedup: one single-CTA kernel up to 4096 pairs (dedup.cu kSmallN), else three
+        dedup_launches = [(1 if b.n_max <= 4096 else 3) if use_dedup else 0 for b in self.blocks]
+        per_block = [(1 if l > 0 else 0) + dedup_launches[l] + 1 + 3 for l in range(self.L)]
         self.launches_per_forward = 1 + sum(per_block) + (1 if use_dedup else 0)
         self._alloc_workspaces()
         self.graph_exec = None

@@ -116,6 +116,88 @@ __global__ void dedup_inverse_kernel(int64_t n_max, const int64_t* n_dev,
     inv[i] = (int32_t)rank[slot_of[i]];
 }
 
+// Small batches (n_max <= kSmallN, e.g. the 3*batch roots of a step): the whole dedup in
+// ONE CTA -- hash table in shared memory, blocked first-occurrence scan, inverse -- one
+// launch instead of two memsets and three kernels.  Same keys, same order (R9).
+constexpr int kSmallThreads = 1024;
+constexpr int kSmallItems = 4;
+constexpr int kSmallN = kSmallThreads * kSmallItems;   // 4096
+constexpr int kSmallLog2Cap = 13;                       // 8192 slots (load <= 1/2)
+constexpr int kSmallSmem = (1 << kSmallLog2Cap) * (8 + 4 + 4);   // keys, first, rank
+
+__global__ void __launch_bounds__(kSmallThreads)
+dedup_small_kernel(int64_t n_max, const int64_t* n_dev, const int32_t* __restrict__ node,
+                   const float* __restrict__ t, int32_t* __restrict__ uniq_node,
+                   float* __restrict__ uniq_t, int64_t* num_uniq_dev, int32_t* __restrict__ inv) {
+  extern __shared__ unsigned long long s_keys[];
+  unsigned int* s_first = reinterpret_cast<unsigned int*>(s_keys + (1 << kSmallLog2Cap));
+  unsigned int* s_rank = s_first + (1 << kSmallLog2Cap);
+  __shared__ int s_warp[kSmallThreads / 32];
+  constexpr uint32_t mask = (1u << kSmallLog2Cap) - 1u;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int n = (int)dev_count(n_dev, n_max);
+  for (int j = tid; j < (1 << kSmallLog2Cap); j += kSmallThreads) {
+    s_keys[j] = 0ull;
+    s_first[j] = 0u;
+  }
+  __syncthreads();
+  uint32_t slot[kSmallItems];
+#pragma unroll
+  for (int r = 0; r < kSmallItems; ++r) {        // blocked: thread owns items tid*4 + r
+    const int i = tid * kSmallItems + r;
+    slot[r] = 0;
+    if (i < n) {
+      const unsigned long long k = pair_key(__ldg(node + i), __ldg(t + i));
+      uint32_t h = slot_hash(k, kSmallLog2Cap);
+      while (true) {
+        const unsigned long long prev = atomicCAS(s_keys + h, 0ull, k);
+        if (prev == 0ull || prev == k) {
+          atomicMax(s_first + h, ~(unsigned int)i);
+          slot[r] = h;
+          break;
+        }
+        h = (h + 1u) & mask;
+      }
+    }
+  }
+  __syncthreads();
+  bool isfirst[kSmallItems];
+  int cnt = 0;
+#pragma unroll
+  for (int r = 0; r < kSmallItems; ++r) {
+    const int i = tid * kSmallItems + r;
+    isfirst[r] = i < n && s_first[slot[r]] == ~(unsigned int)i;
+    cnt += isfirst[r];
+  }
+  const int incl = (int)warp_inclusive_scan((int64_t)cnt, lane);
+  if (lane == 31) s_warp[warp] = incl;
+  __syncthreads();
+  if (warp == 0) {
+    const int wv = s_warp[lane];
+    const int wincl = (int)warp_inclusive_scan((int64_t)wv, lane);
+    s_warp[lane] = wincl - wv;                    // exclusive offset of each warp
+    if (lane == 31) *num_uniq_dev = wincl;
+  }
+  __syncthreads();
+  int pos = s_warp[warp] + incl - cnt;
+#pragma unroll
+  for (int r = 0; r < kSmallItems; ++r) {
+    if (isfirst[r]) {
+      const int i = tid * kSmallItems + r;
+      uniq_node[pos] = node[i];
+      uniq_t[pos] = t[i];
+      s_rank[slot[r]] = (unsigned int)pos;
+      ++pos;
+    }
+  }
+  __syncthreads();
+#pragma unroll
+  for (int r = 0; r < kSmallItems; ++r) {
+    const int i = tid * kSmallItems + r;
+    if (i < n) inv[i] = (int32_t)s_rank[slot[r]];
+  }
+}
+
 static int log2_capacity(int64_t n_max) {
   int64_t want = 2 * (n_max > 32 ? n_max : 32);
   int l = 6;
@@ -152,6 +234,18 @@ extern "C" tgl_status tgl_dedup(int64_t n_max, const int64_t* n_dev, const int32
   TGL_REQUIRE(num_uniq_dev != nullptr, "null num_uniq_dev");
   TGL_REQUIRE(n_max == 0 || (node && t && uniq_node && uniq_t && inv), "null pointer");
   cudaStream_t s = as_stream(stream);
+  if (n_max <= kSmallN) {                        // one CTA, shared-memory table
+    static bool attr = false;
+    if (!attr) {
+      TGL_TRY(cuda_check(cudaFuncSetAttribute(dedup_small_kernel,
+                                              cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                              kSmallSmem), "dedup attr"));
+      attr = true;
+    }
+    dedup_small_kernel<<<1, kSmallThreads, kSmallSmem, s>>>(n_max, n_dev, node, t, uniq_node,
+                                                            uniq_t, num_uniq_dev, inv);
+    return launch_check("dedup_small");
+  }
   char* w = static_cast<char*>(ws);
   // keys/first/rank must start at 0; slot_of is fully overwritten -> clear only what matters
   TGL_TRY(cuda_check(cudaMemsetAsync(w + o_keys, 0, o_slot - o_keys, s), "dedup memset"));

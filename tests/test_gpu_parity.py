@@ -113,7 +113,7 @@ def test_sample_device_count_and_empty(T):
 
 
 # ------------------------------------------------------------------ S3
-@pytest.mark.parametrize("n", [0, 1, 2047, 2048, 2049, 20000, 200001])
+@pytest.mark.parametrize("n", [0, 1, 1800, 2047, 2048, 2049, 4096, 4097, 20000, 200001])
 def test_dedup_bit_exact(T, n):
     rng = np.random.default_rng(n + 1)
     node = rng.integers(0, max(2, n // 8), n).astype(np.int32)
@@ -132,16 +132,17 @@ def test_dedup_bit_exact(T, n):
     assert np.array_equal(np_(inv)[:n], einv)
 
 
-def test_dedup_device_count(T):
+@pytest.mark.parametrize("n_max,n", [(10000, 6001), (4000, 1234)])   # multi-kernel / 1-CTA
+def test_dedup_device_count(T, n_max, n):
     rng = np.random.default_rng(9)
-    node = rng.integers(0, 300, 10000).astype(np.int32)
-    t = rng.integers(0, 30, 10000).astype(np.float32)
-    ndev = torch.tensor([6001], dtype=torch.int64, device="cuda")
+    node = rng.integers(0, 300, n_max).astype(np.int32)
+    t = rng.integers(0, 30, n_max).astype(np.float32)
+    ndev = torch.tensor([n], dtype=torch.int64, device="cuda")
     un, ut, nu, inv = T.dedup(cu(node), cu(t), n_dev=ndev)
-    eu, eut, einv = oracle.dedup(node[:6001], t[:6001])
+    eu, eut, einv = oracle.dedup(node[:n], t[:n])
     U = int(np_(nu)[0])
     assert U == len(eu) and np.array_equal(np_(un)[:U], eu)
-    assert np.array_equal(np_(inv)[:6001], einv)
+    assert np.array_equal(np_(inv)[:n], einv)
 
 
 # ------------------------------------------------------------------ S6

@@ -37,13 +37,26 @@ def main(rep, top=25):
     for k, v in sorted(st, key=lambda x: -x[1])[:10]:
         print(f"{100 * v / tot:5.1f}% {k.replace('smsp__pcsamp_warps_issue_stalled_', '')}")
     src = ncu_csv(rep, "--page", "source", "--print-source", "sass")
-    hs = src[1]
-    rs = [dict(zip(hs, x)) for x in src[2:]]
     key = "Warp Stall Sampling (All Samples)"
-    tot = sum(float(x[key] or 0) for x in rs) or 1
+    hs = next((r for r in src if key in r), None)   # one header row per kernel in the report
+    if hs is None:
+        return
+    rs = []
+    for x in src[src.index(hs) + 1:]:
+        if key in x:                                 # the next kernel's header: stop
+            break
+        rs.append(dict(zip(hs, x)))
+
+    def f(v):
+        try:
+            return float(v or 0)
+        except ValueError:
+            return 0.0
+    tot = sum(f(x.get(key)) for x in rs) or 1
     print("--- top SASS by stall samples")
-    for x in sorted(rs, key=lambda x: -float(x[key] or 0))[:top]:
-        print(f"{100 * float(x[key]) / tot:5.1f}% {x['Address'][-5:]} {x['Source'].strip()[:90]}")
+    for x in sorted(rs, key=lambda x: -f(x.get(key)))[:top]:
+        print(f"{100 * f(x.get(key)) / tot:5.1f}% {x.get('Address', '')[-5:]} "
+              f"{x.get('Source', '').strip()[:90]}")
 
 
 if __name__ == "__main__":
