@@ -29,6 +29,8 @@ __global__ void batch_roots_kernel(int64_t batch, int64_t num_edges, const int64
                                    const float* __restrict__ t, const int32_t* __restrict__ neg,
                                    int32_t* __restrict__ qnode, float* __restrict__ qtime,
                                    int64_t* n_roots_dev) {
+  pdl_wait();     // PDL: predecessor grid complete, its writes visible
+  pdl_trigger();
   int64_t s = start_dev ? *start_dev : 0;
   int64_t b = num_edges - s;
   b = b < 0 ? 0 : (b < batch ? b : batch);
@@ -54,6 +56,8 @@ __global__ void next_block_kernel(int64_t n_dst_max, const int64_t* n_dst_dev,
                                   const int32_t* __restrict__ src_node,
                                   const float* __restrict__ src_t, int32_t* __restrict__ out_node,
                                   float* __restrict__ out_t, int64_t* n_out_dev) {
+  pdl_wait();     // PDL: predecessor grid complete, its writes visible
+  pdl_trigger();
   int64_t nd = dev_count(n_dst_dev, n_dst_max);
   int64_t ns = seg_ptr[nd];
   ns = ns < n_src_max ? ns : n_src_max;
@@ -76,6 +80,8 @@ __global__ void gather_rows_kernel(int64_t n_max, const int64_t* n_dev,
                                    const int32_t* __restrict__ idx,
                                    const float* __restrict__ table, int64_t ld_table, int32_t d,
                                    float* __restrict__ out, int64_t ld_out) {
+  pdl_wait();     // PDL: predecessor grid complete, its writes visible
+  pdl_trigger();
   int64_t n = dev_count(n_dev, n_max);
   int64_t total = n * d;
   for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
@@ -120,7 +126,7 @@ tgl_status tgl_batch_roots(int64_t batch, int64_t num_edges, const int64_t* star
                            int64_t* n_roots_dev, void* stream) {
   TGL_REQUIRE(batch >= 0 && num_edges >= 0, "negative size");
   TGL_REQUIRE(src && dst && t && neg && qnode && qtime, "null pointer");
-  batch_roots_kernel<<<grid_for(batch, 256), 256, 0, as_stream(stream)>>>(
+  launch_pdl(batch_roots_kernel, dim3(grid_for(batch, 256)), dim3(256), 0, as_stream(stream), 
       batch, num_edges, start_dev, src, dst, t, neg, qnode, qtime, n_roots_dev);
   return launch_check("batch_roots");
 }
@@ -133,7 +139,7 @@ tgl_status tgl_next_block(int64_t n_dst_max, const int64_t* n_dst_dev, const int
   TGL_REQUIRE(seg_ptr && out_node && out_t, "null pointer");
   TGL_REQUIRE((n_dst_max == 0 || (dst_node && dst_t)) && (n_src_max == 0 || (src_node && src_t)),
               "null pointer");
-  next_block_kernel<<<grid_for(n_dst_max + n_src_max, 256), 256, 0, as_stream(stream)>>>(
+  launch_pdl(next_block_kernel, dim3(grid_for(n_dst_max + n_src_max, 256)), dim3(256), 0, as_stream(stream), 
       n_dst_max, n_dst_dev, dst_node, dst_t, n_src_max, seg_ptr, src_node, src_t, out_node, out_t,
       n_out_dev);
   return launch_check("next_block");
@@ -145,7 +151,7 @@ tgl_status tgl_gather_rows(int64_t n_max, const int64_t* n_dev, const int32_t* i
   TGL_REQUIRE(n_max >= 0 && d >= 0 && ld_table >= d && ld_out >= d, "bad size");
   if (n_max == 0 || d == 0) return TGL_OK;
   TGL_REQUIRE(idx && table && out, "null pointer");
-  gather_rows_kernel<<<grid_for(n_max * d, 256), 256, 0, as_stream(stream)>>>(
+  launch_pdl(gather_rows_kernel, dim3(grid_for(n_max * d, 256)), dim3(256), 0, as_stream(stream), 
       n_max, n_dev, idx, table, ld_table, d, out, ld_out);
   return launch_check("gather_rows");
 }

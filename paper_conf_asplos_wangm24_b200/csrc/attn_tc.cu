@@ -493,6 +493,8 @@ constexpr int kNPq = 104;   // d_model padded to a multiple of 8 (rows of Wq / W
 
 template <bool kFfn>
 __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
+  pdl_wait();     // PDL: predecessor grid complete, its writes visible
+  pdl_trigger();
   extern __shared__ uint8_t smem_raw[];
   uint8_t* pipe = align1024(smem_raw);
   __shared__ Bars B;
@@ -678,6 +680,8 @@ constexpr int kNPkv = 200;   // [Wk ; Wv] rows (2 * d_model)
 constexpr int kKvEpiBytes = (2 * kMaxDpb * kMaxModel + kBM * 33) * 4;   // s_q, s_r, s_pv
 
 __global__ void __launch_bounds__(kWsThreads, 1) kv_kernel(Args a) {
+  pdl_wait();     // PDL: predecessor grid complete, its writes visible
+  pdl_trigger();
   extern __shared__ uint8_t smem_raw[];
   uint8_t* pipe = align1024(smem_raw);
   __shared__ Bars B;
@@ -1080,6 +1084,8 @@ __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uin
 }
 
 __global__ void __launch_bounds__(kBThreads, 1) kv_bin_kernel(Args a) {
+  pdl_wait();     // PDL: predecessor grid complete, its writes visible
+  pdl_trigger();
   extern __shared__ uint8_t smem_raw[];
   uint8_t* pipe = align1024(smem_raw);
   __shared__ Bars B;
@@ -1410,6 +1416,8 @@ __device__ __forceinline__ float4 ld_row4(const float* base, int row, int64_t ld
 __global__ void __launch_bounds__(kTThreads, 1)
     kv_async_kernel(const Args a, const KvPlan plan, const uint8_t* __restrict__ wkv,
                     const int bdst) {
+  pdl_wait();     // PDL: predecessor grid complete, its writes visible
+  pdl_trigger();
   extern __shared__ uint8_t smem_raw[];
   uint8_t* pipe = align1024(smem_raw);
   __shared__ TBars B;
@@ -1899,6 +1907,8 @@ __device__ __forceinline__ void cp_async_mbar_arrive_noinc(uint64_t* bar) {
 __global__ void __launch_bounds__(kSThreads, 1)
     kv_split_kernel(const Args a, const KvPlan plan, const uint8_t* __restrict__ wkv,
                     const int bdst) {
+  pdl_wait();     // PDL: predecessor grid complete, its writes visible
+  pdl_trigger();
   extern __shared__ uint8_t smem_raw[];
   uint8_t* pipe = align1024(smem_raw);
   __shared__ SBars B;
@@ -2521,7 +2531,7 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
   }
   const int64_t tiles = ceil_div(n_dst_max, kBM);
   const unsigned gq = (unsigned)(tiles < kNumSMs ? tiles : kNumSMs);
-  dense_kernel<false><<<gq, kWsThreads, smem_q, s>>>(a);
+  launch_pdl(dense_kernel<false>, dim3(gq), dim3(kWsThreads), smem_q, s, a);
   TGL_TRY(launch_check("tc q kernel"));
   const bool binned = max_seg > 0 && max_seg <= 32 && P->n_heads == 2;
   const bool async = binned && !(kvsel && strcmp(kvsel, "bin") == 0) &&
@@ -2554,25 +2564,25 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
       set_error("K|V attention: %d K chunks > %d", plan.n, kSMaxChunks);
       return TGL_EUNSUPPORTED;
     }
-    kv_split_kernel<<<gt, kSThreads, kSSmem, s>>>(a, plan, pk + (contig ? PL.okvc : PL.okv64),
+    launch_pdl(kv_split_kernel, dim3(gt), dim3(kSThreads), kSSmem, s, a, plan, pk + (contig ? PL.okvc : PL.okv64),
                                                   bdst);
     kv_kind = contig ? 0 : 1;
   } else if (async) {
     const int bdst = 32 / max_seg;                 // destinations per 32-row bin
     const int64_t ttiles = ceil_div(n_dst_max, 4 * bdst);
     const unsigned gt = (unsigned)(ttiles < kNumSMs ? (ttiles > 0 ? ttiles : 1) : kNumSMs);
-    kv_async_kernel<<<gt, kTThreads, kTSmem, s>>>(a, make_plan(P->d_hsrc, P->d_e, P->d_t),
+    launch_pdl(kv_async_kernel, dim3(gt), dim3(kTThreads), kTSmem, s, a, make_plan(P->d_hsrc, P->d_e, P->d_t),
                                                   pk + PL.okv64, bdst);
     kv_kind = 2;
   } else if (binned) {
     // binned path: whole segments per epilogue warp (no block barriers)
     const unsigned gkv = (unsigned)(n_dst_max < kNumSMs ? (n_dst_max > 0 ? n_dst_max : 1) : kNumSMs);
-    kv_bin_kernel<<<gkv, kBThreads, smem_kvb, s>>>(a);
+    launch_pdl(kv_bin_kernel, dim3(gkv), dim3(kBThreads), smem_kvb, s, a);
     kv_kind = 3;
   } else {
     const int64_t groups = ceil_div(n_dst_max, a.dpb);
     const unsigned gkv = (unsigned)(groups < kNumSMs ? groups : kNumSMs);
-    kv_kernel<<<gkv, kWsThreads, smem_kv, s>>>(a);
+    launch_pdl(kv_kernel, dim3(gkv), dim3(kWsThreads), smem_kv, s, a);
   }
   TGL_TRY(launch_check("tc kv kernel"));
   if (kv_rec) {
@@ -2580,7 +2590,7 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
     g_kv_kind[g_kv_n] = kv_kind;
     ++g_kv_n;
   }
-  dense_kernel<true><<<gq, kWsThreads, smem_q, s>>>(a);
+  launch_pdl(dense_kernel<true>, dim3(gq), dim3(kWsThreads), smem_q, s, a);
   return launch_check("tc ffn kernel");
 }
 

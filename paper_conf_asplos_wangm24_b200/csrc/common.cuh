@@ -67,6 +67,45 @@ constexpr int kNumSMs = 148;
 
 inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
+// ------------------------------------------------------------------ programmatic dependent launch
+// Every kernel of a batch's launch chain is launched with programmatic stream
+// serialisation: its CTAs may start (launch latency, constant staging, barrier init,
+// TMEM allocation) while the previous kernel drains.  pdl_wait() (griddepcontrol.wait)
+// blocks until the previous grid has completed and its writes are visible; EVERY thread
+// of every PDL-launched kernel calls it before touching global data a predecessor wrote
+// (and before exiting), so completion stays transitive along the chain.  pdl_trigger()
+// lets the next kernel's CTAs be scheduled early.  Both are no-ops without the attribute.
+__device__ __forceinline__ void pdl_wait() {
+#ifndef TGL_NO_PDL
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+#endif
+}
+__device__ __forceinline__ void pdl_trigger() {
+#ifndef TGL_NO_PDL
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+#endif
+}
+
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem,
+                              cudaStream_t s, Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+#ifndef TGL_NO_PDL
+  cfg.numAttrs = 1;
+#else
+  cfg.numAttrs = 0;
+#endif
+  return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
+}
+
 // ------------------------------------------------------------------ device helpers
 __device__ __forceinline__ int64_t dev_count(const int64_t* n_dev, int64_t n_max) {
   if (n_dev == nullptr) return n_max;

@@ -28,6 +28,8 @@ __global__ void dedup_insert_kernel(int64_t n_max, const int64_t* n_dev,
                                     const int32_t* __restrict__ node, const float* __restrict__ t,
                                     unsigned long long* keys, unsigned int* first,
                                     uint32_t* __restrict__ slot_of, int log2cap) {
+  pdl_wait();     // PDL: predecessor grid complete, its writes visible
+  pdl_trigger();
   const int64_t n = dev_count(n_dev, n_max);
   const uint32_t mask = (1u << log2cap) - 1u;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
@@ -52,6 +54,8 @@ dedup_compact_kernel(int64_t n_max, const int64_t* n_dev, const int32_t* __restr
                      const uint32_t* __restrict__ slot_of, unsigned int* __restrict__ rank,
                      int32_t* __restrict__ uniq_node, float* __restrict__ uniq_t,
                      int64_t* num_uniq_dev, unsigned long long* status, unsigned int* ticket) {
+  pdl_wait();     // PDL: predecessor grid complete, its writes visible
+  pdl_trigger();
   __shared__ int64_t s_tile;
   __shared__ int64_t s_warp[kDedupThreads / 32];
   __shared__ int64_t s_excl;
@@ -110,6 +114,8 @@ __global__ void dedup_inverse_kernel(int64_t n_max, const int64_t* n_dev,
                                      const uint32_t* __restrict__ slot_of,
                                      const unsigned int* __restrict__ rank,
                                      int32_t* __restrict__ inv) {
+  pdl_wait();     // PDL: predecessor grid complete, its writes visible
+  pdl_trigger();
   const int64_t n = dev_count(n_dev, n_max);
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
        i += (int64_t)gridDim.x * blockDim.x)
@@ -129,6 +135,8 @@ __global__ void __launch_bounds__(kSmallThreads)
 dedup_small_kernel(int64_t n_max, const int64_t* n_dev, const int32_t* __restrict__ node,
                    const float* __restrict__ t, int32_t* __restrict__ uniq_node,
                    float* __restrict__ uniq_t, int64_t* num_uniq_dev, int32_t* __restrict__ inv) {
+  pdl_wait();     // PDL: predecessor grid complete, its writes visible
+  pdl_trigger();
   extern __shared__ unsigned long long s_keys[];
   unsigned int* s_first = reinterpret_cast<unsigned int*>(s_keys + (1 << kSmallLog2Cap));
   unsigned int* s_rank = s_first + (1 << kSmallLog2Cap);
@@ -242,7 +250,7 @@ extern "C" tgl_status tgl_dedup(int64_t n_max, const int64_t* n_dev, const int32
                                               kSmallSmem), "dedup attr"));
       attr = true;
     }
-    dedup_small_kernel<<<1, kSmallThreads, kSmallSmem, s>>>(n_max, n_dev, node, t, uniq_node,
+    launch_pdl(dedup_small_kernel, dim3(1), dim3(kSmallThreads), kSmallSmem, s, n_max, n_dev, node, t, uniq_node,
                                                             uniq_t, num_uniq_dev, inv);
     return launch_check("dedup_small");
   }
@@ -256,13 +264,13 @@ extern "C" tgl_status tgl_dedup(int64_t n_max, const int64_t* n_dev, const int32
   auto slot = reinterpret_cast<uint32_t*>(w + o_slot);
   int64_t g1 = ceil_div(n_max > 0 ? n_max : 1, 256);
   if (g1 > kNumSMs * 8) g1 = kNumSMs * 8;
-  dedup_insert_kernel<<<(unsigned)g1, 256, 0, s>>>(n_max, n_dev, node, t, keys, first, slot, l2);
+  launch_pdl(dedup_insert_kernel, dim3((unsigned)g1), dim3(256), 0, s, n_max, n_dev, node, t, keys, first, slot, l2);
   TGL_TRY(launch_check("dedup_insert"));
-  dedup_compact_kernel<<<(unsigned)tiles, kDedupThreads, 0, s>>>(
+  launch_pdl(dedup_compact_kernel, dim3((unsigned)tiles), dim3(kDedupThreads), 0, s, 
       n_max, n_dev, node, t, first, slot, rank, uniq_node, uniq_t, num_uniq_dev,
       reinterpret_cast<unsigned long long*>(w + o_status),
       reinterpret_cast<unsigned int*>(w + o_ticket));
   TGL_TRY(launch_check("dedup_compact"));
-  dedup_inverse_kernel<<<(unsigned)g1, 256, 0, s>>>(n_max, n_dev, slot, rank, inv);
+  launch_pdl(dedup_inverse_kernel, dim3((unsigned)g1), dim3(256), 0, s, n_max, n_dev, slot, rank, inv);
   return launch_check("dedup_inverse");
 }

@@ -45,6 +45,8 @@ sample_kernel(const int64_t* __restrict__ indptr, const int32_t* __restrict__ nb
               int64_t* __restrict__ seg_ptr, int32_t* __restrict__ out_nbr,
               int32_t* __restrict__ out_eid, float* __restrict__ out_ts,
               unsigned long long* status, unsigned int* ticket) {
+  pdl_wait();     // PDL: predecessor grid complete, its writes visible
+  pdl_trigger();
   __shared__ int64_t s_tile;
   __shared__ int64_t s_start[kSampleTile];
   __shared__ int64_t s_n[kSampleTile];
@@ -198,7 +200,7 @@ extern "C" tgl_status tgl_sample(const tgl_tcsr* g, int64_t nq_max, const int64_
   char* w = static_cast<char*>(ws);
   TGL_TRY(cuda_check(cudaMemsetAsync(w, 0, L.off, s), "sample memset"));
   uint2 key = make_uint2((uint32_t)(seed & 0xFFFFFFFFu), (uint32_t)(seed >> 32));
-  sample_kernel<<<(unsigned)tiles, kSampleWarps * 32, 0, s>>>(
+  launch_pdl(sample_kernel, dim3((unsigned)tiles), dim3(kSampleWarps * 32), 0, s, 
       g->indptr, g->nbr, g->eid, g->ts, nq_max, nq_dev, qnode, qtime, k, strategy, key, layer,
       seg_ptr, out_nbr, out_eid, out_ts, reinterpret_cast<unsigned long long*>(w + o_status),
       reinterpret_cast<unsigned int*>(w + o_ticket));
