@@ -524,8 +524,11 @@ __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
       s_v1[j] = P.bk[j];
     }
   }
+  if (threadIdx.x < 32) s_trace_n[threadIdx.x] = 0;
+  if ((threadIdx.x & 31) == 0) trace(a, 36, 0);     // per-warp start stamp
   ws_init(B, &s_tmem, 2 * kCols);
   const uint32_t tmem = s_tmem;
+  if (threadIdx.x == 0) trace(a, 37, 0);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   DenseSched sched(n);
   int64_t i0;
@@ -536,11 +539,19 @@ __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
       const uint32_t ds = tt % kDSlots;
       wait_free(&B.dempty[ds], tt / kDSlots);
       RowDesc& R = rd[ds];
-      for (int r = lane; r < kBM; r += 32) {
+      int64_t hrows[kBM / 32];                       // all index loads of the warp in flight
+#pragma unroll
+      for (int u = 0; u < kBM / 32; ++u) {
+        const int r = lane + 32 * u;
+        hrows[u] = (r < rows) ? (a.hdst_idx ? (int64_t)a.hdst_idx[i0 + r] : i0 + r) : 0;
+      }
+#pragma unroll
+      for (int u = 0; u < kBM / 32; ++u) {
+        const int r = lane + 32 * u;
         const float *p0 = nullptr, *p1 = nullptr;
         if (r < rows) {
           const int64_t i = i0 + r;
-          const int64_t hrow = a.hdst_idx ? (int64_t)a.hdst_idx[i] : i;
+          const int64_t hrow = hrows[u];
           if (kFfn) {
             p0 = a.rbuf + i * kQLd;                    // [r_i ; h_i]  (eq 7)
             p1 = a.hdst + hrow * a.ld_hdst;
@@ -555,6 +566,7 @@ __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
         R.rdst[r] = r < rows ? r : -1;
       }
       warp_arrive(&B.dfull[ds]);
+      trace(a, 30, tt);
     }
   } else if (warp == kWWarp) {                       // ---------------- weight loader
     uint32_t wit = 0;
@@ -567,6 +579,7 @@ __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
       const uint32_t ds = tt % kDSlots;
       mbar_wait(&B.dfull[ds], (tt / kDSlots) & 1u);
       produce_tile<kNPq, kProdWarp0, kGPT>(sg, split, pipe, B, ait, tt, rd[ds], s_omega, s_phi, a.table);
+      if (warp == kProdWarp0) trace(a, 31, tt);
       warp_arrive(&B.dempty[ds]);
     }
   } else if (warp == kMmaWarp) {                     // ---------------- MMA issuer
@@ -575,12 +588,14 @@ __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
       for (; sched.next(i0, rows); ++tt)
         mma_tile<kNPq, kNPq>(sg, split, pipe, B, tmem + (tt & 1u) * kCols, ait, wit, tt);
     __syncwarp();
+    trace(a, 33, 0);
   } else {                                           // ---------------- epilogue
     const int row = warp * 32 + lane;
     const int D = P.d_model;
     for (; sched.next(i0, rows); ++tt) {
       const uint32_t ab = tt & 1u, ds = tt % kDSlots;
       mbar_wait(&B.tfull[ab], (tt >> 1) & 1u);
+      if (warp == 0) trace(a, 34, tt);
       tc_fence_after();
       warp_arrive(&B.dempty[ds]);                     // descriptors not needed here
       (void)ds;
@@ -619,20 +634,9 @@ __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
           q[D + 1] = qb1;
         }
       } else {
-        // out = LayerNorm(ReLU(acc + bo)): three passes over TMEM (sum, squares, write)
-        float s = 0.f;
-#pragma unroll 1
-        for (int cq = 0; cq < 4; ++cq) {
-          tmem_ld32(ta + cq * 32, v);
-          tmem_wait_ld();
-#pragma unroll
-          for (int j = 0; j < 32; ++j) {
-            const int col = cq * 32 + j;
-            if (col < D) s += fmaxf(v[j] + s_v0[col], 0.f);
-          }
-        }
-        const float mean = s / (float)D;
-        float q2 = 0.f;
+        // out = LayerNorm(ReLU(acc + bo)): two passes over TMEM -- sum and sum of squares
+        // (fp32; the ReLU outputs are O(1), so E[x^2] - mean^2 loses < 1e-6), then write
+        float s = 0.f, s2 = 0.f;
 #pragma unroll 1
         for (int cq = 0; cq < 4; ++cq) {
           tmem_ld32(ta + cq * 32, v);
@@ -641,12 +645,15 @@ __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
           for (int j = 0; j < 32; ++j) {
             const int col = cq * 32 + j;
             if (col < D) {
-              const float d = fmaxf(v[j] + s_v0[col], 0.f) - mean;
-              q2 += d * d;
+              const float y = fmaxf(v[j] + s_v0[col], 0.f);
+              s += y;
+              s2 = fmaf(y, y, s2);
             }
           }
         }
-        const float inv = rsqrtf(q2 / (float)D + P.ln_eps);
+        const float mean = s / (float)D;
+        const float var = fmaxf(s2 / (float)D - mean * mean, 0.f);
+        const float inv = rsqrtf(var + P.ln_eps);
         float* o = a.out + (i0 + row) * D;
 #pragma unroll 1
         for (int cq = 0; cq < 4; ++cq) {
@@ -670,6 +677,7 @@ __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
       }
       tc_fence_before();
       warp_arrive(&B.tempty[ab]);
+      if (warp == 0) trace(a, 35, tt);
     }
   }
   ws_teardown(tmem, 2 * kCols);

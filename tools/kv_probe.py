@@ -123,7 +123,8 @@ if os.environ.get("PROBE_TRACE"):
     k = (v & 0xff).astype(int)
     o = np.argsort(t, kind="stable")
     t0 = t[o[0]]
-    names = {20: "D.build-start", 21: "D.built", 1: "P.load-issued", 3: "P.data-ready", 4: "P.converted", 5: "M.A-ready", 6: "M.issued",
+    names = {30: "Dn.desc-built", 31: "Dn.prod-done", 33: "Dn.mma-done", 34: "Dn.epi-start",
+             35: "Dn.epi-end", 36: "Dn.warp-start", 37: "Dn.init-done", 20: "D.build-start", 21: "D.built", 1: "P.load-issued", 3: "P.data-ready", 4: "P.converted", 5: "M.A-ready", 6: "M.issued",
              7: "M.tile-start", 9: "E.acc-ready", 10: "E.done", 11: "W.issue", 12: "M.B-full"}
     for x in o[:int(os.environ.get('PROBE_TRACE_N', '400'))]:
         print(f"{(t[x] - t0) / 1965:8.2f} us  {names.get(ev[x], ev[x]):14s} {k[x]}")
