@@ -967,7 +967,7 @@ struct BinDesc {
 // Warp w owns TMEM lane quarter w%4 and head w/4; see kv_bin_kernel.
 // kPW: row pitch of the per-warp transpose buffer (33: 32 columns per pass; 17: 16
 // columns per pass, half the shared memory -- the split kernel spends it on stages)
-template <int NS, class D, int kPW = 33>
+template <int NS, class D, int kPW = 33, bool kLowReg = false>
 __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uint64_t* dempty,
                                              uint64_t* tfull, uint64_t* tempty, const D* bd,
                                              uint32_t tmem, float* s_pvf,
@@ -1001,13 +1001,16 @@ __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uin
     const int lo = 31 - __clz(smask & (0xffffffffu >> (31 - lane)));   // last start <= lane
     const int hi = __ffs(emask & (0xffffffffu << lane));              // last end >= lane, +1
     // this row's q (head columns) and q . bk, fetched before waiting for the accumulator
-    float qv[dh];
+    // (kLowReg: read piecewise after the wait instead -- 64-register budget)
     const float* qrow = a.qbuf + (int64_t)(valid ? d : 0) * kQLd;
+    float qv[kLowReg ? 1 : dh];
+    if (!kLowReg) {
 #pragma unroll
-    for (int j = 0; j < dh; j += 2) {
-      const float2 q2 = __ldg(reinterpret_cast<const float2*>(qrow + cb + j));
-      qv[j] = q2.x;
-      qv[j + 1] = q2.y;
+      for (int j = 0; j < dh; j += 2) {
+        const float2 q2 = __ldg(reinterpret_cast<const float2*>(qrow + cb + j));
+        qv[j] = q2.x;
+        qv[j + 1] = q2.y;
+      }
     }
     const float qb = __ldg(qrow + dm + head);
     if (threadIdx.x == 0) tl_mark(a, tt, 5);
@@ -1028,13 +1031,33 @@ __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uin
     float v[32];
     // S10: this head's logit <q_dst, k_row + bk> = <q_dst, k_row> + (q_dst . bk_head)
     float p = qb;
+    if (kLowReg) {
+#pragma unroll 1
+      for (int cq = 0; cq < 4; ++cq) {               // 16-column pieces
+        tmem_ld16(ta + cb + cq * 16, v);
+        float qq[16];
 #pragma unroll
-    for (int cq = 0; cq < 2; ++cq) {
-      tmem_ld32(ta + cb + cq * 32, v);
-      tmem_wait_ld();
+        for (int j = 0; j < 16; j += 2) {
+          const float2 q2 = cq * 16 + j < dh ? __ldg(reinterpret_cast<const float2*>(
+                                                   qrow + cb + cq * 16 + j))
+                                             : make_float2(0.f, 0.f);
+          qq[j] = q2.x;
+          qq[j + 1] = q2.y;
+        }
+        tmem_wait_ld();
 #pragma unroll
-      for (int j = 0; j < 32; ++j)
-        if (cq * 32 + j < dh) p = fmaf(qv[cq * 32 + j], v[j], p);
+        for (int j = 0; j < 16; ++j)
+          if (cq * 16 + j < dh) p = fmaf(qq[j], v[j], p);
+      }
+    } else {
+#pragma unroll
+      for (int cq = 0; cq < 2; ++cq) {
+        tmem_ld32(ta + cb + cq * 32, v);
+        tmem_wait_ld();
+#pragma unroll
+        for (int j = 0; j < 32; ++j)
+          if (cq * 32 + j < dh) p = fmaf(qv[cq * 32 + j], v[j], p);
+      }
     }
     float s = p * P.logit_scale;
     if (P.leaky_slope >= 0.f) s = s < 0.f ? s * P.leaky_slope : s;
@@ -2369,8 +2392,8 @@ __global__ void __launch_bounds__(kSThreads, 1)
       __syncwarp();
     }
   } else if (warp < kBEpi) {                         // ---------------- epilogue warps 0-7
-    bin_epilogue<kSDSlots, TDesc, kSPW>(a, B.dfull, B.dempty, B.tfull, B.tempty, bd, tmem,
-                                        s_pvf, s_bias);
+    bin_epilogue<kSDSlots, TDesc, kSPW, (kSThreads > 768)>(a, B.dfull, B.dempty, B.tfull,
+                                                           B.tempty, bd, tmem, s_pvf, s_bias);
   }
   ws_teardown(tmem, 2 * kCols, kTMma);
 }
