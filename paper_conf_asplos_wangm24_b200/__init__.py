@@ -6,6 +6,6 @@ this package is its ctypes binding (`tgl`) and the host-side TBlock chain
 no CPU fallback.
 """
 from . import tgl  # noqa: F401  (raises ImportError if libtgl.so is missing)
-from .block import TBlock, TGATPipeline, TSampler  # noqa: F401
+from .block import HostStream, TBlock, TGATPipeline, TSampler  # noqa: F401
 
-__all__ = ["tgl", "TBlock", "TGATPipeline", "TSampler"]
+__all__ = ["tgl", "TBlock", "TGATPipeline", "TSampler", "HostStream"]

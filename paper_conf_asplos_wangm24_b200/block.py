@@ -234,6 +234,47 @@ class TGATPipeline:
         return out_h
 
 
+class HostStream:
+    """Serving loop over a staging TGATPipeline: batch i's H2D, graph replay and D2H are
+    enqueued without waiting for batch i-1's result to reach the host.  The root
+    embeddings go through a 2-deep device ring (a D2D copy at the end of the step) and are
+    read back on a side copy stream, so the D2H of batch i overlaps the compute of batch
+    i+1.  Every batch still pays its own H2D (its edges) and D2H (its embeddings)."""
+
+    def __init__(self, pipe: "TGATPipeline", n_out: int, d_out: int):
+        assert pipe.staging and pipe.graph_exec is not None
+        self.p = pipe
+        self.n_out = n_out
+        self.ring = [torch.empty(n_out, d_out, dtype=torch.float32, device=pipe.dev)
+                     for _ in range(2)]
+        self.copy_stream = torch.cuda.Stream()
+        self.d2h_done = [None, None]
+        self.i = 0
+
+    def submit(self, src_h, dst_h, t_h, neg_h, out_h) -> torch.cuda.Event:
+        """Enqueue one batch; returns the event after which out_h holds its embeddings."""
+        p, slot = self.p, self.i % 2
+        self.i += 1
+        cs = torch.cuda.current_stream()
+        n = src_h.shape[0]
+        assert n == p.batch, "staging pipeline is captured for a full batch"
+        for k_, h in (("src", src_h), ("dst", dst_h), ("t", t_h), ("neg", neg_h)):
+            p.stage[k_][:n].copy_(h, non_blocking=True)
+        p.graph_exec.replay()
+        if self.d2h_done[slot] is not None:     # ring slot still being read back
+            cs.wait_event(self.d2h_done[slot])
+        self.ring[slot].copy_(p.graph_out[:self.n_out], non_blocking=True)
+        ready = torch.cuda.Event()
+        ready.record(cs)
+        with torch.cuda.stream(self.copy_stream):
+            self.copy_stream.wait_event(ready)
+            out_h.copy_(self.ring[slot], non_blocking=True)
+            done = torch.cuda.Event()
+            done.record(self.copy_stream)
+        self.d2h_done[slot] = done
+        return done
+
+
 def C_TCSR(t: tgl.TemporalCSR):
     return tgl.C.byref(t.struct)
 

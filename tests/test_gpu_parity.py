@@ -372,3 +372,34 @@ def test_pipeline_lastfm_sampled_roots(T):
     exp = oracle.embed_recursive(tc, g.nfeat, g.efeat, params, cfg.k, opipe.STRATEGY[cfg.strategy],
                                  cfg.seeds["sampler"], qn[pick], qt[pick])
     assert np.abs(emb[pick] - exp).max() <= 1e-3
+
+
+def test_host_stream_matches_graph(T):
+    """The pipelined public host API (HostStream: H2D, replay, D2D ring, D2H on a copy
+    stream) returns, batch by batch, exactly the captured graph's embeddings."""
+    from paper_conf_asplos_wangm24_b200 import HostStream, TGATPipeline, TSampler
+    cfg, g, neg, params = _world("REDDIT", n_edges=60000)
+    ref = _gpu_pipeline(T, cfg, g, neg, params)
+    ref.capture()
+    dev = ref.g
+    ph = TGATPipeline(dev, ref.tcsr, params, cfg.batch,
+                      TSampler(cfg.k, cfg.strategy, cfg.seeds["sampler"]), cfg.dedup,
+                      cfg.precompute, cfg.window, "fp32", staging=True)
+    ph.capture()
+    n0 = 3 * cfg.batch
+    hs = HostStream(ph, n0, cfg.d_model)
+    outs = [torch.empty(n0, cfg.d_model).pin_memory() for _ in range(2)]
+    batches = [60, 61, 62, 63, 64]
+    evs, got = [], []
+    for i, b in enumerate(batches):
+        hb = [torch.from_numpy(np.ascontiguousarray(x)).pin_memory()
+              for x in synth.batch_roots_inputs(g, neg, b)]
+        evs.append(hs.submit(*hb, outs[i % 2]))
+        if i >= 1:
+            evs[i - 1].synchronize()
+            got.append(outs[(i - 1) % 2].numpy().copy())
+    evs[-1].synchronize()
+    got.append(outs[(len(batches) - 1) % 2].numpy().copy())
+    for b, e in zip(batches, got):
+        exp = np_(ref.run_graph(b * cfg.batch))[:n0]
+        assert np.array_equal(e, exp), b
