@@ -113,7 +113,7 @@ def test_sample_device_count_and_empty(T):
 
 
 # ------------------------------------------------------------------ S3
-@pytest.mark.parametrize("n", [0, 1, 1800, 2047, 2048, 2049, 4096, 4097, 20000, 200001])
+@pytest.mark.parametrize("n", [0, 1, 1800, 2047, 2048, 2049, 4096, 4097, 8193, 20000, 32768, 32769, 200001])
 def test_dedup_bit_exact(T, n):
     rng = np.random.default_rng(n + 1)
     node = rng.integers(0, max(2, n // 8), n).astype(np.int32)
