@@ -256,6 +256,54 @@ tgl_status tgl_gather_rows(int64_t n_max, const int64_t* n_dev, const int32_t* i
                            const float* table, int64_t ld_table, int32_t d, float* out,
                            int64_t ld_out, void* stream);
 
+/* ---------------------------------------------------------------------------
+ * N1  Embedding memoisation: the cache() operator ("previously computed
+ * embeddings could be reused and cached"; "cache() will filter destination
+ * node-time pairs to ones that have not been cached and register a hook to
+ * combine computed outputs with cached results"; TGOpt cache_lookup /
+ * cache_store, Listing 1 lines 10-23).  One table per layer (the
+ * listing keys the store by layer); the caller owns it.
+ *
+ * Table: `capacity` slots (a power of two, <= 2^30), keys u64 [capacity] that
+ * the caller zeroes once (0 = empty), vals fp32 [capacity, d] row-major.  A pair
+ * (v, t) is keyed like dedup (node << 32 | order-preserving bits of t, -0 == +0,
+ * R8); a NaN t never hits and is never stored (NaN != NaN).  Linear probing over
+ * at most TGL_CACHE_PROBES slots: a pair that finds no free slot is not stored,
+ * so a full table only costs recomputation, never a wrong row (reading R22).
+ * ------------------------------------------------------------------------- */
+#define TGL_CACHE_PROBES 64
+typedef struct {
+  int64_t capacity;
+  int32_t d;
+  unsigned long long* keys;   /* device [capacity] */
+  float* vals;                /* device [capacity, d] */
+} tgl_cache;
+
+/* Lookup + filter (the pre-processing half of cache()).  For i < n = *n_dev
+ * (NULL -> n_max): slot[i] = the table slot holding (node[i], t[i]) if cached,
+ * else -(1 + j) where j is the rank of i among the misses in input order.  The
+ * misses are compacted, stable: miss_node[j], miss_t[j]; *num_miss_dev = count.
+ * Capacities n_max.  Workspace: scan state (CUB-style protocol). */
+tgl_status tgl_cache_lookup(const tgl_cache* c, int64_t n_max, const int64_t* n_dev,
+                            const int32_t* node, const float* t, int32_t* slot,
+                            int32_t* miss_node, float* miss_t, int64_t* num_miss_dev,
+                            void* ws, size_t* ws_bytes, void* stream);
+
+/* Store (Listing 1 cache_store): for i < n = *n_dev (NULL -> n_max) insert
+ * (node[i], t[i]) -> emb[i][0:d) (row pitch ld_emb floats).  A pair already
+ * present keeps its slot and gets the row rewritten; duplicate pairs inside one
+ * call must carry equal rows (true for dedup'ed or deterministic outputs). */
+tgl_status tgl_cache_store(const tgl_cache* c, int64_t n_max, const int64_t* n_dev,
+                           const int32_t* node, const float* t, const float* emb,
+                           int64_t ld_emb, void* stream);
+
+/* Combine hook (the post-processing half of cache()): for i < n = *n_dev
+ * (NULL -> n_max): out[i] = slot[i] >= 0 ? vals[slot[i]] : computed[-(1 + slot[i])]
+ * (rows of d floats; pitches ld_computed, ld_out). */
+tgl_status tgl_cache_combine(const tgl_cache* c, int64_t n_max, const int64_t* n_dev,
+                             const int32_t* slot, const float* computed, int64_t ld_computed,
+                             float* out, int64_t ld_out, void* stream);
+
 #ifdef __cplusplus
 }
 #endif

@@ -15,7 +15,7 @@ ROOT = os.path.dirname(PKG)
 LIB = os.path.join(PKG, "libtgl.so")
 OBJ = os.path.join(ROOT, "build", "obj")
 
-SOURCES = ["api.cu", "tcsr.cu", "sample.cu", "dedup.cu", "time_encode.cu", "attn.cu",
+SOURCES = ["api.cu", "tcsr.cu", "sample.cu", "dedup.cu", "time_encode.cu", "attn.cu", "cache.cu",
            "attn_tc.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

@@ -26,7 +26,7 @@ SYMBOLS = ["tgl_version", "tgl_status_string", "tgl_last_error", "tgl_build_tcsr
            "tgl_batch_roots", "tgl_dedup", "tgl_sample", "tgl_next_block",
            "tgl_time_precompute", "tgl_time_encode", "tgl_tblock_attn", "tgl_gather_rows",
            "tgl_attn_packed_bytes", "tgl_attn_pack", "tgl_kv_timing", "tgl_kv_timing_ms",
-           "tgl_kv_timing_kernel"]
+           "tgl_kv_timing_kernel", "tgl_cache_lookup", "tgl_cache_store", "tgl_cache_combine"]
 
 
 class TGLError(RuntimeError):
@@ -56,6 +56,9 @@ def _load():
                             vp, i64, i32, vp, vp, sz, vp],
         "tgl_gather_rows": [i64, vp, vp, vp, i64, i32, vp, i64, vp],
         "tgl_attn_pack": [vp, vp, C.c_size_t, vp],
+        "tgl_cache_lookup": [vp, i64, vp, vp, vp, vp, vp, vp, vp, vp, sz, vp],
+        "tgl_cache_store": [vp, i64, vp, vp, vp, vp, i64, vp],
+        "tgl_cache_combine": [vp, i64, vp, vp, vp, i64, vp, i64, vp],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -322,4 +325,59 @@ def gather_rows(idx, table, n_dev=None, n_max=None, out=None, stream=None):
         out = torch.empty(max(n_max, 1), d, dtype=table.dtype, device=table.device)
     _check(_lib.tgl_gather_rows(n_max, _p(n_dev), _p(idx), _p(table), table.stride(0), d,
                                 _p(out), out.stride(0), _s(stream)), "tgl_gather_rows")
+    return out
+
+
+# --------------------------------------------------------------------------- N1 cache()
+class CacheC(C.Structure):
+    _fields_ = [("capacity", C.c_int64), ("d", C.c_int32), ("keys", C.c_void_p),
+                ("vals", C.c_void_p)]
+
+
+class EmbeddingCache:
+    """One layer's memo table (P:297 cache(); include/tgl.h tgl_cache): device keys
+    [capacity] u64 (zeroed here, 0 = empty) and rows [capacity, d] fp32."""
+
+    def __init__(self, capacity: int, d: int, device=None):
+        dev = device or torch.device("cuda")
+        self.keys = torch.zeros(capacity, dtype=torch.int64, device=dev)
+        self.vals = torch.zeros(capacity, d, dtype=torch.float32, device=dev)
+        self.struct = CacheC(capacity, d, self.keys.data_ptr(), self.vals.data_ptr())
+        self.capacity, self.d = capacity, d
+
+    def clear(self):
+        self.keys.zero_()
+
+
+def cache_lookup(cache: EmbeddingCache, node, t, n_dev=None, n_max=None, out=None,
+                 ws: Workspace | None = None, stream=None):
+    """Returns (slot[n_max], miss_node, miss_t, num_miss_dev)."""
+    n_max = node.numel() if n_max is None else n_max
+    dev = node.device
+    if out is None:
+        out = (torch.empty(max(n_max, 1), dtype=torch.int32, device=dev),
+               torch.empty(max(n_max, 1), dtype=torch.int32, device=dev),
+               torch.empty(max(n_max, 1), dtype=torch.float32, device=dev),
+               torch.zeros(1, dtype=torch.int64, device=dev))
+    slot, mn, mt, nm = out
+    _ws_call(_lib.tgl_cache_lookup, [C.byref(cache.struct), n_max, _p(n_dev), _p(node), _p(t),
+                                     _p(slot), _p(mn), _p(mt), _p(nm)], ws, _s(stream),
+             "tgl_cache_lookup")
+    return slot, mn, mt, nm
+
+
+def cache_store(cache: EmbeddingCache, node, t, emb, n_dev=None, n_max=None, stream=None):
+    n_max = node.numel() if n_max is None else n_max
+    _check(_lib.tgl_cache_store(C.byref(cache.struct), n_max, _p(n_dev), _p(node), _p(t),
+                                _p(emb), emb.stride(0), _s(stream)), "tgl_cache_store")
+
+
+def cache_combine(cache: EmbeddingCache, slot, computed, n_dev=None, n_max=None, out=None,
+                  stream=None):
+    n_max = slot.numel() if n_max is None else n_max
+    if out is None:
+        out = torch.empty(max(n_max, 1), cache.d, dtype=torch.float32, device=slot.device)
+    _check(_lib.tgl_cache_combine(C.byref(cache.struct), n_max, _p(n_dev), _p(slot),
+                                  _p(computed), computed.stride(0), _p(out), out.stride(0),
+                                  _s(stream)), "tgl_cache_combine")
     return out
