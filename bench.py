@@ -39,6 +39,8 @@ def parse():
     ap.add_argument("--precision", default="fp32", choices=["fp32", "bf16", "fp32_simt"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--cache", type=int, default=0,
+                    help="cache() table slots per layer (0 = off, the BASELINE configs)")
     return ap.parse_args()
 
 
@@ -365,7 +367,7 @@ def run_ours(args):
     tcsr_ms = ev0.elapsed_time(ev1)
     sampler = TSampler(cfg.k, cfg.strategy, cfg.seeds["sampler"])
     pipe = TGATPipeline(dev, tc, params, cfg.batch, sampler, cfg.dedup, cfg.precompute,
-                        cfg.window, args.precision)
+                        cfg.window, args.precision, cache_capacity=args.cache)
     pipe.capture()
     n0 = 3 * cfg.batch
     gathered = torch.empty(world * n0, cfg.d_model, device="cuda") if world > 1 else None
@@ -497,7 +499,8 @@ def run_ours(args):
     e2e = None
     if world >= 1:
         pipe_h = TGATPipeline(dev, tc, params, cfg.batch, sampler, cfg.dedup, cfg.precompute,
-                              cfg.window, args.precision, staging=True)
+                              cfg.window, args.precision, staging=True,
+                              cache_capacity=args.cache)
         pipe_h.capture()
         from paper_conf_asplos_wangm24_b200 import HostStream
         outs = [torch.empty(n0, cfg.d_model, dtype=torch.float32).pin_memory() for _ in range(2)]
@@ -557,6 +560,7 @@ def run_ours(args):
                            "roots_per_step_all_ranks": world * n0, "layers": cfg.n_layers,
                            "k": cfg.k, "strategy": cfg.strategy, "dedup": cfg.dedup,
                            "precompute": cfg.precompute, "precision": args.precision,
+                           "cache_slots_per_layer": args.cache,
                            "parallelism": f"root-sharded dp{world}" if world > 1 else "single",
                            "l2": "flushed (256 MiB write) between timed steps",
                            "timing": "CUDA events per step on the launch stream; max over ranks"},

@@ -54,7 +54,8 @@ class TGATPipeline:
 
     def __init__(self, graph: dict, tcsr: tgl.TemporalCSR, params: list, batch: int,
                  sampler: TSampler, use_dedup: bool, precompute: bool, window: int = 65536,
-                 precision: str = "fp32", staging: bool = False, device=None):
+                 precision: str = "fp32", staging: bool = False, device=None,
+                 cache_capacity: int = 0):
         self.dev = device or torch.device("cuda")
         self.g = graph
         self.tcsr = tcsr
@@ -95,6 +96,23 @@ class TGATPipeline:
         dedup_launches = [(1 if b.n_max <= 4096 else 3) if use_dedup else 0 for b in self.blocks]
         per_block = [(1 if l > 0 else 0) + dedup_launches[l] + 1 + 3 for l in range(self.L)]
         self.launches_per_forward = 1 + sum(per_block) + (1 if use_dedup else 0)
+        # cache() (TGOpt per-layer store, Listing 1 L23; inference): every
+        # block's dst pairs after dedup are looked up in that layer's table; only the
+        # misses are sampled and computed, then stored, and the combine hook rebuilds the
+        # block's rows in dedup order (b.comb) for the block above / the roots.
+        self.cache_on = bool(cache_capacity)
+        if self.cache_on:
+            assert use_dedup, "cache() sits behind each block's dedup"
+            for b in self.blocks:
+                d = self.attn[b.layer].d_out
+                c = {"table": tgl.EmbeddingCache(cache_capacity, d, self.dev),
+                     "node": z(b.n_max, i32), "t": z(b.n_max, f32), "u": z(1, i64),
+                     "slot": z(b.n_max, i32), "comb": z(b.n_max * d, f32).view(-1, d)}
+                nb = tgl.ws_bytes("tgl_cache_lookup", None, b.n_max, None, None, None, None,
+                                  None, None, None)
+                c["ws"] = torch.empty(max(nb, 256), dtype=torch.uint8, device=self.dev)
+                b.ws["cache"] = c
+            self.launches_per_forward += 3 * self.L
         self._alloc_workspaces()
         self.graph_exec = None
 
@@ -144,12 +162,22 @@ class TGATPipeline:
                 tgl.next_block(p.n_max, p.u_dev, p.uniq_node, p.uniq_t, p.n_max * k, p.seg_ptr,
                                p.nbr, p.ts, b.dst_node, b.dst_t, b.n_dev, stream=s)
                 mark(f"next_block{l}")
+            c = b.ws.get("cache")
             if self.use_dedup:  # S3
+                un, ut, ud = ((c["node"], c["t"], c["u"]) if c is not None
+                              else (b.uniq_node, b.uniq_t, b.u_dev))
                 _call_ws(tgl.lib().tgl_dedup,
                          [b.n_max, tgl._p(b.n_dev), tgl._p(b.dst_node), tgl._p(b.dst_t),
-                          tgl._p(b.uniq_node), tgl._p(b.uniq_t), tgl._p(b.u_dev),
+                          tgl._p(un), tgl._p(ut), tgl._p(ud),
                           tgl._p(b.inv)], b.ws["dedup"], s, "tgl_dedup")
                 mark(f"dedup{l}")
+            if c is not None:  # cache() filter: the misses become the block's dsts
+                _call_ws(tgl.lib().tgl_cache_lookup,
+                         [tgl.C.byref(c["table"].struct), b.n_max, tgl._p(c["u"]),
+                          tgl._p(c["node"]), tgl._p(c["t"]), tgl._p(c["slot"]),
+                          tgl._p(b.uniq_node), tgl._p(b.uniq_t), tgl._p(b.u_dev)],
+                         c["ws"], s, "tgl_cache_lookup")
+                mark(f"cache_lookup{l}")
             # S4 sample
             _call_ws(tgl.lib().tgl_sample,
                      [tgl.C.byref(self.tcsr.struct), b.n_max, tgl._p(b.u_dev),
@@ -166,7 +194,7 @@ class TGATPipeline:
                 hdst, hdst_idx, hsrc, hsrc_idx, off = g["nfeat"], b.uniq_node, g["nfeat"], b.nbr, None
             else:
                 nx = self.blocks[l + 1]
-                hdst = hsrc = nx.out
+                hdst = hsrc = nx.ws["cache"]["comb"] if self.cache_on else nx.out
                 off = b.u_dev        # S14: rows [U_l + e] of the next block hold the sources
                 if self.use_dedup:
                     hdst_idx = hsrc_idx = nx.inv
@@ -189,8 +217,16 @@ class TGATPipeline:
                 ev[1].record(s if s is not None else torch.cuda.current_stream())
                 record[l] = ev
             mark(f"attn{l}")
+            if self.cache_on:  # store the computed misses, then the combine hook
+                c = b.ws["cache"]
+                tgl.cache_store(c["table"], b.uniq_node, b.uniq_t, b.out, n_dev=b.u_dev,
+                                n_max=b.n_max, stream=s)
+                tgl.cache_combine(c["table"], c["slot"], b.out, n_dev=c["u"], n_max=b.n_max,
+                                  out=c["comb"], stream=s)
+                mark(f"cache_merge{l}")
+        head = b0.ws["cache"]["comb"] if self.cache_on else b0.out
         if self.use_dedup:  # S14 at the roots
-            tgl.gather_rows(b0.inv, b0.out, n_dev=b0.n_dev, n_max=b0.n_max, out=self.emb, stream=s)
+            tgl.gather_rows(b0.inv, head, n_dev=b0.n_dev, n_max=b0.n_max, out=self.emb, stream=s)
             mark("gather")
             return self.emb
         return b0.out[:3 * self.batch]

@@ -98,3 +98,46 @@ def test_cache_device_count(T):
         comp_dev = cu(comp) if len(miss) else torch.zeros(1, 100, device="cuda")
         T.cache_store(cache, mn, mt, comp_dev, n_dev=nm, n_max=3000)
         memo.store(node[:n][miss], t[:n][miss], comp)
+
+
+def test_pipeline_root_cache_vs_oracle(T):
+    """TGATPipeline(cache_capacity>0), one table per layer: memoised embeddings over
+    repeated and consecutive batches match the oracle (no cache) within the fp32
+    tolerance; a repeated batch computes nothing at the head block; inner-layer pairs
+    hit across consecutive batches; graph replay == eager."""
+    from oracle import pipeline as opipe
+    import oracle
+    from paper_conf_asplos_wangm24_b200 import TGATPipeline, TSampler
+    from tests.test_gpu_parity import _world
+    cfg, g, neg, params = _world("REDDIT", n_edges=60000)
+    dev = {"src": cu(g.src), "dst": cu(g.dst), "t": cu(g.t), "neg": cu(neg),
+           "nfeat": cu(g.nfeat), "efeat": cu(g.efeat)}
+    tc = T.build_tcsr(cfg.n_nodes, dev["src"], dev["dst"], dev["t"], True, True)
+    pipe = TGATPipeline(dev, tc, params, cfg.batch,
+                        TSampler(cfg.k, cfg.strategy, cfg.seeds["sampler"]), True,
+                        cfg.precompute, cfg.window, "fp32", cache_capacity=1 << 16)
+    otc = oracle.build_tcsr(cfg.n_nodes, g.src, g.dst, g.t, True)
+    n0 = 3 * cfg.batch
+    seen, inner_hits = {}, 0
+    for b in (70, 70, 71, 70, 72):
+        pipe.start_dev.fill_(b * cfg.batch)
+        emb = pipe.forward().cpu().numpy()[:n0].copy()
+        misses = int(pipe.blocks[0].u_dev.item())
+        b1 = pipe.blocks[1]
+        inner_hits += int(b1.ws["cache"]["u"].item()) - int(b1.u_dev.item())
+        if b in seen:
+            assert misses == 0
+            assert np.array_equal(emb, seen[b])
+        exp, _ = opipe.run_batch(otc, g.nfeat, g.efeat, params, cfg.k, cfg.strategy, True,
+                                 cfg.seeds["sampler"], *synth_roots(g, neg, b))
+        assert np.abs(emb - exp).max() <= 1e-3
+        seen[b] = emb
+    assert inner_hits > 0                # layer-1 pairs recur across consecutive batches
+    pipe.capture()                       # replays hit the now-warm cache
+    e_g = pipe.run_graph(72 * cfg.batch).cpu().numpy()[:n0]
+    assert np.array_equal(e_g, seen[72])
+
+
+def synth_roots(g, neg, b):
+    import synth
+    return synth.batch_roots_inputs(g, neg, b)
