@@ -304,6 +304,18 @@ tgl_status tgl_cache_combine(const tgl_cache* c, int64_t n_max, const int64_t* n
                              const int32_t* slot, const float* computed, int64_t ld_computed,
                              float* out, int64_t ld_out, void* stream);
 
+/* Store + combine in one pass (what the TBlock chain launches).  The pairs are
+ * indexed in "dedup space": node[i], t[i], slot[i] as written by tgl_cache_lookup.
+ * For j < n = *n_dev (NULL -> n_max), i = idx ? idx[j] : j:
+ * out[j] = slot[i] >= 0 ? vals[slot[i]] : computed[-(1 + slot[i])], and a miss's
+ * row is inserted under (node[i], t[i]) exactly as tgl_cache_store would.  idx lets
+ * the dedup inverse hook (S14) read the merged rows directly: several j
+ * may share one i; they then store the same row under the same key. */
+tgl_status tgl_cache_merge(const tgl_cache* c, int64_t n_max, const int64_t* n_dev,
+                           const int32_t* idx, const int32_t* node, const float* t,
+                           const int32_t* slot, const float* computed, int64_t ld_computed,
+                           float* out, int64_t ld_out, void* stream);
+
 #ifdef __cplusplus
 }
 #endif

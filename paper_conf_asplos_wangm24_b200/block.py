@@ -112,7 +112,7 @@ class TGATPipeline:
                                   None, None, None)
                 c["ws"] = torch.empty(max(nb, 256), dtype=torch.uint8, device=self.dev)
                 b.ws["cache"] = c
-            self.launches_per_forward += 3 * self.L
+            self.launches_per_forward += 2 * self.L - 1   # lookups + merges - gather
         self._alloc_workspaces()
         self.graph_exec = None
 
@@ -217,14 +217,18 @@ class TGATPipeline:
                 ev[1].record(s if s is not None else torch.cuda.current_stream())
                 record[l] = ev
             mark(f"attn{l}")
-            if self.cache_on:  # store the computed misses, then the combine hook
+            if self.cache_on and l > 0:  # store the misses + combine hook, one launch
                 c = b.ws["cache"]
-                tgl.cache_store(c["table"], b.uniq_node, b.uniq_t, b.out, n_dev=b.u_dev,
-                                n_max=b.n_max, stream=s)
-                tgl.cache_combine(c["table"], c["slot"], b.out, n_dev=c["u"], n_max=b.n_max,
-                                  out=c["comb"], stream=s)
+                tgl.cache_merge(c["table"], c["node"], c["t"], c["slot"], b.out,
+                                n_dev=c["u"], n_max=b.n_max, out=c["comb"], stream=s)
                 mark(f"cache_merge{l}")
-        head = b0.ws["cache"]["comb"] if self.cache_on else b0.out
+        if self.cache_on:  # head: store + combine + S14 inverse in one launch
+            c = b0.ws["cache"]
+            tgl.cache_merge(c["table"], c["node"], c["t"], c["slot"], b0.out, idx=b0.inv,
+                            n_dev=b0.n_dev, n_max=b0.n_max, out=self.emb, stream=s)
+            mark("cache_merge0")
+            return self.emb
+        head = b0.out
         if self.use_dedup:  # S14 at the roots
             tgl.gather_rows(b0.inv, head, n_dev=b0.n_dev, n_max=b0.n_max, out=self.emb, stream=s)
             mark("gather")

@@ -149,6 +149,50 @@ __global__ void cache_combine_kernel(const float* __restrict__ vals, int d, int6
   }
 }
 
+__global__ void cache_merge_kernel(unsigned long long* keys, float* __restrict__ vals,
+                                   int log2cap, int d, int64_t n_max, const int64_t* n_dev,
+                                   const int32_t* __restrict__ idx,
+                                   const int32_t* __restrict__ node, const float* __restrict__ t,
+                                   const int32_t* __restrict__ slot,
+                                   const float* __restrict__ computed, int64_t ld_computed,
+                                   float* __restrict__ out, int64_t ld_out) {
+  pdl_wait();
+  pdl_trigger();
+  const int64_t n = dev_count(n_dev, n_max);
+  const int lane = threadIdx.x & 31;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  const uint64_t mask = (1ull << log2cap) - 1ull;
+  for (int64_t j = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; j < n; j += warps) {
+    const int64_t i = idx ? (int64_t)idx[j] : j;
+    const int32_t s = slot[i];
+    const float* src = s >= 0 ? vals + (int64_t)s * d : computed + (int64_t)(-1 - s) * ld_computed;
+    float* dst = out + j * ld_out;
+    int64_t h = -1;
+    if (s < 0 && lane == 0) {                    // a miss: claim its slot (as cache_store)
+      const float ti = t[i];
+      if (ti == ti) {
+        const unsigned long long k = cache_key(node[i], ti);
+        uint64_t p = cache_hash(k, log2cap);
+        for (int q = 0; q < TGL_CACHE_PROBES; ++q) {
+          const unsigned long long prev = atomicCAS(keys + p, 0ull, k);
+          if (prev == 0ull || prev == k) {
+            h = (int64_t)p;
+            break;
+          }
+          p = (p + 1) & mask;
+        }
+      }
+    }
+    h = __shfl_sync(0xffffffffu, h, 0);
+    float* row = h >= 0 ? vals + h * (int64_t)d : nullptr;
+    for (int c = lane; c < d; c += 32) {
+      const float v = src[c];
+      dst[c] = v;
+      if (row) row[c] = v;
+    }
+  }
+}
+
 static tgl_status cache_check(const tgl_cache* c, int* log2cap) {
   TGL_REQUIRE(c != nullptr && c->keys != nullptr && c->vals != nullptr, "null cache");
   TGL_REQUIRE(c->capacity > 0 && (c->capacity & (c->capacity - 1)) == 0 &&
@@ -224,4 +268,20 @@ extern "C" tgl_status tgl_cache_combine(const tgl_cache* c, int64_t n_max, const
              (const float*)c->vals, (int)c->d, n_max, n_dev, slot, computed, ld_computed, out,
              ld_out);
   return launch_check("cache_combine");
+}
+
+extern "C" tgl_status tgl_cache_merge(const tgl_cache* c, int64_t n_max, const int64_t* n_dev,
+                                      const int32_t* idx, const int32_t* node, const float* t,
+                                      const int32_t* slot, const float* computed,
+                                      int64_t ld_computed, float* out, int64_t ld_out,
+                                      void* stream) {
+  TGL_REQUIRE(n_max >= 0, "negative n_max");
+  int l2 = 0;
+  TGL_TRY(cache_check(c, &l2));
+  TGL_REQUIRE(ld_out >= c->d && ld_computed >= c->d, "row pitch < d");
+  TGL_REQUIRE(n_max == 0 || (node && t && slot && computed && out), "null pointer");
+  launch_pdl(cache_merge_kernel, dim3(warp_grid(n_max)), dim3(256), 0, as_stream(stream),
+             c->keys, c->vals, l2, (int)c->d, n_max, n_dev, idx, node, t, slot, computed,
+             ld_computed, out, ld_out);
+  return launch_check("cache_merge");
 }

@@ -26,7 +26,8 @@ SYMBOLS = ["tgl_version", "tgl_status_string", "tgl_last_error", "tgl_build_tcsr
            "tgl_batch_roots", "tgl_dedup", "tgl_sample", "tgl_next_block",
            "tgl_time_precompute", "tgl_time_encode", "tgl_tblock_attn", "tgl_gather_rows",
            "tgl_attn_packed_bytes", "tgl_attn_pack", "tgl_kv_timing", "tgl_kv_timing_ms",
-           "tgl_kv_timing_kernel", "tgl_cache_lookup", "tgl_cache_store", "tgl_cache_combine"]
+           "tgl_kv_timing_kernel", "tgl_cache_lookup", "tgl_cache_store", "tgl_cache_combine",
+           "tgl_cache_merge"]
 
 
 class TGLError(RuntimeError):
@@ -59,6 +60,7 @@ def _load():
         "tgl_cache_lookup": [vp, i64, vp, vp, vp, vp, vp, vp, vp, vp, sz, vp],
         "tgl_cache_store": [vp, i64, vp, vp, vp, vp, i64, vp],
         "tgl_cache_combine": [vp, i64, vp, vp, vp, i64, vp, i64, vp],
+        "tgl_cache_merge": [vp, i64, vp, vp, vp, vp, vp, vp, i64, vp, i64, vp],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -380,4 +382,16 @@ def cache_combine(cache: EmbeddingCache, slot, computed, n_dev=None, n_max=None,
     _check(_lib.tgl_cache_combine(C.byref(cache.struct), n_max, _p(n_dev), _p(slot),
                                   _p(computed), computed.stride(0), _p(out), out.stride(0),
                                   _s(stream)), "tgl_cache_combine")
+    return out
+
+
+def cache_merge(cache: EmbeddingCache, node, t, slot, computed, idx=None, n_dev=None,
+                n_max=None, out=None, stream=None):
+    """Store + combine in one launch; out[j] = merged row idx[j] (identity if None)."""
+    n_max = (slot.numel() if idx is None else idx.numel()) if n_max is None else n_max
+    if out is None:
+        out = torch.empty(max(n_max, 1), cache.d, dtype=torch.float32, device=slot.device)
+    _check(_lib.tgl_cache_merge(C.byref(cache.struct), n_max, _p(n_dev), _p(idx), _p(node),
+                                _p(t), _p(slot), _p(computed), computed.stride(0), _p(out),
+                                out.stride(0), _s(stream)), "tgl_cache_merge")
     return out

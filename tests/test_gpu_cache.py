@@ -141,3 +141,28 @@ def test_pipeline_root_cache_vs_oracle(T):
 def synth_roots(g, neg, b):
     import synth
     return synth.batch_roots_inputs(g, neg, b)
+
+
+def test_cache_merge_equals_store_then_combine(T):
+    """tgl_cache_merge (the launch the chain uses) == tgl_cache_store + tgl_cache_combine,
+    read through an index (the S14 inverse) with repeated entries."""
+    rng = np.random.default_rng(7)
+    d = 100
+    cache = T.EmbeddingCache(1 << 14, d)
+    memo = Memo()
+    for n in (3000, 2500, 4000):
+        node = np.unique(rng.integers(0, 600, n)).astype(np.int32)   # dedup space: unique pairs
+        t = np.full(len(node), 5.0, np.float32)
+        slot, mn, mt, nm = T.cache_lookup(cache, cu(node), cu(t))
+        hit, miss = memo.lookup(node, t)
+        assert np.array_equal(slot.cpu().numpy()[:len(node)] >= 0, hit)
+        comp = rows_of(node[miss], t[miss], d)
+        comp_dev = cu(comp) if len(miss) else torch.zeros(1, d, device="cuda")
+        idx = rng.integers(0, len(node), 2 * len(node)).astype(np.int32)
+        out = T.cache_merge(cache, cu(node), cu(t), slot, comp_dev, idx=cu(idx)).cpu().numpy()
+        memo.store(node[miss], t[miss], comp)
+        exp = memo.combine(node, t, hit, comp)[idx]
+        assert np.array_equal(bits(out[:len(idx)]), bits(exp))
+    # every pair merged so far is now a hit
+    slot, _, _, nm = T.cache_lookup(cache, cu(node), cu(t))
+    assert int(nm.item()) == 0
