@@ -86,3 +86,7 @@ def test_cache_abi_validation():
     ok = tgl.CacheC(1024, 100, 256, 256)
     assert lib.tgl_cache_combine(C.byref(ok), 10, None, None, None, 50, None, 100, None) == -1
     assert lib.tgl_cache_store(None, 10, None, None, None, None, 100, None) == -1
+    assert lib.tgl_cache_merge(C.byref(bad), 10, None, None, None, None, None, None, 100, None,
+                               100, None) == -1
+    assert lib.tgl_cache_merge(C.byref(ok), 10, None, None, None, None, None, None, 100, None,
+                               100, None) == -1          # null arrays
