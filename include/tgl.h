@@ -310,7 +310,9 @@ tgl_status tgl_cache_combine(const tgl_cache* c, int64_t n_max, const int64_t* n
  * out[j] = slot[i] >= 0 ? vals[slot[i]] : computed[-(1 + slot[i])], and a miss's
  * row is inserted under (node[i], t[i]) exactly as tgl_cache_store would.  idx lets
  * the dedup inverse hook (S14) read the merged rows directly: several j
- * may share one i; they then store the same row under the same key. */
+ * may share one i; they then store the same row under the same key.  Only the
+ * misses some j reads are stored: idx must be onto [0, U) (the dedup inverse is)
+ * for the table to receive every computed row. */
 tgl_status tgl_cache_merge(const tgl_cache* c, int64_t n_max, const int64_t* n_dev,
                            const int32_t* idx, const int32_t* node, const float* t,
                            const int32_t* slot, const float* computed, int64_t ld_computed,

@@ -158,7 +158,9 @@ def test_cache_merge_equals_store_then_combine(T):
         assert np.array_equal(slot.cpu().numpy()[:len(node)] >= 0, hit)
         comp = rows_of(node[miss], t[miss], d)
         comp_dev = cu(comp) if len(miss) else torch.zeros(1, d, device="cuda")
-        idx = rng.integers(0, len(node), 2 * len(node)).astype(np.int32)
+        # surjective like the dedup inverse: every pair is read (and so stored) at least once
+        idx = np.concatenate([rng.permutation(len(node)),
+                              rng.integers(0, len(node), len(node))]).astype(np.int32)
         out = T.cache_merge(cache, cu(node), cu(t), slot, comp_dev, idx=cu(idx)).cpu().numpy()
         memo.store(node[miss], t[miss], comp)
         exp = memo.combine(node, t, hit, comp)[idx]
