@@ -30,9 +30,12 @@ def main(path):
             cur = []
         if cur is not None and "Fill" not in name:
             cur.append((name, v))
-    if cur and any("gather_rows" in n for n, _ in cur):
+    # a full step ends with the S14 gather (or, with cache(), the root cache_merge); torch
+    # kernels (the bench's per-step counters, outside the timed region) are left out
+    done = lambda st: any("gather_rows" in n or "cache_merge" in n for n, _ in st)
+    if cur and done(cur):
         steps.append(cur)
-    steps = [s for s in steps if any("gather_rows" in n for n, _ in s)]
+    steps = [[(n, v) for n, v in s if "at::" not in n] for s in steps if done(s)]
     tot = [sum(v for _, v in s) for s in steps]
     med = sorted(range(len(steps)), key=lambda i: tot[i])[len(steps) // 2]
     s = steps[med]
