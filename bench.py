@@ -358,6 +358,9 @@ def run_ours(args):
         cfg, g, neg, params = load_world(args.config)
         dev = {"src": cu(g.src), "dst": cu(g.dst), "t": cu(g.t), "neg": cu(neg),
                "nfeat": cu(g.nfeat), "efeat": cu(g.efeat)}
+    if args.cache and not cfg.dedup:                 # cache() sits behind each block's dedup
+        from dataclasses import replace
+        cfg = replace(cfg, dedup=True)               # (the paper pairs them at inference)
     torch.cuda.synchronize()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     ev0.record()
