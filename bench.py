@@ -39,6 +39,8 @@ def parse():
     ap.add_argument("--precision", default="fp32", choices=["fp32", "bf16", "fp32_simt"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--dedup", default="config", choices=["config", "on", "off"],
+                    help="override the config's dedup setting (ablation only)")
     ap.add_argument("--cache", type=int, default=0,
                     help="cache() table slots per layer (0 = off, the BASELINE configs)")
     return ap.parse_args()
@@ -358,9 +360,9 @@ def run_ours(args):
         cfg, g, neg, params = load_world(args.config)
         dev = {"src": cu(g.src), "dst": cu(g.dst), "t": cu(g.t), "neg": cu(neg),
                "nfeat": cu(g.nfeat), "efeat": cu(g.efeat)}
-    if args.cache and not cfg.dedup:                 # cache() sits behind each block's dedup
-        from dataclasses import replace
-        cfg = replace(cfg, dedup=True)               # (the paper pairs them at inference)
+    if args.dedup != "config" or (args.cache and not cfg.dedup):
+        from dataclasses import replace              # cache() sits behind each block's dedup
+        cfg = replace(cfg, dedup=args.dedup == "on" or bool(args.cache))   # (P:578 pairs them)
     torch.cuda.synchronize()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     ev0.record()
