@@ -168,3 +168,32 @@ def test_cache_merge_equals_store_then_combine(T):
     # every pair merged so far is now a hit
     slot, _, _, nm = T.cache_lookup(cache, cu(node), cu(t))
     assert int(nm.item()) == 0
+
+
+def test_pipeline_cache_full_reddit_vs_oracle(T):
+    """Full-size REDDIT in the bench's launch configuration (graph replay, consecutive
+    batches from 70 % of the stream, a warm per-layer cache) against the uncached
+    oracle: max abs <= 1e-3 on every root."""
+    from oracle import pipeline as opipe
+    import oracle
+    import synth
+    from paper_conf_asplos_wangm24_b200 import TGATPipeline, TSampler
+    from tests.test_gpu_parity import _world
+    cfg, g, neg, params = _world("REDDIT")
+    dev = {"src": cu(g.src), "dst": cu(g.dst), "t": cu(g.t), "neg": cu(neg),
+           "nfeat": cu(g.nfeat), "efeat": cu(g.efeat)}
+    tc = T.build_tcsr(cfg.n_nodes, dev["src"], dev["dst"], dev["t"], True, True)
+    pipe = TGATPipeline(dev, tc, params, cfg.batch,
+                        TSampler(cfg.k, cfg.strategy, cfg.seeds["sampler"]), True,
+                        cfg.precompute, cfg.window, "fp32", cache_capacity=1 << 20)
+    pipe.capture()
+    otc = oracle.build_tcsr(cfg.n_nodes, g.src, g.dst, g.t, True)
+    b0 = int(0.7 * cfg.n_batches)
+    n0 = 3 * cfg.batch
+    for b in range(b0, b0 + 6):
+        emb = pipe.run_graph(b * cfg.batch).cpu().numpy()[:n0]
+        if b < b0 + 4:
+            continue                       # warm the cache like the bench's warm-up
+        exp, _ = opipe.run_batch(otc, g.nfeat, g.efeat, params, cfg.k, cfg.strategy, True,
+                                 cfg.seeds["sampler"], *synth.batch_roots_inputs(g, neg, b))
+        assert np.abs(emb - exp).max() <= 1e-3
