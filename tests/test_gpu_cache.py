@@ -143,11 +143,11 @@ def synth_roots(g, neg, b):
     return synth.batch_roots_inputs(g, neg, b)
 
 
-def test_cache_merge_equals_store_then_combine(T):
+@pytest.mark.parametrize("d", [100, 37])   # float4 copies / scalar copies
+def test_cache_merge_equals_store_then_combine(T, d):
     """tgl_cache_merge (the launch the chain uses) == tgl_cache_store + tgl_cache_combine,
     read through an index (the S14 inverse) with repeated entries."""
     rng = np.random.default_rng(7)
-    d = 100
     cache = T.EmbeddingCache(1 << 14, d)
     memo = Memo()
     for n in (3000, 2500, 4000):
