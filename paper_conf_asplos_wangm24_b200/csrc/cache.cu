@@ -155,7 +155,7 @@ __global__ void cache_merge_kernel(unsigned long long* keys, float* __restrict__
                                    const int32_t* __restrict__ node, const float* __restrict__ t,
                                    const int32_t* __restrict__ slot,
                                    const float* __restrict__ computed, int64_t ld_computed,
-                                   float* __restrict__ out, int64_t ld_out, bool vec4) {
+                                   float* __restrict__ out, int64_t ld_out) {
   pdl_wait();
   pdl_trigger();
   const int64_t n = dev_count(n_dev, n_max);
@@ -185,17 +185,6 @@ __global__ void cache_merge_kernel(unsigned long long* keys, float* __restrict__
     }
     h = __shfl_sync(0xffffffffu, h, 0);
     float* row = h >= 0 ? vals + h * (int64_t)d : nullptr;
-    if (vec4) {                                  // 16-byte rows and pitches: float4 copies
-      const float4* s4 = reinterpret_cast<const float4*>(src);
-      float4* d4 = reinterpret_cast<float4*>(dst);
-      float4* r4 = reinterpret_cast<float4*>(row);
-      for (int c = lane; c < (d >> 2); c += 32) {
-        const float4 v = s4[c];
-        d4[c] = v;
-        if (row) r4[c] = v;
-      }
-      continue;
-    }
     for (int c = lane; c < d; c += 32) {
       const float v = src[c];
       dst[c] = v;
@@ -291,11 +280,8 @@ extern "C" tgl_status tgl_cache_merge(const tgl_cache* c, int64_t n_max, const i
   TGL_TRY(cache_check(c, &l2));
   TGL_REQUIRE(ld_out >= c->d && ld_computed >= c->d, "row pitch < d");
   TGL_REQUIRE(n_max == 0 || (node && t && slot && computed && out), "null pointer");
-  auto a16 = [](const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; };
-  const bool vec4 = (c->d % 4 == 0) && (ld_computed % 4 == 0) && (ld_out % 4 == 0) &&
-                    a16(c->vals) && a16(computed) && a16(out);
   launch_pdl(cache_merge_kernel, dim3(warp_grid(n_max)), dim3(256), 0, as_stream(stream),
              c->keys, c->vals, l2, (int)c->d, n_max, n_dev, idx, node, t, slot, computed,
-             ld_computed, out, ld_out, vec4);
+             ld_computed, out, ld_out);
   return launch_check("cache_merge");
 }
