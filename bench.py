@@ -1,22 +1,31 @@
 #!/usr/bin/env python
 """Benchmark of the TBlock hot path (BASELINE.json metric) -- one JSON line on rank 0.
 
-    python bench.py [--gpus N --steps K --warmup W --config REDDIT --precision fp32]
+    python bench.py [--gpus N --steps K --warmup W --config GDELT --precision fp32]
     python bench.py --impl reference ...      # the CPU oracle on the host cores
 
-A step = one batch through every §8(a) row: roots (S2) -> [dedup (S3)] ->
-sample (S4) -> next block (S5) -> ... -> TBlock attention tail..head (S6-S13,
-S15) -> dedup inverse at the roots (S14), replayed as one CUDA graph with the
-graph, features and batch edges resident in HBM.  Between timed steps L2 is
-flushed by writing a 256 MiB buffer (outside the timed events).  With N GPUs
-(torchrun) every rank runs its own batch of the stream (weak scaling) and the
-root embeddings of all ranks are all-gathered over NCCL inside the step (S16).
+A step = one batch through every §8(a) row: roots (S2) -> [dedup (S3)] -> sample (S4)
+-> next block (S5) -> ... -> TBlock attention tail..head (S6-S13, S15) -> dedup
+inverse at the roots (S14), replayed as a captured CUDA graph with the graph,
+features and batch edges resident in HBM.
+
+Default workload: GDELT (configs[3]), the config `north_star` quotes at 1/2/4/8 B200.
+With N GPUs (torchrun, or `--gpus N` which self-launches N ranks) the roots of every
+batch are sharded across the ranks (S16): each rank computes its slice
+of the (deduped) roots, the slices are all-gathered over NCCL on a comm stream that
+overlaps the next batch, and the batch's embeddings are rebuilt on every rank
+(`"scaling": "strong"`: the batch is fixed, N GPUs share it).
+
+L2: GDELT / MAG read edge-feature tables (142 GB / 62 GB) far larger than L2, so their
+steps run back to back with no flush and the timed region is the whole K-step loop;
+WIKI / REDDIT / LASTFM flush L2 (256 MiB write) between steps, outside per-step events.
 """
 from __future__ import annotations
 
 import argparse
 import json
 import os
+import platform
 import statistics
 import subprocess
 import sys
@@ -27,23 +36,42 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "sampled edges/s and TBlock embeddings/s at 1/2/4/8 B200; % HBM roofline"
+BIG = ("GDELT", "MAG")            # generated on the device (synth.gpu)
+FLUSH_DEFAULT = {"WIKI": True, "REDDIT": True, "LASTFM": True, "GDELT": False, "MAG": False}
 
 
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="REDDIT")
+    ap.add_argument("--config", default="GDELT")
     ap.add_argument("--precision", default="fp32", choices=["fp32", "bf16", "fp32_simt"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--cpu-seconds", type=float, default=10.0,
+                    help="oracle work per cpu_baseline leg (all cores, then 1 thread)")
+    ap.add_argument("--ref-seconds", type=float, default=120.0,
+                    help="budget of the --impl reference timed steps (sizes its sample)")
     ap.add_argument("--dedup", default="config", choices=["config", "on", "off"],
                     help="override the config's dedup setting (ablation only)")
     ap.add_argument("--cache", type=int, default=0,
                     help="cache() table slots per layer (0 = off, the BASELINE configs)")
+    ap.add_argument("--l2-flush", default="auto", choices=["auto", "on", "off"])
+    ap.add_argument("--kv-kernel", default="auto",
+                    choices=["auto", "split", "split_pad", "async", "bin", "general"])
+    ap.add_argument("--no-e2e", action="store_true")
     return ap.parse_args()
+
+
+def cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return platform.processor() or "unknown"
 
 
 # ---------------------------------------------------------------------- clocks
@@ -100,7 +128,15 @@ class ClockSampler:
                 "samples": len(sm), "reasons": sorted(reasons)}
 
 
-# ---------------------------------------------------------------------- shared inputs
+# ---------------------------------------------------------------------- inputs
+class HostGraph:
+    """Host view of a device-generated graph: what batch slicing and the oracle need."""
+
+    def __init__(self, cfg, src, dst, t):
+        self.cfg, self.src, self.dst, self.t, self.num_edges = cfg, src, dst, t, cfg.n_edges
+        self.nfeat = self.efeat = None        # regenerated row by row (synth.feature_rows)
+
+
 def load_world(cfg_name: str):
     import synth
     cfg = synth.get_config(cfg_name)
@@ -110,43 +146,9 @@ def load_world(cfg_name: str):
     return cfg, g, neg, params
 
 
-def oracle_rate(cfg, g, neg, params, batches, seconds: float):
-    """CPU oracle (as it stands) on whole batches until `seconds` of CPU work."""
-    import oracle
-    from oracle import pipeline as opipe
-    t0 = time.perf_counter()
-    tc = oracle.build_tcsr(cfg.n_nodes, g.src, g.dst, g.t, True)
-    t_build = time.perf_counter() - t0
-    done, edges, t_run, nb = 0, 0, 0.0, 0
-    for b in batches:
-        nb += 1
-        t0 = time.perf_counter()
-        emb, blocks = opipe.run_batch(tc, g.nfeat, g.efeat, params, cfg.k, cfg.strategy,
-                                      cfg.dedup, cfg.seeds["sampler"],
-                                      *synth_batch(g, neg, b))
-        t_run += time.perf_counter() - t0
-        done += emb.shape[0]
-        edges += sum(int(bl.seg_ptr[-1]) for bl in blocks)
-        if t_run >= seconds:
-            break
-    return {"emb_per_s": done / t_run, "edges_per_s": edges / t_run, "batches": nb,
-            "roots": done, "seconds": t_run,
-        "cores": oracle.num_threads(), "tcsr_build_s": t_build}
-
-
-BIG = ("GDELT", "MAG")   # generated on the device (synth.gpu); host RAM holds only the COO
-
-
-class HostGraph:
-    """Host view of a device-generated graph: what batch slicing and the oracle need."""
-
-    def __init__(self, cfg, src, dst, t):
-        self.cfg, self.src, self.dst, self.t, self.num_edges = cfg, src, dst, t, cfg.n_edges
-
-
 def load_world_device(cfg_name: str):
     """GDELT/MAG: COO, negatives and feature tables generated on cuda (synth.gpu, the
-    same counter-based values as synth.make_graph), host copies of the COO only."""
+    same counter-based values as synth.feature_rows), host copies of the COO only."""
     import synth
     import torch
     from synth import gpu as sg
@@ -166,10 +168,110 @@ def load_world_device(cfg_name: str):
     return cfg, g, neg_h, synth.gen.model_params(cfg), dev
 
 
-def oracle_rate_big(cfg, g, neg, params, batches, seconds: float, frac: int = 0):
-    """Listing 1's recursion (oracle/big.py) root by root on whole-graph-free segments:
-    the whole-graph oracle cannot hold GDELT/MAG.  Bounded by `seconds` of CPU work."""
-    import oracle
+def host_graph_for_reference(cfg):
+    """The COO the GPU arm uses: synth.gpu on a GPU box (input generation only), else the
+    numpy generator (CPU-only machines; same recipe, another draw)."""
+    import synth
+    import torch
+    if cfg.name in BIG and torch.cuda.is_available():
+        from synth import gpu as sg
+        d = torch.device("cuda")
+        src, dst, t = sg.device_graph(cfg, d)
+        g = HostGraph(cfg, src.cpu().numpy(), dst.cpu().numpy(), t.cpu().numpy())
+        neg = sg.device_negatives(cfg, d).cpu().numpy()
+        del src, dst, t
+        torch.cuda.empty_cache()
+        return g, neg
+    if cfg.name in BIG:
+        g = synth.make_graph(cfg, with_features=False)
+        g.nfeat = g.efeat = None
+        return g, synth.make_negatives(cfg)
+    return synth.make_graph(cfg), synth.make_negatives(cfg)
+
+
+def synth_batch(g, neg, b):
+    import synth
+    return synth.batch_roots_inputs(g, neg, b)
+
+
+def config_dict(cfg, args, world: int, flush: bool) -> dict:
+    """The workload description both arms print (identical dicts: same_config)."""
+    return {"workload": cfg.name, "batch_edges": cfg.batch, "roots_per_step": 3 * cfg.batch,
+            "layers": cfg.n_layers, "k": cfg.k, "strategy": cfg.strategy, "dedup": cfg.dedup,
+            "precompute": cfg.precompute, "precision": args.precision,
+            "cache_slots_per_layer": args.cache,
+            "parallelism": (f"root-sharded x{world} (each rank: slice of the batch's roots; "
+                            f"NCCL all-gather of root embeddings)" if world > 1 else "single"),
+            "l2": ("flushed (256 MiB write) between timed steps, outside per-step events"
+                   if flush else "not flushed: per-step inputs are gathered from feature "
+                                 "tables far larger than L2; steps back to back"),
+            "timing": ("CUDA events per step on the launch stream; max over ranks" if flush else
+                       "CUDA events around the whole K-step loop; max over ranks")}
+
+
+# ---------------------------------------------------------------------- oracle legs
+class OracleRunner:
+    """The whole-graph CPU oracle (oracle.c) on whole batches: T-CSR once, then Listing 2's
+    block chain per batch (oracle/pipeline.py).  GDELT's edge features (142 GB) are never
+    materialised on the host: the rows a batch samples are regenerated by
+    synth.feature_rows (input generation, outside the timed region)."""
+
+    def __init__(self, cfg, g, params):
+        import numpy as np
+        import oracle
+        import synth
+        self.cfg, self.g, self.params = cfg, g, params
+        t0 = time.perf_counter()
+        self.tc = oracle.build_tcsr(cfg.n_nodes, g.src, g.dst, g.t, True)
+        self.tcsr_s = time.perf_counter() - t0
+        self.nfeat = (g.nfeat if g.nfeat is not None else
+                      synth.feature_rows(cfg.seeds["feat"], np.arange(cfg.n_nodes), cfg.d_v))
+        self.lazy_e = g.efeat is None
+
+    def batch(self, src_b, dst_b, t_b, neg_b):
+        """(roots, sampled edges, oracle seconds) of one (possibly partial) batch."""
+        import numpy as np
+        import synth
+        from oracle import pipeline as opipe
+        cfg = self.cfg
+        t0 = time.perf_counter()
+        qn, qt = opipe.roots(src_b, dst_b, t_b, neg_b)
+        blocks = opipe.build_blocks(self.tc, qn, qt, len(self.params), cfg.k, cfg.strategy,
+                                    cfg.dedup, cfg.seeds["sampler"])
+        t1 = time.perf_counter()
+        if self.lazy_e and cfg.d_e > 0:      # the sampled edges' feature rows only
+            eids = np.unique(np.concatenate([bl.eid[:bl.seg_ptr[-1]] for bl in blocks]))
+            ef = synth.feature_rows(cfg.seeds["feat"] + 7919, eids, cfg.d_e)
+            for bl in blocks:
+                bl.eid = np.searchsorted(eids, bl.eid).astype(np.int32)
+        else:
+            ef = self.g.efeat if self.g.efeat is not None else np.zeros((1, 0), np.float32)
+        t2 = time.perf_counter()
+        opipe.aggregate(blocks, self.params, self.nfeat, ef)
+        t3 = time.perf_counter()
+        return 3 * len(src_b), sum(int(bl.seg_ptr[-1]) for bl in blocks), (t1 - t0) + (t3 - t2)
+
+
+def oracle_rate(runner, g, neg, batches, seconds: float, edges_per_call: int | None = None):
+    """Oracle throughput over whole batches (or their first `edges_per_call` edges) until
+    `seconds` of oracle work."""
+    roots = edges = 0
+    t_run, nb = 0.0, 0
+    for b in batches:
+        src_b, dst_b, t_b, neg_b = synth_batch(g, neg, b)
+        if edges_per_call:
+            src_b, dst_b, t_b, neg_b = (x[:edges_per_call] for x in (src_b, dst_b, t_b, neg_b))
+        r, e, dt = runner.batch(src_b, dst_b, t_b, neg_b)
+        roots, edges, t_run, nb = roots + r, edges + e, t_run + dt, nb + 1
+        if t_run >= seconds:
+            break
+    return {"emb_per_s": roots / t_run, "edges_per_s": edges / t_run, "batches": nb,
+            "roots": roots, "seconds": t_run}
+
+
+def oracle_rate_mag(cfg, g, neg, params, batches, seconds: float):
+    """MAG (2.6B CSR entries: no whole-graph oracle): Listing 1's recursion
+    (oracle/big.py) root by root, bounded by `seconds` of oracle work."""
     from oracle import big
     from oracle import pipeline as opipe
     segs, done, t_run, nb = {}, 0, 0.0, 0
@@ -187,131 +289,112 @@ def oracle_rate_big(cfg, g, neg, params, batches, seconds: float, frac: int = 0)
         if t_run >= seconds:
             break
     return {"emb_per_s": done / t_run, "batches": nb, "roots": done, "seconds": t_run,
-            "cores": oracle.num_threads(), "edges_per_s": float("nan")}
+            "edges_per_s": float("nan")}
 
 
-def synth_batch(g, neg, b):
-    import synth
-    return synth.batch_roots_inputs(g, neg, b)
+def cpu_baseline(cfg, g, neg, params, batches, seconds: float, runner=None) -> dict:
+    """The oracle as it stands on this host: all cores (OpenMP), then one thread."""
+    import oracle
+    ncores = oracle.num_threads()
+    legs = {}
+    for threads in (ncores, 1):
+        oracle.set_num_threads(threads)
+        if cfg.name == "MAG":
+            r = oracle_rate_mag(cfg, g, neg, params, batches, seconds)
+            smp = (f"{r['roots']} roots from {r['batches']} batch(es) at 70% of the stream, one "
+                   f"at a time by Listing 1's recursion (oracle/big.py), {r['seconds']:.1f} s")
+        else:
+            # whole batches when one fits the budget, else the first edges of each batch
+            per = None if threads > 1 or cfg.name not in BIG else max(1, cfg.batch // 20)
+            r = oracle_rate(runner, g, neg, batches, seconds, per)
+            smp = (f"{r['batches']} {'whole batch(es)' if per is None else f'x first {per} edges of a batch'}"
+                   f" ({r['roots']} roots) from 70% of the stream, {r['seconds']:.1f} s")
+        legs[threads] = (r, smp)
+    oracle.set_num_threads(ncores)
+    r, smp = legs[ncores]
+    r1, smp1 = legs[1]
+    out = {"value": r["emb_per_s"], "unit": "embeddings/s", "cores": ncores, "kind": "oracle",
+           "sample": smp, "sampled_edges_per_s": r["edges_per_s"],
+           "single_thread": {"value": r1["emb_per_s"], "unit": "embeddings/s", "cores": 1,
+                             "sample": smp1, "sampled_edges_per_s": r1["edges_per_s"]},
+           "cpu_model": cpu_model(), "host_cpus": os.cpu_count()}
+    if runner is not None:
+        out["tcsr_build_s"] = runner.tcsr_s
+    return out
 
 
 # ---------------------------------------------------------------------- reference arm
 def run_reference(args):
+    """--impl reference: the CPU oracle (there is no reference code: the reference is a
+    paper) on this host's cores, on our arm's config and metric; each timed step is one
+    batch of the same stream -- whole when the budget allows, else its first edges."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
-    if args.config.upper() in BIG:
-        return run_reference_big(args)
-    cfg, g, neg, params = load_world(args.config)
-    import oracle
-    from oracle import pipeline as opipe
-    tc = oracle.build_tcsr(cfg.n_nodes, g.src, g.dst, g.t, True)
-    b0 = int(0.7 * cfg.n_batches)
-    # bounded sample: a slice of each batch's roots (first `frac` of its edges)
-    frac_edges = max(1, cfg.batch // 8)
-    times, roots, edges = [], 0, 0
-    for i in range(args.warmup + args.steps):
-        b = b0 + i
-        src_b, dst_b, t_b, neg_b = synth_batch(g, neg, b)
-        sl = slice(0, frac_edges)
-        t0 = time.perf_counter()
-        emb, blocks = opipe.run_batch(tc, g.nfeat, g.efeat, params, cfg.k, cfg.strategy,
-                                      cfg.dedup, cfg.seeds["sampler"], src_b[sl], dst_b[sl],
-                                      t_b[sl], neg_b[sl])
-        dt = time.perf_counter() - t0
-        if i >= args.warmup:
-            times.append(dt)
-            roots += emb.shape[0]
-            edges += sum(int(bl.seg_ptr[-1]) for bl in blocks)
-    T = sum(times)
-    val = roots / T
-    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "embeddings/s",
-            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": 1e3 * T / args.steps, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": cfg.name, "batch_edges_per_step": frac_edges,
-                       "roots_per_step": 3 * frac_edges, "layers": cfg.n_layers, "k": cfg.k,
-                       "strategy": cfg.strategy, "dedup": cfg.dedup,
-                       "precompute": cfg.precompute},
-            "sampled_edges_per_s": edges / T,
-            "cpu_baseline": {"value": val, "unit": "embeddings/s",
-                             "cores": oracle.num_threads(), "kind": "oracle",
-                             "sample": f"first {frac_edges} of each {cfg.batch}-edge batch "
-                                       f"({3 * frac_edges} roots) from 70% of the stream"},
-            "e2e": {"value": val, "unit": "embeddings/s", "h2d_bytes_per_step": 0,
-                    "d2h_bytes_per_step": 0}}
-    print(json.dumps(line), flush=True)
-    return 0
-
-
-def run_reference_big(args):
-    """--impl reference on GDELT/MAG: the oracle's recursion (oracle/big.py) on a few roots
-    per step; the COO comes from the same seeded generator as our arm (synth.gpu on a
-    GPU box -- input generation only -- else synth.make_graph)."""
     import oracle
     import synth
-    from oracle import big
-    from oracle import pipeline as opipe
-    import torch
     cfg = synth.get_config(args.config.upper())
-    if torch.cuda.is_available():                   # the same COO our arm generates
-        from synth import gpu as sg
-        d = torch.device("cuda")
-        src, dst, t = sg.device_graph(cfg, d)
-        gg = HostGraph(cfg, src.cpu().numpy(), dst.cpu().numpy(), t.cpu().numpy())
-        neg = sg.device_negatives(cfg, d).cpu().numpy()
-        del src, dst, t
-    else:
-        gg = synth.make_graph(cfg, with_features=False)
-        neg = synth.make_negatives(cfg)
+    if args.dedup != "config":
+        from dataclasses import replace
+        cfg = replace(cfg, dedup=args.dedup == "on")
+    flush = FLUSH_DEFAULT[cfg.name] if args.l2_flush == "auto" else args.l2_flush == "on"
+    g, neg = host_graph_for_reference(cfg)
     params = synth.gen.model_params(cfg)
     b0 = int(0.7 * cfg.n_batches)
-    per_step = 2                                    # roots per step (bounded sample)
-    times, roots, segs = [], 0, {}
+    nb_avail = cfg.n_batches - b0
+    if cfg.name == "MAG":
+        runner = None
+        per = 2                                   # roots per step (Listing 1 recursion)
+    else:
+        runner = OracleRunner(cfg, g, params)
+        # size the step: whole batches if K of them fit the budget, else first edges
+        r, _, dt = runner.batch(*synth_batch(g, neg, b0))
+        per = cfg.batch
+        while per > 1 and dt * args.steps * per / cfg.batch > args.ref_seconds:
+            per //= 2
+    from oracle import big
+    from oracle import pipeline as opipe
+    times, roots, edges, segs = [], 0, 0, {}
     for i in range(args.warmup + args.steps):
-        qn, qt = opipe.roots(*synth_batch(gg, neg, b0 + i))
-        t0 = time.perf_counter()
-        big.embed_recursive(gg.src, gg.dst, gg.t, cfg, params, qn[:per_step], qt[:per_step],
-                            cfg.seeds["sampler"], segs=segs)
-        dt = time.perf_counter() - t0
+        b = b0 + (i % nb_avail)
+        if cfg.name == "MAG":
+            qn, qt = opipe.roots(*synth_batch(g, neg, b))
+            t0 = time.perf_counter()
+            big.embed_recursive(g.src, g.dst, g.t, cfg, params, qn[:per], qt[:per],
+                                cfg.seeds["sampler"], segs=segs)
+            dt, rr, ee = time.perf_counter() - t0, per, 0
+        else:
+            src_b, dst_b, t_b, neg_b = (x[:per] for x in synth_batch(g, neg, b))
+            rr, ee, dt = runner.batch(src_b, dst_b, t_b, neg_b)
         if i >= args.warmup:
             times.append(dt)
-            roots += per_step
+            roots += rr
+            edges += ee
     T = sum(times)
     val = roots / T
+    sample = (f"first {per} roots of each batch, Listing 1's recursion (oracle/big.py)"
+              if cfg.name == "MAG" else
+              ("whole batches" if per == cfg.batch else f"first {per} of each {cfg.batch}-edge "
+               f"batch ({3 * per} roots)") + " from 70% of the stream, whole-graph oracle")
     line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "embeddings/s",
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": 1e3 * T / args.steps, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": cfg.name, "roots_per_step": per_step, "layers": cfg.n_layers,
-                       "k": cfg.k, "strategy": cfg.strategy, "dedup": cfg.dedup,
-                       "precompute": cfg.precompute},
-            "cpu_baseline": {"value": val, "unit": "embeddings/s",
-                             "cores": oracle.num_threads(), "kind": "oracle",
-                             "sample": f"first {per_step} roots of each batch from 70% of the "
-                                       f"stream, Listing 1's recursion (oracle/big.py)"},
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": config_dict(cfg, args, args.gpus, flush),
+            "sampled_edges_per_s": edges / T if edges else None,
+            "cpu_baseline": {"value": val, "unit": "embeddings/s", "cores": oracle.num_threads(),
+                             "kind": "oracle", "sample": sample, "cpu_model": cpu_model()},
             "e2e": {"value": val, "unit": "embeddings/s", "h2d_bytes_per_step": 0,
                     "d2h_bytes_per_step": 0}}
+    if runner is not None:
+        line["cpu_baseline"]["tcsr_build_s"] = runner.tcsr_s
     print(json.dumps(line), flush=True)
     return 0
 
 
 # ---------------------------------------------------------------------- our arm
-def algorithmic_attn(cfg, n_dst: int, n_edges: int, d_hdst: int, d_hsrc: int):
-    """Per tgl_tblock_attn call: FLOPs and bytes the method must do."""
-    dm, dt, de = cfg.d_model, cfg.d_t, cfg.d_e
-    kkv = d_hsrc + de + dt
-    flops = (n_edges * 2 * (2 * dm) * kkv          # K and V projections (S9)
-             + n_dst * 2 * dm * (d_hdst + dt)       # Q (S8)
-             + n_dst * 2 * dm * (dm + d_hdst)       # FFN (S13)
-             + n_edges * 4 * dm)                    # logits + weighted sum (S10-S12)
-    bytes_ = (n_edges * (4 * (d_hsrc + de) + 4 + 4 + 4 + 8)   # gathers + nbr/eid/ts + idx
-              + n_dst * (4 * d_hdst * 2 + 8 + 8 + 4 * cfg.d_model))  # h_dst (Q and FFN), t, seg, out
-    return flops, bytes_
-
-
 def algorithmic_kv(cfg, n_dst: float, n_edges: float, d_hsrc: int):
-    """Per launch of the K|V attention kernel (S6, S7, S9-S12; DESIGN.md §7):
+    """Per launch of the K|V attention kernel (S6, S7, S9-S12; SURVEY §8(d), DESIGN §7):
     FLOPs = E * (2 * 2*d_model * K) for [K;V] = W [h ; e ; Phi] (K = d_hs + d_e + d_t)
             + E * 4 * d_model for the logits and the alpha-weighted sum;
     bytes = E * (4 (d_hs + d_e) + 12)  (gathered rows + nbr/eid/ts; Phi computed or
@@ -327,15 +410,26 @@ def algorithmic_kv(cfg, n_dst: float, n_edges: float, d_hsrc: int):
 def ncu_traffic(config: str, precision: str):
     """dram__bytes_read.sum + dram__bytes_write.sum per launch of the K|V kernel from the
     committed `ncu --set full` capture of this config and precision (profiles/), or None."""
-    try:
-        d = json.load(open(os.path.join(ROOT, "profiles", "r01_kv_split_traffic.json")))
-        return d[config][precision]
-    except Exception:
-        return None
+    for name in ("r02_kv_traffic.json", "r01_kv_split_traffic.json"):
+        try:
+            d = json.load(open(os.path.join(ROOT, "profiles", name)))
+            return d[config][precision]
+        except Exception:
+            continue
+    return None
 
 
-KV_KERNELS = {0: "kv_split_kernel (contiguous K plan)", 1: "kv_split_kernel (padded K plan)",
-              2: "kv_async_kernel", 3: "kv_bin_kernel", 4: "kv_kernel (general)"}
+def relaunch(args) -> int:
+    """`--gpus N` without torchrun: start N ranks on this node (127.0.0.1 rendezvous)."""
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+           f"--nproc-per-node={args.gpus}", "--master-addr", "127.0.0.1",
+           "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
 
 
 def run_ours(args):
@@ -351,43 +445,62 @@ def run_ours(args):
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     import synth
     from paper_conf_asplos_wangm24_b200 import TGATPipeline, TSampler, tgl
-    from paper_conf_asplos_wangm24_b200 import dist as pdist
+    from paper_conf_asplos_wangm24_b200.dist import ShardedRunner
 
     cu = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
-    if args.config.upper() in BIG:
-        cfg, g, neg, params, dev = load_world_device(args.config.upper())
+    name = args.config.upper()
+    if name in BIG:
+        cfg, g, neg, params, dev = load_world_device(name)
     else:
-        cfg, g, neg, params = load_world(args.config)
+        cfg, g, neg, params = load_world(name)
         dev = {"src": cu(g.src), "dst": cu(g.dst), "t": cu(g.t), "neg": cu(neg),
                "nfeat": cu(g.nfeat), "efeat": cu(g.efeat)}
     if args.dedup != "config" or (args.cache and not cfg.dedup):
         from dataclasses import replace              # cache() sits behind each block's dedup
         cfg = replace(cfg, dedup=args.dedup == "on" or bool(args.cache))   # (P:578 pairs them)
+    flush = FLUSH_DEFAULT[cfg.name] if args.l2_flush == "auto" else args.l2_flush == "on"
+    want_cpu = rank == 0 and world == 1 and not args.no_cpu_baseline
+
+    # the whole-graph oracle's T-CSR (a C qsort of 2E entries: ~2 min on GDELT) builds on a
+    # host thread while the GPU is measured (ctypes releases the GIL)
+    oracle_box = {}
+    if want_cpu and cfg.name != "MAG":
+        def _build():
+            oracle_box["runner"] = OracleRunner(cfg, g, params)
+        oth = threading.Thread(target=_build, daemon=True)
+        oth.start()
+
+    # S1 T-CSR: one warm-up build (module load, first-touch), then the timed build
+    tgl.build_tcsr(cfg.n_nodes, dev["src"], dev["dst"], dev["t"], True, True)
     torch.cuda.synchronize()
+    torch.cuda.empty_cache()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     ev0.record()
     tc = tgl.build_tcsr(cfg.n_nodes, dev["src"], dev["dst"], dev["t"], True, True)
     ev1.record()
     torch.cuda.synchronize()
     tcsr_ms = ev0.elapsed_time(ev1)
+    M = 2 * cfg.n_edges
+    tcsr_bytes = cfg.n_edges * 12 + M * 12 + (cfg.n_nodes + 1) * 8   # SURVEY §8(d) per edge
+
     sampler = TSampler(cfg.k, cfg.strategy, cfg.seeds["sampler"])
+    shard = (rank, world) if world > 1 else None
     pipe = TGATPipeline(dev, tc, params, cfg.batch, sampler, cfg.dedup, cfg.precompute,
-                        cfg.window, args.precision, cache_capacity=args.cache)
+                        cfg.window, args.precision, cache_capacity=args.cache, shard=shard)
+    for a in pipe.attn:
+        a.set_kv_kernel(args.kv_kernel)
     pipe.capture()
     n0 = 3 * cfg.batch
-    gathered = torch.empty(world * n0, cfg.d_model, device="cuda") if world > 1 else None
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    flush_buf = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     b0 = int(0.7 * cfg.n_batches)
     nb_avail = cfg.n_batches - b0
 
     def batch_of(i):
-        return pdist.rank_batch(i, rank, world, b0, nb_avail)
+        return b0 + (i % nb_avail)
 
-    # per-step device counters read after timing (outside the events)
-    cnt_e = torch.zeros(args.warmup + args.steps, dtype=torch.int64, device="cuda")
+    runner = ShardedRunner(pipe) if shard else None
     stream = torch.cuda.current_stream()
-    starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-    ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    cnt_e = torch.zeros(args.warmup + args.steps, dtype=torch.int64, device="cuda")
 
     def counts_into(i):
         tot = torch.zeros((), dtype=torch.int64, device="cuda")
@@ -395,12 +508,17 @@ def run_ours(args):
             tot = tot + b.seg_ptr.index_select(0, b.u_dev.clamp(max=b.n_max)).squeeze()
         cnt_e[i] = tot
 
+    def one_step(j):
+        if runner is not None:
+            runner.step(batch_of(j) * cfg.batch)
+        else:
+            pipe.start_dev.fill_(batch_of(j) * cfg.batch)
+            pipe.run_graph()
+
     for i in range(args.warmup):
-        pipe.start_dev.fill_(batch_of(i) * cfg.batch)
-        out = pipe.run_graph()
-        if world > 1:
-            pdist.allgather_embeddings(out[:n0], gathered)
-        counts_into(i)
+        one_step(i)
+    if runner is not None:
+        runner.drain()
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
@@ -408,173 +526,153 @@ def run_ours(args):
     clk.start()
     time.sleep(0.3)
     torch.cuda.synchronize()
-    for i in range(args.steps):
-        j = args.warmup + i
-        flush.zero_()                                  # L2 flush, outside the events
-        pipe.start_dev.fill_(batch_of(j) * cfg.batch)
-        starts[i].record(stream)
-        out = pipe.run_graph()
-        if world > 1:
-            pdist.allgather_embeddings(out[:n0], gathered)   # S16
-        ends[i].record(stream)
-        counts_into(j)
-    torch.cuda.synchronize()
+    if flush:
+        starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+        ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+        for i in range(args.steps):
+            j = args.warmup + i
+            flush_buf.zero_()
+            starts[i].record(stream)
+            if runner is not None:
+                runner.step(batch_of(j) * cfg.batch)
+                runner.drain()
+            else:
+                pipe.start_dev.fill_(batch_of(j) * cfg.batch)
+                pipe.run_graph()
+            ends[i].record(stream)
+        torch.cuda.synchronize()
+        step_ms = [s.elapsed_time(e) for s, e in zip(starts, ends)]
+        total_ms = sum(step_ms)
+    else:
+        e_start, e_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e_start.record(stream)
+        for i in range(args.steps):
+            one_step(args.warmup + i)
+        if runner is not None:
+            runner.drain()
+        e_end.record(stream)
+        torch.cuda.synchronize()
+        total_ms = e_start.elapsed_time(e_end)
+        step_ms = None
     if world > 1:
         dist.barrier()
     clocks = clk.stop()
-    step_ms = [s.elapsed_time(e) for s, e in zip(starts, ends)]
-    total_ms = sum(step_ms)
+    # sampled edges of the timed batches: the same batches replayed once more, untimed
+    # (the chain is deterministic), each followed by its device-side count
+    for i in range(args.steps):
+        one_step(args.warmup + i)
+        if runner is not None:
+            runner.drain()
+        counts_into(args.warmup + i)
+    torch.cuda.synchronize()
     t_max = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
     if world > 1:
         dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
     total_ms = float(t_max.item())
-    edges_local = int(cnt_e[args.warmup:].sum().item())
-    e_tot = torch.tensor([edges_local], dtype=torch.int64, device="cuda")
+    e_tot = cnt_e[args.warmup:].sum().reshape(1)
     if world > 1:
         dist.all_reduce(e_tot)
-    roots_all = world * n0 * args.steps
-    emb_per_s = roots_all / (total_ms / 1e3)
+    emb_per_s = n0 * args.steps / (total_ms / 1e3)
     edges_per_s = int(e_tot.item()) / (total_ms / 1e3)
 
-    # ---- dominant call: tgl_tblock_attn on the tail block, timed eagerly with events
-    rec_ms, rec_shape, brk, kv_ms = [], None, {}, []
-    lib = tgl.lib()
-    for i in range(max(3, min(args.steps, 20))):
-        flush.zero_()
-        pipe.start_dev.fill_(batch_of(args.warmup + i) * cfg.batch)
+    # ---- eager probes on batches the timed loop did not run (fresh, L2 flushed):
+    # the K|V kernel (CUDA events recorded by the library on its own stream), the
+    # per-step breakdown and the sampler alone
+    tail = pipe.L - 1
+    probe = tgl.KvProbe()
+    n_probe = max(3, min(args.steps, 10))
+    kv_ms, kinds, shapes, brk, smp_ms, smp_edges = [], set(), [], {}, 0.0, 0
+    for i in range(n_probe):
+        j = args.warmup + args.steps + i
+        flush_buf.zero_()
+        pipe.start_dev.fill_(batch_of(j) * cfg.batch)
         rec = {}
-        lib.tgl_kv_timing(1)          # CUDA events around each K|V kernel, on its stream
+        pipe.attn[tail].attach_probe(probe)
         pipe.forward(record=rec)
+        pipe.attn[tail].attach_probe(None)
         torch.cuda.synchronize()
-        kv_ms.append(lib.tgl_kv_timing_ms(0))   # the tail block runs first
-        tail = pipe.L - 1
-        rec_ms.append(rec[tail][0].elapsed_time(rec[tail][1]))
+        kv_ms.append(probe.ms())
+        kinds.add(probe.kernel)
         mk = rec["_marks"]
         for (n0_, e0_), (n1_, e1_) in zip(mk[:-1], mk[1:]):
-            brk.setdefault(n1_, []).append(e0_.elapsed_time(e1_))
+            dt_ = e0_.elapsed_time(e1_)
+            brk.setdefault(n1_, []).append(dt_)
+            if n1_.startswith("sample"):
+                smp_ms += dt_
+        for b in pipe.blocks:
+            U = int(b.u_dev.item())
+            smp_edges += int(b.seg_ptr[U].item())
         bt = pipe.blocks[tail]
         U = int(bt.u_dev.item())
-        E = int(bt.seg_ptr[U].item())
-        rec_shape = (rec_shape or []) + [(U, E)]
-    U_avg = sum(u for u, _ in rec_shape) / len(rec_shape)
-    E_avg = sum(e for _, e in rec_shape) / len(rec_shape)
-    fl, by = algorithmic_attn(cfg, U_avg, E_avg, cfg.d_v, cfg.d_v)
-    attn_ms = sum(rec_ms) / len(rec_ms)
-    lib.tgl_kv_timing(0)
+        shapes.append((U, int(bt.seg_ptr[U].item())))
+    U_avg = sum(u for u, _ in shapes) / len(shapes)
+    E_avg = sum(e for _, e in shapes) / len(shapes)
+    kv_avg = sum(kv_ms) / len(kv_ms)
     kv_fl, kv_by = algorithmic_kv(cfg, U_avg, E_avg, cfg.d_v)
-    kv_ok = [m for m in kv_ms if m > 0]
-    kv_avg = sum(kv_ok) / len(kv_ok) if kv_ok else float("nan")
     peaks = {}
     try:
         peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
     except Exception:
         pass
-    sm_max = clocks.get("sm_max_mhz") or peaks.get("sm_max_mhz", 1965.0)
     hbm_peak = peaks.get("hbm_gbs", 6545.9)
     bf16_peak = peaks.get("bf16_tflops", 1613.6)
+    tf32_peak = bf16_peak * 1.1 / 2.25            # fp32-operand tensor peak (guide's ratio)
+    passes = {"fp32": 3, "bf16": 1, "fp32_simt": 0}[args.precision]
     kv_tf = kv_fl / (kv_avg / 1e3) / 1e12
     kv_gbs = kv_by / (kv_avg / 1e3) / 1e9
-    if args.precision == "fp32_simt":
-        peak = 148 * 128 * 2 * sm_max * 1e6 / 1e12     # TFLOP/s, FFMA on all SMs
-        bound, unit, ach = "alu", "TFLOP/s", kv_tf
-        note = "FP32 FFMA peak = 148 SM x 128 lanes x 2 x clocks.max.sm (derived)"
-    elif args.precision == "fp32":
-        # fp32 = 3 bf16 MMA passes per algorithmic FLOP: the tensor roofline for fp32
-        # operands is the measured bf16 burst peak / 3; it binds before HBM
-        peak, bound, unit, ach = bf16_peak / 3, "tensor", "TFLOP/s", kv_tf
-        note = "measured cuBLAS bf16 burst peak (MEASURED_PEAKS.json) / 3 passes"
-    else:
-        peak, bound, unit, ach = hbm_peak, "hbm", "GB/s", kv_gbs
-        note = "measured HBM copy bandwidth (MEASURED_PEAKS.json); bf16 MMA time < HBM time"
     tr = ncu_traffic(cfg.name, args.precision)
-    kname = KV_KERNELS.get(int(lib.tgl_kv_timing_kernel(0)), "?")
-    roofline = {"kernel": f"{kname}: K|V attention of the tail block (S6,S7,S9-S12)",
-                "bound": bound, "achieved": ach, "peak": peak, "unit": unit,
-                "frac": ach / peak,
+    roofline = {"kernel": f"{tgl.KV_KERNEL_NAME.get(min(kinds), '?')}: K|V attention of the "
+                          f"tail block (S6, S7, S9-S12)",
+                "bound": "hbm", "achieved": kv_gbs, "peak": hbm_peak, "unit": "GB/s",
+                "frac": kv_gbs / hbm_peak,
                 "traffic": tr["dram_bytes_per_launch"] if tr else None,
                 "traffic_note": (f"ncu --set full, {tr['source']}" if tr else None),
-                "per_launch_ms": kv_avg, "launches_timed": len(kv_ok),
-                "algorithmic_flops": kv_fl, "algorithmic_bytes": kv_by,
-                "tensor_tflops": kv_tf, "tensor_frac_bf16_peak": kv_tf / bf16_peak,
-                "hbm_gbs": kv_gbs, "hbm_frac": kv_gbs / hbm_peak,
-                "n_dst_avg": U_avg, "n_edges_avg": E_avg, "peak_note": note,
-                "attn_call_ms": attn_ms, "attn_call_tflops": fl / (attn_ms / 1e3) / 1e12}
+                "peak_note": "measured HBM copy bandwidth (MEASURED_PEAKS.json hbm_gbs)",
+                "per_launch_ms": kv_avg, "launches_timed": len(kv_ms),
+                "algorithmic_bytes": kv_by, "algorithmic_flops": kv_fl,
+                "n_dst_avg": U_avg, "n_edges_avg": E_avg,
+                "tensor": {"achieved_tflops": kv_tf, "fp32_operand_peak_tflops": tf32_peak,
+                           "frac_fp32_operand_peak": kv_tf / tf32_peak,
+                           "mma_passes": passes,
+                           "pipe_frac_bf16_peak": passes * kv_tf / bf16_peak,
+                           "note": "fp32 mode issues 3 bf16 MMAs (hi*hi + lo*hi + hi*lo) per "
+                                   "algorithmic FLOP; pipe_frac = issued bf16 work / measured "
+                                   "bf16 peak"}}
+    sampler_line = {"sampled_edges_per_s": smp_edges / (smp_ms / 1e3) if smp_ms else None,
+                    "ms_per_step": smp_ms / n_probe, "sampled_edges_per_step": smp_edges / n_probe,
+                    "timing": "tgl_sample launches alone (CUDA events, eager, L2 flushed)"}
 
     # ---- e2e through the public API: pinned host batch -> device -> host embeddings
     e2e = None
-    if world >= 1:
-        pipe_h = TGATPipeline(dev, tc, params, cfg.batch, sampler, cfg.dedup, cfg.precompute,
-                              cfg.window, args.precision, staging=True,
-                              cache_capacity=args.cache)
-        pipe_h.capture()
-        from paper_conf_asplos_wangm24_b200 import HostStream
-        outs = [torch.empty(n0, cfg.d_model, dtype=torch.float32).pin_memory() for _ in range(2)]
-        host_batches = []
-        for i in range(args.steps):
-            sb, db, tb, nb_ = synth.batch_roots_inputs(g, neg, batch_of(args.warmup + i))
-            host_batches.append(tuple(torch.from_numpy(np.ascontiguousarray(x)).pin_memory()
-                                      for x in (sb, db, tb, nb_)))
-        hs = HostStream(pipe_h, n0, cfg.d_model)
-        for i in range(min(3, args.steps)):
-            hs.submit(*host_batches[i], outs[i % 2]).synchronize()
-        torch.cuda.synchronize()
-        if world > 1:
-            dist.barrier()
-        # serving loop: batch i's embeddings are on the host (event synchronised) before
-        # batch i+1's are requested; the D2H of batch i overlaps batch i+1's compute
-        t0 = time.perf_counter()
-        prev = None
-        for i in range(args.steps):
-            done = hs.submit(*host_batches[i], outs[i % 2])
-            if world > 1:
-                pdist.allgather_embeddings(pipe_h.graph_out[:n0], gathered)
-            if prev is not None:
-                prev.synchronize()
-            prev = done
-        prev.synchronize()
-        torch.cuda.synchronize()
-        el = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device="cuda")
-        if world > 1:
-            dist.all_reduce(el, op=dist.ReduceOp.MAX)
-        h2d = cfg.batch * (4 + 4 + 4 + 4)
-        e2e = {"value": world * n0 * args.steps / float(el.item()), "unit": "embeddings/s",
-               "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": n0 * cfg.d_model * 4,
-               "timing": "host wall clock over the serving loop (HostStream): per batch H2D "
-                         "of its edges, graph replay, D2H of its embeddings on a copy stream, "
-                         "host waits for batch i before batch i+2 is submitted"}
+    if not args.no_e2e:
+        e2e = run_e2e(args, cfg, g, neg, params, dev, tc, sampler, batch_of, world, rank, shard)
 
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        rate = oracle_rate_big if cfg.name in BIG else oracle_rate
-        r = rate(cfg, g, neg, params, [batch_of(i) for i in range(200)], args.cpu_seconds)
-        smp = (f"{r['roots']} roots of {r['batches']} batch(es) from 70% of the stream, one "
-               f"at a time by Listing 1's recursion (oracle/big.py), {r['seconds']:.1f} s"
-               if cfg.name in BIG else
-               f"{r['batches']} whole batch(es) ({r['roots']} roots) from 70% of the stream, "
-               f"{r['seconds']:.1f} s")
-        cpu = {"value": r["emb_per_s"], "unit": "embeddings/s", "cores": r["cores"],
-               "kind": "oracle", "sample": smp, "sampled_edges_per_s": r["edges_per_s"]}
+    if want_cpu:
+        if cfg.name != "MAG":
+            oth.join()
+        cpu = cpu_baseline(cfg, g, neg, params, [batch_of(i) for i in range(200)],
+                           args.cpu_seconds, oracle_box.get("runner"))
 
     if rank == 0:
         line = {"metric": METRIC, "value": emb_per_s, "unit": "embeddings/s",
                 "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
                 "ms_per_step": total_ms / args.steps, "higher_is_better": True,
-                "scaling": "weak", "vs_baseline": None, "dtype": {"fp32": "f32 (3-pass bf16 tensor-core split)",
-                                             "bf16": "bf16", "fp32_simt": "f32"}[args.precision], "data": "synthetic",
-                "config": {"workload": cfg.name, "batch_edges": cfg.batch, "roots_per_step": n0,
-                           "roots_per_step_all_ranks": world * n0, "layers": cfg.n_layers,
-                           "k": cfg.k, "strategy": cfg.strategy, "dedup": cfg.dedup,
-                           "precompute": cfg.precompute, "precision": args.precision,
-                           "cache_slots_per_layer": args.cache,
-                           "parallelism": f"root-sharded dp{world}" if world > 1 else "single",
-                           "l2": "flushed (256 MiB write) between timed steps",
-                           "timing": "CUDA events per step on the launch stream; max over ranks"},
+                "scaling": "strong", "vs_baseline": None,
+                "dtype": {"fp32": "f32 (3-pass bf16 tensor-core split)", "bf16": "bf16",
+                          "fp32_simt": "f32"}[args.precision],
+                "data": "synthetic (seeded generators shaped like PAPER.md Table 3)",
+                "config": config_dict(cfg, args, world, flush),
                 "sampled_edges_per_s": edges_per_s,
-                "tcsr_build_ms": tcsr_ms,
+                "sampler": sampler_line,
+                "tcsr": {"build_ms": tcsr_ms, "entries": M,
+                         "algorithmic_bytes": tcsr_bytes,
+                         "hbm_frac": tcsr_bytes / (tcsr_ms / 1e3) / 1e9 / hbm_peak,
+                         "timing": "second build (the first warms module load / first touch)"},
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
                 "gpu_launches": pipe.launches_per_forward * args.steps,
                 "gpu_launches_per_step": pipe.launches_per_forward,
-                "step_ms_p50": statistics.median(step_ms),
+                "step_ms_p50": statistics.median(step_ms) if step_ms else None,
                 "breakdown_ms_eager": {k_: statistics.median(v_) for k_, v_ in brk.items()}}
         print(json.dumps(line), flush=True)
     if world > 1:
@@ -582,10 +680,78 @@ def run_ours(args):
     return 0
 
 
+def run_e2e(args, cfg, g, neg, params, dev, tc, sampler, batch_of, world, rank, shard):
+    """The public serving loop: per batch the H2D of its edges from pinned host memory,
+    the captured chain, and the D2H of its root embeddings (rank 0 with N > 1), timed by
+    the host wall clock (max over ranks).  Warm-up batches are not among the timed ones."""
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    from paper_conf_asplos_wangm24_b200 import HostStream, TGATPipeline
+    from paper_conf_asplos_wangm24_b200.dist import ShardedRunner
+    n0 = 3 * cfg.batch
+    pipe_h = TGATPipeline(dev, tc, params, cfg.batch, sampler, cfg.dedup, cfg.precompute,
+                          cfg.window, args.precision, staging=True, cache_capacity=args.cache,
+                          shard=shard)
+    for a in pipe_h.attn:
+        a.set_kv_kernel(args.kv_kernel)
+    pipe_h.capture()
+    outs = [torch.empty(n0, cfg.d_model, dtype=torch.float32).pin_memory() for _ in range(2)]
+    n_warm = min(3, args.steps)
+    host_batches = []
+    for i in range(n_warm + args.steps):     # warm-up on batches the timed loop never sees
+        j = args.warmup + args.steps + 16 + i if i < n_warm else args.warmup + (i - n_warm)
+        sb, db, tb, nb_ = synth_batch(g, neg, batch_of(j))
+        host_batches.append(tuple(torch.from_numpy(np.ascontiguousarray(x)).pin_memory()
+                                  for x in (sb, db, tb, nb_)))
+    if shard is None:
+        hs = HostStream(pipe_h, n0, cfg.d_model)
+        submit = lambda i: hs.submit(*host_batches[i], outs[i % 2])
+    else:
+        run = ShardedRunner(pipe_h)
+        copy_stream = torch.cuda.Stream()
+
+        def submit(i):
+            for k_, h in zip(("src", "dst", "t", "neg"), host_batches[i]):
+                pipe_h.stage[k_].copy_(h, non_blocking=True)
+            e = run.step(0)
+            done = torch.cuda.Event()
+            with torch.cuda.stream(run.comm):
+                if rank == 0:
+                    outs[i % 2].copy_(e, non_blocking=True)
+                done.record(run.comm)
+            return done
+    for i in range(n_warm):
+        submit(i).synchronize()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    t0 = time.perf_counter()
+    prev = None
+    for i in range(n_warm, n_warm + args.steps):
+        done = submit(i)
+        if prev is not None:
+            prev.synchronize()
+        prev = done
+    prev.synchronize()
+    torch.cuda.synchronize()
+    el = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(el, op=dist.ReduceOp.MAX)
+    h2d = cfg.batch * (4 + 4 + 4 + 4)
+    return {"value": n0 * args.steps / float(el.item()), "unit": "embeddings/s",
+            "h2d_bytes_per_step": h2d * world, "d2h_bytes_per_step": n0 * cfg.d_model * 4,
+            "timing": "host wall clock over the serving loop: per batch H2D of its edges "
+                      "(every rank), graph replay, D2H of its embeddings on a copy stream; "
+                      "the host waits for batch i before batch i+2 is submitted"}
+
+
 def main():
     args = parse()
     if args.impl == "reference":
         return run_reference(args)
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return relaunch(args)
     return run_ours(args)
 
 

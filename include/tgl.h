@@ -202,6 +202,29 @@ tgl_status tgl_time_encode(int64_t n, const float* dt, int32_t d_t, const float*
  * Precision: TGL_FP32 splits every fp32 operand into bf16 hi + lo and runs three
  * MMA passes (hi*hi + lo*hi + hi*lo) with fp32 accumulation; TGL_BF16 one pass.
  * ------------------------------------------------------------------------- */
+/* Which K|V attention kernel runs (S6, S7, S9-S12; the dominant kernel).  AUTO picks
+ * SPLIT when every row table has a 16-byte pitch and max_seg <= 32, BIN for other
+ * pitches, GENERAL for max_seg > 32.  The others are kept as tested baselines. */
+#define TGL_KV_AUTO 0
+#define TGL_KV_SPLIT 1        /* split-role tcgen05 kernel; K chunks cut contiguously over
+                                 [h | e | Phi] when d_hsrc, d_e are multiples of 4, else
+                                 per-segment padded (reported as TGL_KV_SPLIT_PAD) */
+#define TGL_KV_SPLIT_PAD 2    /* split-role, per-segment padded K chunks */
+#define TGL_KV_ASYNC 3        /* single-role cp.async producers */
+#define TGL_KV_BIN 4          /* register-gather producers (any row pitch) */
+#define TGL_KV_GENERAL 5      /* any segment length */
+#define TGL_KV_SIMT 6         /* (reported only) the TGL_FP32_SIMT kernel */
+
+/* Measurement record (bench.py): when tgl_attn_params.probe != NULL the call records
+ * ev_start / ev_stop (cudaEvent_t, created by the caller) on its stream immediately
+ * before and after the K|V kernel and writes the TGL_KV_* id of the kernel that ran to
+ * `kernel`.  Never set it while capturing a CUDA graph. */
+typedef struct {
+  void* ev_start;
+  void* ev_stop;
+  int32_t kernel;
+} tgl_kv_probe;
+
 typedef struct {
   int32_t d_hdst, d_hsrc, d_e, d_t, d_model, n_heads, d_out;
   const float *Wq, *bq;           /* [d_model][d_hdst + d_t]          */
@@ -215,6 +238,9 @@ typedef struct {
   int32_t precision;              /* TGL_FP32 | TGL_BF16 | TGL_FP32_SIMT */
   const void* packed;             /* optional tgl_attn_pack() output for these weights and
                                      this precision; NULL = pack inside every call */
+  int32_t kv_kernel;              /* TGL_KV_AUTO (0) or a specific K|V kernel (TGL_KV_*);
+                                     a kernel that cannot take the call -> EUNSUPPORTED */
+  tgl_kv_probe* probe;            /* optional (NULL): caller-owned measurement record */
 } tgl_attn_params;
 
 /* Weight layout transform for the tensor-core path, done once per layer (the
@@ -235,19 +261,6 @@ tgl_status tgl_tblock_attn(const tgl_attn_params* P, int64_t n_dst_max, const in
                            int32_t max_seg, float* out, void* ws, size_t* ws_bytes,
                            void* stream);
 
-/* Measurement hook (bench.py): while armed (arm = 1; arming resets the records),
- * the first 8 tensor-core tgl_tblock_attn calls each record a pair of CUDA events
- * on their stream around their K|V attention kernel (S6, S7, S9-S12; the dominant
- * kernel).  tgl_kv_timing_ms(i) synchronises on the i-th stop event and returns
- * that kernel's duration in ms (negative if call i was not recorded).  Host-side
- * state, not thread-safe; measurement only (never armed during graph capture). */
-int tgl_kv_timing(int arm);
-float tgl_kv_timing_ms(int i);
-/* Which K|V kernel call i ran: 0 split-role (contiguous K chunks), 1 split-role (per-
- * segment padded K chunks), 2 single-role cp.async, 3 register-gather (rows without a
- * 16-byte pitch), 4 general (segments > 32 rows); -1 if call i was not recorded. */
-int tgl_kv_timing_kernel(int i);
-
 /* ---------------------------------------------------------------------------
  * S14  Dedup inverse applied to rows (the hook of P:279 / TGOpt dedup_invert
  * P:179): out[j][:] = table[idx[j]][:] for j < n, n = *n_dev (NULL -> n_max).
@@ -255,6 +268,31 @@ int tgl_kv_timing_kernel(int i);
 tgl_status tgl_gather_rows(int64_t n_max, const int64_t* n_dev, const int32_t* idx,
                            const float* table, int64_t ld_table, int32_t d, float* out,
                            int64_t ld_out, void* stream);
+
+/* ---------------------------------------------------------------------------
+ * S16  Root sharding across G ranks (the paper is single-GPU, P:424,
+ * and TGL's multi-GPU training is the contrast it names).  Every rank holds the
+ * whole graph, features and weights, forms the batch's roots (and dedups them when
+ * enabled) redundantly, and computes S4-S15 for the contiguous slice
+ * [r*c, min((r+1)*c, U)) of the U unique roots, c = ceil(U / world); embeddings
+ * depend only on <node, t> (content-keyed sampling, R6), so the slices compose.
+ *
+ * tgl_shard_slice: out[i] = (node, t)[lo + i] for the slice of `rank`; U = *n_dev
+ * (NULL -> n_max); capacities out_node/out_t[ceil(n_max / world)]; *out_n_dev = its
+ * length (device).
+ * tgl_shard_gather: after an all-gather of every rank's slice outputs padded to c_max
+ * rows (`gathered` = [world * c_max, d], rank-major), rebuild row j < n = *n_dev (NULL
+ * -> n_max): i = idx ? idx[j] : j (idx = the roots' dedup inverse, S14), out[j] =
+ * gathered[(i / c) * c_max + i % c] with c = ceil(U / world), U = *u_dev (NULL ->
+ * u_max).  Requires c_max >= ceil(u_max / world).  Errors: EINVAL.
+ * ------------------------------------------------------------------------- */
+tgl_status tgl_shard_slice(int64_t n_max, const int64_t* n_dev, const int32_t* node,
+                           const float* t, int32_t rank, int32_t world, int32_t* out_node,
+                           float* out_t, int64_t* out_n_dev, void* stream);
+tgl_status tgl_shard_gather(int64_t n_max, const int64_t* n_dev, const int32_t* idx,
+                            int64_t u_max, const int64_t* u_dev, int32_t world,
+                            const float* gathered, int64_t c_max, int32_t d, float* out,
+                            int64_t ld_out, void* stream);
 
 /* ---------------------------------------------------------------------------
  * N1  Embedding memoisation: the cache() operator ("previously computed
@@ -266,8 +304,8 @@ tgl_status tgl_gather_rows(int64_t n_max, const int64_t* n_dev, const int32_t* i
  *
  * Table: `capacity` slots (a power of two, <= 2^30), keys u64 [capacity] that
  * the caller zeroes once (0 = empty), vals fp32 [capacity, d] row-major.  A pair
- * (v, t) is keyed like dedup (node << 32 | order-preserving bits of t, -0 == +0,
- * R8); a NaN t never hits and is never stored (NaN != NaN).  Linear probing over
+ * (v, t) is keyed like dedup (node << 32 | raw fp32 bits of t with -0 canonicalised
+ * to +0, R8); a NaN t never hits and is never stored (NaN != NaN).  Linear probing over
  * at most TGL_CACHE_PROBES slots: a pair that finds no free slot is not stored,
  * so a full table only costs recomputation, never a wrong row (reading R22).
  * ------------------------------------------------------------------------- */

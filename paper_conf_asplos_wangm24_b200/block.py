@@ -55,7 +55,13 @@ class TGATPipeline:
     def __init__(self, graph: dict, tcsr: tgl.TemporalCSR, params: list, batch: int,
                  sampler: TSampler, use_dedup: bool, precompute: bool, window: int = 65536,
                  precision: str = "fp32", staging: bool = False, device=None,
-                 cache_capacity: int = 0):
+                 cache_capacity: int = 0, shard: tuple | None = None):
+        """shard = (rank, world): root sharding (S16).  The batch's roots
+        (deduped when use_dedup) are formed on every rank; this pipeline computes the
+        contiguous slice `rank` of them (tgl_shard_slice) and forward(slot) returns the
+        slice's embeddings [c_max, d_out] in `send[slot]`; `combine(slot, gathered)`
+        rebuilds the whole batch from the all-gathered slices (tgl_shard_gather).  Two
+        slots (two captured graphs) let batch b's all-gather overlap batch b+1."""
         self.dev = device or torch.device("cuda")
         self.g = graph
         self.tcsr = tcsr
@@ -73,9 +79,23 @@ class TGATPipeline:
         self.start_dev = torch.zeros(1, dtype=i64, device=self.dev)
         self.blocks = []
         n_max = 3 * batch
+        self.shard = shard
+        if shard is not None:
+            rank, world = shard
+            assert 0 <= rank < world and cache_capacity == 0
+            self.world = world
+            self.c_max = -(-n_max // world)          # rows per rank slice (padded)
+            # per slot: the batch's roots (S2) and, with dedup, their unique pairs + inverse
+            self.roots = []
+            for _ in range(2):
+                r = {"node": z(n_max, i32), "t": z(n_max, f32), "n": z(1, i64)}
+                if use_dedup:
+                    r.update(unode=z(n_max, i32), ut=z(n_max, f32), u=z(1, i64), inv=z(n_max, i32))
+                self.roots.append(r)
+            n_max = self.c_max
         for l in range(self.L):
             b = TBlock(l, n_max, z(n_max, i32), z(n_max, f32), z(1, i64))
-            if use_dedup:
+            if use_dedup and not (shard is not None and l == 0):   # sharded head: roots
                 b.uniq_node, b.uniq_t, b.u_dev, b.inv = z(n_max, i32), z(n_max, f32), z(1, i64), z(n_max, i32)
             else:
                 b.uniq_node, b.uniq_t, b.u_dev = b.dst_node, b.dst_t, b.n_dev
@@ -85,6 +105,9 @@ class TGATPipeline:
             self.blocks.append(b)
             n_max = n_max + n_max * k
         self.emb = z(3 * batch * self.attn[0].d_out, f32).view(-1, self.attn[0].d_out)
+        if shard is not None:   # the head block writes the slice into send[slot]
+            d0 = self.attn[0].d_out
+            self.send = [z(self.c_max * d0, f32).view(-1, d0) for _ in range(2)]
         # staging mode: the batch's edges arrive from host memory each step (public API)
         self.staging = staging
         if staging:
@@ -94,8 +117,11 @@ class TGATPipeline:
         # kernels launched per forward (libtgl only; memsets excluded)
         # dedup: one single-CTA kernel up to 4096 pairs (dedup.cu kSmallN), else three
         dedup_launches = [(1 if b.n_max <= 4096 else 3) if use_dedup else 0 for b in self.blocks]
+        if shard is not None:   # roots' dedup (before the slice) replaces block 0's + slice
+            dedup_launches[0] = ((1 if 3 * batch <= 4096 else 3) if use_dedup else 0) + 1
         per_block = [(1 if l > 0 else 0) + dedup_launches[l] + 1 + 3 for l in range(self.L)]
-        self.launches_per_forward = 1 + sum(per_block) + (1 if use_dedup else 0)
+        self.launches_per_forward = 1 + sum(per_block) + (1 if use_dedup and shard is None
+                                                          else 0)
         # cache() (TGOpt per-layer store, Listing 1 L23; inference): every
         # block's dst pairs after dedup are looked up in that layer's table; only the
         # misses are sampled and computed, then stored, and the combine hook rebuilds the
@@ -119,8 +145,12 @@ class TGATPipeline:
     # ------------------------------------------------------------------ workspaces
     def _alloc_workspaces(self):
         k = self.sampler.k
+        if self.shard is not None and self.use_dedup:
+            nb = tgl.ws_bytes("tgl_dedup", 3 * self.batch, None, None, None, None, None, None,
+                              None)
+            self.roots_ws = torch.empty(max(nb, 256), dtype=torch.uint8, device=self.dev)
         for b in self.blocks:
-            if self.use_dedup:
+            if self.use_dedup and b.inv is not None:
                 nb = tgl.ws_bytes("tgl_dedup", b.n_max, None, None, None, None, None, None, None)
                 b.ws["dedup"] = torch.empty(max(nb, 256), dtype=torch.uint8, device=self.dev)
             nb = tgl.ws_bytes("tgl_sample", C_TCSR(self.tcsr), b.n_max, None, None, None, k, 0,
@@ -132,13 +162,16 @@ class TGATPipeline:
             b.ws["attn"] = torch.empty(max(nb, 256), dtype=torch.uint8, device=self.dev)
 
     # ------------------------------------------------------------------ the batch
-    def forward(self, stream=None, record: dict | None = None):
+    def forward(self, stream=None, record: dict | None = None, slot: int = 0):
         """Enqueue one batch (edges [start, start+batch) with start = self.start_dev).
 
         record: optional dict; eager mode only -- CUDA events around each
-        tgl_tblock_attn call are stored as record[layer] = (start, end)."""
+        tgl_tblock_attn call are stored as record[layer] = (start, end).
+        slot: sharded mode only -- which roots / send buffers this batch uses."""
         g, k, s = self.g, self.sampler.k, stream
         b0 = self.blocks[0]
+        if self.shard is not None:
+            return self._forward_sharded(slot, s, record)
         marks = None if record is None else record.setdefault("_marks", [])
 
         def mark(name):
@@ -156,6 +189,12 @@ class TGATPipeline:
             tgl.batch_roots(self.batch, self.E, self.start_dev, g["src"], g["dst"], g["t"],
                             g["neg"], b0.dst_node, b0.dst_t, b0.n_dev, stream=s)
         mark("roots")
+        return self._chain(s, record, mark)
+
+    def _chain(self, s, record, mark):
+        """S3-S15 from block 0's dst pairs to the head output (b0.out / the roots)."""
+        g, k = self.g, self.sampler.k
+        b0 = self.blocks[0]
         for l, b in enumerate(self.blocks):
             if l > 0:  # S5 next_block (R14): [dst after dedup ; sampled src]
                 p = self.blocks[l - 1]
@@ -163,7 +202,7 @@ class TGATPipeline:
                                p.nbr, p.ts, b.dst_node, b.dst_t, b.n_dev, stream=s)
                 mark(f"next_block{l}")
             c = b.ws.get("cache")
-            if self.use_dedup:  # S3
+            if self.use_dedup and b.inv is not None:  # S3
                 un, ut, ud = ((c["node"], c["t"], c["u"]) if c is not None
                               else (b.uniq_node, b.uniq_t, b.u_dev))
                 _call_ws(tgl.lib().tgl_dedup,
@@ -222,6 +261,8 @@ class TGATPipeline:
                 tgl.cache_merge(c["table"], c["node"], c["t"], c["slot"], b.out,
                                 n_dev=c["u"], n_max=b.n_max, out=c["comb"], stream=s)
                 mark(f"cache_merge{l}")
+        if self.shard is not None:
+            return b0.out
         if self.cache_on:  # head: store + combine + S14 inverse in one launch
             c = b0.ws["cache"]
             tgl.cache_merge(c["table"], c["node"], c["t"], c["slot"], b0.out, idx=b0.inv,
@@ -235,6 +276,51 @@ class TGATPipeline:
             return self.emb
         return b0.out[:3 * self.batch]
 
+    def _forward_sharded(self, slot, s, record):
+        b0 = self.blocks[0]
+        marks = None if record is None else record.setdefault("_marks", [])
+
+        def mark(name):
+            if marks is not None:
+                ev = torch.cuda.Event(enable_timing=True)
+                ev.record(s if s is not None else torch.cuda.current_stream())
+                marks.append((name, ev))
+
+        mark("start")
+        r = self.roots[slot]
+        g = self.stage if self.staging else self.g
+        tgl.batch_roots(self.batch, self.stage_n if self.staging else self.E,
+                        None if self.staging else self.start_dev, g["src"], g["dst"], g["t"],
+                        g["neg"], r["node"], r["t"], r["n"], stream=s)
+        mark("roots")
+        un, ut, un_dev = r["node"], r["t"], r["n"]
+        if self.use_dedup:   # the roots' dedup, redundant on every rank (S3)
+            _call_ws(tgl.lib().tgl_dedup,
+                     [3 * self.batch, tgl._p(r["n"]), tgl._p(r["node"]), tgl._p(r["t"]),
+                      tgl._p(r["unode"]), tgl._p(r["ut"]), tgl._p(r["u"]), tgl._p(r["inv"])],
+                     self.roots_ws, s, "tgl_dedup")
+            un, ut, un_dev = r["unode"], r["ut"], r["u"]
+            mark("dedup_roots")
+        rank, world = self.shard
+        tgl.shard_slice(un, ut, rank, world, n_dev=un_dev, n_max=3 * self.batch,
+                        out=(b0.dst_node, b0.dst_t, b0.n_dev), stream=s)
+        mark("shard_slice")
+        b0.out = self.send[slot]
+        return self._chain(s, record, mark)
+
+    def combine(self, slot: int, gathered: torch.Tensor, out: torch.Tensor | None = None,
+                stream=None):
+        """Root embeddings of the batch in `slot` from the all-gathered slices
+        ([world * c_max, d], rank-major): S14 through the roots' inverse."""
+        r = self.roots[slot]
+        out = self.emb if out is None else out
+        n0 = 3 * self.batch
+        if self.use_dedup:
+            return tgl.shard_gather(gathered, self.c_max, self.world, n0, u_dev=r["u"],
+                                    idx=r["inv"], n_max=n0, n_dev=r["n"], out=out, stream=stream)
+        return tgl.shard_gather(gathered, self.c_max, self.world, n0, u_dev=r["n"], idx=None,
+                                n_max=n0, n_dev=r["n"], out=out, stream=stream)
+
     # ------------------------------------------------------------------ CUDA graph
     def capture(self):
         torch.cuda.synchronize()
@@ -245,6 +331,15 @@ class TGATPipeline:
                 self.forward()
         torch.cuda.current_stream().wait_stream(s)
         torch.cuda.synchronize()
+        if self.shard is not None:        # one graph per slot (its own roots / send)
+            self.graphs = []
+            for slot in range(2):
+                gs = torch.cuda.CUDAGraph()
+                with torch.cuda.graph(gs):
+                    self.forward(slot=slot)
+                self.graphs.append(gs)
+            self.graph_exec, self.graph_out = self.graphs[0], self.send[0]
+            return self.graphs
         g = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g):
             out = self.forward()
@@ -252,9 +347,12 @@ class TGATPipeline:
         self.graph_out = out
         return g
 
-    def run_graph(self, start: int | None = None):
+    def run_graph(self, start: int | None = None, slot: int = 0):
         if start is not None:
             self.start_dev.fill_(start)
+        if self.shard is not None:
+            self.graphs[slot].replay()
+            return self.send[slot]
         self.graph_exec.replay()
         return self.graph_out
 

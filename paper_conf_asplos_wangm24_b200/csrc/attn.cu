@@ -10,9 +10,9 @@
 //                   segmented softmax (S11) and the alpha-weighted scatter-sum
 //                   (S12) finish in shared memory; only r_i leaves the SM.
 //   3. out_ffn    : out_i = LayerNorm(ReLU(Wo [r_i ; h_i] + bo))      (S13)
-// This file is the SIMT (FFMA) implementation used for TGL_FP32; projections run
-// on CUDA cores with fp32 accumulation.  TGL_BF16 rounds the projection operands
-// to bf16 (RNE) before the same FMAs.
+// This file is the SIMT (FFMA) implementation, selected by TGL_FP32_SIMT (exact fp32
+// products on the CUDA cores, fp32 accumulation; the slow reference mode).  TGL_FP32
+// and TGL_BF16 run on the tensor cores (attn_tc.cu); tgl_tblock_attn below dispatches.
 #include <cuda_bf16.h>
 
 #include "common.cuh"
@@ -526,8 +526,14 @@ extern "C" tgl_status tgl_tblock_attn(const tgl_attn_params* P, int64_t n_dst_ma
   const unsigned g64 = (unsigned)ceil_div(n_dst_max, kTBM);
   q_proj_kernel<<<g64, kAttnThreads, 0, s>>>(a);
   TGL_TRY(launch_check("q_proj"));
+  tgl_kv_probe* probe = P->probe;
+  if (probe) probe->kernel = TGL_KV_SIMT;
+  if (probe && probe->ev_start)
+    TGL_TRY(cuda_check(cudaEventRecord(static_cast<cudaEvent_t>(probe->ev_start), s), "probe"));
   kv_attn_kernel<<<(unsigned)ceil_div(n_dst_max, a.dpb), kAttnThreads, 0, s>>>(a);
   TGL_TRY(launch_check("kv_attn"));
+  if (probe && probe->ev_stop)
+    TGL_TRY(cuda_check(cudaEventRecord(static_cast<cudaEvent_t>(probe->ev_stop), s), "probe"));
   out_ffn_kernel<<<g64, kAttnThreads, 0, s>>>(a);
   return launch_check("out_ffn");
 }

@@ -184,6 +184,10 @@ struct Pipe {
   }
 };
 
+// ---- profiling instrumentation: compiled only into probe builds (-DTGL_PROBE, tools/);
+// product builds have no debug state, read no environment and take no debug branches
+#ifdef TGL_PROBE
+#define TGL_DBG(a) ((a).dbg)
 // ---- profiling timeline (TGL_DEBUG_MASK & 32): [cta][tile][event] globaltimer stamps
 constexpr int kTlTiles = 32, kTlEvents = 8;
 __device__ unsigned long long g_timeline[kNumSMs * kTlTiles * kTlEvents];
@@ -216,6 +220,16 @@ __device__ __forceinline__ void tl_mark(const Args& a, uint32_t tt, int ev) {
     g_timeline[(blockIdx.x * kTlTiles + tt) * kTlEvents + ev] = t;
   }
 }
+
+#define TGL_TRACE_RESET() \
+  if (threadIdx.x < 32) s_trace_n[threadIdx.x] = 0
+#else
+#define TGL_DBG(a) 0
+#define TGL_TRACE_RESET() (void)0
+__device__ __forceinline__ void trace(const Args&, int, uint32_t) {}
+__device__ __forceinline__ void prof_add(const Args&, int, long long) {}
+__device__ __forceinline__ void tl_mark(const Args&, uint32_t, int) {}
+#endif
 
 __device__ __forceinline__ void named_bar(int id, int n) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
@@ -524,7 +538,7 @@ __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
       s_v1[j] = P.bk[j];
     }
   }
-  if (threadIdx.x < 32) s_trace_n[threadIdx.x] = 0;
+  TGL_TRACE_RESET();
   if ((threadIdx.x & 31) == 0) trace(a, 36, 0);     // per-warp start stamp
   ws_init(B, &s_tmem, 2 * kCols);
   const uint32_t tmem = s_tmem;
@@ -771,7 +785,7 @@ __global__ void __launch_bounds__(kWsThreads, 1) kv_kernel(Args a) {
       const uint32_t ds = tt % kDSlots;
       mbar_wait(&B.dfull[ds], (tt / kDSlots) & 1u);
       produce_tile<kNPkv, kProdWarp0, kGPT>(a.skv, split, pipe, B, ait, tt, rd[ds], s_omega,
-                                            s_phi, a.table, (a.dbg & 2) != 0);
+                                            s_phi, a.table, (TGL_DBG(a) & 2) != 0);
       warp_arrive(&B.dempty[ds]);
     }
   } else if (warp == kMmaWarp) {                     // ---------------- MMA issuer
@@ -779,7 +793,7 @@ __global__ void __launch_bounds__(kWsThreads, 1) kv_kernel(Args a) {
     if (lane == 0)
       for (; sched.next(t0, rows); ++tt)
         mma_tile<kNPkv, kNPkv>(a.skv, split, pipe, B, tmem + (tt & 1u) * kCols, ait, wit, tt,
-                               (a.dbg & 4) != 0);
+                               (TGL_DBG(a) & 4) != 0);
     __syncwarp();
   } else {                                           // ---------------- epilogue (128 threads)
     const int tid = threadIdx.x;                      // 0..127
@@ -830,7 +844,7 @@ __global__ void __launch_bounds__(kWsThreads, 1) kv_kernel(Args a) {
         tc_fence_after();
         const int d = rd[ds].rdst[row];
         warp_arrive(&B.dempty[ds]);
-        if (a.dbg & 1) {
+        if (TGL_DBG(a) & 1) {
           tc_fence_before();
           warp_arrive(&B.tempty[ab]);
           continue;
@@ -1022,7 +1036,7 @@ __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uin
     if (warp == 0) prof_add(a, 11, e1c - e0c);      // epilogue: wait for the accumulator
     tc_fence_after();
     if (threadIdx.x == 0) tl_mark(a, tt, 6);
-    if (a.dbg & 1) {
+    if (TGL_DBG(a) & 1) {
       tc_fence_before();
       warp_arrive(&tempty[ab]);
       continue;
@@ -1208,11 +1222,11 @@ __global__ void __launch_bounds__(kBThreads, 1) kv_bin_kernel(Args a) {
         float et[4];
 #pragma unroll
         for (int u = 0; u < 4; ++u) {              // all loads of the lane's 4 rows in flight
-          const bool ok = dst[u] >= 0 && !(a.dbg & 16);
+          const bool ok = dst[u] >= 0 && !(TGL_DBG(a) & 16);
           hi[u] = ok ? (a.hsrc_idx ? a.hsrc_idx[hoff + e[u]] : (int32_t)(hoff + e[u])) : 0;
           ei[u] = (ok && P.d_e > 0) ? a.eid[e[u]] : 0;
-          if (a.dbg & 128) ei[u] &= 0x3FF;            // profiling: edge rows in 700 KB
-          if (a.dbg & 256) hi[u] &= 0x3FF;
+          if (TGL_DBG(a) & 128) ei[u] &= 0x3FF;            // profiling: edge rows in 700 KB
+          if (TGL_DBG(a) & 256) hi[u] &= 0x3FF;
           et[u] = ok ? a.edge_t[e[u]] : 0.f;
         }
 #pragma unroll
@@ -1238,7 +1252,7 @@ __global__ void __launch_bounds__(kBThreads, 1) kv_bin_kernel(Args a) {
       const int live = bd[ds].live;
       warp_arrive(&B.dempty[ds]);
       if (!live) break;
-      if (lane == 0 && !(a.dbg & 8)) wload_tile<kNPkv>(a.skv, pipe, B, a.wkv, wl, tt);
+      if (lane == 0 && !(TGL_DBG(a) & 8)) wload_tile<kNPkv>(a.skv, pipe, B, a.wkv, wl, tt);
       __syncwarp();
     }
   } else if (warp >= kBProd0) {                      // ---------------- producers
@@ -1252,7 +1266,7 @@ __global__ void __launch_bounds__(kBThreads, 1) kv_bin_kernel(Args a) {
       }
       if (threadIdx.x == kBProd0 * 32) tl_mark(a, tt, 2);
       produce_tile<kNPkv, kBProd0, kBGPT>(a.skv, split, pipe, B, ait, tt, bd[ds], s_omega,
-                                          s_phi, a.table, (a.dbg & 2) != 0, a.dbg);
+                                          s_phi, a.table, (TGL_DBG(a) & 2) != 0, TGL_DBG(a));
       if (threadIdx.x == kBProd0 * 32) tl_mark(a, tt, 3);
       warp_arrive(&B.dempty[ds]);
     }
@@ -1267,7 +1281,7 @@ __global__ void __launch_bounds__(kBThreads, 1) kv_bin_kernel(Args a) {
       if (lane == 0) tl_mark(a, tt, 4);
       if (lane == 0)
         mma_tile<kNPkv, kNPkv>(a.skv, split, pipe, B, tmem + (tt & 1u) * kCols, ait, wl, tt,
-                               (a.dbg & 4) != 0, (a.dbg & 8) != 0);
+                               (TGL_DBG(a) & 4) != 0, (TGL_DBG(a) & 8) != 0);
       __syncwarp();
     }
   } else {                                           // ---------------- epilogue warps 0-7
@@ -1488,7 +1502,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
     }
     fence_mbar_init();
   }
-  if (threadIdx.x < 32) s_trace_n[threadIdx.x] = 0;
+  TGL_TRACE_RESET();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (warp == kTMma) tmem_alloc(&s_tmem, 2 * kCols);
   tc_fence_before();
@@ -1566,12 +1580,12 @@ __global__ void __launch_bounds__(kTThreads, 1)
       float et[4];
 #pragma unroll
       for (int u = 0; u < 4; ++u) {                   // all loads of the lane's 4 rows in flight
-        const bool ok = dr[u] >= 0 && !(a.dbg & 16);
+        const bool ok = dr[u] >= 0 && !(TGL_DBG(a) & 16);
         hi[u] = ok ? (a.hsrc_idx ? a.hsrc_idx[hoff + er[u]] : (int32_t)(hoff + er[u])) : 0;
         ei[u] = (ok && P.d_e > 0) ? a.eid[er[u]] : 0;
         et[u] = ok ? a.edge_t[er[u]] : 0.f;
-        if (a.dbg & 128) ei[u] &= 0x3FF;              // profiling: edge rows in 700 KB
-        if (a.dbg & 256) hi[u] &= 0x3FF;
+        if (TGL_DBG(a) & 128) ei[u] &= 0x3FF;              // profiling: edge rows in 700 KB
+        if (TGL_DBG(a) & 256) hi[u] &= 0x3FF;
       }
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
@@ -1604,7 +1618,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
           const uint32_t k = wl + (i - r0);
           const uint32_t sw = k % kTWStages;
           wait_free_sleep(&B.wempty[sw], k / kTWStages, 500);
-          if (a.dbg & 8) {
+          if (TGL_DBG(a) & 8) {
             mbar_arrive(&B.wfull[sw]);
             continue;
           }
@@ -1661,7 +1675,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
           const uint32_t sb = pipe_s + s * kTAStage + rw0 * 128 + j * 16;
           const int cb = col + 4 * j;                // first fp32 column of this lane
           const uint32_t nb = cb >= width ? 0u : (uint32_t)min(16, (width - cb) * 4);
-          if (!(a.dbg & 2)) {
+          if (!(TGL_DBG(a) & 2)) {
             const float* base = seg == 0 ? a.hsrc : (seg == 1 ? a.efeat : a.table);
             const int64_t ld = seg == 0 ? a.ld_hsrc : (seg == 1 ? a.ld_e : (int64_t)P.d_t);
             const int x0 = seg == 0 ? hr0 : (seg == 1 ? er0 : tr0);
@@ -1716,7 +1730,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
       for (int q = 0; q < 2; ++q) {
         if (q >= cnt) break;
         const int c = chunk_of(ct, i0 + q, nch);
-        if (c >= plan.c[0] + plan.c[1] && !(a.dbg & 1024)) {   // time chunk: Phi where the table misses
+        if (c >= plan.c[0] + plan.c[1] && !(TGL_DBG(a) & 1024)) {   // time chunk: Phi where the table misses
           const int cc = col_of_time(plan, c) + 4 * j;
           float w[4], f[4];
 #pragma unroll
@@ -1740,7 +1754,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
         }
       }
       __syncwarp();
-      if (!(a.dbg & 64)) {
+      if (!(TGL_DBG(a) & 64)) {
         const uint32_t o0 = sw64_off(rr, 4 * j), o1 = sw64_off(rr + 4, 4 * j);
 #pragma unroll
         for (int q = 0; q < 2; ++q) {
@@ -1760,7 +1774,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
 #undef TGL_SPLIT_STORE
         }
       }
-      if (!(a.dbg & 2048)) fence_proxy_async_smem();   // 2048: profiling only (unsafe)
+      if (!(TGL_DBG(a) & 2048)) fence_proxy_async_smem();   // 2048: profiling only (unsafe)
       __syncwarp();
       if (pw == 0) trace(a, 4, uc);
       if (lane == 0) {
@@ -1823,7 +1837,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
             if (q >= cnt) break;
             const uint32_t ab = pipe_s + st[q] * kTAStage;
             const uint32_t wb = w_s + (kw[q] % kTWStages) * kTWStage;
-            const int nk = (a.dbg & 4) ? 0 : plan_ksteps(plan, cc[q]);
+            const int nk = (TGL_DBG(a) & 4) ? 0 : plan_ksteps(plan, cc[q]);
             for (int ks = 0; ks < nk; ++ks) {
               const uint64_t ah = desc_sw64(ab + ks * 32, 1024), bh = desc_sw64(wb + ks * 32, 512);
               mma_bf16(acc, ah, bh, idesc, ((i + q) | ks) != 0);
@@ -1997,7 +2011,7 @@ __global__ void __launch_bounds__(kSThreads, 1)
     }
     fence_mbar_init();
   }
-  if (threadIdx.x < 32) s_trace_n[threadIdx.x] = 0;
+  TGL_TRACE_RESET();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (warp == kTMma) tmem_alloc(&s_tmem, 2 * kCols);
   tc_fence_before();
@@ -2104,7 +2118,7 @@ __global__ void __launch_bounds__(kSThreads, 1)
           const uint32_t sw = k % kSW;
           wait_free_sleep(&B.wempty[sw], k / kSW, TGL_SLEEP_W);
           trace(a, 11, k);
-          if (a.dbg & 8) {                           // profiling: no weight bytes
+          if (TGL_DBG(a) & 8) {                           // profiling: no weight bytes
             mbar_arrive(&B.wfull[sw]);
             continue;
           }
@@ -2163,7 +2177,7 @@ __global__ void __launch_bounds__(kSThreads, 1)
         TGL_PROF_CLK(l1);
         const uint32_t dst = f_s + sf * kSStage + lofs;
 #pragma unroll
-        if (!(a.dbg & 2))                            // profiling: no gathers
+        if (!(TGL_DBG(a) & 2))                            // profiling: no gathers
 #pragma unroll
           for (int k = 0; k < 8; ++k)
             if (x[k] >= 0) cp_async16_zfill(dst + k * 512, b + (int64_t)x[k] * ld, nb);
@@ -2225,7 +2239,7 @@ __global__ void __launch_bounds__(kSThreads, 1)
         if (cw == 0) trace(a, 3, g);
         float4 x[kSKc];
         const uint32_t src = f_s + sf * kSStage + lofs;
-        if (a.dbg & 64) {                            // profiling: no conversion work
+        if (TGL_DBG(a) & 64) {                            // profiling: no conversion work
           wait_free(&B.bempty[sb], g / kSB);
           __syncwarp();
           if (lane == 0) {
@@ -2363,7 +2377,7 @@ __global__ void __launch_bounds__(kSThreads, 1)
           // 14-bit start-address field (addr >> 4) by plain adds (no carry: smem < 256 KB)
           const uint64_t a0 = desc_sw64(b_s + sb * kSStage, 1024);
           const uint64_t w0 = desc_sw64(w_s + (kw % kSW) * kTWStage, 512);
-          if (!(a.dbg & 4)) {                        // profiling: no MMAs
+          if (!(TGL_DBG(a) & 4)) {                        // profiling: no MMAs
 #pragma unroll
             for (int ks = 0; ks < 2; ++ks) {
               if (ks < nk) {
@@ -2377,7 +2391,7 @@ __global__ void __launch_bounds__(kSThreads, 1)
             }
           }
           const bool keep = (nch >= 4) && (i >= nch - 2);   // reused by the next tile
-          if (a.dbg & 8192) {                        // profiling: plain arrives, no commit
+          if (TGL_DBG(a) & 8192) {                        // profiling: plain arrives, no commit
             mbar_arrive(&B.bempty[sb]);
             if (!keep) mbar_arrive(&B.wempty[kw % kSW]);
           } else {
@@ -2455,15 +2469,32 @@ static bool rows_16b(const float* base, int width, int64_t ld) {
 
 }  // namespace tca
 
-// host entry used by tgl_tblock_attn (attn.cu) for TGL_FP32 / TGL_BF16
-// measurement hook state (tgl_kv_timing): host-side only, armed by bench.py
-constexpr int kKvEvMax = 8;
-static bool g_kv_armed = false;
-static int g_kv_n = 0;                               // K|V launches recorded since arming
-static cudaEvent_t g_kv_ev[kKvEvMax][2] = {};
-static int g_kv_kind[kKvEvMax] = {};                 // 0 split/contig, 1 split/padded, 2 async,
-                                                     // 3 bin, 4 general
+// dynamic shared memory opt-in of every tensor-core kernel (per device, once)
+static tgl_status set_smem_attrs(int smem_q, int smem_kv, int smem_kvb) {
+  using namespace tca;
+  static PerDeviceOnce once;
+  return cuda_check(once.run([=] {
+    cudaError_t e = cudaFuncSetAttribute(dense_kernel<false>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, smem_q);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(dense_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               smem_q);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(kv_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_kv);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(kv_bin_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               smem_kvb);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(kv_async_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               kTSmem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(kv_split_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               kSSmem);
+    return e;
+  }), "smem attributes");
+}
 
+// host entry used by tgl_tblock_attn (attn.cu) for TGL_FP32 / TGL_BF16
 size_t tc_attn_ws_bytes(const tgl_attn_params* P, int64_t n_dst_max, size_t* o_q, size_t* o_r,
                         size_t* o_pack) {
   using namespace tca;
@@ -2530,97 +2561,83 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
   int dpb = kBM / ms;
   a.dpb = dpb < 1 ? 1 : (dpb > kMaxDpb ? kMaxDpb : dpb);
   a.split = P->precision == TGL_FP32 ? 1 : 0;
-  a.dbg = getenv("TGL_DEBUG_MASK") ? atoi(getenv("TGL_DEBUG_MASK")) : 0;
+#ifdef TGL_PROBE
+  a.dbg = getenv("TGL_DEBUG_MASK") ? atoi(getenv("TGL_DEBUG_MASK")) : 0;   // probe builds only
+#else
+  a.dbg = 0;
+#endif
 
   const int smem_q = Pipe<kNPq>::kBytes + 1024;
   const int smem_kv = Pipe<kNPkv>::kBytes + 1024 + kKvEpiBytes;
   const int smem_kvb = Pipe<kNPkv>::kBytes + 1024 + kBEpi * 32 * 33 * 4;
-  // TGL_KV (tests / probes only): "bin" forces the register-gather kernel, "async" the
-  // single-role LDGSTS kernel, "split" / "split_pad" the split-role kernel with the
-  // contiguous / per-segment-padded K plan (default: split, contiguous when possible)
-  const char* kvsel = getenv("TGL_KV");
-  static bool attr_done = false;   // cached cudaFuncSetAttribute (idempotent)
-  if (!attr_done) {
-    TGL_TRY(cuda_check(cudaFuncSetAttribute(dense_kernel<false>,
-                                            cudaFuncAttributeMaxDynamicSharedMemorySize, smem_q),
-                       "attr q"));
-    TGL_TRY(cuda_check(cudaFuncSetAttribute(dense_kernel<true>,
-                                            cudaFuncAttributeMaxDynamicSharedMemorySize, smem_q),
-                       "attr ffn"));
-    TGL_TRY(cuda_check(cudaFuncSetAttribute(kv_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                            smem_kv), "attr kv"));
-    TGL_TRY(cuda_check(cudaFuncSetAttribute(kv_bin_kernel,
-                                            cudaFuncAttributeMaxDynamicSharedMemorySize, smem_kvb),
-                       "attr kv bin"));
-    TGL_TRY(cuda_check(cudaFuncSetAttribute(kv_async_kernel,
-                                            cudaFuncAttributeMaxDynamicSharedMemorySize, kTSmem),
-                       "attr kv async"));
-    TGL_TRY(cuda_check(cudaFuncSetAttribute(kv_split_kernel,
-                                            cudaFuncAttributeMaxDynamicSharedMemorySize, kSSmem),
-                       "attr kv split"));
-    attr_done = true;
-  }
+  TGL_TRY(set_smem_attrs(smem_q, smem_kv, smem_kvb));
   const int64_t tiles = ceil_div(n_dst_max, kBM);
   const unsigned gq = (unsigned)(tiles < kNumSMs ? tiles : kNumSMs);
   launch_pdl(dense_kernel<false>, dim3(gq), dim3(kWsThreads), smem_q, s, a);
   TGL_TRY(launch_check("tc q kernel"));
+  const int sel = P->kv_kernel;
+  if (sel < TGL_KV_AUTO || sel > TGL_KV_GENERAL) {
+    set_error("kv_kernel %d: not a TGL_KV_* id", sel);
+    return TGL_EINVAL;
+  }
   const bool binned = max_seg > 0 && max_seg <= 32 && P->n_heads == 2;
-  const bool async = binned && !(kvsel && strcmp(kvsel, "bin") == 0) &&
-                     rows_16b(hsrc, P->d_hsrc, ld_hsrc) && rows_16b(efeat, P->d_e, ld_e) &&
+  const bool async = binned && rows_16b(hsrc, P->d_hsrc, ld_hsrc) && rows_16b(efeat, P->d_e, ld_e) &&
                      rows_16b(table, table ? P->d_t : 0, P->d_t);
-  // default: the split-role kernel; TGL_KV=async keeps the single-role LDGSTS producers
-  const bool use_split = async && !(kvsel && strcmp(kvsel, "async") == 0);
-  if (kvsel && (strcmp(kvsel, "async") == 0 || strcmp(kvsel, "split") == 0 ||
-                strcmp(kvsel, "split_pad") == 0) && !async) {
-    set_error("TGL_KV=async: the async-gather path cannot take this call (16-B row pitch / "
-              "max_seg <= 32 / 2 heads)");
-    return TGL_EUNSUPPORTED;
+  const bool contig = contig_ok(P->d_hsrc, P->d_e);
+  int kind;
+  if (sel == TGL_KV_AUTO) {
+    kind = async ? TGL_KV_SPLIT : (binned ? TGL_KV_BIN : TGL_KV_GENERAL);
+  } else {
+    kind = sel;
+    const bool ok = (sel == TGL_KV_GENERAL) || (sel == TGL_KV_BIN && binned) ||
+                    ((sel == TGL_KV_SPLIT || sel == TGL_KV_SPLIT_PAD || sel == TGL_KV_ASYNC) &&
+                     async);
+    if (!ok) {
+      set_error("kv_kernel %d cannot take this call (16-byte row pitches, max_seg <= 32, "
+                "2 heads)", sel);
+      return TGL_EUNSUPPORTED;
+    }
   }
-  const bool kv_rec = g_kv_armed && g_kv_n < kKvEvMax;
-  int kv_kind = 4;
-  if (kv_rec) {
-    for (int e = 0; e < 2; ++e)
-      if (g_kv_ev[g_kv_n][e] == nullptr)
-        TGL_TRY(cuda_check(cudaEventCreate(&g_kv_ev[g_kv_n][e]), "event"));
-    TGL_TRY(cuda_check(cudaEventRecord(g_kv_ev[g_kv_n][0], s), "event record"));
+  if (kind == TGL_KV_SPLIT && !contig) kind = TGL_KV_SPLIT_PAD;   // plan follows the widths
+  tgl_kv_probe* probe = P->probe;
+  if (probe) {
+    probe->kernel = kind;
+    if (probe->ev_start)
+      TGL_TRY(cuda_check(cudaEventRecord(static_cast<cudaEvent_t>(probe->ev_start), s),
+                         "probe event"));
   }
-  if (use_split) {
+  if (kind == TGL_KV_SPLIT || kind == TGL_KV_SPLIT_PAD) {
     const int bdst = 32 / max_seg;                 // destinations per 32-row bin
     const int64_t ttiles = ceil_div(n_dst_max, 4 * bdst);
     const unsigned gt = (unsigned)(ttiles < kNumSMs ? (ttiles > 0 ? ttiles : 1) : kNumSMs);
-    const bool contig = contig_ok(P->d_hsrc, P->d_e) && !(kvsel && strcmp(kvsel, "split_pad") == 0);
-    const KvPlan plan = contig ? make_plan_contig(P->d_hsrc, P->d_e, P->d_t)
-                               : make_plan(P->d_hsrc, P->d_e, P->d_t);
+    const bool cplan = kind == TGL_KV_SPLIT;
+    const KvPlan plan = cplan ? make_plan_contig(P->d_hsrc, P->d_e, P->d_t)
+                              : make_plan(P->d_hsrc, P->d_e, P->d_t);
     if (plan.n > kSMaxChunks) {
       set_error("K|V attention: %d K chunks > %d", plan.n, kSMaxChunks);
       return TGL_EUNSUPPORTED;
     }
-    launch_pdl(kv_split_kernel, dim3(gt), dim3(kSThreads), kSSmem, s, a, plan, pk + (contig ? PL.okvc : PL.okv64),
-                                                  bdst);
-    kv_kind = contig ? 0 : 1;
-  } else if (async) {
+    launch_pdl(kv_split_kernel, dim3(gt), dim3(kSThreads), kSSmem, s, a, plan,
+               pk + (cplan ? PL.okvc : PL.okv64), bdst);
+  } else if (kind == TGL_KV_ASYNC) {
     const int bdst = 32 / max_seg;                 // destinations per 32-row bin
     const int64_t ttiles = ceil_div(n_dst_max, 4 * bdst);
     const unsigned gt = (unsigned)(ttiles < kNumSMs ? (ttiles > 0 ? ttiles : 1) : kNumSMs);
-    launch_pdl(kv_async_kernel, dim3(gt), dim3(kTThreads), kTSmem, s, a, make_plan(P->d_hsrc, P->d_e, P->d_t),
-                                                  pk + PL.okv64, bdst);
-    kv_kind = 2;
-  } else if (binned) {
+    launch_pdl(kv_async_kernel, dim3(gt), dim3(kTThreads), kTSmem, s, a,
+               make_plan(P->d_hsrc, P->d_e, P->d_t), pk + PL.okv64, bdst);
+  } else if (kind == TGL_KV_BIN) {
     // binned path: whole segments per epilogue warp (no block barriers)
     const unsigned gkv = (unsigned)(n_dst_max < kNumSMs ? (n_dst_max > 0 ? n_dst_max : 1) : kNumSMs);
     launch_pdl(kv_bin_kernel, dim3(gkv), dim3(kBThreads), smem_kvb, s, a);
-    kv_kind = 3;
   } else {
     const int64_t groups = ceil_div(n_dst_max, a.dpb);
     const unsigned gkv = (unsigned)(groups < kNumSMs ? groups : kNumSMs);
     launch_pdl(kv_kernel, dim3(gkv), dim3(kWsThreads), smem_kv, s, a);
   }
   TGL_TRY(launch_check("tc kv kernel"));
-  if (kv_rec) {
-    TGL_TRY(cuda_check(cudaEventRecord(g_kv_ev[g_kv_n][1], s), "event record"));
-    g_kv_kind[g_kv_n] = kv_kind;
-    ++g_kv_n;
-  }
+  if (probe && probe->ev_stop)
+    TGL_TRY(cuda_check(cudaEventRecord(static_cast<cudaEvent_t>(probe->ev_stop), s),
+                       "probe event"));
   launch_pdl(dense_kernel<true>, dim3(gq), dim3(kWsThreads), smem_q, s, a);
   return launch_check("tc ffn kernel");
 }
@@ -2628,32 +2645,6 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
 }  // namespace tgl
 
 using namespace tgl;
-
-// profiling aid (not part of the documented ABI): copy the per-tile timeline
-extern "C" int tgl_debug_timeline(unsigned long long* host, size_t n) {
-  const size_t cap = sizeof(tca::g_timeline) / sizeof(unsigned long long);
-  return (int)cudaMemcpyFromSymbol(host, tca::g_timeline,
-                                   (n < cap ? n : cap) * sizeof(unsigned long long));
-}
-
-extern "C" int tgl_kv_timing(int arm) {
-  tgl::g_kv_armed = arm != 0;
-  if (arm) tgl::g_kv_n = 0;                        // disarming keeps the records
-  return 0;
-}
-
-extern "C" int tgl_kv_timing_kernel(int i) {
-  return (i < 0 || i >= tgl::g_kv_n) ? -1 : tgl::g_kv_kind[i];
-}
-
-extern "C" float tgl_kv_timing_ms(int i) {
-  if (i < 0 || i >= tgl::g_kv_n) return -1.f;
-  float ms = -1.f;
-  if (cudaEventSynchronize(tgl::g_kv_ev[i][1]) != cudaSuccess) return -1.f;
-  if (cudaEventElapsedTime(&ms, tgl::g_kv_ev[i][0], tgl::g_kv_ev[i][1]) != cudaSuccess)
-    return -1.f;
-  return ms;
-}
 
 extern "C" size_t tgl_attn_packed_bytes(const tgl_attn_params* P) {
   if (P == nullptr || !tc_attn_supported(P)) return 0;
@@ -2676,6 +2667,14 @@ extern "C" tgl_status tgl_attn_pack(const tgl_attn_params* P, void* packed, size
   return tca::launch_pack(P, static_cast<uint8_t*>(packed), as_stream(stream));
 }
 
+#ifdef TGL_PROBE
+// probe builds only (tools/): read back the instrumentation buffers
+extern "C" int tgl_debug_timeline(unsigned long long* host, size_t n) {
+  const size_t cap = sizeof(tca::g_timeline) / sizeof(unsigned long long);
+  return (int)cudaMemcpyFromSymbol(host, tca::g_timeline,
+                                   (n < cap ? n : cap) * sizeof(unsigned long long));
+}
+
 extern "C" int tgl_debug_prof(unsigned long long* host, int reset) {
   if (reset) {
     static unsigned long long z[tgl::kNumSMs * 16];
@@ -2691,3 +2690,4 @@ extern "C" int tgl_debug_trace(unsigned long long* host, int reset) {
   }
   return (int)cudaMemcpyFromSymbol(host, tgl::tca::g_trace, sizeof(unsigned long long) * 8192);
 }
+#endif  // TGL_PROBE

@@ -243,13 +243,12 @@ extern "C" tgl_status tgl_dedup(int64_t n_max, const int64_t* n_dev, const int32
   TGL_REQUIRE(n_max == 0 || (node && t && uniq_node && uniq_t && inv), "null pointer");
   cudaStream_t s = as_stream(stream);
   if (n_max <= kSmallN) {                        // one CTA, shared-memory table
-    static bool attr = false;
-    if (!attr) {
-      TGL_TRY(cuda_check(cudaFuncSetAttribute(dedup_small_kernel,
-                                              cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                              kSmallSmem), "dedup attr"));
-      attr = true;
-    }
+    static PerDeviceOnce attr;
+    TGL_TRY(cuda_check(attr.run([] {
+                         return cudaFuncSetAttribute(dedup_small_kernel,
+                                                     cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                     kSmallSmem);
+                       }), "dedup attr"));
     launch_pdl(dedup_small_kernel, dim3(1), dim3(kSmallThreads), kSmallSmem, s, n_max, n_dev, node, t, uniq_node,
                                                             uniq_t, num_uniq_dev, inv);
     return launch_check("dedup_small");

@@ -19,15 +19,19 @@ TGL_UNDIRECTED = 1
 TGL_INPUT_TIME_SORTED = 2
 RECENT, UNIFORM = 0, 1
 FP32, BF16, FP32_SIMT = 0, 1, 2
+# tgl_attn_params.kv_kernel (include/tgl.h TGL_KV_*)
+KV_KERNEL = {"auto": 0, "split": 1, "split_pad": 2, "async": 3, "bin": 4, "general": 5}
+KV_KERNEL_NAME = {1: "kv_split_kernel (contiguous K plan)", 2: "kv_split_kernel (padded K plan)",
+                  3: "kv_async_kernel", 4: "kv_bin_kernel", 5: "kv_kernel (general)",
+                  6: "kv_attn_kernel (SIMT)"}
 STRATEGY = {"recent": RECENT, "uniform": UNIFORM}
 PRECISION = {"fp32": FP32, "bf16": BF16, "fp32_simt": FP32_SIMT}
 
 SYMBOLS = ["tgl_version", "tgl_status_string", "tgl_last_error", "tgl_build_tcsr",
            "tgl_batch_roots", "tgl_dedup", "tgl_sample", "tgl_next_block",
            "tgl_time_precompute", "tgl_time_encode", "tgl_tblock_attn", "tgl_gather_rows",
-           "tgl_attn_packed_bytes", "tgl_attn_pack", "tgl_kv_timing", "tgl_kv_timing_ms",
-           "tgl_kv_timing_kernel", "tgl_cache_lookup", "tgl_cache_store", "tgl_cache_combine",
-           "tgl_cache_merge"]
+           "tgl_attn_packed_bytes", "tgl_attn_pack", "tgl_cache_lookup", "tgl_cache_store", "tgl_cache_combine",
+           "tgl_cache_merge", "tgl_shard_slice", "tgl_shard_gather"]
 
 
 class TGLError(RuntimeError):
@@ -61,6 +65,8 @@ def _load():
         "tgl_cache_store": [vp, i64, vp, vp, vp, vp, i64, vp],
         "tgl_cache_combine": [vp, i64, vp, vp, vp, i64, vp, i64, vp],
         "tgl_cache_merge": [vp, i64, vp, vp, vp, vp, vp, vp, i64, vp, i64, vp],
+        "tgl_shard_slice": [i64, vp, vp, vp, i32, i32, vp, vp, vp, vp],
+        "tgl_shard_gather": [i64, vp, vp, i64, vp, i32, vp, i64, i32, vp, i64, vp],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -68,12 +74,6 @@ def _load():
         f.restype = i32
     lib.tgl_attn_packed_bytes.argtypes = [vp]
     lib.tgl_attn_packed_bytes.restype = C.c_size_t
-    lib.tgl_kv_timing.argtypes = [C.c_int]
-    lib.tgl_kv_timing.restype = C.c_int
-    lib.tgl_kv_timing_ms.argtypes = [C.c_int]
-    lib.tgl_kv_timing_ms.restype = C.c_float
-    lib.tgl_kv_timing_kernel.argtypes = [C.c_int]
-    lib.tgl_kv_timing_kernel.restype = C.c_int
     return lib
 
 
@@ -261,7 +261,31 @@ class AttnParamsC(C.Structure):
                 ("ln_beta", C.c_void_p), ("ln_eps", C.c_float),
                 ("omega", C.c_void_p), ("phi", C.c_void_p),
                 ("leaky_slope", C.c_float), ("logit_scale", C.c_float),
-                ("precision", C.c_int32), ("packed", C.c_void_p)]
+                ("precision", C.c_int32), ("packed", C.c_void_p),
+                ("kv_kernel", C.c_int32), ("probe", C.c_void_p)]
+
+
+class KvProbeC(C.Structure):
+    _fields_ = [("ev_start", C.c_void_p), ("ev_stop", C.c_void_p), ("kernel", C.c_int32)]
+
+
+class KvProbe:
+    """Caller-owned measurement record (tgl.h tgl_kv_probe): two CUDA events the call
+    records around its K|V attention kernel, and which kernel ran.  Attach with
+    `AttnParams.attach_probe(p)` for eager calls only (never inside graph capture)."""
+
+    def __init__(self):
+        self.start = torch.cuda.Event(enable_timing=True)
+        self.stop = torch.cuda.Event(enable_timing=True)
+        self.struct = KvProbeC(self.start.cuda_event, self.stop.cuda_event, -1)
+
+    def ms(self) -> float:
+        self.stop.synchronize()
+        return self.start.elapsed_time(self.stop)
+
+    @property
+    def kernel(self) -> int:
+        return int(self.struct.kernel)
 
 
 _WEIGHTS = ("Wq", "bq", "Wk", "bk", "Wv", "bv", "Wo", "bo", "ln_gamma", "ln_beta", "omega", "phi")
@@ -273,7 +297,8 @@ class AttnParams:
     pack=True runs tgl_attn_pack once (tensor-core weight layout) so that every
     tgl_tblock_attn call streams the packed weights instead of re-packing them."""
 
-    def __init__(self, p: dict, device=None, precision="fp32", pack: bool = False):
+    def __init__(self, p: dict, device=None, precision="fp32", pack: bool = False,
+                 kv_kernel: str | int = "auto"):
         device = device or torch.device("cuda")
         self.host = p
         self.t = {k: torch.as_tensor(p[k], dtype=torch.float32).contiguous().to(device)
@@ -287,7 +312,8 @@ class AttnParams:
                                   *[_p(self.t[k]) for k in _WEIGHTS[:10]], float(p["ln_eps"]),
                                   _p(self.t["omega"]), _p(self.t["phi"]),
                                   float(p["leaky_slope"]), float(p["logit_scale"]),
-                                  self.precision, None)
+                                  self.precision, None,
+                                  KV_KERNEL.get(kv_kernel, kv_kernel), None)
         self.packed = None
         if pack and self.precision != FP32_SIMT:
             nb = _lib.tgl_attn_packed_bytes(C.byref(self.struct))
@@ -295,6 +321,15 @@ class AttnParams:
             _check(_lib.tgl_attn_pack(C.byref(self.struct), _p(self.packed), nb, _s()),
                    "tgl_attn_pack")
             self.struct.packed = _p(self.packed)
+
+    def attach_probe(self, probe: "KvProbe | None"):
+        """Record the next calls' K|V kernel into `probe` (None detaches)."""
+        self._probe = probe
+        self.struct.probe = None if probe is None else C.cast(C.pointer(probe.struct),
+                                                              C.c_void_p).value
+
+    def set_kv_kernel(self, kv_kernel: str | int):
+        self.struct.kv_kernel = KV_KERNEL.get(kv_kernel, kv_kernel)
 
 
 def tblock_attn(P: AttnParams, seg_ptr, dst_t, hdst, hdst_idx, hsrc, hsrc_idx, efeat, eid,
@@ -394,4 +429,35 @@ def cache_merge(cache: EmbeddingCache, node, t, slot, computed, idx=None, n_dev=
     _check(_lib.tgl_cache_merge(C.byref(cache.struct), n_max, _p(n_dev), _p(idx), _p(node),
                                 _p(t), _p(slot), _p(computed), computed.stride(0), _p(out),
                                 out.stride(0), _s(stream)), "tgl_cache_merge")
+    return out
+
+
+# --------------------------------------------------------------------------- S16 sharding
+def shard_slice(node, t, rank: int, world: int, n_dev=None, n_max=None, out=None, stream=None):
+    """Slice `rank` of the U = *n_dev unique roots: returns (node, t, n_dev) with capacity
+    ceil(n_max / world)."""
+    n_max = node.numel() if n_max is None else n_max
+    cap = max(1, -(-n_max // world))
+    dev = node.device
+    if out is None:
+        out = (torch.empty(cap, dtype=torch.int32, device=dev),
+               torch.empty(cap, dtype=torch.float32, device=dev),
+               torch.zeros(1, dtype=torch.int64, device=dev))
+    on, ot, od = out
+    _check(_lib.tgl_shard_slice(n_max, _p(n_dev), _p(node), _p(t), rank, world, _p(on), _p(ot),
+                                _p(od), _s(stream)), "tgl_shard_slice")
+    return on, ot, od
+
+
+def shard_gather(gathered, c_max: int, world: int, u_max: int, u_dev=None, idx=None,
+                 n_max=None, n_dev=None, out=None, stream=None):
+    """Rebuild the batch's root rows from the all-gathered slices (rank-major, c_max rows
+    each), through the roots' dedup inverse `idx` (None = identity)."""
+    d = gathered.shape[1]
+    n_max = (idx.numel() if idx is not None else u_max) if n_max is None else n_max
+    if out is None:
+        out = torch.empty(max(n_max, 1), d, dtype=torch.float32, device=gathered.device)
+    _check(_lib.tgl_shard_gather(n_max, _p(n_dev), _p(idx), u_max, _p(u_dev), world,
+                                 _p(gathered), c_max, d, _p(out), out.stride(0), _s(stream)),
+           "tgl_shard_gather")
     return out

@@ -90,3 +90,27 @@ def test_no_cpu_fallback_in_product():
         if fn.endswith(".py"):
             src = open(os.path.join(pkg, fn)).read()
             assert "import oracle" not in src and "from oracle" not in src, fn
+
+
+def test_product_library_has_no_debug_surface():
+    """Product builds export exactly the tgl.h entry points (the probe-only tgl_debug_*
+    readers and any timing hooks exist only in -DTGL_PROBE builds) and read no
+    environment variables (kernel choice is tgl_attn_params.kv_kernel)."""
+    import subprocess
+    out = subprocess.run(["nm", "-D", "--defined-only", tgl.LIB_PATH], capture_output=True,
+                         text=True).stdout
+    exported = {ln.split()[-1] for ln in out.splitlines() if ln.split()[-1].startswith("tgl_")}
+    assert exported == set(declared_symbols()), exported ^ set(declared_symbols())
+    blob = open(tgl.LIB_PATH, "rb").read()      # (cudart itself calls getenv: check ours)
+    for var in (b"TGL_DEBUG_MASK", b"TGL_KV\x00"):
+        assert var not in blob, var
+
+
+def test_shard_validation_errors():
+    lib = tgl.lib()
+    # rank outside [0, world)
+    st = lib.tgl_shard_slice(10, None, None, None, 2, 2, None, None, None, None)
+    assert st == -1 and b"rank" in lib.tgl_last_error()
+    # c_max smaller than ceil(u_max / world)
+    st = lib.tgl_shard_gather(10, None, None, 10, None, 4, None, 2, 100, None, 100, None)
+    assert st == -1 and b"c_max" in lib.tgl_last_error()

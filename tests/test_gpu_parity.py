@@ -216,20 +216,25 @@ def cu_pad(a, mult=4):
                                                           (200, 10, 100, 0, 0),
                                                           (333, 10, 413, 186, 0),
                                                           (517, 10, 128, 0, 0),
-                                                          (150, 10, 24, 12, 7)])
+                                                          (150, 10, 24, 12, 7),
+                                                          (148 * 12 + 37, 10, 413, 186, 0)])
 def test_attention_vs_oracle(T, monkeypatch, precision, kv, n_dst, kmax, d_h, d_e, long_every):
-    """TGL_KV selects the K|V kernel: "split" (default: loader / converter warps, K chunks
-    cut contiguously over [h | e | Phi] when the widths are multiples of 4), "split_pad"
-    (the same kernel with every segment padded to 32 columns), "async" (single-role
-    cp.async producers) -- all three need 16-B row pitches: the odd GDELT widths 413/186
-    go in row-padded views -- or "bin" (register gathers)."""
+    """tgl_attn_params.kv_kernel selects the K|V kernel: "split" (default: loader /
+    converter warps, K chunks cut contiguously over [h | e | Phi] when the widths are
+    multiples of 4, else per-segment padded), "split_pad" (the same kernel with every
+    segment padded to 32 columns), "async" (single-role cp.async producers) -- all three
+    need 16-B row pitches: the odd GDELT widths 413/186 go in row-padded views -- or "bin"
+    (register gathers).  The 413/186 case with 1,813 destinations is 14k edges, ~120
+    tiles: several tiles per CTA, so the persistent loop runs the padded plan through
+    the alternating-K weight reuse (the path the GDELT bench times)."""
     rng = np.random.default_rng(n_dst + kmax)
     p, seg, dst_t, nfeat, dn, sn, ef, eid, et = attn_case(rng, n_dst, kmax, d_h, d_e,
                                                           long_every=long_every)
-    if kv and np.diff(seg).max() <= 32:      # longer segments take the general kernel
-        monkeypatch.setenv("TGL_KV", kv)
+    sel = kv if (kv and np.diff(seg).max() <= 32) else "auto"   # longer: general kernel
     exp = oracle.tblock_attn(p, seg, dst_t, nfeat, dn, nfeat, sn, ef, eid, et)
-    P = T.AttnParams(p, precision=precision, pack=(n_dst % 2 == 1))
+    P = T.AttnParams(p, precision=precision, pack=(n_dst % 2 == 1), kv_kernel=sel)
+    probe = T.KvProbe()
+    P.attach_probe(probe)
     tab = T.time_precompute(65536, P.t["omega"], P.t["phi"])
     put = cu_pad if kv in ("async", "split", "split_pad") else cu
     nf = put(nfeat)
@@ -239,21 +244,28 @@ def test_attention_vs_oracle(T, monkeypatch, precision, kv, n_dst, kmax, d_h, d_
                             table=table, max_seg=int(np.diff(seg).max()))
         err = np.abs(np_(got)[:n_dst] - exp).max()
         assert err <= TOL[precision], err
+        if sel != "auto" and precision != "fp32_simt":   # the requested kernel really ran
+            want = T.KV_KERNEL[sel]
+            if sel == "split" and (d_h % 4 or d_e % 4):
+                want = T.KV_KERNEL["split_pad"]
+            assert probe.kernel == want, (probe.kernel, want)
 
 
 def test_attention_async_rejects_unaligned_pitch(T, monkeypatch):
-    """TGL_KV=async on a 413-float row pitch (1652 B, not a multiple of 16): EUNSUPPORTED,
-    while the default dispatch falls back to the register-gather kernel."""
+    """kv_kernel=async on a 413-float row pitch (1652 B, not a multiple of 16):
+    EUNSUPPORTED, while the default dispatch falls back to the register-gather kernel."""
     rng = np.random.default_rng(5)
     p, seg, dst_t, nfeat, dn, sn, ef, eid, et = attn_case(rng, 64, 10, 413, 186)
     exp = oracle.tblock_attn(p, seg, dst_t, nfeat, dn, nfeat, sn, ef, eid, et)
-    P = T.AttnParams(p)
-    args = (P, cu(seg), cu(dst_t), cu(nfeat), cu(dn), cu(nfeat), cu(sn), cu(ef), cu(eid), cu(et))
-    monkeypatch.setenv("TGL_KV", "async")
+    P = T.AttnParams(p, kv_kernel="async")
+    args = (cu(seg), cu(dst_t), cu(nfeat), cu(dn), cu(nfeat), cu(sn), cu(ef), cu(eid), cu(et))
     with pytest.raises(T.TGLError):
-        T.tblock_attn(*args, max_seg=10)
-    monkeypatch.delenv("TGL_KV")
-    got = T.tblock_attn(*args, max_seg=10)
+        T.tblock_attn(P, *args, max_seg=10)
+    P.set_kv_kernel("auto")
+    probe = T.KvProbe()
+    P.attach_probe(probe)
+    got = T.tblock_attn(P, *args, max_seg=10)
+    assert probe.kernel == T.KV_KERNEL["bin"]
     assert np.abs(np_(got)[:64] - exp).max() <= 1e-3
 
 

@@ -19,12 +19,16 @@ from paper_conf_asplos_wangm24_b200.block import _call_ws
 
 prec = sys.argv[1] if len(sys.argv) > 1 else "fp32"
 cfg = synth.get_config(os.environ.get("CFG", "REDDIT"))
-g = synth.make_graph(cfg)
-neg = synth.make_negatives(cfg)
-params = synth.gen.model_params(cfg)
-cu = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
-dev = {"src": cu(g.src), "dst": cu(g.dst), "t": cu(g.t), "neg": cu(neg), "nfeat": cu(g.nfeat),
-       "efeat": cu(g.efeat)}
+if cfg.name in ("GDELT", "MAG"):     # device-generated, 16-byte row pitch (as bench.py)
+    import bench
+    cfg, g, neg, params, dev = bench.load_world_device(cfg.name)
+else:
+    g = synth.make_graph(cfg)
+    neg = synth.make_negatives(cfg)
+    params = synth.gen.model_params(cfg)
+    cu = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    dev = {"src": cu(g.src), "dst": cu(g.dst), "t": cu(g.t), "neg": cu(neg),
+           "nfeat": cu(g.nfeat), "efeat": cu(g.efeat)}
 tc = tgl.build_tcsr(cfg.n_nodes, dev["src"], dev["dst"], dev["t"], True, True)
 pipe = TGATPipeline(dev, tc, params, cfg.batch, TSampler(cfg.k, cfg.strategy, cfg.seeds["sampler"]),
                     cfg.dedup, cfg.precompute, cfg.window, prec)
