@@ -51,7 +51,7 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0,
                     help="oracle work per cpu_baseline leg (all cores, then 1 thread)")
-    ap.add_argument("--ref-seconds", type=float, default=120.0,
+    ap.add_argument("--ref-seconds", type=float, default=60.0,
                     help="budget of the --impl reference timed steps (sizes its sample)")
     ap.add_argument("--dedup", default="config", choices=["config", "on", "off"],
                     help="override the config's dedup setting (ablation only)")
@@ -252,6 +252,16 @@ class OracleRunner:
         return 3 * len(src_b), sum(int(bl.seg_ptr[-1]) for bl in blocks), (t1 - t0) + (t3 - t2)
 
 
+def size_sample(runner, g, neg, b, budget_s: float, batch: int) -> int:
+    """Edges of a batch the oracle processes in about `budget_s` (a power of two, at most
+    the whole batch): timed on a 16-edge probe, scaled linearly."""
+    _, _, dt = runner.batch(*(x[:16] for x in synth_batch(g, neg, b)))
+    per = batch
+    while per > 16 and dt * per / 16 > budget_s:
+        per //= 2
+    return per
+
+
 def oracle_rate(runner, g, neg, batches, seconds: float, edges_per_call: int | None = None):
     """Oracle throughput over whole batches (or their first `edges_per_call` edges) until
     `seconds` of oracle work."""
@@ -305,7 +315,8 @@ def cpu_baseline(cfg, g, neg, params, batches, seconds: float, runner=None) -> d
                    f"at a time by Listing 1's recursion (oracle/big.py), {r['seconds']:.1f} s")
         else:
             # whole batches when one fits the budget, else the first edges of each batch
-            per = None if threads > 1 or cfg.name not in BIG else max(1, cfg.batch // 20)
+            per = size_sample(runner, g, neg, batches[0], seconds / 3, cfg.batch)
+            per = None if per >= cfg.batch else per
             r = oracle_rate(runner, g, neg, batches, seconds, per)
             smp = (f"{r['batches']} {'whole batch(es)' if per is None else f'x first {per} edges of a batch'}"
                    f" ({r['roots']} roots) from 70% of the stream, {r['seconds']:.1f} s")
@@ -348,10 +359,7 @@ def run_reference(args):
     else:
         runner = OracleRunner(cfg, g, params)
         # size the step: whole batches if K of them fit the budget, else first edges
-        r, _, dt = runner.batch(*synth_batch(g, neg, b0))
-        per = cfg.batch
-        while per > 1 and dt * args.steps * per / cfg.batch > args.ref_seconds:
-            per //= 2
+        per = size_sample(runner, g, neg, b0, args.ref_seconds / args.steps, cfg.batch)
     from oracle import big
     from oracle import pipeline as opipe
     times, roots, edges, segs = [], 0, 0, {}
@@ -661,7 +669,7 @@ def run_ours(args):
                 "scaling": "strong", "vs_baseline": None,
                 "dtype": {"fp32": "f32 (3-pass bf16 tensor-core split)", "bf16": "bf16",
                           "fp32_simt": "f32"}[args.precision],
-                "data": "synthetic (seeded generators shaped like PAPER.md Table 3)",
+                "data": "synthetic",
                 "config": config_dict(cfg, args, world, flush),
                 "sampled_edges_per_s": edges_per_s,
                 "sampler": sampler_line,

@@ -49,6 +49,13 @@ def _compile(src: str, verbose: bool) -> str:
 
 def build(verbose: bool = False, force: bool = False) -> str:
     os.makedirs(OBJ, exist_ok=True)
+    # objects built with other flags (e.g. a -DTGL_PROBE profiling build) are stale
+    stamp = os.path.join(OBJ, "flags.txt")
+    want = " ".join(f for f in FLAGS if not f.startswith("/"))   # not the checkout path
+    if not os.path.exists(stamp) or open(stamp).read() != want:
+        force = True
+        if os.path.exists(stamp):
+            os.remove(stamp)
     srcs = [s for s in SOURCES if os.path.exists(os.path.join(CSRC, s))]
     if force:
         for s in srcs:
@@ -65,6 +72,8 @@ def build(verbose: bool = False, force: bool = False) -> str:
         if r.returncode != 0:
             raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")
         os.replace(tmp, LIB)
+    with open(stamp, "w") as f:
+        f.write(want)
     return LIB
 
 

@@ -277,6 +277,9 @@ class KvProbe:
     def __init__(self):
         self.start = torch.cuda.Event(enable_timing=True)
         self.stop = torch.cuda.Event(enable_timing=True)
+        self.start.record()                 # torch creates the CUDA events lazily
+        self.stop.record()
+        assert self.start.cuda_event and self.stop.cuda_event
         self.struct = KvProbeC(self.start.cuda_event, self.stop.cuda_event, -1)
 
     def ms(self) -> float:

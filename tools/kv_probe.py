@@ -1,4 +1,7 @@
-"""Time the REDDIT tail-block tgl_tblock_attn call per K|V kernel and debug mask.
+"""Time the tail-block tgl_tblock_attn call per K|V kernel and debug mask (CFG=REDDIT|GDELT|...).
+
+Needs a probe build: TGL_NVCC_EXTRA="-DTGL_PROBE [-DTGL_KV_PROF]" (the debug mask and the
+instrumentation readers exist only there).
 
     python tools/kv_probe.py [precision]
 
@@ -67,7 +70,7 @@ for kv in KVS:
     for mask in MASKS:
         if kv == "bin" and mask & 64:
             continue
-        os.environ["TGL_KV"] = kv
+        a.set_kv_kernel(kv)
         os.environ["TGL_DEBUG_MASK"] = str(mask)
         ts = []
         for it in range(8):
@@ -93,7 +96,7 @@ if os.environ.get("PROBE_PROF"):
     lib.tgl_debug_prof.argtypes = [C.c_void_p, C.c_int]
     host = (C.c_ulonglong * (148 * 16))()
     for kv in (os.environ.get("PROBE_PROF_KV", "split"),):
-        os.environ["TGL_KV"] = kv
+        a.set_kv_kernel(kv)
         os.environ["TGL_DEBUG_MASK"] = str(512 | int(os.environ.get("PROBE_PROF_MASK", "0")))
         call(); torch.cuda.synchronize()
         lib.tgl_debug_prof(None, 1)
@@ -114,7 +117,7 @@ if os.environ.get("PROBE_TRACE"):
     import ctypes as C
     lib.tgl_debug_trace.argtypes = [C.c_void_p, C.c_int]
     host = (C.c_ulonglong * 8192)()
-    os.environ["TGL_KV"] = os.environ.get("PROBE_TRACE_KV", "split")
+    a.set_kv_kernel(os.environ.get("PROBE_TRACE_KV", "split"))
     os.environ["TGL_DEBUG_MASK"] = str(4096 | int(os.environ.get("PROBE_TRACE_MASK", "0")))
     call(); torch.cuda.synchronize()
     lib.tgl_debug_trace(None, 1)
