@@ -38,6 +38,9 @@ sys.path.insert(0, ROOT)
 METRIC = "sampled edges/s and TBlock embeddings/s at 1/2/4/8 B200; % HBM roofline"
 BIG = ("GDELT", "MAG")            # generated on the device (synth.gpu)
 FLUSH_DEFAULT = {"WIKI": True, "REDDIT": True, "LASTFM": True, "GDELT": False, "MAG": False}
+# operand layout of the K|V gathers: split16 tables (kv_pre) everywhere but MAG, whose 62 GB
+# node table cannot be held twice next to its 32 GB T-CSR (fp32 rows, converted in the SM)
+LAYOUT = {"MAG": "fp32"}
 
 
 def parse():
@@ -156,15 +159,22 @@ def load_world_device(cfg_name: str):
     d = torch.device("cuda")
     src, dst, t = sg.device_graph(cfg, d)
     neg = sg.device_negatives(cfg, d)
-    # 16-byte row pitch (GDELT's 413 / 186 floats padded to 416 / 188): the K|V kernel's
-    # cp.async gathers need it; the values are the same counter-based features
+    from paper_conf_asplos_wangm24_b200 import tgl
+    # node features: fp32 rows with a 16-byte pitch (h_dst of the Q / FFN kernels) and the
+    # split16 operand table the K|V kernel gathers; edge features: split16 only, built
+    # chunk by chunk from the same counter-based values (the fp32 table never exists)
     nfeat = sg.device_feature_table(cfg.seeds["feat"], cfg.n_nodes, cfg.d_v, d, pitch_mult=4)
-    efeat = (sg.device_feature_table(cfg.seeds["feat"] + 7919, cfg.n_edges, cfg.d_e, d,
-                                     pitch_mult=4)
-             if cfg.d_e else torch.zeros((0, 0), dtype=torch.float32, device=d))
+    dev = {"src": src, "dst": dst, "t": t, "neg": neg, "nfeat": nfeat, "efeat": None}
+    if LAYOUT.get(cfg.name, "split") == "split":
+        dev["nfeat_split"] = tgl.split_rows(nfeat)
+    if cfg.d_e:
+        dev["efeat_split"] = tgl.split_table(
+            cfg.n_edges, cfg.d_e,
+            lambda r0, r1: sg.feature_rows_torch(cfg.seeds["feat"] + 7919,
+                                                 torch.arange(r0, r1, device=d), cfg.d_e))
+    torch.cuda.synchronize()
     g = HostGraph(cfg, src.cpu().numpy(), dst.cpu().numpy(), t.cpu().numpy())
     neg_h = neg.cpu().numpy()
-    dev = {"src": src, "dst": dst, "t": t, "neg": neg, "nfeat": nfeat, "efeat": efeat}
     return cfg, g, neg_h, synth.gen.model_params(cfg), dev
 
 
@@ -199,6 +209,9 @@ def config_dict(cfg, args, world: int, flush: bool) -> dict:
     return {"workload": cfg.name, "batch_edges": cfg.batch, "roots_per_step": 3 * cfg.batch,
             "layers": cfg.n_layers, "k": cfg.k, "strategy": cfg.strategy, "dedup": cfg.dedup,
             "precompute": cfg.precompute, "precision": args.precision,
+            "operand_layout": ("fp32 rows" if args.precision == "fp32_simt" or
+                               LAYOUT.get(cfg.name, "split") == "fp32" else
+                               "split16 (bf16 hi/lo tables, tgl_split_rows)"),
             "cache_slots_per_layer": args.cache,
             "parallelism": (f"root-sharded x{world} (each rank: slice of the batch's roots; "
                             f"NCCL all-gather of root embeddings)" if world > 1 else "single"),
@@ -493,8 +506,10 @@ def run_ours(args):
 
     sampler = TSampler(cfg.k, cfg.strategy, cfg.seeds["sampler"])
     shard = (rank, world) if world > 1 else None
+    layout = "fp32" if args.precision == "fp32_simt" else LAYOUT.get(cfg.name, "split")
     pipe = TGATPipeline(dev, tc, params, cfg.batch, sampler, cfg.dedup, cfg.precompute,
-                        cfg.window, args.precision, cache_capacity=args.cache, shard=shard)
+                        cfg.window, args.precision, cache_capacity=args.cache, shard=shard,
+                        layout=layout)
     for a in pipe.attn:
         a.set_kv_kernel(args.kv_kernel)
     pipe.capture()
@@ -653,7 +668,8 @@ def run_ours(args):
     # ---- e2e through the public API: pinned host batch -> device -> host embeddings
     e2e = None
     if not args.no_e2e:
-        e2e = run_e2e(args, cfg, g, neg, params, dev, tc, sampler, batch_of, world, rank, shard)
+        e2e = run_e2e(args, cfg, g, neg, params, dev, tc, sampler, batch_of, world, rank, shard,
+                      layout)
 
     cpu = None
     if want_cpu:
@@ -688,7 +704,7 @@ def run_ours(args):
     return 0
 
 
-def run_e2e(args, cfg, g, neg, params, dev, tc, sampler, batch_of, world, rank, shard):
+def run_e2e(args, cfg, g, neg, params, dev, tc, sampler, batch_of, world, rank, shard, layout):
     """The public serving loop: per batch the H2D of its edges from pinned host memory,
     the captured chain, and the D2H of its root embeddings (rank 0 with N > 1), timed by
     the host wall clock (max over ranks).  Warm-up batches are not among the timed ones."""
@@ -700,7 +716,7 @@ def run_e2e(args, cfg, g, neg, params, dev, tc, sampler, batch_of, world, rank, 
     n0 = 3 * cfg.batch
     pipe_h = TGATPipeline(dev, tc, params, cfg.batch, sampler, cfg.dedup, cfg.precompute,
                           cfg.window, args.precision, staging=True, cache_capacity=args.cache,
-                          shard=shard)
+                          shard=shard, layout=layout)
     for a in pipe_h.attn:
         a.set_kv_kernel(args.kv_kernel)
     pipe_h.capture()

@@ -214,6 +214,16 @@ tgl_status tgl_time_encode(int64_t n, const float* dt, int32_t d_t, const float*
 #define TGL_KV_BIN 4          /* register-gather producers (any row pitch) */
 #define TGL_KV_GENERAL 5      /* any segment length */
 #define TGL_KV_SIMT 6         /* (reported only) the TGL_FP32_SIMT kernel */
+#define TGL_KV_PRE 7          /* pre-split h_src / e tables (tgl_split_rows): loaders move
+                                 the bf16 hi / lo operands straight into the MMA's shared-
+                                 memory stages, no conversion in the SM (AUTO picks it
+                                 whenever input_layout marks the gathered tables split) */
+
+/* tgl_attn_params.input_layout bits: the table is in the split16 layout of
+ * tgl_split_rows (its leading dimension still counts 4-byte words). */
+#define TGL_SPLIT_HSRC 1
+#define TGL_SPLIT_E 2
+#define TGL_SPLIT_TABLE 4   /* tenc_table is split16 [window, round_up(d_t, 8)] (kv_pre only) */
 
 /* Measurement record (bench.py): when tgl_attn_params.probe != NULL the call records
  * ev_start / ev_stop (cudaEvent_t, created by the caller) on its stream immediately
@@ -241,6 +251,9 @@ typedef struct {
   int32_t kv_kernel;              /* TGL_KV_AUTO (0) or a specific K|V kernel (TGL_KV_*);
                                      a kernel that cannot take the call -> EUNSUPPORTED */
   tgl_kv_probe* probe;            /* optional (NULL): caller-owned measurement record */
+  int32_t input_layout;           /* TGL_SPLIT_* bits: hsrc / efeat / tenc_table are
+                                     split16 tables (tensor-core precisions, max_seg <= 32,
+                                     2 heads) */
 } tgl_attn_params;
 
 /* Weight layout transform for the tensor-core path, done once per layer (the
@@ -260,6 +273,16 @@ tgl_status tgl_tblock_attn(const tgl_attn_params* P, int64_t n_dst_max, const in
                            const float* edge_t, const float* tenc_table, int64_t window,
                            int32_t max_seg, float* out, void* ws, size_t* ws_bytes,
                            void* stream);
+
+/* Split16 feature layout for the gathered operands of the tensor-core K|V path: row r
+ * of dst (pitch ld_dst 4-byte words, 16-byte aligned rows) holds bf16 RNE(x) for the
+ * dp = round_up(d, 8) columns (zeros past d), then bf16 RNE(x - hi) for the same
+ * columns -- 4 bytes per column like fp32, written once per table (features) or per
+ * layer output, so the K|V kernel gathers MMA operands without converting them.
+ * hi + lo equals x to 2^-17 relative; the 3-pass product is the fp32 mode's.  Errors:
+ * EINVAL (ld_dst < dp, ld_dst % 4 != 0, unaligned dst). */
+tgl_status tgl_split_rows(int64_t n_rows, int32_t d, const float* src, int64_t ld_src,
+                          void* dst, int64_t ld_dst, void* stream);
 
 /* ---------------------------------------------------------------------------
  * S14  Dedup inverse applied to rows (the hook of P:279 / TGOpt dedup_invert

@@ -35,6 +35,7 @@ class TBlock:
     eid: torch.Tensor = None
     ts: torch.Tensor = None
     out: torch.Tensor = None       # layer output [n_max, d_out]
+    out_split: torch.Tensor = None  # the same rows as a split16 table (layout="split")
     ws: dict = field(default_factory=dict)
 
 
@@ -55,13 +56,20 @@ class TGATPipeline:
     def __init__(self, graph: dict, tcsr: tgl.TemporalCSR, params: list, batch: int,
                  sampler: TSampler, use_dedup: bool, precompute: bool, window: int = 65536,
                  precision: str = "fp32", staging: bool = False, device=None,
-                 cache_capacity: int = 0, shard: tuple | None = None):
+                 cache_capacity: int = 0, shard: tuple | None = None,
+                 layout: str | None = None):
         """shard = (rank, world): root sharding (S16).  The batch's roots
         (deduped when use_dedup) are formed on every rank; this pipeline computes the
         contiguous slice `rank` of them (tgl_shard_slice) and forward(slot) returns the
         slice's embeddings [c_max, d_out] in `send[slot]`; `combine(slot, gathered)`
         rebuilds the whole batch from the all-gathered slices (tgl_shard_gather).  Two
-        slots (two captured graphs) let batch b's all-gather overlap batch b+1."""
+        slots (two captured graphs) let batch b's all-gather overlap batch b+1.
+
+        layout: "split" (default for the tensor-core precisions) gathers the K|V operands
+        from split16 tables (tgl_split_rows: bf16 hi / lo halves, the kv_pre kernel) --
+        graph["nfeat_split"] / graph["efeat_split"] when given, else split here once --
+        and every inner layer output is split once for the layer above; "fp32" gathers
+        fp32 rows and converts in the SM (kv_split)."""
         self.dev = device or torch.device("cuda")
         self.g = graph
         self.tcsr = tcsr
@@ -73,6 +81,23 @@ class TGATPipeline:
         self.attn = [tgl.AttnParams(p, self.dev, precision, pack=True) for p in params]
         self.tables = [tgl.time_precompute(window, a.t["omega"], a.t["phi"]) if precompute else None
                        for a in self.attn]
+        if layout is None:
+            layout = "fp32" if precision == "fp32_simt" else "split"
+        self.split = layout == "split"
+        if self.split:
+            assert precision != "fp32_simt", "split16 tables feed the tensor-core path"
+            nf = graph.get("nfeat_split")
+            if nf is None:
+                nf = tgl.split_rows(graph["nfeat"])
+            ef = graph.get("efeat_split")
+            if ef is None and graph.get("efeat") is not None and graph["efeat"].numel():
+                ef = tgl.split_rows(graph["efeat"])
+            self.nfeat_split, self.efeat_split = nf, ef
+            for l, a in enumerate(self.attn):
+                a.struct.input_layout = (tgl.SPLIT_HSRC | (tgl.SPLIT_E if a.host["d_e"] else 0) |
+                                         tgl.SPLIT_TABLE)
+            # the precompute tables as split16 rows too: gathered like features
+            self.tables = [None if t is None else tgl.split_rows(t) for t in self.tables]
         k = sampler.k
         i32, f32, i64 = torch.int32, torch.float32, torch.int64
         z = lambda n, dt: torch.zeros(max(int(n), 1), dtype=dt, device=self.dev)
@@ -102,6 +127,9 @@ class TGATPipeline:
             b.seg_ptr = z(n_max + 1, i64)
             b.nbr, b.eid, b.ts = z(n_max * k, i32), z(n_max * k, i32), z(n_max * k, f32)
             b.out = z(n_max * self.attn[l].d_out, f32).view(-1, self.attn[l].d_out)
+            if self.split and l > 0:       # the layer above gathers its rows split
+                dpo = tgl.split_width(self.attn[l].d_out)
+                b.out_split = z(n_max * dpo, f32).view(-1, dpo)
             self.blocks.append(b)
             n_max = n_max + n_max * k
         self.emb = z(3 * batch * self.attn[0].d_out, f32).view(-1, self.attn[0].d_out)
@@ -119,7 +147,9 @@ class TGATPipeline:
         dedup_launches = [(1 if b.n_max <= 4096 else 3) if use_dedup else 0 for b in self.blocks]
         if shard is not None:   # roots' dedup (before the slice) replaces block 0's + slice
             dedup_launches[0] = ((1 if 3 * batch <= 4096 else 3) if use_dedup else 0) + 1
-        per_block = [(1 if l > 0 else 0) + dedup_launches[l] + 1 + 3 for l in range(self.L)]
+        per_block = [(1 if l > 0 else 0) + dedup_launches[l] + 1 + 3 + (1 if self.split and l > 0
+                                                                         else 0)
+                     for l in range(self.L)]
         self.launches_per_forward = 1 + sum(per_block) + (1 if use_dedup and shard is None
                                                           else 0)
         # cache() (TGOpt per-layer store, Listing 1 L23; inference): every
@@ -231,16 +261,20 @@ class TGATPipeline:
             a = self.attn[l]
             if l == self.L - 1:
                 hdst, hdst_idx, hsrc, hsrc_idx, off = g["nfeat"], b.uniq_node, g["nfeat"], b.nbr, None
+                if self.split:
+                    hsrc = self.nfeat_split
             else:
                 nx = self.blocks[l + 1]
                 hdst = hsrc = nx.ws["cache"]["comb"] if self.cache_on else nx.out
+                if self.split:
+                    hsrc = nx.out_split
                 off = b.u_dev        # S14: rows [U_l + e] of the next block hold the sources
                 if self.use_dedup:
                     hdst_idx = hsrc_idx = nx.inv
                 else:
                     hdst_idx = hsrc_idx = None
-            ef = g["efeat"]
-            ld_e = ef.stride(0) if (ef.dim() == 2 and ef.shape[1] > 0) else 0
+            ef = self.efeat_split if self.split else g["efeat"]
+            ld_e = ef.stride(0) if (ef is not None and ef.dim() == 2 and ef.shape[1] > 0) else 0
             if record is not None:
                 ev = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
                 ev[0].record(s if s is not None else torch.cuda.current_stream())
@@ -261,6 +295,10 @@ class TGATPipeline:
                 tgl.cache_merge(c["table"], c["node"], c["t"], c["slot"], b.out,
                                 n_dev=c["u"], n_max=b.n_max, out=c["comb"], stream=s)
                 mark(f"cache_merge{l}")
+            if self.split and l > 0:     # the operands the layer above gathers (split16)
+                tgl.split_rows(b.ws["cache"]["comb"] if self.cache_on else b.out,
+                               out=b.out_split, n_rows=b.n_max, stream=s)
+                mark(f"split{l}")
         if self.shard is not None:
             return b0.out
         if self.cache_on:  # head: store + combine + S14 inverse in one launch

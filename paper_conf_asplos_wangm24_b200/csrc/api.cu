@@ -2,6 +2,8 @@
 #include <stdarg.h>
 #include <string.h>
 
+#include <cuda_bf16.h>
+
 #include "common.cuh"
 
 namespace tgl {
@@ -92,6 +94,39 @@ __global__ void gather_rows_kernel(int64_t n_max, const int64_t* n_dev,
   }
 }
 
+// ---------------------------------------------------------------- split16 rows
+// dst row r (pitch ld_dst 4-byte words): bf16 hi of columns [0, dp) then bf16 lo of the
+// same columns, dp = d rounded up to 8 (zero columns past d); hi = RNE(x),
+// lo = RNE(x - hi) -- the operand split of the 3-pass tensor-core path.  One thread per
+// 8-column group: 16-byte stores.
+__global__ void split_rows_kernel(int64_t n_rows, int32_t d, const float* __restrict__ src,
+                                  int64_t ld_src, uint8_t* __restrict__ dst, int64_t ld_dst) {
+  pdl_wait();
+  pdl_trigger();
+  const int dp = (d + 7) & ~7;
+  const int groups = dp >> 3;
+  const int64_t total = n_rows * groups;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = x / groups;
+    const int g = (int)(x - r * groups);
+    const float* sp = src + r * ld_src + 8 * g;
+    uint32_t h[4], l[4];
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      const int c = 8 * g + 2 * e;
+      const float x0 = c < d ? sp[2 * e] : 0.f, x1 = c + 1 < d ? sp[2 * e + 1] : 0.f;
+      __nv_bfloat162 hh = __floats2bfloat162_rn(x0, x1);
+      __nv_bfloat162 ll = __floats2bfloat162_rn(x0 - __low2float(hh), x1 - __high2float(hh));
+      h[e] = *reinterpret_cast<uint32_t*>(&hh);
+      l[e] = *reinterpret_cast<uint32_t*>(&ll);
+    }
+    uint8_t* row = dst + r * ld_dst * 4;
+    *reinterpret_cast<uint4*>(row + 16 * g) = make_uint4(h[0], h[1], h[2], h[3]);
+    *reinterpret_cast<uint4*>(row + 2 * dp + 16 * g) = make_uint4(l[0], l[1], l[2], l[3]);
+  }
+}
+
 static int grid_for(int64_t n, int threads) {
   int64_t g = ceil_div(n > 0 ? n : 1, threads);
   int64_t cap = (int64_t)kNumSMs * 16;
@@ -154,6 +189,19 @@ tgl_status tgl_gather_rows(int64_t n_max, const int64_t* n_dev, const int32_t* i
   launch_pdl(gather_rows_kernel, dim3(grid_for(n_max * d, 256)), dim3(256), 0, as_stream(stream), 
       n_max, n_dev, idx, table, ld_table, d, out, ld_out);
   return launch_check("gather_rows");
+}
+
+tgl_status tgl_split_rows(int64_t n_rows, int32_t d, const float* src, int64_t ld_src,
+                          void* dst, int64_t ld_dst, void* stream) {
+  TGL_REQUIRE(n_rows >= 0 && d >= 0, "negative size");
+  const int64_t dp = (d + 7) & ~7;
+  TGL_REQUIRE(ld_src >= d && ld_dst >= dp && ld_dst % 4 == 0, "bad leading dim");
+  if (n_rows == 0 || d == 0) return TGL_OK;
+  TGL_REQUIRE(src && dst, "null pointer");
+  TGL_REQUIRE((reinterpret_cast<uintptr_t>(dst) & 15) == 0, "dst must be 16-byte aligned");
+  launch_pdl(split_rows_kernel, dim3(grid_for(n_rows * (dp / 8), 256)), dim3(256), 0,
+             as_stream(stream), n_rows, d, src, ld_src, static_cast<uint8_t*>(dst), ld_dst);
+  return launch_check("split_rows");
 }
 
 }  // extern "C"

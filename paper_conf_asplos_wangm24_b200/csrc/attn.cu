@@ -469,6 +469,10 @@ extern "C" tgl_status tgl_tblock_attn(const tgl_attn_params* P, int64_t n_dst_ma
                   P->precision == TGL_FP32_SIMT,
               "unknown precision");
   const bool use_tc = P->precision != TGL_FP32_SIMT;
+  if (!use_tc && P->input_layout != 0) {
+    set_error("split16 inputs (input_layout) feed the tensor-core path only");
+    return TGL_EUNSUPPORTED;
+  }
   if (use_tc && !tc_attn_supported(P)) {
     set_error("tensor-core path needs d_model == d_out == 100 (use TGL_FP32_SIMT otherwise)");
     return TGL_EUNSUPPORTED;

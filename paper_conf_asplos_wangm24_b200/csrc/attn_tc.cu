@@ -576,7 +576,9 @@ __global__ void __launch_bounds__(kWsThreads, 1) dense_kernel(Args a) {
         R.p0[r] = p0;
         R.p1[r] = p1;
         R.dt[r] = 0.f;
-        R.trow[r] = (!kFfn && a.table != nullptr) ? 0 : -1;   // precomputed_zeros = row 0
+        // precomputed_zeros = table row 0 (fp32 tables only; a split16 table is read by
+        // kv_pre alone, so Phi(0) = cos(phi) is evaluated -- bit-identical, R11)
+        R.trow[r] = (!kFfn && a.table != nullptr && !(P.input_layout & TGL_SPLIT_TABLE)) ? 0 : -1;
         R.rdst[r] = r < rows ? r : -1;
       }
       warp_arrive(&B.dfull[ds]);
@@ -2412,13 +2414,476 @@ __global__ void __launch_bounds__(kSThreads, 1)
   ws_teardown(tmem, 2 * kCols, kTMma);
 }
 
+
+// ------------------------------------------------------------------ pre-split K|V kernel
+// kv_pre_kernel: the split-role design without the converter stage.  The gathered
+// feature tables (h_src, e) are stored PRE-SPLIT (tgl_split_rows: per row the bf16 hi
+// halves of its columns, then the bf16 lo halves, every segment padded to 8 columns),
+// i.e. the exact operands the converters of kv_split_kernel produced on every gather
+// -- so loaders move 16-byte hi / lo pieces with LDGSTS straight into the swizzled
+// SW64 A stages the MMA reads, and completion is an mbarrier arrival
+// (cp.async.mbarrier.arrive.noinc; CUTLASS's sm100 cp.async + UMMA mainloop relies on
+// the same ordering).  Only the time columns are produced in the SM: 4 time warps
+// evaluate Phi(dt) (table row or direct), split and store them.  K is the contiguous
+// concatenation K' = [h (dp0) | e (dp1) | Phi (dpt)] of 8-column groups, cut into
+// 32-column chunks; [Wk ; Wv] is packed in the same K' order (zero rows for padding).
+// In bf16 mode only the hi halves are loaded (half the gather bytes).
+// Roles: epilogue warps 0-7 (bin_epilogue), MMA 8, weights 9, tile descriptors 10-11,
+// loaders 12-15, time warps 16-19: 640 threads.
+#ifndef TGL_KV_PRE_ASTAGES
+#define TGL_KV_PRE_ASTAGES 8
+#endif
+constexpr int kPAStages = TGL_KV_PRE_ASTAGES;         // A stages (hi | lo, 16 KB each)
+constexpr int kPAStage = kBM * kTC * 4;                // 16 KB
+constexpr int kPW = 2;                                 // weight stages (25.6 KB each)
+constexpr int kPLoad0 = 12, kPLoadWarps = 4;
+constexpr int kPTime0 = 16, kPTimeWarps = 4;
+constexpr int kPThreads = (kPTime0 + kPTimeWarps) * 32;   // 640
+constexpr int kPPipeBytes = kPAStages * kPAStage + kPW * kTWStage;
+constexpr int kPSmem = 1024 + kPPipeBytes + kBEpi * 32 * kSPW * 4;
+constexpr int kPMaxChunks = 64;
+
+struct PrePlan {      // K' = [h: dp0 | e: dp1 | Phi: dpt], 8-column groups, 32-column chunks
+  int d0, d1, dt;     // true widths
+  int dp0, dp1, dpt;  // padded to multiples of 8
+  int k;              // dp0 + dp1 + dpt
+  int n;              // chunks
+  // issue order of the chunks inside a tile: the chunks holding time columns (produced by
+  // the time warps, the slowest producer) spread evenly among the gathered ones, so they
+  // never queue back to back at a tile boundary; odd tiles walk the order backwards
+  unsigned char order[64];
+};
+static int pad8h(int x) { return (x + 7) & ~7; }
+static PrePlan make_pre_plan(int d0, int d1, int dt) {
+  PrePlan p;
+  p.d0 = d0; p.d1 = d1; p.dt = dt;
+  p.dp0 = pad8h(d0); p.dp1 = pad8h(d1); p.dpt = pad8h(dt);
+  p.k = p.dp0 + p.dp1 + p.dpt;
+  p.n = (p.k + kTC - 1) / kTC;
+  const int ct = (p.dp0 + p.dp1) / kTC;            // first chunk holding time columns
+  const int nt = p.n - ct, nf = ct;
+  int pos = 0, f = 0, t = 0;
+  for (int i = 0; i < p.n && i < 64; ++i) {
+    // time chunk j goes to position floor((j + 0.5) n / nt)
+    const bool take_t = t < nt && (f >= nf || i >= (int)((t + 0.5) * p.n / (nt > 0 ? nt : 1)));
+    p.order[pos++] = (unsigned char)(take_t ? ct + t++ : f++);
+  }
+  return p;
+}
+
+__global__ void pack_kv_pre_kernel(const float* Wk, const float* Wv, int dm, int ksrc, PrePlan p,
+                                   uint8_t* out) {
+  const int kw = p.n * kTC;
+  const int64_t total = (int64_t)kNPkv * kw;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const int n = (int)(x / kw), kp = (int)(x % kw);
+    const int c = kp / kTC, cc = kp % kTC;
+    int src = -1;                                   // column of [h | e | Phi] in W
+    if (kp < p.dp0) {
+      if (kp < p.d0) src = kp;
+    } else if (kp < p.dp0 + p.dp1) {
+      if (kp - p.dp0 < p.d1) src = p.d0 + (kp - p.dp0);
+    } else if (kp < p.k) {
+      if (kp - p.dp0 - p.dp1 < p.dt) src = p.d0 + p.d1 + (kp - p.dp0 - p.dp1);
+    }
+    float v = 0.f;
+    if (n < 2 * dm && src >= 0)
+      v = n < dm ? Wk[(int64_t)n * ksrc + src] : Wv[(int64_t)(n - dm) * ksrc + src];
+    const __nv_bfloat16 hi = __float2bfloat16_rn(v);
+    const __nv_bfloat16 lo = __float2bfloat16_rn(v - __bfloat162float(hi));
+    const int64_t off = (int64_t)c * kTWStage + (n >> 3) * 512 + sw64_off(n, cc);
+    *reinterpret_cast<__nv_bfloat16*>(out + off) = hi;
+    *reinterpret_cast<__nv_bfloat16*>(out + off + kTWHalf) = lo;
+  }
+}
+
+struct PBars {
+  uint64_t afull[kPAStages], aempty[kPAStages];
+  uint64_t wfull[kPW], wempty[kPW];
+  uint64_t dfull[kSDSlots], dempty[kSDSlots];
+  uint64_t tfull[2], tempty[2];
+};
+
+__global__ void __launch_bounds__(kPThreads, 1)
+    kv_pre_kernel(const Args a, const PrePlan plan, const uint8_t* __restrict__ wkv,
+                  const int bdst) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* pipe = align1024(smem_raw);
+  __shared__ PBars B;
+  __shared__ uint32_t s_tmem;
+  __shared__ TDesc bd[kSDSlots];
+  __shared__ float s_omega[256], s_phi[256];
+  __shared__ float s_bias[2 * kMaxModel];
+  __shared__ int64_t s_seg[kTDescWarps][4 * 32 + 1];
+  __shared__ float s_td[kTDescWarps][4 * 32];
+  float* s_pvf = reinterpret_cast<float*>(pipe + kPPipeBytes);
+  constexpr uint32_t kCols = 256;
+  constexpr int dm = 100;
+  const tgl_attn_params& P = a.P;
+  const bool split = a.split != 0;
+  const int nch = plan.n;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  // prologue independent of the predecessor grid (PDL): barriers, TMEM, constants
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < kPAStages; ++s) {
+      mbar_init(&B.afull[s], kPLoadWarps * 32 + kPTimeWarps);
+      mbar_init(&B.aempty[s], 1);
+    }
+    for (int s = 0; s < kPW; ++s) {
+      mbar_init(&B.wfull[s], 1);
+      mbar_init(&B.wempty[s], 1);
+    }
+    for (int s = 0; s < kSDSlots; ++s) {
+      mbar_init(&B.dfull[s], 1);
+      mbar_init(&B.dempty[s], kBEpi + kPLoadWarps + kPTimeWarps + 2);
+    }
+    for (int s = 0; s < 2; ++s) {
+      mbar_init(&B.tfull[s], 1);
+      mbar_init(&B.tempty[s], kBEpi);
+    }
+    fence_mbar_init();
+  }
+  TGL_TRACE_RESET();
+  if (warp == kTMma) tmem_alloc(&s_tmem, 2 * kCols);
+  for (int j = threadIdx.x; j < P.d_t; j += blockDim.x) {
+    s_omega[j] = P.omega[j];
+    s_phi[j] = P.phi[j];
+  }
+  for (int j = threadIdx.x; j < 2 * dm; j += blockDim.x) s_bias[j] = j < dm ? P.bk[j] : P.bv[j - dm];
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  pdl_wait();     // PDL: predecessor grid complete, its writes visible
+  pdl_trigger();
+  const int64_t n = dev_count(a.n_dst_dev, a.n_dst_max);
+  const uint32_t tmem = s_tmem;
+  const uint32_t pipe_s = smem_u32(pipe);
+  const uint32_t a_s = pipe_s;                                  // A ring
+  const uint32_t w_s = pipe_s + kPAStages * kPAStage;           // weight ring
+  uint32_t tt = 0;
+  const int kt0 = plan.dp0 + plan.dp1;                          // first time column of K'
+
+  if (warp >= kTDesc0 && warp < kTDesc0 + kTDescWarps) {   // ------- tile builders
+    const int dw = warp - kTDesc0;
+    const int64_t hoff = a.hsrc_off_dev ? *a.hsrc_off_dev : 0;
+    const int dpt = 4 * bdst;
+    const int64_t ntiles = (n + dpt - 1) / dpt;
+    int64_t* sg = s_seg[dw];
+    float* stdv = s_td[dw];
+    for (tt = dw;; tt += kTDescWarps) {
+      const uint32_t ds = tt % kSDSlots;
+      wait_free_sleep(&B.dempty[ds], tt / kSDSlots, TGL_SLEEP_DESC);
+      TDesc& R = bd[ds];
+      const int64_t T = blockIdx.x + (int64_t)tt * gridDim.x;
+      if (T >= ntiles) {
+        if (lane == 0) R.live = 0;
+        warp_arrive(&B.dfull[ds]);
+        break;
+      }
+      const int64_t d0 = T * dpt;
+      const int nd = (int)((n - d0) < dpt ? (n - d0) : dpt);
+      for (int j = lane; j <= nd; j += 32) sg[j] = a.seg_ptr[d0 + j];
+      for (int j = lane; j < nd; j += 32) stdv[j] = a.dst_t[d0 + j];
+      __syncwarp();
+      int64_t er[4] = {0, 0, 0, 0};
+      float tr[4] = {0.f, 0.f, 0.f, 0.f};
+      int dr[4] = {-1, -1, -1, -1};
+      unsigned ovf_bins = 0;
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int j0 = u * bdst;
+        if (j0 >= nd) continue;
+        const int j1 = (j0 + bdst) < nd ? j0 + bdst : nd;
+        const int64_t e0 = sg[j0], e1 = sg[j1];
+        if (e1 - e0 > 32) {
+          ovf_bins |= 1u << u;
+          continue;
+        }
+        const int64_t e = e0 + lane;
+        if (e < e1) {
+          int j = j0;
+          while (sg[j + 1] <= e) ++j;
+          dr[u] = (int)(d0 + j);
+          er[u] = e;
+          tr[u] = stdv[j];
+        }
+      }
+      for (int j = 0; j < nd; ++j) {
+        const bool ovf = (ovf_bins >> (j / bdst)) & 1u;
+        if (sg[j + 1] == sg[j] || ovf) {
+          const float fill = ovf ? __int_as_float(0x7fc00000) : 0.f;
+          for (int c = lane; c < dm; c += 32) a.rbuf[(d0 + j) * kQLd + c] = fill;
+        }
+      }
+      R.live = 1;
+      int32_t hi[4], ei[4];
+      float et[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const bool ok = dr[u] >= 0;
+        hi[u] = ok ? (a.hsrc_idx ? a.hsrc_idx[hoff + er[u]] : (int32_t)(hoff + er[u])) : 0;
+        ei[u] = (ok && P.d_e > 0) ? a.eid[er[u]] : 0;
+        et[u] = ok ? a.edge_t[er[u]] : 0.f;
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int r = 32 * u + lane;
+        const bool ok = dr[u] >= 0;
+        const float dt = tr[u] - et[u];               // fp32 delta (R18)
+        R.hrow[r] = ok ? hi[u] : -1;
+        R.erow[r] = ok ? ei[u] : -1;
+        R.dt[r] = ok ? dt : 0.f;
+        R.trow[r] = ok ? (int)tenc_table_row(dt, a.table, a.window) : -1;
+        R.rdst[r] = dr[u];
+      }
+      warp_arrive(&B.dfull[ds]);
+    }
+  } else if (warp == kTW) {                          // ---------------- weight loader
+    uint32_t wl = 0;
+    const uint32_t wbytes = split ? kTWStage : kTWHalf;
+    for (;; ++tt) {
+      const uint32_t ds = tt % kSDSlots;
+      mbar_wait_sleep(&B.dfull[ds], (tt / kSDSlots) & 1u, TGL_SLEEP_W);
+      const int live = bd[ds].live;
+      warp_arrive(&B.dempty[ds]);
+      if (!live) break;
+      if (lane == 0) {
+        const int r0 = (tt > 0 && nch >= 4) ? 2 : 0;
+        for (int i = r0; i < nch; ++i) {
+          const uint32_t k = wl + (i - r0);
+          const uint32_t sw = k % kPW;
+          wait_free_sleep(&B.wempty[sw], k / kPW, TGL_SLEEP_W);
+          mbar_arrive_expect_tx(&B.wfull[sw], wbytes);
+          bulk_g2s(pipe + kPAStages * kPAStage + sw * kTWStage,
+                   wkv + (size_t)plan.order[chunk_of(tt, i, nch)] * kTWStage, wbytes, &B.wfull[sw]);
+        }
+        wl += nch - r0;
+      }
+      __syncwarp();
+    }
+  } else if (warp >= kPLoad0 && warp < kPLoad0 + kPLoadWarps) {   // ---------- loaders
+    // lane: rows lw*32 + (lane>>3) + 4k (k = 0..7); piece pc = lane & 7 of the row's
+    // 32-column chunk: hi group pc (pc < 4) or lo group pc - 4, 16 bytes each
+    const int lw = warp - kPLoad0;
+    const int r0 = lw * 32 + (lane >> 3), pc = lane & 7;
+    const bool lo_piece = pc >= 4;
+    const int j = pc & 3;
+    const uint32_t ofs0 = (uint32_t)(r0 >> 3) * 1024 + (lo_piece ? 512 : 0);
+    const bool active = split || !lo_piece;         // bf16 mode: hi halves only
+    // split16 precompute table: its rows are gathered like features (time warps only
+    // evaluate Phi for the rows the table misses)
+    const bool tsplit = (P.input_layout & TGL_SPLIT_TABLE) && a.table != nullptr;
+    const uint8_t* hbase = reinterpret_cast<const uint8_t*>(a.hsrc);
+    const uint8_t* ebase = reinterpret_cast<const uint8_t*>(a.efeat);
+    const uint8_t* tbase = reinterpret_cast<const uint8_t*>(a.table);
+    const int64_t hld = 4 * a.ld_hsrc, eld = 4 * a.ld_e, tld = 4 * plan.dpt;
+    uint32_t g = 0;
+    for (;; ++tt) {
+      const uint32_t ds = tt % kSDSlots;
+      mbar_wait_sleep(&B.dfull[ds], (tt / kSDSlots) & 1u, TGL_SLEEP_LOAD);
+      const TDesc& R = bd[ds];
+      if (!R.live) {
+        warp_arrive(&B.dempty[ds]);
+        break;
+      }
+      int hrow[8], erow[8], trw[8];
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        hrow[k] = R.hrow[r0 + 4 * k];
+        erow[k] = R.erow[r0 + 4 * k];
+        trw[k] = (tsplit && R.rdst[r0 + 4 * k] >= 0) ? R.trow[r0 + 4 * k] : -1;
+      }
+      __syncwarp();
+      warp_arrive(&B.dempty[ds]);
+      for (int i = 0; i < nch; ++i, ++g) {
+        const int c = plan.order[chunk_of(tt, i, nch)];
+        const int col = c * kTC + 8 * j;             // K' column of this piece
+        const int ks = (plan.k - c * kTC) > 16 ? 2 : 1;   // K steps the MMA issues
+        const uint32_t sa = g % kPAStages;
+        wait_free_sleep(&B.aempty[sa], g / kPAStages, TGL_SLEEP_LOAD);
+        const bool in_k = active && col < c * kTC + 16 * ks && !(TGL_DBG(a) & 2);
+        const uint32_t dst = a_s + sa * kPAStage + ofs0;
+        if (in_k && col < kt0) {                     // a gathered feature piece
+          const bool seg_h = col < plan.dp0;
+          const uint8_t* base = seg_h ? hbase : ebase;
+          const int64_t ldb = seg_h ? hld : eld;
+          const uint32_t pofs = seg_h ? (uint32_t)(lo_piece ? 2 * plan.dp0 : 0) + 2 * col
+                                      : (uint32_t)(lo_piece ? 2 * plan.dp1 : 0) +
+                                            2 * (col - plan.dp0);
+#pragma unroll
+          for (int k = 0; k < 8; ++k) {
+            const int row = seg_h ? hrow[k] : erow[k];
+            const int rr = (r0 + 4 * k) & 7;
+            const uint32_t d = dst + (uint32_t)(k >> 1) * 1024 + rr * 64 +
+                               (((j ^ (rr >> 1)) & 3) << 4);
+            cp_async16_zfill(d, base + (row >= 0 ? (int64_t)row * ldb + pofs : 0),
+                             row >= 0 ? 16u : 0u);
+          }
+        } else if (in_k && tsplit && col < plan.k) {  // a time piece of a table row
+          const uint32_t pofs = (uint32_t)(lo_piece ? 2 * plan.dpt : 0) + 2 * (col - kt0);
+#pragma unroll
+          for (int k = 0; k < 8; ++k) {
+            if (trw[k] < 0) continue;                  // Phi evaluated by the time warps
+            const int rr = (r0 + 4 * k) & 7;
+            const uint32_t d = dst + (uint32_t)(k >> 1) * 1024 + rr * 64 +
+                               (((j ^ (rr >> 1)) & 3) << 4);
+            cp_async16_zfill(d, tbase + (int64_t)trw[k] * tld + pofs, 16u);
+          }
+        }                                            // (other time + K padding: time warps)
+        cp_async_mbar_arrive_noinc(&B.afull[sa]);
+      }
+    }
+  } else if (warp >= kPTime0 && warp < kPTime0 + kPTimeWarps) {   // -------- time warps
+    // thread: row w*32 + lane, the 8-column groups of every chunk that holds time
+    // columns: Phi (eq 8, R10 argument; reduced + SFU cosine, the accurate cosf only
+    // where a row's |argument| >= 1e9) -> bf16 hi / lo -> the A stage
+    const int tw = warp - kPTime0;
+    const int r = tw * 32 + lane;
+    const int rr = r & 7;
+    const bool tsplit = (P.input_layout & TGL_SPLIT_TABLE) && a.table != nullptr;
+    const uint32_t rofs = (uint32_t)(r >> 3) * 1024 + rr * 64;
+    uint32_t g = 0;
+    for (;; ++tt) {
+      const uint32_t ds = tt % kSDSlots;
+      mbar_wait_sleep(&B.dfull[ds], (tt / kSDSlots) & 1u, TGL_SLEEP_LOAD);
+      const TDesc& R = bd[ds];
+      if (!R.live) {
+        warp_arrive(&B.dempty[ds]);
+        break;
+      }
+      const float dtr = R.dt[r];
+      // 0: evaluate Phi; 1: table row (split16: gathered by the loaders, fp32: read here);
+      // 2: padding row (zeros)
+      const int trow = R.trow[r];
+      const int mode = R.rdst[r] < 0 ? 2 : (trow >= 0 ? 1 : 0);
+      __syncwarp();
+      warp_arrive(&B.dempty[ds]);
+      for (int i = 0; i < nch; ++i, ++g) {
+        const int c = plan.order[chunk_of(tt, i, nch)];
+        const int ks = (plan.k - c * kTC) > 16 ? 2 : 1;
+        const uint32_t sa = g % kPAStages;
+        const bool has_time = (c + 1) * kTC > kt0 && !(TGL_DBG(a) & 64);
+        if (has_time) {
+          wait_free(&B.aempty[sa], g / kPAStages);
+          const uint32_t dst = a_s + sa * kPAStage + rofs;
+#pragma unroll
+          for (int jj = 0; jj < 4; ++jj) {
+            const int col = c * kTC + 8 * jj;
+            if (col < kt0 || col >= c * kTC + 16 * ks) continue;     // warp-uniform
+            const int tc = col - kt0;                 // time column of the group
+            if (tsplit && mode == 1 && col < plan.k) continue;   // gathered from the table
+            float x[8];
+            if (mode == 0) {
+              bool bad = false;
+#pragma unroll
+              for (int e = 0; e < 8; ++e) {
+                const float bb = __fadd_rn(__fmul_rn(s_omega[tc + e], dtr), s_phi[tc + e]);
+                bad |= !(fabsf(bb) < 1e9f);
+                x[e] = tenc_cos_reduced(bb);
+              }
+              if (bad) {                              // rare: |b| >= 1e9 or non-finite
+#pragma unroll
+                for (int e = 0; e < 8; ++e) x[e] = tenc_fast(dtr, s_omega[tc + e], s_phi[tc + e]);
+              }
+            } else if (mode == 1 && !tsplit) {
+#pragma unroll
+              for (int e = 0; e < 8; ++e)
+                x[e] = tc + e < P.d_t ? __ldg(a.table + (int64_t)trow * P.d_t + tc + e) : 0.f;
+            } else {
+#pragma unroll
+              for (int e = 0; e < 8; ++e) x[e] = 0.f;
+            }
+            if (tc + 8 > P.d_t) {                     // padding columns of the time segment
+#pragma unroll
+              for (int e = 0; e < 8; ++e)
+                if (tc + e >= P.d_t) x[e] = 0.f;
+            }
+            uint32_t h[4], l[4];
+#pragma unroll
+            for (int e = 0; e < 4; ++e) split2(x[2 * e], x[2 * e + 1], h[e], l[e]);
+            const uint32_t po = (uint32_t)(((jj ^ (rr >> 1)) & 3) << 4);
+            st_shared_v4(dst + po, h[0], h[1], h[2], h[3]);
+            if (split) st_shared_v4(dst + 512 + po, l[0], l[1], l[2], l[3]);
+          }
+          fence_proxy_async_smem();
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&B.afull[sa]);
+        } else {
+          // no time columns: arrive once the stage's previous use is released, so the
+          // arrival counts toward this chunk's phase
+          if (lane == 0) {
+            wait_free(&B.aempty[sa], g / kPAStages);
+            mbar_arrive(&B.afull[sa]);
+          }
+          __syncwarp();
+        }
+      }
+    }
+  } else if (warp == kTMma) {                        // ---------------- MMA issuer
+    uint32_t g = 0, wl = 0;
+    constexpr uint32_t idesc = idesc_bf16(kBM, kNPkv);
+    for (;; ++tt) {
+      const uint32_t ds = tt % kSDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kSDSlots) & 1u);
+      const int live = bd[ds].live;
+      warp_arrive(&B.dempty[ds]);
+      if (!live) break;
+      const uint32_t acc = tmem + (tt & 1u) * kCols;
+      wait_free(&B.tempty[tt & 1u], tt >> 1);
+      tc_fence_after();
+      const int r0 = (tt > 0 && nch >= 4) ? 2 : 0;
+      for (int i = 0; i < nch; ++i, ++g) {
+        const int c = plan.order[chunk_of(tt, i, nch)];
+        const int nk = (plan.k - c * kTC) > 16 ? 2 : 1;
+        const uint32_t sa = g % kPAStages;
+        mbar_wait(&B.afull[sa], (g / kPAStages) & 1u);
+        uint32_t kw;
+        if (i < r0) {
+          kw = wl - 1 - i;                           // resident from the previous tile
+        } else {
+          kw = wl + (i - r0);
+          mbar_wait(&B.wfull[kw % kPW], (kw / kPW) & 1u);
+        }
+        tc_fence_after();
+        if (elect_one()) {
+          const uint64_t a0 = desc_sw64(a_s + sa * kPAStage, 1024);
+          const uint64_t w0 = desc_sw64(w_s + (kw % kPW) * kTWStage, 512);
+#pragma unroll
+          for (int ks = 0; ks < 2; ++ks) {
+            if (ks < nk && !(TGL_DBG(a) & 4)) {
+              const uint64_t ah = a0 + 2 * ks, bh = w0 + 2 * ks;
+              mma_bf16(acc, ah, bh, idesc, (i | ks) != 0);
+              if (split) {
+                mma_bf16(acc, ah + (512 >> 4), bh, idesc, 1u);
+                mma_bf16(acc, ah, bh + (kTWHalf >> 4), idesc, 1u);
+              }
+            }
+          }
+          const bool keep = (nch >= 4) && (i >= nch - 2);   // reused by the next tile
+          mma_commit(&B.aempty[sa]);
+          if (!keep) mma_commit(&B.wempty[kw % kPW]);
+        }
+        __syncwarp();
+      }
+      wl += nch - r0;
+      if (elect_one()) mma_commit(&B.tfull[tt & 1u]);
+      __syncwarp();
+    }
+  } else if (warp < kBEpi) {                         // ---------------- epilogue warps 0-7
+    bin_epilogue<kSDSlots, TDesc, kSPW, false>(a, B.dfull, B.dempty, B.tfull, B.tempty, bd,
+                                               tmem, s_pvf, s_bias);
+  }
+  ws_teardown(tmem, 2 * kCols, kTMma);
+}
+
 }  // namespace tca
 
 // ------------------------------------------------------------------ host side
 namespace tca {
 
 struct PackedLayout {
-  size_t oq, okv, oo, okv64, okvc, total;
+  size_t oq, okv, oo, okv64, okvc, okvp, total;
 };
 
 static PackedLayout packed_layout(const tgl_attn_params* P) {
@@ -2432,6 +2897,7 @@ static PackedLayout packed_layout(const tgl_attn_params* P) {
   L.oo = W.take((size_t)so.nchunks * 2 * kNPq * 128);
   L.okv64 = W.take((size_t)make_plan(P->d_hsrc, P->d_e, P->d_t).n * kTWStage);
   L.okvc = W.take((size_t)make_plan_contig(P->d_hsrc, P->d_e, P->d_t).n * kTWStage);
+  L.okvp = W.take((size_t)make_pre_plan(P->d_hsrc, P->d_e, P->d_t).n * kTWStage);
   L.total = W.off;
   return L;
 }
@@ -2453,7 +2919,11 @@ static tgl_status launch_pack(const tgl_attn_params* P, uint8_t* base, cudaStrea
   pack_kv64_kernel<<<64, 256, 0, s>>>(P->Wk, P->Wv, P->d_model, P->d_hsrc + P->d_e + P->d_t,
                                       make_plan_contig(P->d_hsrc, P->d_e, P->d_t),
                                       base + L.okvc);
-  return launch_check("pack_kv64 contiguous");
+  TGL_TRY(launch_check("pack_kv64 contiguous"));
+  pack_kv_pre_kernel<<<64, 256, 0, s>>>(P->Wk, P->Wv, P->d_model, P->d_hsrc + P->d_e + P->d_t,
+                                        make_pre_plan(P->d_hsrc, P->d_e, P->d_t),
+                                        base + L.okvp);
+  return launch_check("pack_kv_pre");
 }
 
 }  // namespace tca
@@ -2490,6 +2960,9 @@ static tgl_status set_smem_attrs(int smem_q, int smem_kv, int smem_kvb) {
     if (e == cudaSuccess)
       e = cudaFuncSetAttribute(kv_split_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                kSSmem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(kv_pre_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               kPSmem);
     return e;
   }), "smem attributes");
 }
@@ -2576,9 +3049,44 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
   launch_pdl(dense_kernel<false>, dim3(gq), dim3(kWsThreads), smem_q, s, a);
   TGL_TRY(launch_check("tc q kernel"));
   const int sel = P->kv_kernel;
-  if (sel < TGL_KV_AUTO || sel > TGL_KV_GENERAL) {
+  if (sel < TGL_KV_AUTO || sel > TGL_KV_PRE || sel == TGL_KV_SIMT) {
     set_error("kv_kernel %d: not a TGL_KV_* id", sel);
     return TGL_EINVAL;
+  }
+  const bool pre_in = (P->input_layout & (TGL_SPLIT_HSRC | TGL_SPLIT_E | TGL_SPLIT_TABLE)) != 0;
+  if (pre_in || sel == TGL_KV_PRE) {
+    // pre-split h_src / e tables (tgl_split_rows): every gathered table present must be
+    // split, rows 16-byte aligned; max_seg <= 32 and 2 heads (the binned epilogue)
+    const PrePlan plan = make_pre_plan(P->d_hsrc, P->d_e, P->d_t);
+    const bool hs_ok = P->d_hsrc == 0 || ((P->input_layout & TGL_SPLIT_HSRC) &&
+                                          ld_hsrc >= plan.dp0 && rows_16b(hsrc, 1, ld_hsrc));
+    const bool e_ok = P->d_e == 0 || ((P->input_layout & TGL_SPLIT_E) && ld_e >= plan.dp1 &&
+                                      rows_16b(efeat, 1, ld_e));
+    const bool t_ok = !(P->input_layout & TGL_SPLIT_TABLE) || table == nullptr ||
+                      rows_16b(table, 1, plan.dpt);
+    if (!(sel == TGL_KV_AUTO || sel == TGL_KV_PRE) || !hs_ok || !e_ok || !t_ok ||
+        !(max_seg > 0 && max_seg <= 32 && P->n_heads == 2) || plan.n > kPMaxChunks) {
+      set_error("pre-split inputs: kv_kernel must be AUTO/PRE, every gathered table split "
+                "(input_layout), 16-byte rows, ld >= padded width, max_seg <= 32, 2 heads");
+      return TGL_EUNSUPPORTED;
+    }
+    tgl_kv_probe* probe = P->probe;
+    if (probe) {
+      probe->kernel = TGL_KV_PRE;
+      if (probe->ev_start)
+        TGL_TRY(cuda_check(cudaEventRecord(static_cast<cudaEvent_t>(probe->ev_start), s),
+                           "probe event"));
+    }
+    const int bdst = 32 / max_seg;
+    const int64_t ttiles = ceil_div(n_dst_max, 4 * bdst);
+    const unsigned gt = (unsigned)(ttiles < kNumSMs ? (ttiles > 0 ? ttiles : 1) : kNumSMs);
+    launch_pdl(kv_pre_kernel, dim3(gt), dim3(kPThreads), kPSmem, s, a, plan, pk + PL.okvp, bdst);
+    TGL_TRY(launch_check("tc kv pre kernel"));
+    if (probe && probe->ev_stop)
+      TGL_TRY(cuda_check(cudaEventRecord(static_cast<cudaEvent_t>(probe->ev_stop), s),
+                         "probe event"));
+    launch_pdl(dense_kernel<true>, dim3(gq), dim3(kWsThreads), smem_q, s, a);
+    return launch_check("tc ffn kernel");
   }
   const bool binned = max_seg > 0 && max_seg <= 32 && P->n_heads == 2;
   const bool async = binned && rows_16b(hsrc, P->d_hsrc, ld_hsrc) && rows_16b(efeat, P->d_e, ld_e) &&

@@ -20,10 +20,12 @@ TGL_INPUT_TIME_SORTED = 2
 RECENT, UNIFORM = 0, 1
 FP32, BF16, FP32_SIMT = 0, 1, 2
 # tgl_attn_params.kv_kernel (include/tgl.h TGL_KV_*)
-KV_KERNEL = {"auto": 0, "split": 1, "split_pad": 2, "async": 3, "bin": 4, "general": 5}
+KV_KERNEL = {"auto": 0, "split": 1, "split_pad": 2, "async": 3, "bin": 4, "general": 5,
+             "pre": 7}
+SPLIT_HSRC, SPLIT_E, SPLIT_TABLE = 1, 2, 4
 KV_KERNEL_NAME = {1: "kv_split_kernel (contiguous K plan)", 2: "kv_split_kernel (padded K plan)",
                   3: "kv_async_kernel", 4: "kv_bin_kernel", 5: "kv_kernel (general)",
-                  6: "kv_attn_kernel (SIMT)"}
+                  6: "kv_attn_kernel (SIMT)", 7: "kv_pre_kernel (pre-split operands)"}
 STRATEGY = {"recent": RECENT, "uniform": UNIFORM}
 PRECISION = {"fp32": FP32, "bf16": BF16, "fp32_simt": FP32_SIMT}
 
@@ -31,7 +33,7 @@ SYMBOLS = ["tgl_version", "tgl_status_string", "tgl_last_error", "tgl_build_tcsr
            "tgl_batch_roots", "tgl_dedup", "tgl_sample", "tgl_next_block",
            "tgl_time_precompute", "tgl_time_encode", "tgl_tblock_attn", "tgl_gather_rows",
            "tgl_attn_packed_bytes", "tgl_attn_pack", "tgl_cache_lookup", "tgl_cache_store", "tgl_cache_combine",
-           "tgl_cache_merge", "tgl_shard_slice", "tgl_shard_gather"]
+           "tgl_cache_merge", "tgl_shard_slice", "tgl_shard_gather", "tgl_split_rows"]
 
 
 class TGLError(RuntimeError):
@@ -67,6 +69,7 @@ def _load():
         "tgl_cache_merge": [vp, i64, vp, vp, vp, vp, vp, vp, i64, vp, i64, vp],
         "tgl_shard_slice": [i64, vp, vp, vp, i32, i32, vp, vp, vp, vp],
         "tgl_shard_gather": [i64, vp, vp, i64, vp, i32, vp, i64, i32, vp, i64, vp],
+        "tgl_split_rows": [i64, i32, vp, i64, vp, i64, vp],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -262,7 +265,8 @@ class AttnParamsC(C.Structure):
                 ("omega", C.c_void_p), ("phi", C.c_void_p),
                 ("leaky_slope", C.c_float), ("logit_scale", C.c_float),
                 ("precision", C.c_int32), ("packed", C.c_void_p),
-                ("kv_kernel", C.c_int32), ("probe", C.c_void_p)]
+                ("kv_kernel", C.c_int32), ("probe", C.c_void_p),
+                ("input_layout", C.c_int32)]
 
 
 class KvProbeC(C.Structure):
@@ -316,7 +320,7 @@ class AttnParams:
                                   _p(self.t["omega"]), _p(self.t["phi"]),
                                   float(p["leaky_slope"]), float(p["logit_scale"]),
                                   self.precision, None,
-                                  KV_KERNEL.get(kv_kernel, kv_kernel), None)
+                                  KV_KERNEL.get(kv_kernel, kv_kernel), None, 0)
         self.packed = None
         if pack and self.precision != FP32_SIMT:
             nb = _lib.tgl_attn_packed_bytes(C.byref(self.struct))
@@ -463,4 +467,40 @@ def shard_gather(gathered, c_max: int, world: int, u_max: int, u_dev=None, idx=N
     _check(_lib.tgl_shard_gather(n_max, _p(n_dev), _p(idx), u_max, _p(u_dev), world,
                                  _p(gathered), c_max, d, _p(out), out.stride(0), _s(stream)),
            "tgl_shard_gather")
+    return out
+
+
+# --------------------------------------------------------------------------- split16 tables
+def split_width(d: int) -> int:
+    """Row pitch (4-byte words) of a split16 table of d columns."""
+    return (d + 7) // 8 * 8
+
+
+def split_rows(src, out=None, n_rows=None, stream=None):
+    """fp32 [n, d] (unit column stride) -> split16 table viewed as float32 [n, dp]
+    (bf16 hi of dp columns, then bf16 lo; tgl_split_rows)."""
+    n = src.shape[0] if n_rows is None else n_rows
+    d = src.shape[1]
+    dp = split_width(d)
+    if out is None:
+        out = torch.empty(max(n, 1), dp, dtype=torch.float32, device=src.device)
+    assert out.stride(1) == 1 and out.shape[1] >= dp
+    _check(_lib.tgl_split_rows(n, d, _prow(src), src.stride(0), out.data_ptr(), out.stride(0),
+                               _s(stream)), "tgl_split_rows")
+    return out
+
+
+def split_table(n_rows: int, d: int, make_rows, chunk_rows: int = 1 << 20, device=None,
+                stream=None):
+    """A split16 table of n_rows x d built chunk by chunk: make_rows(r0, r1) returns the fp32
+    rows [r0, r1) on the device; each chunk is split into place, so the fp32 table never
+    exists whole (GDELT's 142 GB of edge features)."""
+    device = device or torch.device("cuda")
+    dp = split_width(d)
+    out = torch.empty(max(n_rows, 1), dp, dtype=torch.float32, device=device)
+    for r0 in range(0, n_rows, chunk_rows):
+        r1 = min(n_rows, r0 + chunk_rows)
+        rows = make_rows(r0, r1)
+        split_rows(rows, out=out[r0:r1], stream=stream)
+        del rows
     return out

@@ -95,24 +95,32 @@ def _run(name, host_gb, dev_gb):
     segs = _check_tcsr(cfg, src, dst, t, tc, src_h, dst_h, t_h, rng)
     torch.cuda.empty_cache()
 
-    # the bench's layout: rows padded to a 16-byte pitch (GDELT 413 / 186 -> 416 / 188), so
-    # the split-role K|V kernel runs with the per-segment padded K plan it times
+    # the bench's layout (bench.load_world_device): fp32 node rows with a 16-byte pitch
+    # for h_dst, split16 operand tables for the K|V gathers (edge features built chunk by
+    # chunk: the fp32 table never exists), so the kernel the bench times runs here
+    split = name != "MAG"     # MAG: fp32 rows (no room for a second 62 GB node table)
     nfeat = sg.device_feature_table(cfg.seeds["feat"], cfg.n_nodes, cfg.d_v, dev, pitch_mult=4)
-    efeat = (sg.device_feature_table(cfg.seeds["feat"] + 7919, cfg.n_edges, cfg.d_e, dev,
-                                     pitch_mult=4)
-             if cfg.d_e else torch.zeros((0, 0), dtype=torch.float32, device=dev))
+    efeat = None
+    efeat_split = (tgl.split_table(cfg.n_edges, cfg.d_e,
+                                   lambda r0, r1: sg.feature_rows_torch(
+                                       cfg.seeds["feat"] + 7919, torch.arange(r0, r1, device=dev),
+                                       cfg.d_e))
+                   if cfg.d_e else None)
     rows = rng.integers(0, cfg.n_nodes, 5)
     assert np.array_equal(nfeat[torch.from_numpy(rows).to(dev)].cpu().numpy(),
                           synth.feature_rows(cfg.seeds["feat"], rows, cfg.d_v))
     params = synth.gen.model_params(cfg)
-    graph = {"src": src, "dst": dst, "t": t, "neg": neg, "nfeat": nfeat, "efeat": efeat}
+    graph = {"src": src, "dst": dst, "t": t, "neg": neg, "nfeat": nfeat, "efeat": efeat,
+             "nfeat_split": tgl.split_rows(nfeat) if split else None,
+             "efeat_split": efeat_split}
+    layout = "split" if split else "fp32"
     pipe = TGATPipeline(graph, tc, params, cfg.batch,
                         TSampler(cfg.k, cfg.strategy, cfg.seeds["sampler"]), cfg.dedup,
-                        cfg.precompute, cfg.window, "fp32")
+                        cfg.precompute, cfg.window, "fp32", layout=layout)
     pipe.capture()
     pipe16 = TGATPipeline(graph, tc, params, cfg.batch,
                           TSampler(cfg.k, cfg.strategy, cfg.seeds["sampler"]), cfg.dedup,
-                          cfg.precompute, cfg.window, "bf16")
+                          cfg.precompute, cfg.window, "bf16", layout=layout)
     pipe16.capture()
     # the K|V kernel the bench times on this layout
     probe = tgl.KvProbe()
@@ -122,7 +130,7 @@ def _run(name, host_gb, dev_gb):
     pipe.forward()
     torch.cuda.synchronize()
     pipe.attn[tail].attach_probe(None)
-    want = "split" if (cfg.d_v % 4 == 0 and cfg.d_e % 4 == 0) else "split_pad"
+    want = "pre" if split else ("split" if cfg.d_v % 4 == 0 else "split_pad")
     assert probe.kernel == tgl.KV_KERNEL[want], (probe.kernel, want)
 
     class _G:   # host view for batch slicing
@@ -164,7 +172,7 @@ def _run(name, host_gb, dev_gb):
         torch.cuda.synchronize()
         err16 = np.abs(e16.cpu().numpy()[pick] - exp).max()
         assert err16 <= 5e-2, err16
-    del pipe, pipe16, graph, nfeat, efeat, tc, src, dst, t, neg
+    del pipe, pipe16, graph, nfeat, efeat, efeat_split, tc, src, dst, t, neg
     torch.cuda.empty_cache()
 
 

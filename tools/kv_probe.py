@@ -50,11 +50,16 @@ if os.environ.get("PROBE_WINDOW"):          # 0 = direct evaluation, else a smal
     tab = tgl.time_precompute(w, a.t["omega"], a.t["phi"]) if w > 0 else None
 
 
+hs = pipe.nfeat_split if pipe.split else nf          # operand tables of the pipeline layout
+if pipe.split:
+    ef = pipe.efeat_split
+
+
 def call():
     _call_ws(lib.tgl_tblock_attn,
              [tgl.C.byref(a.struct), b.n_max, tgl._p(b.u_dev), tgl._p(b.seg_ptr), tgl._p(b.uniq_t),
-              tgl._prow(nf), tgl._p(b.uniq_node), nf.stride(0), tgl._prow(nf), tgl._p(b.nbr), None,
-              nf.stride(0), tgl._prow(ef), tgl._p(b.eid), ef.stride(0), tgl._p(b.ts),
+              tgl._prow(nf), tgl._p(b.uniq_node), nf.stride(0), tgl._prow(hs), tgl._p(b.nbr), None,
+              hs.stride(0), tgl._prow(ef), tgl._p(b.eid), ef.stride(0), tgl._p(b.ts),
               tgl._p(tab), 0 if tab is None else tab.shape[0], cfg.k, tgl._p(b.out)],
              b.ws["attn"], None, "tail attn")
 
