@@ -2701,7 +2701,11 @@ __global__ void __launch_bounds__(kPThreads, 1)
         const int col = c * kTC + 8 * j;             // K' column of this piece
         const int ks = (plan.k - c * kTC) > 16 ? 2 : 1;   // K steps the MMA issues
         const uint32_t sa = g % kPAStages;
+        TGL_PROF_CLK(l0);
         wait_free_sleep(&B.aempty[sa], g / kPAStages, TGL_SLEEP_LOAD);
+#ifdef TGL_KV_PROF
+        if (lw == 0) prof_add(a, 5, clock64() - l0);  // loader: wait for a free stage
+#endif
         const bool in_k = active && col < c * kTC + 16 * ks && !(TGL_DBG(a) & 2);
         const uint32_t dst = a_s + sa * kPAStage + ofs0;
         if (in_k && col < kt0) {                     // a gathered feature piece
@@ -2765,7 +2769,9 @@ __global__ void __launch_bounds__(kPThreads, 1)
         const uint32_t sa = g % kPAStages;
         const bool has_time = (c + 1) * kTC > kt0 && !(TGL_DBG(a) & 64);
         if (has_time) {
+          TGL_PROF_CLK(t0);
           wait_free(&B.aempty[sa], g / kPAStages);
+          TGL_PROF_CLK(t1);
           const uint32_t dst = a_s + sa * kPAStage + rofs;
 #pragma unroll
           for (int jj = 0; jj < 4; ++jj) {
@@ -2808,6 +2814,12 @@ __global__ void __launch_bounds__(kPThreads, 1)
           }
           fence_proxy_async_smem();
           __syncwarp();
+#ifdef TGL_KV_PROF
+          if (tw == 0) {
+            prof_add(a, 0, t1 - t0);                   // time warp: wait for a free stage
+            prof_add(a, 1, clock64() - t1);            // time warp: Phi + split + store
+          }
+#endif
           if (lane == 0) mbar_arrive(&B.afull[sa]);
         } else {
           // no time columns: arrive once the stage's previous use is released, so the
@@ -2830,14 +2842,21 @@ __global__ void __launch_bounds__(kPThreads, 1)
       warp_arrive(&B.dempty[ds]);
       if (!live) break;
       const uint32_t acc = tmem + (tt & 1u) * kCols;
+      TGL_PROF_CLK(mt0);
       wait_free(&B.tempty[tt & 1u], tt >> 1);
+      TGL_PROF_CLK(mt1);
+#ifdef TGL_KV_PROF
+      prof_add(a, 7, mt1 - mt0);                     // MMA: wait for an accumulator
+#endif
       tc_fence_after();
       const int r0 = (tt > 0 && nch >= 4) ? 2 : 0;
       for (int i = 0; i < nch; ++i, ++g) {
         const int c = plan.order[chunk_of(tt, i, nch)];
         const int nk = (plan.k - c * kTC) > 16 ? 2 : 1;
         const uint32_t sa = g % kPAStages;
+        TGL_PROF_CLK(ma0);
         mbar_wait(&B.afull[sa], (g / kPAStages) & 1u);
+        TGL_PROF_CLK(ma1);
         uint32_t kw;
         if (i < r0) {
           kw = wl - 1 - i;                           // resident from the previous tile
@@ -2845,6 +2864,10 @@ __global__ void __launch_bounds__(kPThreads, 1)
           kw = wl + (i - r0);
           mbar_wait(&B.wfull[kw % kPW], (kw / kPW) & 1u);
         }
+#ifdef TGL_KV_PROF
+        prof_add(a, (c + 1) * kTC > kt0 ? 9 : 8, ma1 - ma0);   // MMA: A wait (time / gathered)
+        prof_add(a, 10, clock64() - ma1);            // MMA: W wait
+#endif
         tc_fence_after();
         if (elect_one()) {
           const uint64_t a0 = desc_sw64(a_s + sa * kPAStage, 1024);

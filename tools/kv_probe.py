@@ -108,7 +108,10 @@ if os.environ.get("PROBE_PROF"):
         call(); torch.cuda.synchronize()
         lib.tgl_debug_prof(host, 0)
         v = np.frombuffer(host, dtype=np.uint64).reshape(148, 16).astype(np.float64)
-        names = (["C:ffull-wait", "C:lds+phi", "C:bempty-wait", "C:cvt+sts", "C:fence",
+        names = (["T:aempty-wait", "T:phi+split+st", "2", "3", "4", "L:aempty-wait", "6",
+                  "M:tempty-wait", "M:afull-wait(gathered)", "M:afull-wait(time)",
+                  "M:wfull-wait", "E:acc-wait", "E:work"] if kv == "pre" else
+                 ["C:ffull-wait", "C:lds+phi", "C:bempty-wait", "C:cvt+sts", "C:fence",
                   "L:fempty-wait", "L:issue", "M:bfull-wait", "M:wfull-wait", "9", "10",
                   "E:acc-wait", "E:work"] if kv == "split" else
                  ["P:stage-free", "P:issue", "P:data-wait", "P:convert", "P:fence+arrive",
