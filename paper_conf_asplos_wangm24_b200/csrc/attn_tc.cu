@@ -2431,11 +2431,17 @@ __global__ void __launch_bounds__(kSThreads, 1)
 // Roles: epilogue warps 0-7 (bin_epilogue), MMA 8, weights 9, tile descriptors 10-11,
 // loaders 12-15, time warps 16-19: 640 threads.
 #ifndef TGL_KV_PRE_ASTAGES
-#define TGL_KV_PRE_ASTAGES 8
+#define TGL_KV_PRE_ASTAGES 7
+#endif
+#ifndef TGL_KV_PRE_WSTAGES
+#define TGL_KV_PRE_WSTAGES 3
 #endif
 constexpr int kPAStages = TGL_KV_PRE_ASTAGES;         // A stages (hi | lo, 16 KB each)
 constexpr int kPAStage = kBM * kTC * 4;                // 16 KB
-constexpr int kPW = 2;                                 // weight stages (25.6 KB each)
+// weight stages (25.6 KB each): 3, so that a chunk can stream in while the two chunks
+// kept across the tile boundary (alternating K order) are still being read -- with 2
+// stages the MMA waited ~18 % of the kernel for weights (probe counters, GDELT)
+constexpr int kPW = TGL_KV_PRE_WSTAGES;
 constexpr int kPLoad0 = 12, kPLoadWarps = 4;
 constexpr int kPTime0 = 16, kPTimeWarps = 4;
 constexpr int kPThreads = (kPTime0 + kPTimeWarps) * 32;   // 640
@@ -2497,6 +2503,16 @@ __global__ void pack_kv_pre_kernel(const float* Wk, const float* Wv, int dm, int
     *reinterpret_cast<__nv_bfloat16*>(out + off + kTWHalf) = lo;
   }
 }
+
+// kv_pre waits: test_wait + nanosleep back-off (default) or the suspend-hint try_wait
+// (-DTGL_PRE_SUSPEND: the waiting warp sleeps in hardware, no polling instructions)
+#ifdef TGL_PRE_SUSPEND
+#define PRE_WAIT_SLEEP(bar, par, ns) mbar_wait(bar, par)
+#define PRE_FREE_SLEEP(bar, u, ns) wait_free(bar, u)
+#else
+#define PRE_WAIT_SLEEP(bar, par, ns) mbar_wait_sleep(bar, par, ns)
+#define PRE_FREE_SLEEP(bar, u, ns) wait_free_sleep(bar, u, ns)
+#endif
 
 struct PBars {
   uint64_t afull[kPAStages], aempty[kPAStages];
@@ -2573,7 +2589,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
     float* stdv = s_td[dw];
     for (tt = dw;; tt += kTDescWarps) {
       const uint32_t ds = tt % kSDSlots;
-      wait_free_sleep(&B.dempty[ds], tt / kSDSlots, TGL_SLEEP_DESC);
+      PRE_FREE_SLEEP(&B.dempty[ds], tt / kSDSlots, TGL_SLEEP_DESC);
       TDesc& R = bd[ds];
       const int64_t T = blockIdx.x + (int64_t)tt * gridDim.x;
       if (T >= ntiles) {
@@ -2644,7 +2660,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
     const uint32_t wbytes = split ? kTWStage : kTWHalf;
     for (;; ++tt) {
       const uint32_t ds = tt % kSDSlots;
-      mbar_wait_sleep(&B.dfull[ds], (tt / kSDSlots) & 1u, TGL_SLEEP_W);
+      PRE_WAIT_SLEEP(&B.dfull[ds], (tt / kSDSlots) & 1u, TGL_SLEEP_W);
       const int live = bd[ds].live;
       warp_arrive(&B.dempty[ds]);
       if (!live) break;
@@ -2653,7 +2669,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
         for (int i = r0; i < nch; ++i) {
           const uint32_t k = wl + (i - r0);
           const uint32_t sw = k % kPW;
-          wait_free_sleep(&B.wempty[sw], k / kPW, TGL_SLEEP_W);
+          PRE_FREE_SLEEP(&B.wempty[sw], k / kPW, TGL_SLEEP_W);
           mbar_arrive_expect_tx(&B.wfull[sw], wbytes);
           bulk_g2s(pipe + kPAStages * kPAStage + sw * kTWStage,
                    wkv + (size_t)plan.order[chunk_of(tt, i, nch)] * kTWStage, wbytes, &B.wfull[sw]);
@@ -2681,7 +2697,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
     uint32_t g = 0;
     for (;; ++tt) {
       const uint32_t ds = tt % kSDSlots;
-      mbar_wait_sleep(&B.dfull[ds], (tt / kSDSlots) & 1u, TGL_SLEEP_LOAD);
+      PRE_WAIT_SLEEP(&B.dfull[ds], (tt / kSDSlots) & 1u, TGL_SLEEP_LOAD);
       const TDesc& R = bd[ds];
       if (!R.live) {
         warp_arrive(&B.dempty[ds]);
@@ -2702,7 +2718,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
         const int ks = (plan.k - c * kTC) > 16 ? 2 : 1;   // K steps the MMA issues
         const uint32_t sa = g % kPAStages;
         TGL_PROF_CLK(l0);
-        wait_free_sleep(&B.aempty[sa], g / kPAStages, TGL_SLEEP_LOAD);
+        PRE_FREE_SLEEP(&B.aempty[sa], g / kPAStages, TGL_SLEEP_LOAD);
 #ifdef TGL_KV_PROF
         if (lw == 0) prof_add(a, 5, clock64() - l0);  // loader: wait for a free stage
 #endif
@@ -2750,7 +2766,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
     uint32_t g = 0;
     for (;; ++tt) {
       const uint32_t ds = tt % kSDSlots;
-      mbar_wait_sleep(&B.dfull[ds], (tt / kSDSlots) & 1u, TGL_SLEEP_LOAD);
+      PRE_WAIT_SLEEP(&B.dfull[ds], (tt / kSDSlots) & 1u, TGL_SLEEP_LOAD);
       const TDesc& R = bd[ds];
       if (!R.live) {
         warp_arrive(&B.dempty[ds]);
