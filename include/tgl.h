@@ -90,7 +90,19 @@ typedef struct {
   const int32_t* nbr;    /* [num_entries] */
   const int32_t* eid;    /* [num_entries] */
   const float* ts;       /* [num_entries], sorted inside each segment */
+  const float* ts_coarse; /* optional (NULL): ts_coarse[p] = ts[32 p], p < ceil(M / 32) -- a
+                             1/32 fence index the sampler searches first, so a query's
+                             DRAM probes shrink to one 128-byte window of its segment */
+  const void* entries;    /* optional (NULL): int32x4 {nbr, eid, bits(ts), 0} per entry --
+                             the sampler's picks fetch one 16-byte record (one DRAM
+                             sector) instead of three arrays */
 } tgl_tcsr;
+
+/* Sampler indexes of a T-CSR (once per graph, after tgl_build_tcsr; either output may be
+ * NULL): ts_coarse [ceil(M/32)] floats as above, entries [M] x 16 bytes (16-byte
+ * aligned).  The caller owns both and stores them in the tgl_tcsr it passes to
+ * tgl_sample; results are bit-identical with or without them. */
+tgl_status tgl_tcsr_index(const tgl_tcsr* g, float* ts_coarse, void* entries, void* stream);
 
 /* ---------------------------------------------------------------------------
  * S2  Roots of a batch (head TBlock).  P:235 (L2.8) `head = batch.block(ctx)`;

@@ -147,7 +147,8 @@ class TGATPipeline:
         dedup_launches = [(1 if b.n_max <= 4096 else 3) if use_dedup else 0 for b in self.blocks]
         if shard is not None:   # roots' dedup (before the slice) replaces block 0's + slice
             dedup_launches[0] = ((1 if 3 * batch <= 4096 else 3) if use_dedup else 0) + 1
-        per_block = [(1 if l > 0 else 0) + dedup_launches[l] + 1 + 3 + (1 if self.split and l > 0
+        # per block: next_block, dedup, sample (count + scan + pick), Q + K|V + FFN, split
+        per_block = [(1 if l > 0 else 0) + dedup_launches[l] + 3 + 3 + (1 if self.split and l > 0
                                                                          else 0)
                      for l in range(self.L)]
         self.launches_per_forward = 1 + sum(per_block) + (1 if use_dedup and shard is None

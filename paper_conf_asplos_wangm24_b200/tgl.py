@@ -33,7 +33,8 @@ SYMBOLS = ["tgl_version", "tgl_status_string", "tgl_last_error", "tgl_build_tcsr
            "tgl_batch_roots", "tgl_dedup", "tgl_sample", "tgl_next_block",
            "tgl_time_precompute", "tgl_time_encode", "tgl_tblock_attn", "tgl_gather_rows",
            "tgl_attn_packed_bytes", "tgl_attn_pack", "tgl_cache_lookup", "tgl_cache_store", "tgl_cache_combine",
-           "tgl_cache_merge", "tgl_shard_slice", "tgl_shard_gather", "tgl_split_rows"]
+           "tgl_cache_merge", "tgl_shard_slice", "tgl_shard_gather", "tgl_split_rows",
+           "tgl_tcsr_index"]
 
 
 class TGLError(RuntimeError):
@@ -70,6 +71,7 @@ def _load():
         "tgl_shard_slice": [i64, vp, vp, vp, i32, i32, vp, vp, vp, vp],
         "tgl_shard_gather": [i64, vp, vp, i64, vp, i32, vp, i64, i32, vp, i64, vp],
         "tgl_split_rows": [i64, i32, vp, i64, vp, i64, vp],
+        "tgl_tcsr_index": [vp, vp, vp, vp],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -154,15 +156,32 @@ def ws_bytes(fn_name: str, *args_before_ws) -> int:
 # --------------------------------------------------------------------------- S1
 class TCSR(C.Structure):
     _fields_ = [("num_nodes", C.c_int64), ("num_entries", C.c_int64), ("indptr", C.c_void_p),
-                ("nbr", C.c_void_p), ("eid", C.c_void_p), ("ts", C.c_void_p)]
+                ("nbr", C.c_void_p), ("eid", C.c_void_p), ("ts", C.c_void_p),
+                ("ts_coarse", C.c_void_p), ("entries", C.c_void_p)]
 
 
 class TemporalCSR:
     """Device-resident T-CSR + the host struct the ABI takes."""
 
-    def __init__(self, indptr, nbr, eid, ts):
+    def __init__(self, indptr, nbr, eid, ts, coarse: bool = True, packed: bool = True,
+                 stream=None):
+        """coarse / packed: build the sampler's fence index (M/32 floats) and the packed
+        16-byte entry records (16 B per entry) with tgl_tcsr_index."""
         self.indptr, self.nbr, self.eid, self.ts = indptr, nbr, eid, ts
-        self.struct = TCSR(indptr.numel() - 1, nbr.numel(), _p(indptr), _p(nbr), _p(eid), _p(ts))
+        M = nbr.numel()
+        self.ts_coarse = self.entries = None
+        self.struct = TCSR(indptr.numel() - 1, M, _p(indptr), _p(nbr), _p(eid), _p(ts), None,
+                           None)
+        if M > 0 and (coarse or packed):
+            if coarse:
+                self.ts_coarse = torch.empty((M + 31) // 32, dtype=torch.float32,
+                                             device=ts.device)
+            if packed:
+                self.entries = torch.empty(M, 4, dtype=torch.int32, device=ts.device)
+            _check(_lib.tgl_tcsr_index(C.byref(self.struct), _p(self.ts_coarse),
+                                       _p(self.entries), _s(stream)), "tgl_tcsr_index")
+            self.struct.ts_coarse = _p(self.ts_coarse)
+            self.struct.entries = _p(self.entries)
 
     @property
     def num_nodes(self):
@@ -170,7 +189,8 @@ class TemporalCSR:
 
 
 def build_tcsr(num_nodes: int, src, dst, t, undirected=True, time_sorted=False,
-               ws: Workspace | None = None, stream=None) -> TemporalCSR:
+               ws: Workspace | None = None, stream=None, coarse: bool = True,
+               packed: bool = True) -> TemporalCSR:
     dev = src.device
     E = src.numel()
     M = 2 * E if undirected else E
@@ -181,7 +201,7 @@ def build_tcsr(num_nodes: int, src, dst, t, undirected=True, time_sorted=False,
     flags = (TGL_UNDIRECTED if undirected else 0) | (TGL_INPUT_TIME_SORTED if time_sorted else 0)
     _ws_call(_lib.tgl_build_tcsr, [num_nodes, E, _p(src), _p(dst), _p(t), flags, _p(indptr),
                                    _p(nbr), _p(eid), _p(ts)], ws, _s(stream), "tgl_build_tcsr")
-    return TemporalCSR(indptr, nbr, eid, ts)
+    return TemporalCSR(indptr, nbr, eid, ts, coarse=coarse, packed=packed, stream=stream)
 
 
 # --------------------------------------------------------------------------- S2

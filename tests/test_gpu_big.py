@@ -89,7 +89,7 @@ def _run(name, host_gb, dev_gb):
     neg = sg.device_negatives(cfg, dev)
     src_h, dst_h, t_h, neg_h = (x.cpu().numpy() for x in (src, dst, t, neg))
     torch.cuda.empty_cache()
-    tc = tgl.build_tcsr(cfg.n_nodes, src, dst, t, True, True)
+    tc = tgl.build_tcsr(cfg.n_nodes, src, dst, t, True, True, packed=name != "MAG")
     torch.cuda.synchronize()
     torch.cuda.empty_cache()
     segs = _check_tcsr(cfg, src, dst, t, tc, src_h, dst_h, t_h, rng)

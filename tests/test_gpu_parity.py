@@ -68,16 +68,20 @@ def test_tcsr_full_configs(T, name):
 
 
 # ------------------------------------------------------------------ S4
+@pytest.mark.parametrize("index", ["coarse+packed", "none", "coarse"])
 @pytest.mark.parametrize("strategy", ["recent", "uniform"])
 @pytest.mark.parametrize("k", [1, 10, 20, 45])
-def test_sample_bit_exact(T, strategy, k):
+def test_sample_bit_exact(T, strategy, k, index):
+    """Bit-exact against the oracle with and without the sampler indexes of
+    tgl_tcsr_index (fence index ts_coarse, packed 16-byte entries)."""
     rng = np.random.default_rng(k)
     N, E = 400, 60000
     src, dst, t = rand_graph(rng, N, E, 5000)
     src[:20000] = 7  # one huge segment (multi-round search)
     o = np.argsort(t, kind="stable")
     src, dst, t = src[o], dst[o], t[o]
-    g = T.build_tcsr(N, cu(src), cu(dst), cu(t), True, True)
+    g = T.build_tcsr(N, cu(src), cu(dst), cu(t), True, True, coarse="coarse" in index,
+                     packed="packed" in index)
     tc = oracle.build_tcsr(N, src, dst, t, True)
     nq = 3001
     qn = rng.integers(0, N, nq).astype(np.int32)
