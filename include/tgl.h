@@ -297,6 +297,33 @@ tgl_status tgl_split_rows(int64_t n_rows, int32_t d, const float* src, int64_t l
                           void* dst, int64_t ld_dst, void* stream);
 
 /* ---------------------------------------------------------------------------
+ * N2  Backward of one TBlock attention layer (training is the paper's
+ * headline workload).  Given dL/d(out) for the n = *n_dst_dev destinations
+ * of a tgl_tblock_attn call (same arguments, fp32 row tables, input_layout 0), adds
+ * (+=) dL/dtheta for every parameter of the layer into G (shapes of the weights) and,
+ * when the pointers are non-NULL, dL/dh into grad_hdst (row hdst_idx[i]) and grad_hsrc
+ * (row hsrc_idx[o + e]) -- the rows the forward gathered; several destinations / edges
+ * may hit one row (atomic adds).  The time encoder Phi_j(dt) = cos(omega_j dt + phi_j)
+ * (R10 fp32 argument b) contributes domega_j = sum -sin(b) dt dPhi, dphi_j = sum -sin(b)
+ * dPhi (including Phi(0) of eq 4).  The forward is recomputed in fp32 (exact fp32
+ * products); n_edges_max bounds seg_ptr[n].  Workspace: O(n_dst_max * (d_hdst + d_t +
+ * d_model) + n_edges_max * (d_hsrc + d_e + d_t + d_model)) floats.
+ * Errors: EINVAL (d_out != d_model, d_model > 128, > 2 heads, split inputs, nulls).
+ * ------------------------------------------------------------------------- */
+typedef struct {
+  float *dWq, *dbq, *dWk, *dbk, *dWv, *dbv, *dWo, *dbo, *dgamma, *dbeta, *domega, *dphi;
+} tgl_attn_grads;
+
+tgl_status tgl_tblock_attn_backward(
+    const tgl_attn_params* P, int64_t n_dst_max, const int64_t* n_dst_dev, int64_t n_edges_max,
+    const int64_t* seg_ptr, const float* dst_t, const float* hdst, const int32_t* hdst_idx,
+    int64_t ld_hdst, const float* hsrc, const int32_t* hsrc_idx, const int64_t* hsrc_off_dev,
+    int64_t ld_hsrc, const float* efeat, const int32_t* eid, int64_t ld_e, const float* edge_t,
+    const float* grad_out, int64_t ld_gout, const tgl_attn_grads* G, float* grad_hdst,
+    int64_t ld_ghdst, float* grad_hsrc, int64_t ld_ghsrc, void* ws, size_t* ws_bytes,
+    void* stream);
+
+/* ---------------------------------------------------------------------------
  * S14  Dedup inverse applied to rows (the hook of P:279 / TGOpt dedup_invert
  * P:179): out[j][:] = table[idx[j]][:] for j < n, n = *n_dev (NULL -> n_max).
  * ------------------------------------------------------------------------- */

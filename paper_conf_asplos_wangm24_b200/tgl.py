@@ -34,7 +34,7 @@ SYMBOLS = ["tgl_version", "tgl_status_string", "tgl_last_error", "tgl_build_tcsr
            "tgl_time_precompute", "tgl_time_encode", "tgl_tblock_attn", "tgl_gather_rows",
            "tgl_attn_packed_bytes", "tgl_attn_pack", "tgl_cache_lookup", "tgl_cache_store", "tgl_cache_combine",
            "tgl_cache_merge", "tgl_shard_slice", "tgl_shard_gather", "tgl_split_rows",
-           "tgl_tcsr_index"]
+           "tgl_tcsr_index", "tgl_tblock_attn_backward"]
 
 
 class TGLError(RuntimeError):
@@ -72,6 +72,8 @@ def _load():
         "tgl_shard_gather": [i64, vp, vp, i64, vp, i32, vp, i64, i32, vp, i64, vp],
         "tgl_split_rows": [i64, i32, vp, i64, vp, i64, vp],
         "tgl_tcsr_index": [vp, vp, vp, vp],
+        "tgl_tblock_attn_backward": [vp, i64, vp, i64, vp, vp, vp, vp, i64, vp, vp, vp, i64, vp,
+                                     vp, i64, vp, vp, i64, vp, vp, i64, vp, i64, vp, sz, vp],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -524,3 +526,39 @@ def split_table(n_rows: int, d: int, make_rows, chunk_rows: int = 1 << 20, devic
         split_rows(rows, out=out[r0:r1], stream=stream)
         del rows
     return out
+
+
+# --------------------------------------------------------------------------- N2 backward
+GRAD_NAMES = ("Wq", "bq", "Wk", "bk", "Wv", "bv", "Wo", "bo", "ln_gamma", "ln_beta", "omega",
+              "phi")
+
+
+class AttnGradsC(C.Structure):
+    _fields_ = [(f"d{n}", C.c_void_p) for n in ("Wq", "bq", "Wk", "bk", "Wv", "bv", "Wo", "bo",
+                                                 "gamma", "beta", "omega", "phi")]
+
+
+def zero_grads(P: AttnParams) -> dict:
+    """Gradient accumulators (zeros) shaped like the layer's weights."""
+    return {n: torch.zeros_like(P.t[n]) for n in GRAD_NAMES}
+
+
+def tblock_attn_backward(P: AttnParams, seg_ptr, dst_t, hdst, hdst_idx, hsrc, hsrc_idx, efeat,
+                         eid, edge_t, grad_out, grads: dict, grad_hdst=None, grad_hsrc=None,
+                         n_dst_max=None, n_dst_dev=None, n_edges_max=None, hsrc_off_dev=None,
+                         ws: Workspace | None = None, stream=None):
+    """Backward of tgl_tblock_attn (N2): accumulates into `grads` (zero_grads) and, when
+    given, into grad_hdst / grad_hsrc (row tables shaped like hdst / hsrc)."""
+    n_dst_max = seg_ptr.numel() - 1 if n_dst_max is None else n_dst_max
+    n_edges_max = (int(edge_t.numel()) if n_edges_max is None else n_edges_max)
+    G = AttnGradsC(*[_p(grads[n]) for n in GRAD_NAMES])
+    ld_e = efeat.stride(0) if (efeat is not None and efeat.dim() == 2 and efeat.shape[1]) else 0
+    _ws_call(_lib.tgl_tblock_attn_backward,
+             [C.byref(P.struct), n_dst_max, _p(n_dst_dev), n_edges_max, _p(seg_ptr), _p(dst_t),
+              _prow(hdst), _p(hdst_idx), hdst.stride(0), _prow(hsrc), _p(hsrc_idx),
+              _p(hsrc_off_dev), hsrc.stride(0), _prow(efeat) if ld_e else None,
+              _p(eid) if ld_e else None, ld_e, _p(edge_t), _prow(grad_out), grad_out.stride(0),
+              C.byref(G), _prow(grad_hdst), grad_hdst.stride(0) if grad_hdst is not None else 0,
+              _prow(grad_hsrc), grad_hsrc.stride(0) if grad_hsrc is not None else 0], ws,
+             _s(stream), "tgl_tblock_attn_backward")
+    return grads
