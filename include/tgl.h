@@ -299,7 +299,8 @@ tgl_status tgl_split_rows(int64_t n_rows, int32_t d, const float* src, int64_t l
 /* ---------------------------------------------------------------------------
  * N2  Backward of one TBlock attention layer (training is the paper's
  * headline workload).  Given dL/d(out) for the n = *n_dst_dev destinations
- * of a tgl_tblock_attn call (same arguments, fp32 row tables, input_layout 0), adds
+ * of a tgl_tblock_attn call (same arguments, but fp32 row tables for h_dst, h_src and e:
+ * P->input_layout and P->kv_kernel are ignored), adds
  * (+=) dL/dtheta for every parameter of the layer into G (shapes of the weights) and,
  * when the pointers are non-NULL, dL/dh into grad_hdst (row hdst_idx[i]) and grad_hsrc
  * (row hsrc_idx[o + e]) -- the rows the forward gathered; several destinations / edges
@@ -308,11 +309,17 @@ tgl_status tgl_split_rows(int64_t n_rows, int32_t d, const float* src, int64_t l
  * dPhi (including Phi(0) of eq 4).  The forward is recomputed in fp32 (exact fp32
  * products); n_edges_max bounds seg_ptr[n].  Workspace: O(n_dst_max * (d_hdst + d_t +
  * d_model) + n_edges_max * (d_hsrc + d_e + d_t + d_model)) floats.
- * Errors: EINVAL (d_out != d_model, d_model > 128, > 2 heads, split inputs, nulls).
+ * Errors: EINVAL (d_out != d_model, d_model > 128, > 2 heads, nulls).
  * ------------------------------------------------------------------------- */
 typedef struct {
   float *dWq, *dbq, *dWk, *dbk, *dWv, *dbv, *dWo, *dbo, *dgamma, *dbeta, *domega, *dphi;
 } tgl_attn_grads;
+
+/* Adjoint of the S14 gather (the dedup inverse hook in the backward): out[idx[j]][:] +=
+ * src[j][:] for j < n = *n_dev (NULL -> n_max); idx NULL = identity; atomic adds. */
+tgl_status tgl_scatter_add_rows(int64_t n_max, const int64_t* n_dev, const int32_t* idx,
+                                const float* src, int64_t ld_src, int32_t d, float* out,
+                                int64_t ld_out, void* stream);
 
 tgl_status tgl_tblock_attn_backward(
     const tgl_attn_params* P, int64_t n_dst_max, const int64_t* n_dst_dev, int64_t n_edges_max,

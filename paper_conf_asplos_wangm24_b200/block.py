@@ -360,6 +360,52 @@ class TGATPipeline:
         return tgl.shard_gather(gathered, self.c_max, self.world, n0, u_dev=r["n"], idx=None,
                                 n_max=n0, n_dev=r["n"], out=out, stream=stream)
 
+    # ------------------------------------------------------------------ N2 backward
+    def backward(self, grad_emb: torch.Tensor, grads: list | None = None, stream=None):
+        """Training step of the TBlock chain: given dL/d(root embeddings)
+        [3B, d_out] of the batch the last forward() ran, accumulate every layer's parameter
+        gradients (grads[l]: tgl.zero_grads(attn[l]), created when None) -- the head block
+        first, its input-row gradients routed to the block below through the same dedup
+        hooks the forward used (S14 / S15 adjoints), down to the tail (raw features get
+        none).  Needs fp32 feature tables (layout="fp32" or both tables present)."""
+        assert self.shard is None and not self.cache_on, "backward: unsharded, no cache()"
+        g = self.g
+        assert g.get("efeat") is not None or self.attn[-1].host["d_e"] == 0, \
+            "backward gathers fp32 edge rows"
+        s = stream
+        if grads is None:
+            grads = [tgl.zero_grads(a) for a in self.attn]
+        b0 = self.blocks[0]
+        d0 = self.attn[0].d_out
+        # S14 adjoint at the roots: dL/d(head rows) = scatter-add of dL/d(emb) through inv_0
+        g_out = torch.zeros(b0.n_max, d0, device=self.dev)
+        if self.use_dedup:
+            tgl.scatter_add_rows(b0.inv, grad_emb, g_out, n_dev=b0.n_dev, n_max=b0.n_max,
+                                 stream=s)
+        else:
+            tgl.scatter_add_rows(None, grad_emb, g_out, n_dev=b0.n_dev, n_max=b0.n_max,
+                                 stream=s)
+        k = self.sampler.k
+        for l, b in enumerate(self.blocks):
+            a = self.attn[l]
+            tail = l == self.L - 1
+            ef = g["efeat"] if a.host["d_e"] else None
+            if tail:
+                hdst = hsrc = g["nfeat"]
+                hdst_idx, hsrc_idx, off, g_next = b.uniq_node, b.nbr, None, None
+            else:
+                nx = self.blocks[l + 1]
+                hdst = hsrc = nx.out
+                hdst_idx = hsrc_idx = nx.inv if self.use_dedup else None
+                off = b.u_dev
+                g_next = torch.zeros_like(nx.out)     # dL/d(rows of the block below)
+            tgl.tblock_attn_backward(a, b.seg_ptr, b.uniq_t, hdst, hdst_idx, hsrc, hsrc_idx, ef,
+                                     b.eid if ef is not None else None, b.ts, g_out, grads[l],
+                                     g_next, g_next, n_dst_max=b.n_max, n_dst_dev=b.u_dev,
+                                     n_edges_max=b.n_max * k, hsrc_off_dev=off, stream=s)
+            g_out = g_next
+        return grads
+
     # ------------------------------------------------------------------ CUDA graph
     def capture(self):
         torch.cuda.synchronize()

@@ -94,6 +94,25 @@ __global__ void gather_rows_kernel(int64_t n_max, const int64_t* n_dev,
   }
 }
 
+// ---------------------------------------------------------------- N2 row scatter-add
+// out[idx[j]][:] += src[j][:] for j < n (the adjoint of the S14 gather); atomic adds.
+__global__ void scatter_add_rows_kernel(int64_t n_max, const int64_t* n_dev,
+                                        const int32_t* __restrict__ idx,
+                                        const float* __restrict__ src, int64_t ld_src, int32_t d,
+                                        float* __restrict__ out, int64_t ld_out) {
+  pdl_wait();
+  pdl_trigger();
+  const int64_t n = dev_count(n_dev, n_max);
+  const int64_t total = n * d;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t j = x / d;
+    const int c = (int)(x - j * d);
+    const int64_t r = idx ? (int64_t)idx[j] : j;
+    atomicAdd(out + r * ld_out + c, src[j * ld_src + c]);
+  }
+}
+
 // ---------------------------------------------------------------- split16 rows
 // dst row r (pitch ld_dst 4-byte words): bf16 hi of columns [0, dp) then bf16 lo of the
 // same columns, dp = d rounded up to 8 (zero columns past d); hi = RNE(x),
@@ -189,6 +208,17 @@ tgl_status tgl_gather_rows(int64_t n_max, const int64_t* n_dev, const int32_t* i
   launch_pdl(gather_rows_kernel, dim3(grid_for(n_max * d, 256)), dim3(256), 0, as_stream(stream), 
       n_max, n_dev, idx, table, ld_table, d, out, ld_out);
   return launch_check("gather_rows");
+}
+
+tgl_status tgl_scatter_add_rows(int64_t n_max, const int64_t* n_dev, const int32_t* idx,
+                                const float* src, int64_t ld_src, int32_t d, float* out,
+                                int64_t ld_out, void* stream) {
+  TGL_REQUIRE(n_max >= 0 && d >= 0 && ld_src >= d && ld_out >= d, "bad size");
+  if (n_max == 0 || d == 0) return TGL_OK;
+  TGL_REQUIRE(src && out, "null pointer");
+  launch_pdl(scatter_add_rows_kernel, dim3(grid_for(n_max * d, 256)), dim3(256), 0,
+             as_stream(stream), n_max, n_dev, idx, src, ld_src, d, out, ld_out);
+  return launch_check("scatter_add_rows");
 }
 
 tgl_status tgl_split_rows(int64_t n_rows, int32_t d, const float* src, int64_t ld_src,

@@ -419,7 +419,6 @@ extern "C" tgl_status tgl_tblock_attn_backward(
   TGL_REQUIRE(G->dWq && G->dbq && G->dWk && G->dbk && G->dWv && G->dbv && G->dWo && G->dbo &&
                   G->dgamma && G->dbeta && G->domega && G->dphi,
               "null gradient buffer");
-  TGL_REQUIRE(P->input_layout == 0, "backward takes fp32 row tables (input_layout 0)");
   cudaStream_t s = as_stream(stream);
   char* w = static_cast<char*>(ws);
   // zero-padded rows beyond the device counts must contribute nothing to the GEMMs

@@ -34,7 +34,7 @@ SYMBOLS = ["tgl_version", "tgl_status_string", "tgl_last_error", "tgl_build_tcsr
            "tgl_time_precompute", "tgl_time_encode", "tgl_tblock_attn", "tgl_gather_rows",
            "tgl_attn_packed_bytes", "tgl_attn_pack", "tgl_cache_lookup", "tgl_cache_store", "tgl_cache_combine",
            "tgl_cache_merge", "tgl_shard_slice", "tgl_shard_gather", "tgl_split_rows",
-           "tgl_tcsr_index", "tgl_tblock_attn_backward"]
+           "tgl_tcsr_index", "tgl_tblock_attn_backward", "tgl_scatter_add_rows"]
 
 
 class TGLError(RuntimeError):
@@ -72,6 +72,7 @@ def _load():
         "tgl_shard_gather": [i64, vp, vp, i64, vp, i32, vp, i64, i32, vp, i64, vp],
         "tgl_split_rows": [i64, i32, vp, i64, vp, i64, vp],
         "tgl_tcsr_index": [vp, vp, vp, vp],
+        "tgl_scatter_add_rows": [i64, vp, vp, vp, i64, i32, vp, i64, vp],
         "tgl_tblock_attn_backward": [vp, i64, vp, i64, vp, vp, vp, vp, i64, vp, vp, vp, i64, vp,
                                      vp, i64, vp, vp, i64, vp, vp, i64, vp, i64, vp, sz, vp],
     }
@@ -562,3 +563,12 @@ def tblock_attn_backward(P: AttnParams, seg_ptr, dst_t, hdst, hdst_idx, hsrc, hs
               _prow(grad_hsrc), grad_hsrc.stride(0) if grad_hsrc is not None else 0], ws,
              _s(stream), "tgl_tblock_attn_backward")
     return grads
+
+
+def scatter_add_rows(idx, src, out, n_dev=None, n_max=None, stream=None):
+    """out[idx[j]] += src[j] for j < n (identity when idx is None)."""
+    n_max = (src.shape[0] if idx is None else idx.numel()) if n_max is None else n_max
+    _check(_lib.tgl_scatter_add_rows(n_max, _p(n_dev), _p(idx), _prow(src), src.stride(0),
+                                     src.shape[1], _prow(out), out.stride(0), _s(stream)),
+           "tgl_scatter_add_rows")
+    return out

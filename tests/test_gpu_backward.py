@@ -107,3 +107,76 @@ def test_backward_device_counts_and_offset():
     for n in tgl.GRAD_NAMES:
         _close(grads[n].cpu().numpy() / 2, exp[n], n)
     _close(gh.cpu().numpy() / 2, exp["hdst"] + exp["hsrc"], "h rows (dst + src, one table)")
+
+
+def _oracle_chain_grads(cfg, g, neg, params, b, G):
+    """Listing 2's block chain forward (oracle.pipeline's routing) with backward tapes,
+    then the chain rule from the roots down: dL/d(emb) -> head rows (S14 adjoint) -> each
+    block's input rows -> the block below."""
+    import oracle
+    from oracle import pipeline as opipe
+    tc = oracle.build_tcsr(cfg.n_nodes, g.src, g.dst, g.t, True)
+    qn, qt = opipe.roots(*synth.batch_roots_inputs(g, neg, b))
+    blocks = opipe.build_blocks(tc, qn, qt, len(params), cfg.k, cfg.strategy, cfg.dedup,
+                                cfg.seeds["sampler"])
+    L = len(blocks)
+    tapes, tables = [None] * L, [None] * L
+    for l in range(L - 1, -1, -1):
+        bl = blocks[l]
+        if l == L - 1:
+            hd, hd_idx, hs, hs_idx = g.nfeat, bl.uniq_node, g.nfeat, bl.nbr
+        else:
+            nxt = blocks[l + 1]
+            tab = tables[l + 1].astype(np.float32)            # fp32 between layers (R17)
+            U = bl.uniq_node.shape[0]
+            if nxt.inv is not None:
+                hd_idx, hs_idx = nxt.inv[:U], nxt.inv[U:]
+            else:
+                hd_idx = np.arange(U)
+                hs_idx = np.arange(U, nxt.dst_node.shape[0])
+            hd = hs = tab
+        out, tape = ob.tblock_forward(params[l], bl.seg_ptr, bl.uniq_t, hd, hd_idx, hs, hs_idx,
+                                      g.efeat, bl.eid, bl.ts)
+        tapes[l], tables[l] = tape, out
+    b0 = blocks[0]
+    U0 = b0.uniq_node.shape[0]
+    g_out = np.zeros((U0, params[0]["d_out"]))
+    if b0.inv is not None:
+        np.add.at(g_out, b0.inv, G)
+    else:
+        g_out += G
+    res = []
+    for l in range(L):
+        rows = tables[l + 1].shape[0] if l + 1 < L else g.nfeat.shape[0]
+        gr = ob.tblock_backward(params[l], tapes[l], g_out, rows, rows)
+        res.append(gr)
+        g_out = gr["hdst"] + gr["hsrc"]
+    return res
+
+
+@pytest.mark.parametrize("name,dedup", [("REDDIT", True), ("REDDIT", False), ("WIKI", False)])
+def test_pipeline_backward_vs_oracle_chain(name, dedup):
+    """TGATPipeline.backward: every layer's parameter gradients of a whole batch (the
+    training step of the chain) against the oracle's chain rule over the same blocks."""
+    from dataclasses import replace
+    from paper_conf_asplos_wangm24_b200 import TGATPipeline, TSampler, tgl
+    cfg = replace(synth.get_config(name).scaled(30000, batch=200), dedup=dedup)
+    g = synth.make_graph(cfg)
+    neg = synth.make_negatives(cfg)
+    params = synth.gen.model_params(cfg)
+    dev = {"src": cu(g.src), "dst": cu(g.dst), "t": cu(g.t), "neg": cu(neg),
+           "nfeat": cu(g.nfeat), "efeat": cu(g.efeat)}
+    tc = tgl.build_tcsr(cfg.n_nodes, dev["src"], dev["dst"], dev["t"], True, True)
+    pipe = TGATPipeline(dev, tc, params, cfg.batch, TSampler(cfg.k, cfg.strategy,
+                                                             cfg.seeds["sampler"]),
+                        cfg.dedup, cfg.precompute, cfg.window, "fp32")
+    b = int(0.7 * cfg.n_batches)
+    pipe.start_dev.fill_(b * cfg.batch)
+    pipe.forward()
+    G = np.random.default_rng(4).standard_normal((3 * cfg.batch, cfg.d_model)).astype(np.float32)
+    grads = pipe.backward(cu(G))
+    torch.cuda.synchronize()
+    exp = _oracle_chain_grads(cfg, g, neg, params, b, G.astype(np.float64))
+    for l in range(len(params)):
+        for n in tgl.GRAD_NAMES:
+            _close(grads[l][n].cpu().numpy(), exp[l][n], f"layer {l} {n}")
