@@ -62,7 +62,8 @@ def parse():
                     help="cache() table slots per layer (0 = off, the BASELINE configs)")
     ap.add_argument("--l2-flush", default="auto", choices=["auto", "on", "off"])
     ap.add_argument("--kv-kernel", default="auto",
-                    choices=["auto", "split", "split_pad", "async", "bin", "general"])
+                    choices=["auto", "pre", "pre2", "split", "split_pad", "async", "bin",
+                             "general"])
     ap.add_argument("--no-e2e", action="store_true")
     return ap.parse_args()
 
@@ -431,7 +432,7 @@ def algorithmic_kv(cfg, n_dst: float, n_edges: float, d_hsrc: int):
 def ncu_traffic(config: str, precision: str):
     """dram__bytes_read.sum + dram__bytes_write.sum per launch of the K|V kernel from the
     committed `ncu --set full` capture of this config and precision (profiles/), or None."""
-    for name in ("r02_kv_traffic.json", "r01_kv_split_traffic.json"):
+    for name in ("r02_kv_traffic.json",):
         try:
             d = json.load(open(os.path.join(ROOT, "profiles", name)))
             return d[config][precision]

@@ -226,6 +226,8 @@ tgl_status tgl_time_encode(int64_t n, const float* dt, int32_t d_t, const float*
 #define TGL_KV_BIN 4          /* register-gather producers (any row pitch) */
 #define TGL_KV_GENERAL 5      /* any segment length */
 #define TGL_KV_SIMT 6         /* (reported only) the TGL_FP32_SIMT kernel */
+#define TGL_KV_PRE2 8         /* kv_pre on a CTA pair: one tcgen05.mma.cta_group::2 (M = 256)
+                                 per K step, each SM streams half of the weights */
 #define TGL_KV_PRE 7          /* pre-split h_src / e tables (tgl_split_rows): loaders move
                                  the bf16 hi / lo operands straight into the MMA's shared-
                                  memory stages, no conversion in the SM (AUTO picks it

@@ -987,7 +987,20 @@ template <int NS, class D, int kPW = 33, bool kLowReg = false>
 __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uint64_t* dempty,
                                              uint64_t* tfull, uint64_t* tempty, const D* bd,
                                              uint32_t tmem, float* s_pvf,
-                                             const float* s_bias) {
+                                             const float* s_bias, uint32_t tempty_cl = 0) {
+  // tempty_cl != 0: the accumulator barriers live in the leader CTA of a pair (2-SM MMA);
+  // release them there with cluster-scope remote arrives
+  auto release = [&](uint32_t ab) {
+    if (tempty_cl) {
+      __syncwarp();
+      if ((threadIdx.x & 31) == 0)
+        asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(
+                         tempty_cl + ab * 8)
+                     : "memory");
+    } else {
+      warp_arrive(&tempty[ab]);
+    }
+  };
   constexpr uint32_t kCols = 256;
   constexpr int dm = 100, dh = 50;
   const tgl_attn_params& P = a.P;
@@ -1040,7 +1053,7 @@ __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uin
     if (threadIdx.x == 0) tl_mark(a, tt, 6);
     if (TGL_DBG(a) & 1) {
       tc_fence_before();
-      warp_arrive(&tempty[ab]);
+      release(ab);
       continue;
     }
     const uint32_t ta = tmem + ab * kCols + ((uint32_t)(q4 * 32) << 16);
@@ -1125,7 +1138,7 @@ __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uin
     tc_fence_before();
     if (warp == 0) trace(a, 10, tt);
     if (warp == 0) prof_add(a, 12, clock64() - e1c);   // epilogue: tile work
-    warp_arrive(&tempty[ab]);
+    release(ab);
     if (threadIdx.x == 0) tl_mark(a, tt, 7);
   }
 }
@@ -2916,13 +2929,532 @@ __global__ void __launch_bounds__(kPThreads, 1)
   ws_teardown(tmem, 2 * kCols, kTMma);
 }
 
+
+// ------------------------------------------------------------------ 2-SM pre-split K|V kernel
+// kv_pre2_kernel: kv_pre on a CTA pair (cluster of 2 on one TPC), one
+// tcgen05.mma.cta_group::2 of M = 256 per K step: rows 0-127 are the leader's tile, rows
+// 128-255 the peer's (two independent 128-row tiles), and the weight chunk's N = 208
+// rows ([Wk ; Wv] padded with 8 zero rows) are split between the two shared memories
+// (104 rows each), so every SM reads and fills HALF of the weight stream -- per 32-column
+// chunk ~72 KB of shared-memory traffic per SM instead of ~104 KB, below the MMA time.
+// The leader issues the MMAs; the peer's MMA warp relays its A / W readiness to the
+// leader (local barrier wait, then a cluster-scope remote arrive); MMA completion is
+// committed to both CTAs' barriers (multicast); the peer's epilogue releases the
+// leader's accumulator barrier remotely.  Each CTA's epilogue reads its own TMEM rows.
+#ifndef TGL_KV_PRE2_ASTAGES
+#define TGL_KV_PRE2_ASTAGES 8
+#endif
+#ifndef TGL_KV_PRE2_WSTAGES
+#define TGL_KV_PRE2_WSTAGES 4
+#endif
+constexpr int kP2AStages = TGL_KV_PRE2_ASTAGES;
+#ifndef TGL_KV_PRE_AUTO_PAIR
+#define TGL_KV_PRE_AUTO_PAIR 0
+#endif
+constexpr bool kPreAutoPair = TGL_KV_PRE_AUTO_PAIR != 0;   // AUTO picks the pair kernel
+constexpr int kP2N = 208;                              // N of the pair MMA (multiple of 16)
+constexpr int kP2Half = (kP2N / 2) * 64;               // 6656 B: one of hi / lo per CTA
+constexpr int kP2WStage = 2 * kP2Half;                 // 13312 B per CTA per chunk
+constexpr int kP2W = TGL_KV_PRE2_WSTAGES;
+constexpr int kP2PipeBytes = kP2AStages * kPAStage + kP2W * kP2WStage;
+constexpr int kP2Smem = 1024 + kP2PipeBytes + kBEpi * 32 * kSPW * 4;
+
+__global__ void pack_kv_pre2_kernel(const float* Wk, const float* Wv, int dm, int ksrc,
+                                    PrePlan p, uint8_t* out) {
+  const int kw = p.n * kTC;
+  const int64_t total = (int64_t)kP2N * kw;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const int n = (int)(x / kw), kp = (int)(x % kw);
+    const int c = kp / kTC, cc = kp % kTC;
+    int src = -1;
+    if (kp < p.dp0) {
+      if (kp < p.d0) src = kp;
+    } else if (kp < p.dp0 + p.dp1) {
+      if (kp - p.dp0 < p.d1) src = p.d0 + (kp - p.dp0);
+    } else if (kp < p.k) {
+      if (kp - p.dp0 - p.dp1 < p.dt) src = p.d0 + p.d1 + (kp - p.dp0 - p.dp1);
+    }
+    float v = 0.f;
+    if (n < 2 * dm && src >= 0)
+      v = n < dm ? Wk[(int64_t)n * ksrc + src] : Wv[(int64_t)(n - dm) * ksrc + src];
+    const __nv_bfloat16 hi = __float2bfloat16_rn(v);
+    const __nv_bfloat16 lo = __float2bfloat16_rn(v - __bfloat162float(hi));
+    const int r = n / (kP2N / 2), nn = n % (kP2N / 2);
+    const int64_t off = (int64_t)c * 2 * kP2WStage + r * kP2WStage + (nn >> 3) * 512 +
+                        sw64_off(nn, cc);
+    *reinterpret_cast<__nv_bfloat16*>(out + off) = hi;
+    *reinterpret_cast<__nv_bfloat16*>(out + off + kP2Half) = lo;
+  }
+}
+
+__device__ __forceinline__ uint32_t cluster_ctarank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ uint32_t mapa_shared(uint32_t saddr, uint32_t rank) {
+  uint32_t d;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(d) : "r"(saddr), "r"(rank));
+  return d;
+}
+__device__ __forceinline__ void mbar_arrive_remote(uint32_t cl_addr) {
+  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cl_addr)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity) {
+  const uint32_t a = smem_u32(bar);
+  uint32_t done = 0;
+  do {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.b32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(a), "r"(parity)
+        : "memory");
+  } while (!done);
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;"
+               ::: "memory");
+}
+__device__ __forceinline__ void mma_bf16_pair(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc,
+                                              uint32_t idesc, uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+__device__ __forceinline__ void mma_commit_pair(uint64_t* bar) {
+  asm volatile(
+      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64"
+      " [%0], %1;" ::"r"(smem_u32(bar)), "h"((uint16_t)3)
+      : "memory");
+}
+
+struct P2Bars {
+  uint64_t afull[kP2AStages], aempty[kP2AStages], pfull[kP2AStages];
+  uint64_t wfull[kP2W], wempty[kP2W];
+  uint64_t dfull[kSDSlots], dempty[kSDSlots];
+  uint64_t tfull[2], tempty[2];
+};
+
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
+    kv_pre2_kernel(const Args a, const PrePlan plan, const uint8_t* __restrict__ wkv,
+                   const int bdst) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* pipe = align1024(smem_raw);
+  __shared__ P2Bars B;
+  __shared__ uint32_t s_tmem;
+  __shared__ TDesc bd[kSDSlots];
+  __shared__ float s_omega[256], s_phi[256];
+  __shared__ float s_bias[2 * kMaxModel];
+  __shared__ int64_t s_seg[kTDescWarps][4 * 32 + 1];
+  __shared__ float s_td[kTDescWarps][4 * 32];
+  float* s_pvf = reinterpret_cast<float*>(pipe + kP2PipeBytes);
+  constexpr uint32_t kCols = 256;
+  constexpr int dm = 100;
+  const tgl_attn_params& P = a.P;
+  const bool split = a.split != 0;
+  const int nch = plan.n;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = cluster_ctarank();
+  const bool leader = rank == 0;
+  const int64_t pair = blockIdx.x >> 1, npairs = gridDim.x >> 1;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < kP2AStages; ++s) {
+      mbar_init(&B.afull[s], kPLoadWarps * 32 + kPTimeWarps);
+      mbar_init(&B.aempty[s], 1);
+      mbar_init(&B.pfull[s], 1);
+    }
+    for (int s = 0; s < kP2W; ++s) {
+      mbar_init(&B.wfull[s], 1);
+      mbar_init(&B.wempty[s], 1);
+    }
+    for (int s = 0; s < kSDSlots; ++s) {
+      mbar_init(&B.dfull[s], 1);
+      mbar_init(&B.dempty[s], kBEpi + kPLoadWarps + kPTimeWarps + 2);
+    }
+    for (int s = 0; s < 2; ++s) {
+      mbar_init(&B.tfull[s], 1);
+      mbar_init(&B.tempty[s], 2 * kBEpi);             // both CTAs' epilogues
+    }
+    fence_mbar_init();
+  }
+  TGL_TRACE_RESET();
+  if (warp == kTMma) {                               // paired TMEM allocation
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(&s_tmem)),
+                 "r"(2 * kCols)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+  }
+  for (int j = threadIdx.x; j < P.d_t; j += blockDim.x) {
+    s_omega[j] = P.omega[j];
+    s_phi[j] = P.phi[j];
+  }
+  for (int j = threadIdx.x; j < 2 * dm; j += blockDim.x) s_bias[j] = j < dm ? P.bk[j] : P.bv[j - dm];
+  tc_fence_before();
+  cluster_sync_all();                                // peer barriers initialised
+  tc_fence_after();
+  pdl_wait();
+  pdl_trigger();
+  const int64_t n = dev_count(a.n_dst_dev, a.n_dst_max);
+  const uint32_t tmem = s_tmem;
+  const uint32_t pipe_s = smem_u32(pipe);
+  const uint32_t a_s = pipe_s;
+  const uint32_t w_s = pipe_s + kP2AStages * kPAStage;
+  const int dpt = 4 * bdst;
+  const int64_t ntiles = (n + dpt - 1) / dpt;
+  const int64_t npt = (ntiles + 1) / 2;               // pair tiles
+  uint32_t tt = 0;
+  const int kt0 = plan.dp0 + plan.dp1;
+
+  if (warp >= kTDesc0 && warp < kTDesc0 + kTDescWarps) {   // ------- tile builders
+    const int dw = warp - kTDesc0;
+    const int64_t hoff = a.hsrc_off_dev ? *a.hsrc_off_dev : 0;
+    int64_t* sg = s_seg[dw];
+    float* stdv = s_td[dw];
+    for (tt = dw;; tt += kTDescWarps) {
+      const uint32_t ds = tt % kSDSlots;
+      PRE_FREE_SLEEP(&B.dempty[ds], tt / kSDSlots, TGL_SLEEP_DESC);
+      TDesc& R = bd[ds];
+      const int64_t PT = pair + (int64_t)tt * npairs;
+      if (PT >= npt) {
+        if (lane == 0) R.live = 0;
+        warp_arrive(&B.dfull[ds]);
+        break;
+      }
+      const int64_t T = 2 * PT + rank;                 // this CTA's 128-row tile
+      const int64_t d0 = T * dpt;
+      int nd = (int)((n - d0) < dpt ? (n - d0) : dpt);
+      nd = nd < 0 ? 0 : nd;
+      for (int j = lane; j <= nd; j += 32) sg[j] = a.seg_ptr[d0 + j];
+      for (int j = lane; j < nd; j += 32) stdv[j] = a.dst_t[d0 + j];
+      __syncwarp();
+      int64_t er[4] = {0, 0, 0, 0};
+      float tr[4] = {0.f, 0.f, 0.f, 0.f};
+      int dr[4] = {-1, -1, -1, -1};
+      unsigned ovf_bins = 0;
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int j0 = u * bdst;
+        if (j0 >= nd) continue;
+        const int j1 = (j0 + bdst) < nd ? j0 + bdst : nd;
+        const int64_t e0 = sg[j0], e1 = sg[j1];
+        if (e1 - e0 > 32) {
+          ovf_bins |= 1u << u;
+          continue;
+        }
+        const int64_t e = e0 + lane;
+        if (e < e1) {
+          int j = j0;
+          while (sg[j + 1] <= e) ++j;
+          dr[u] = (int)(d0 + j);
+          er[u] = e;
+          tr[u] = stdv[j];
+        }
+      }
+      for (int j = 0; j < nd; ++j) {
+        const bool ovf = (ovf_bins >> (j / bdst)) & 1u;
+        if (sg[j + 1] == sg[j] || ovf) {
+          const float fill = ovf ? __int_as_float(0x7fc00000) : 0.f;
+          for (int c = lane; c < dm; c += 32) a.rbuf[(d0 + j) * kQLd + c] = fill;
+        }
+      }
+      R.live = 1;
+      int32_t hi[4], ei[4];
+      float et[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const bool ok = dr[u] >= 0;
+        hi[u] = ok ? (a.hsrc_idx ? a.hsrc_idx[hoff + er[u]] : (int32_t)(hoff + er[u])) : 0;
+        ei[u] = (ok && P.d_e > 0) ? a.eid[er[u]] : 0;
+        et[u] = ok ? a.edge_t[er[u]] : 0.f;
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int r = 32 * u + lane;
+        const bool ok = dr[u] >= 0;
+        const float dt = tr[u] - et[u];
+        R.hrow[r] = ok ? hi[u] : -1;
+        R.erow[r] = ok ? ei[u] : -1;
+        R.dt[r] = ok ? dt : 0.f;
+        R.trow[r] = ok ? (int)tenc_table_row(dt, a.table, a.window) : -1;
+        R.rdst[r] = dr[u];
+      }
+      warp_arrive(&B.dfull[ds]);
+    }
+  } else if (warp == kTW) {                          // ---------------- weight loader (half)
+    uint32_t wl = 0;
+    const uint32_t wbytes = split ? kP2WStage : kP2Half;
+    for (;; ++tt) {
+      const uint32_t ds = tt % kSDSlots;
+      PRE_WAIT_SLEEP(&B.dfull[ds], (tt / kSDSlots) & 1u, TGL_SLEEP_W);
+      const int live = bd[ds].live;
+      warp_arrive(&B.dempty[ds]);
+      if (!live) break;
+      if (lane == 0) {
+        const int r0 = (tt > 0 && nch >= 4) ? 2 : 0;
+        for (int i = r0; i < nch; ++i) {
+          const uint32_t k = wl + (i - r0);
+          const uint32_t sw = k % kP2W;
+          PRE_FREE_SLEEP(&B.wempty[sw], k / kP2W, TGL_SLEEP_W);
+          mbar_arrive_expect_tx(&B.wfull[sw], wbytes);
+          bulk_g2s(pipe + kP2AStages * kPAStage + sw * kP2WStage,
+                   wkv + (size_t)plan.order[chunk_of(tt, i, nch)] * 2 * kP2WStage +
+                       rank * kP2WStage,
+                   wbytes, &B.wfull[sw]);
+        }
+        wl += nch - r0;
+      }
+      __syncwarp();
+    }
+  } else if (warp >= kPLoad0 && warp < kPLoad0 + kPLoadWarps) {   // ---------- loaders
+    const int lw = warp - kPLoad0;
+    const int r0 = lw * 32 + (lane >> 3), pc = lane & 7;
+    const bool lo_piece = pc >= 4;
+    const int j = pc & 3;
+    const uint32_t ofs0 = (uint32_t)(r0 >> 3) * 1024 + (lo_piece ? 512 : 0);
+    const bool active = split || !lo_piece;
+    const bool tsplit = (P.input_layout & TGL_SPLIT_TABLE) && a.table != nullptr;
+    const uint8_t* hbase = reinterpret_cast<const uint8_t*>(a.hsrc);
+    const uint8_t* ebase = reinterpret_cast<const uint8_t*>(a.efeat);
+    const uint8_t* tbase = reinterpret_cast<const uint8_t*>(a.table);
+    const int64_t hld = 4 * a.ld_hsrc, eld = 4 * a.ld_e, tld = 4 * plan.dpt;
+    uint32_t g = 0;
+    for (;; ++tt) {
+      const uint32_t ds = tt % kSDSlots;
+      PRE_WAIT_SLEEP(&B.dfull[ds], (tt / kSDSlots) & 1u, TGL_SLEEP_LOAD);
+      const TDesc& R = bd[ds];
+      if (!R.live) {
+        warp_arrive(&B.dempty[ds]);
+        break;
+      }
+      int hrow[8], erow[8], trw[8];
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        hrow[k] = R.hrow[r0 + 4 * k];
+        erow[k] = R.erow[r0 + 4 * k];
+        trw[k] = (tsplit && R.rdst[r0 + 4 * k] >= 0) ? R.trow[r0 + 4 * k] : -1;
+      }
+      __syncwarp();
+      warp_arrive(&B.dempty[ds]);
+      for (int i = 0; i < nch; ++i, ++g) {
+        const int c = plan.order[chunk_of(tt, i, nch)];
+        const int col = c * kTC + 8 * j;
+        const int ks = (plan.k - c * kTC) > 16 ? 2 : 1;
+        const uint32_t sa = g % kP2AStages;
+        PRE_FREE_SLEEP(&B.aempty[sa], g / kP2AStages, TGL_SLEEP_LOAD);
+        const bool in_k = active && col < c * kTC + 16 * ks;
+        const uint32_t dst = a_s + sa * kPAStage + ofs0;
+        if (in_k && col < kt0) {
+          const bool seg_h = col < plan.dp0;
+          const uint8_t* base = seg_h ? hbase : ebase;
+          const int64_t ldb = seg_h ? hld : eld;
+          const uint32_t pofs = seg_h ? (uint32_t)(lo_piece ? 2 * plan.dp0 : 0) + 2 * col
+                                      : (uint32_t)(lo_piece ? 2 * plan.dp1 : 0) +
+                                            2 * (col - plan.dp0);
+#pragma unroll
+          for (int k = 0; k < 8; ++k) {
+            const int row = seg_h ? hrow[k] : erow[k];
+            const int rr = (r0 + 4 * k) & 7;
+            const uint32_t d = dst + (uint32_t)(k >> 1) * 1024 + rr * 64 +
+                               (((j ^ (rr >> 1)) & 3) << 4);
+            cp_async16_zfill(d, base + (row >= 0 ? (int64_t)row * ldb + pofs : 0),
+                             row >= 0 ? 16u : 0u);
+          }
+        } else if (in_k && tsplit && col < plan.k) {
+          const uint32_t pofs = (uint32_t)(lo_piece ? 2 * plan.dpt : 0) + 2 * (col - kt0);
+#pragma unroll
+          for (int k = 0; k < 8; ++k) {
+            if (trw[k] < 0) continue;
+            const int rr = (r0 + 4 * k) & 7;
+            const uint32_t d = dst + (uint32_t)(k >> 1) * 1024 + rr * 64 +
+                               (((j ^ (rr >> 1)) & 3) << 4);
+            cp_async16_zfill(d, tbase + (int64_t)trw[k] * tld + pofs, 16u);
+          }
+        }
+        cp_async_mbar_arrive_noinc(&B.afull[sa]);
+      }
+    }
+  } else if (warp >= kPTime0 && warp < kPTime0 + kPTimeWarps) {   // -------- time warps
+    const int tw = warp - kPTime0;
+    const int r = tw * 32 + lane;
+    const int rr = r & 7;
+    const bool tsplit = (P.input_layout & TGL_SPLIT_TABLE) && a.table != nullptr;
+    const uint32_t rofs = (uint32_t)(r >> 3) * 1024 + rr * 64;
+    uint32_t g = 0;
+    for (;; ++tt) {
+      const uint32_t ds = tt % kSDSlots;
+      PRE_WAIT_SLEEP(&B.dfull[ds], (tt / kSDSlots) & 1u, TGL_SLEEP_LOAD);
+      const TDesc& R = bd[ds];
+      if (!R.live) {
+        warp_arrive(&B.dempty[ds]);
+        break;
+      }
+      const float dtr = R.dt[r];
+      const int trow = R.trow[r];
+      const int mode = R.rdst[r] < 0 ? 2 : (trow >= 0 ? 1 : 0);
+      __syncwarp();
+      warp_arrive(&B.dempty[ds]);
+      for (int i = 0; i < nch; ++i, ++g) {
+        const int c = plan.order[chunk_of(tt, i, nch)];
+        const int ks = (plan.k - c * kTC) > 16 ? 2 : 1;
+        const uint32_t sa = g % kP2AStages;
+        const bool has_time = (c + 1) * kTC > kt0;
+        if (has_time) {
+          wait_free(&B.aempty[sa], g / kP2AStages);
+          const uint32_t dst = a_s + sa * kPAStage + rofs;
+#pragma unroll
+          for (int jj = 0; jj < 4; ++jj) {
+            const int col = c * kTC + 8 * jj;
+            if (col < kt0 || col >= c * kTC + 16 * ks) continue;
+            const int tc = col - kt0;
+            if (tsplit && mode == 1 && col < plan.k) continue;
+            float x[8];
+            if (mode == 0) {
+              bool bad = false;
+#pragma unroll
+              for (int e = 0; e < 8; ++e) {
+                const float bb = __fadd_rn(__fmul_rn(s_omega[tc + e], dtr), s_phi[tc + e]);
+                bad |= !(fabsf(bb) < 1e9f);
+                x[e] = tenc_cos_reduced(bb);
+              }
+              if (bad) {
+#pragma unroll
+                for (int e = 0; e < 8; ++e) x[e] = tenc_fast(dtr, s_omega[tc + e], s_phi[tc + e]);
+              }
+            } else if (mode == 1 && !tsplit) {
+#pragma unroll
+              for (int e = 0; e < 8; ++e)
+                x[e] = tc + e < P.d_t ? __ldg(a.table + (int64_t)trow * P.d_t + tc + e) : 0.f;
+            } else {
+#pragma unroll
+              for (int e = 0; e < 8; ++e) x[e] = 0.f;
+            }
+            if (tc + 8 > P.d_t) {
+#pragma unroll
+              for (int e = 0; e < 8; ++e)
+                if (tc + e >= P.d_t) x[e] = 0.f;
+            }
+            uint32_t h[4], l[4];
+#pragma unroll
+            for (int e = 0; e < 4; ++e) split2(x[2 * e], x[2 * e + 1], h[e], l[e]);
+            const uint32_t po = (uint32_t)(((jj ^ (rr >> 1)) & 3) << 4);
+            st_shared_v4(dst + po, h[0], h[1], h[2], h[3]);
+            if (split) st_shared_v4(dst + 512 + po, l[0], l[1], l[2], l[3]);
+          }
+          fence_proxy_async_smem();
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&B.afull[sa]);
+        } else {
+          if (lane == 0) {
+            wait_free(&B.aempty[sa], g / kP2AStages);
+            mbar_arrive(&B.afull[sa]);
+          }
+          __syncwarp();
+        }
+      }
+    }
+  } else if (warp == kTMma && !leader) {             // ---------------- peer relay
+    // the leader's MMA reads this CTA's A stage and weight half: tell it when both landed
+    uint32_t g = 0, wl = 0;
+    const uint32_t pfull0 = mapa_shared(smem_u32(&B.pfull[0]), 0);
+    for (;; ++tt) {
+      const uint32_t ds = tt % kSDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kSDSlots) & 1u);
+      const int live = bd[ds].live;
+      warp_arrive(&B.dempty[ds]);
+      if (!live) break;
+      const int r0 = (tt > 0 && nch >= 4) ? 2 : 0;
+      for (int i = 0; i < nch; ++i, ++g) {
+        const uint32_t sa = g % kP2AStages;
+        mbar_wait(&B.afull[sa], (g / kP2AStages) & 1u);
+        if (i >= r0) {
+          const uint32_t kw = wl + (i - r0);
+          mbar_wait(&B.wfull[kw % kP2W], (kw / kP2W) & 1u);
+        }
+        if (lane == 0) mbar_arrive_remote(pfull0 + sa * 8);
+        __syncwarp();
+      }
+      wl += nch - r0;
+    }
+  } else if (warp == kTMma) {                        // ---------------- MMA issuer (leader)
+    uint32_t g = 0, wl = 0;
+    constexpr uint32_t idesc = idesc_bf16(2 * kBM, kP2N);
+    for (;; ++tt) {
+      const uint32_t ds = tt % kSDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kSDSlots) & 1u);
+      const int live = bd[ds].live;
+      warp_arrive(&B.dempty[ds]);
+      if (!live) break;
+      const uint32_t acc = tmem + (tt & 1u) * kCols;
+      if (tt >= 2) mbar_wait_cluster(&B.tempty[tt & 1u], ((tt >> 1) - 1) & 1u);
+      tc_fence_after();
+      const int r0 = (tt > 0 && nch >= 4) ? 2 : 0;
+      for (int i = 0; i < nch; ++i, ++g) {
+        const int c = plan.order[chunk_of(tt, i, nch)];
+        const int nk = (plan.k - c * kTC) > 16 ? 2 : 1;
+        const uint32_t sa = g % kP2AStages;
+        mbar_wait(&B.afull[sa], (g / kP2AStages) & 1u);
+        mbar_wait_cluster(&B.pfull[sa], (g / kP2AStages) & 1u);
+        uint32_t kw;
+        if (i < r0) {
+          kw = wl - 1 - i;
+        } else {
+          kw = wl + (i - r0);
+          mbar_wait(&B.wfull[kw % kP2W], (kw / kP2W) & 1u);
+        }
+        tc_fence_after();
+        if (elect_one()) {
+          const uint64_t a0 = desc_sw64(a_s + sa * kPAStage, 1024);
+          const uint64_t w0 = desc_sw64(w_s + (kw % kP2W) * kP2WStage, 512);
+#pragma unroll
+          for (int ks = 0; ks < 2; ++ks) {
+            if (ks < nk) {
+              const uint64_t ah = a0 + 2 * ks, bh = w0 + 2 * ks;
+              mma_bf16_pair(acc, ah, bh, idesc, (i | ks) != 0);
+              if (split) {
+                mma_bf16_pair(acc, ah + (512 >> 4), bh, idesc, 1u);
+                mma_bf16_pair(acc, ah, bh + (kP2Half >> 4), idesc, 1u);
+              }
+            }
+          }
+          const bool keep = (nch >= 4) && (i >= nch - 2);
+          mma_commit_pair(&B.aempty[sa]);
+          if (!keep) mma_commit_pair(&B.wempty[kw % kP2W]);
+        }
+        __syncwarp();
+      }
+      wl += nch - r0;
+      if (elect_one()) mma_commit_pair(&B.tfull[tt & 1u]);
+      __syncwarp();
+    }
+  } else if (warp < kBEpi) {                         // ---------------- epilogue warps 0-7
+    bin_epilogue<kSDSlots, TDesc, kSPW, false>(a, B.dfull, B.dempty, B.tfull, B.tempty, bd, tmem,
+                                               s_pvf, s_bias,
+                                               mapa_shared(smem_u32(&B.tempty[0]), 0));
+  }
+  tc_fence_before();
+  __syncthreads();
+  cluster_sync_all();                                // the peer's smem / barriers stay valid
+  if (warp == kTMma)
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem),
+                 "r"(2 * kCols)
+                 : "memory");
+}
+
 }  // namespace tca
 
 // ------------------------------------------------------------------ host side
 namespace tca {
 
 struct PackedLayout {
-  size_t oq, okv, oo, okv64, okvc, okvp, total;
+  size_t oq, okv, oo, okv64, okvc, okvp, okvp2, total;
 };
 
 static PackedLayout packed_layout(const tgl_attn_params* P) {
@@ -2937,6 +3469,7 @@ static PackedLayout packed_layout(const tgl_attn_params* P) {
   L.okv64 = W.take((size_t)make_plan(P->d_hsrc, P->d_e, P->d_t).n * kTWStage);
   L.okvc = W.take((size_t)make_plan_contig(P->d_hsrc, P->d_e, P->d_t).n * kTWStage);
   L.okvp = W.take((size_t)make_pre_plan(P->d_hsrc, P->d_e, P->d_t).n * kTWStage);
+  L.okvp2 = W.take((size_t)make_pre_plan(P->d_hsrc, P->d_e, P->d_t).n * 2 * kP2WStage);
   L.total = W.off;
   return L;
 }
@@ -2962,7 +3495,11 @@ static tgl_status launch_pack(const tgl_attn_params* P, uint8_t* base, cudaStrea
   pack_kv_pre_kernel<<<64, 256, 0, s>>>(P->Wk, P->Wv, P->d_model, P->d_hsrc + P->d_e + P->d_t,
                                         make_pre_plan(P->d_hsrc, P->d_e, P->d_t),
                                         base + L.okvp);
-  return launch_check("pack_kv_pre");
+  TGL_TRY(launch_check("pack_kv_pre"));
+  pack_kv_pre2_kernel<<<64, 256, 0, s>>>(P->Wk, P->Wv, P->d_model, P->d_hsrc + P->d_e + P->d_t,
+                                         make_pre_plan(P->d_hsrc, P->d_e, P->d_t),
+                                         base + L.okvp2);
+  return launch_check("pack_kv_pre2");
 }
 
 }  // namespace tca
@@ -3002,6 +3539,9 @@ static tgl_status set_smem_attrs(int smem_q, int smem_kv, int smem_kvb) {
     if (e == cudaSuccess)
       e = cudaFuncSetAttribute(kv_pre_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                kPSmem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(kv_pre2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               kP2Smem);
     return e;
   }), "smem attributes");
 }
@@ -3088,12 +3628,12 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
   launch_pdl(dense_kernel<false>, dim3(gq), dim3(kWsThreads), smem_q, s, a);
   TGL_TRY(launch_check("tc q kernel"));
   const int sel = P->kv_kernel;
-  if (sel < TGL_KV_AUTO || sel > TGL_KV_PRE || sel == TGL_KV_SIMT) {
+  if (sel < TGL_KV_AUTO || sel > TGL_KV_PRE2 || sel == TGL_KV_SIMT) {
     set_error("kv_kernel %d: not a TGL_KV_* id", sel);
     return TGL_EINVAL;
   }
   const bool pre_in = (P->input_layout & (TGL_SPLIT_HSRC | TGL_SPLIT_E | TGL_SPLIT_TABLE)) != 0;
-  if (pre_in || sel == TGL_KV_PRE) {
+  if (pre_in || sel == TGL_KV_PRE || sel == TGL_KV_PRE2) {
     // pre-split h_src / e tables (tgl_split_rows): every gathered table present must be
     // split, rows 16-byte aligned; max_seg <= 32 and 2 heads (the binned epilogue)
     const PrePlan plan = make_pre_plan(P->d_hsrc, P->d_e, P->d_t);
@@ -3103,15 +3643,17 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
                                       rows_16b(efeat, 1, ld_e));
     const bool t_ok = !(P->input_layout & TGL_SPLIT_TABLE) || table == nullptr ||
                       rows_16b(table, 1, plan.dpt);
-    if (!(sel == TGL_KV_AUTO || sel == TGL_KV_PRE) || !hs_ok || !e_ok || !t_ok ||
+    if (!(sel == TGL_KV_AUTO || sel == TGL_KV_PRE || sel == TGL_KV_PRE2) || !hs_ok || !e_ok ||
+        !t_ok ||
         !(max_seg > 0 && max_seg <= 32 && P->n_heads == 2) || plan.n > kPMaxChunks) {
       set_error("pre-split inputs: kv_kernel must be AUTO/PRE, every gathered table split "
                 "(input_layout), 16-byte rows, ld >= padded width, max_seg <= 32, 2 heads");
       return TGL_EUNSUPPORTED;
     }
+    const bool pair = sel == TGL_KV_PRE2 || (sel == TGL_KV_AUTO && kPreAutoPair);
     tgl_kv_probe* probe = P->probe;
     if (probe) {
-      probe->kernel = TGL_KV_PRE;
+      probe->kernel = pair ? TGL_KV_PRE2 : TGL_KV_PRE;
       if (probe->ev_start)
         TGL_TRY(cuda_check(cudaEventRecord(static_cast<cudaEvent_t>(probe->ev_start), s),
                            "probe event"));
@@ -3119,7 +3661,15 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
     const int bdst = 32 / max_seg;
     const int64_t ttiles = ceil_div(n_dst_max, 4 * bdst);
     const unsigned gt = (unsigned)(ttiles < kNumSMs ? (ttiles > 0 ? ttiles : 1) : kNumSMs);
-    launch_pdl(kv_pre_kernel, dim3(gt), dim3(kPThreads), kPSmem, s, a, plan, pk + PL.okvp, bdst);
+    if (pair) {                                    // CTA pairs: even grid of <= 148 CTAs
+      const int64_t npt = ceil_div(ttiles > 0 ? ttiles : 1, 2);
+      const unsigned gp = 2u * (unsigned)(npt < kNumSMs / 2 ? npt : kNumSMs / 2);
+      launch_pdl(kv_pre2_kernel, dim3(gp), dim3(kPThreads), kP2Smem, s, a, plan, pk + PL.okvp2,
+                 bdst);
+    } else {
+      launch_pdl(kv_pre_kernel, dim3(gt), dim3(kPThreads), kPSmem, s, a, plan, pk + PL.okvp,
+                 bdst);
+    }
     TGL_TRY(launch_check("tc kv pre kernel"));
     if (probe && probe->ev_stop)
       TGL_TRY(cuda_check(cudaEventRecord(static_cast<cudaEvent_t>(probe->ev_stop), s),

@@ -210,7 +210,8 @@ def cu_pad(a, mult=4):
     return t[:, :d]
 
 
-@pytest.mark.parametrize("precision,kv", [("fp32", "pre"), ("bf16", "pre"),
+@pytest.mark.parametrize("precision,kv", [("fp32", "pre"), ("bf16", "pre"), ("fp32", "pre2"),
+                                          ("bf16", "pre2"),
                                           ("fp32", "split"), ("bf16", "split"),
                                           ("fp32", "split_pad"), ("bf16", "split_pad"),
                                           ("fp32", "async"), ("bf16", "async"), ("fp32", "bin"),
@@ -235,7 +236,7 @@ def test_attention_vs_oracle(T, monkeypatch, precision, kv, n_dst, kmax, d_h, d_
     rng = np.random.default_rng(n_dst + kmax)
     p, seg, dst_t, nfeat, dn, sn, ef, eid, et = attn_case(rng, n_dst, kmax, d_h, d_e,
                                                           long_every=long_every)
-    if kv == "pre" and np.diff(seg).max() > 32:
+    if kv in ("pre", "pre2") and np.diff(seg).max() > 32:
         pytest.skip("the pre-split kernel takes segments <= 32 rows (binned epilogue)")
     sel = kv if (kv and np.diff(seg).max() <= 32) else "auto"   # longer: general kernel
     exp = oracle.tblock_attn(p, seg, dst_t, nfeat, dn, nfeat, sn, ef, eid, et)
@@ -247,7 +248,7 @@ def test_attention_vs_oracle(T, monkeypatch, precision, kv, n_dst, kmax, d_h, d_
     nf = put(nfeat)
     hs, efd = nf, (put(ef) if d_e else None)
     tables = [(None, 0), (tab, 0)]
-    if kv == "pre":            # split16 operand tables (tgl_split_rows), fp32 h_dst
+    if kv in ("pre", "pre2"):  # split16 operand tables (tgl_split_rows), fp32 h_dst
         hs = T.split_rows(nf)
         efd = T.split_rows(efd) if d_e else None
         base = T.SPLIT_HSRC | (T.SPLIT_E if d_e else 0)
@@ -259,7 +260,7 @@ def test_attention_vs_oracle(T, monkeypatch, precision, kv, n_dst, kmax, d_h, d_
                             table=table, max_seg=int(np.diff(seg).max()))
         err = np.abs(np_(got)[:n_dst] - exp).max()
         assert err <= TOL[precision], err
-        if kv == "pre" and sel == "auto":             # long segments: no split path
+        if kv in ("pre", "pre2") and sel == "auto":   # long segments: no split path
             continue
         if sel != "auto" and precision != "fp32_simt":   # the requested kernel really ran
             want = T.KV_KERNEL[sel]
