@@ -238,6 +238,9 @@ tgl_status tgl_time_encode(int64_t n, const float* dt, int32_t d_t, const float*
 #define TGL_SPLIT_HSRC 1
 #define TGL_SPLIT_E 2
 #define TGL_SPLIT_TABLE 4   /* tenc_table is split16 [window, round_up(d_t, 8)] (kv_pre only) */
+#define TGL_SPLIT_HDST 8    /* hdst is split16 too: the Q / FFN projections gather converter-
+                               free operands (Phi(0) folded into the Q bias); needs the
+                               pre-split K|V path and d_model == 100 */
 
 /* Measurement record (bench.py): when tgl_attn_params.probe != NULL the call records
  * ev_start / ev_stop (cudaEvent_t, created by the caller) on its stream immediately

@@ -95,7 +95,7 @@ class TGATPipeline:
             self.nfeat_split, self.efeat_split = nf, ef
             for l, a in enumerate(self.attn):
                 a.struct.input_layout = (tgl.SPLIT_HSRC | (tgl.SPLIT_E if a.host["d_e"] else 0) |
-                                         tgl.SPLIT_TABLE)
+                                         tgl.SPLIT_TABLE | tgl.SPLIT_HDST)
             # the precompute tables as split16 rows too: gathered like features
             self.tables = [None if t is None else tgl.split_rows(t) for t in self.tables]
         k = sampler.k
@@ -263,12 +263,12 @@ class TGATPipeline:
             if l == self.L - 1:
                 hdst, hdst_idx, hsrc, hsrc_idx, off = g["nfeat"], b.uniq_node, g["nfeat"], b.nbr, None
                 if self.split:
-                    hsrc = self.nfeat_split
+                    hdst = hsrc = self.nfeat_split
             else:
                 nx = self.blocks[l + 1]
                 hdst = hsrc = nx.ws["cache"]["comb"] if self.cache_on else nx.out
                 if self.split:
-                    hsrc = nx.out_split
+                    hdst = hsrc = nx.out_split
                 off = b.u_dev        # S14: rows [U_l + e] of the next block hold the sources
                 if self.use_dedup:
                     hdst_idx = hsrc_idx = nx.inv

@@ -37,6 +37,7 @@ constexpr int kChunk = 64;                 // bf16 K elements per chunk (one 128
 constexpr int kAPart = kBM * 128;          // bytes of A_hi (or A_lo) per stage
 constexpr int kMaxDpb = 16;
 constexpr int kQLd = 128;                  // q / r scratch leading dim (floats)
+constexpr int kDPN = 104;                  // d_model padded to 8: N of dense_pre, r split16 width
 constexpr int kMaxModel = 128;
 
 __host__ __device__ __forceinline__ int pad8(int x) { return (x + 7) & ~7; }
@@ -121,6 +122,7 @@ struct Args {
   float* out;
   float* qbuf;
   float* rbuf;
+  uint8_t* rsplit;     // split16 r rows [n_dst_max][104 words] for dense_pre FFN (or null)
   const uint8_t* wq;   // packed
   const uint8_t* wkv;
   const uint8_t* wo;
@@ -130,6 +132,23 @@ struct Args {
   int split;           // 1 = 3-pass fp32 mode
   int dbg;             // TGL_DEBUG_MASK (profiling only): 1 skip epilogue math, 2 skip gathers, 4 skip MMAs
 };
+
+// an empty (0) or overflowed (NaN) segment's r row, called by one warp: fp32 scratch row, or
+// the split16 row dense_pre gathers (hi = value, lo = 0, padding columns 100..103 zero)
+__device__ __forceinline__ void fill_r_row(const Args& a, int64_t row, float fill, int lane,
+                                           int dm) {
+  if (a.rsplit == nullptr) {
+    for (int c = lane; c < dm; c += 32) a.rbuf[row * kQLd + c] = fill;
+    return;
+  }
+  uint16_t* rp = reinterpret_cast<uint16_t*>(a.rsplit + row * (4 * kDPN));
+  const __nv_bfloat16 h = __float2bfloat16_rn(fill);
+  const uint16_t hb = *reinterpret_cast<const uint16_t*>(&h);
+  for (int c = lane; c < kDPN; c += 32) {
+    rp[c] = c < dm ? hb : (uint16_t)0;
+    rp[kDPN + c] = c < dm && fill != fill ? hb : (uint16_t)0;
+  }
+}
 
 // offset (not integer round-trip) so the compiler keeps the shared address space
 __device__ __forceinline__ uint8_t* align1024(uint8_t* p) {
@@ -1130,7 +1149,22 @@ __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uin
           const int dr = __shfl_sync(0xffffffffu, d, slo);
           float acc = 0.f;
           for (int r = slo; r < shi; ++r) acc += pvw[r * kPW + (lane & (kCW - 1))];
-          if (act) a.rbuf[(int64_t)dr * kQLd + cb + c] = acc + bvc;
+          if (act) {
+            const float rv = acc + bvc;
+            if (a.rsplit != nullptr) {                 // split16 operand row for dense_pre
+              uint8_t* rp = a.rsplit + (int64_t)dr * (4 * kDPN);
+              const __nv_bfloat16 rh = __float2bfloat16_rn(rv);
+              const __nv_bfloat16 rl = __float2bfloat16_rn(rv - __bfloat162float(rh));
+              *reinterpret_cast<__nv_bfloat16*>(rp + 2 * (cb + c)) = rh;
+              *reinterpret_cast<__nv_bfloat16*>(rp + 2 * kDPN + 2 * (cb + c)) = rl;
+              if (cb + c < kDPN - dm) {                // zero the padding columns 100..103
+                *reinterpret_cast<uint16_t*>(rp + 2 * (dm + cb + c)) = 0;
+                *reinterpret_cast<uint16_t*>(rp + 2 * kDPN + 2 * (dm + cb + c)) = 0;
+              }
+            } else {
+              a.rbuf[(int64_t)dr * kQLd + cb + c] = rv;
+            }
+          }
         }
         __syncwarp();
       }
@@ -1407,6 +1441,32 @@ __device__ __forceinline__ void cp_async16_zfill(uint32_t dst, const void* src, 
                "r"(src_bytes)
                : "memory");
 }
+// L2 cache policies (createpolicy): streamed-once rows evict first, reused operands last
+__device__ __forceinline__ uint64_t l2_policy_evict_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t l2_policy_evict_last() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ void cp_async16_zfill_hint(uint32_t dst, const void* src,
+                                                      uint32_t src_bytes, uint64_t pol) {
+  asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;" ::"r"(dst),
+               "l"(src), "r"(src_bytes), "l"(pol)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_g2s_hint(void* dst_smem, const void* src_gmem, uint32_t bytes,
+                                              uint64_t* bar, uint64_t pol) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], "
+      "[%1], %2, [%3], %4;" ::"r"(smem_u32(dst_smem)),
+      "l"(src_gmem), "r"(bytes), "r"(smem_u32(bar)), "l"(pol)
+      : "memory");
+}
+
 __device__ __forceinline__ void cp_async_wait_dyn(int pending) {   // <= pending groups left
   switch (pending) {
     case 0: cp_async_wait<0>(); break;
@@ -1587,7 +1647,7 @@ __global__ void __launch_bounds__(kTThreads, 1)
         const bool ovf = (ovf_bins >> (j / bdst)) & 1u;
         if (sg[j + 1] == sg[j] || ovf) {
           const float fill = ovf ? __int_as_float(0x7fc00000) : 0.f;
-          for (int c = lane; c < dm; c += 32) a.rbuf[(d0 + j) * kQLd + c] = fill;
+          fill_r_row(a, d0 + j, fill, lane, dm);
         }
       }
       R.live = 1;
@@ -2090,7 +2150,7 @@ __global__ void __launch_bounds__(kSThreads, 1)
         const bool ovf = (ovf_bins >> (j / bdst)) & 1u;
         if (sg[j + 1] == sg[j] || ovf) {
           const float fill = ovf ? __int_as_float(0x7fc00000) : 0.f;
-          for (int c = lane; c < dm; c += 32) a.rbuf[(d0 + j) * kQLd + c] = fill;
+          fill_r_row(a, d0 + j, fill, lane, dm);
         }
       }
       R.live = 1;
@@ -2455,6 +2515,12 @@ constexpr int kPAStage = kBM * kTC * 4;                // 16 KB
 // kept across the tile boundary (alternating K order) are still being read -- with 2
 // stages the MMA waited ~18 % of the kernel for weights (probe counters, GDELT)
 constexpr int kPW = TGL_KV_PRE_WSTAGES;
+// weight chunks kept across a tile boundary (the K order alternates per tile).  Kept
+// chunks pin weight stages at the boundary, so the next loads queue behind them.
+#ifndef TGL_KV_PRE_REUSE
+#define TGL_KV_PRE_REUSE 2
+#endif
+constexpr int kPreReuse = TGL_KV_PRE_REUSE;
 constexpr int kPLoad0 = 12, kPLoadWarps = 4;
 constexpr int kPTime0 = 16, kPTimeWarps = 4;
 constexpr int kPThreads = (kPTime0 + kPTimeWarps) * 32;   // 640
@@ -2642,7 +2708,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
         const bool ovf = (ovf_bins >> (j / bdst)) & 1u;
         if (sg[j + 1] == sg[j] || ovf) {
           const float fill = ovf ? __int_as_float(0x7fc00000) : 0.f;
-          for (int c = lane; c < dm; c += 32) a.rbuf[(d0 + j) * kQLd + c] = fill;
+          fill_r_row(a, d0 + j, fill, lane, dm);
         }
       }
       R.live = 1;
@@ -2670,6 +2736,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
     }
   } else if (warp == kTW) {                          // ---------------- weight loader
     uint32_t wl = 0;
+    const uint64_t wpol = l2_policy_evict_last();    // weights: re-read by every tile
     const uint32_t wbytes = split ? kTWStage : kTWHalf;
     for (;; ++tt) {
       const uint32_t ds = tt % kSDSlots;
@@ -2678,14 +2745,15 @@ __global__ void __launch_bounds__(kPThreads, 1)
       warp_arrive(&B.dempty[ds]);
       if (!live) break;
       if (lane == 0) {
-        const int r0 = (tt > 0 && nch >= 4) ? 2 : 0;
+        const int r0 = (tt > 0 && nch >= 4) ? kPreReuse : 0;
         for (int i = r0; i < nch; ++i) {
           const uint32_t k = wl + (i - r0);
           const uint32_t sw = k % kPW;
           PRE_FREE_SLEEP(&B.wempty[sw], k / kPW, TGL_SLEEP_W);
           mbar_arrive_expect_tx(&B.wfull[sw], wbytes);
-          bulk_g2s(pipe + kPAStages * kPAStage + sw * kTWStage,
-                   wkv + (size_t)plan.order[chunk_of(tt, i, nch)] * kTWStage, wbytes, &B.wfull[sw]);
+          bulk_g2s_hint(pipe + kPAStages * kPAStage + sw * kTWStage,
+                        wkv + (size_t)plan.order[chunk_of(tt, i, nch)] * kTWStage, wbytes,
+                        &B.wfull[sw], wpol);
         }
         wl += nch - r0;
       }
@@ -2707,6 +2775,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
     const uint8_t* ebase = reinterpret_cast<const uint8_t*>(a.efeat);
     const uint8_t* tbase = reinterpret_cast<const uint8_t*>(a.table);
     const int64_t hld = 4 * a.ld_hsrc, eld = 4 * a.ld_e, tld = 4 * plan.dpt;
+    const uint64_t epol = l2_policy_evict_first();
     uint32_t g = 0;
     for (;; ++tt) {
       const uint32_t ds = tt % kSDSlots;
@@ -2750,8 +2819,11 @@ __global__ void __launch_bounds__(kPThreads, 1)
             const int rr = (r0 + 4 * k) & 7;
             const uint32_t d = dst + (uint32_t)(k >> 1) * 1024 + rr * 64 +
                                (((j ^ (rr >> 1)) & 3) << 4);
-            cp_async16_zfill(d, base + (row >= 0 ? (int64_t)row * ldb + pofs : 0),
-                             row >= 0 ? 16u : 0u);
+            const void* src = base + (row >= 0 ? (int64_t)row * ldb + pofs : 0);
+            if (seg_h)
+              cp_async16_zfill(d, src, row >= 0 ? 16u : 0u);
+            else                                       // edge rows: streamed once
+              cp_async16_zfill_hint(d, src, row >= 0 ? 16u : 0u, epol);
           }
         } else if (in_k && tsplit && col < plan.k) {  // a time piece of a table row
           const uint32_t pofs = (uint32_t)(lo_piece ? 2 * plan.dpt : 0) + 2 * (col - kt0);
@@ -2878,7 +2950,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
       prof_add(a, 7, mt1 - mt0);                     // MMA: wait for an accumulator
 #endif
       tc_fence_after();
-      const int r0 = (tt > 0 && nch >= 4) ? 2 : 0;
+      const int r0 = (tt > 0 && nch >= 4) ? kPreReuse : 0;
       for (int i = 0; i < nch; ++i, ++g) {
         const int c = plan.order[chunk_of(tt, i, nch)];
         const int nk = (plan.k - c * kTC) > 16 ? 2 : 1;
@@ -2912,7 +2984,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
               }
             }
           }
-          const bool keep = (nch >= 4) && (i >= nch - 2);   // reused by the next tile
+          const bool keep = (nch >= 4) && (i >= nch - kPreReuse);   // reused by the next tile
           mma_commit(&B.aempty[sa]);
           if (!keep) mma_commit(&B.wempty[kw % kPW]);
         }
@@ -2929,6 +3001,381 @@ __global__ void __launch_bounds__(kPThreads, 1)
   ws_teardown(tmem, 2 * kCols, kTMma);
 }
 
+
+// ------------------------------------------------------------------ S8 / S13 on split16 rows
+// dense_pre_kernel<kFfn>: the dense projections with converter-free operands, the same
+// scheme as kv_pre.  A = [seg0 | seg1] of split16 rows (8-column groups, 32-column
+// chunks), gathered by LDGSTS straight into the SW64 stages; the MMA is M=128 N=104.
+//   Q   (kFfn = 0): seg0 = h_dst (hdst split16, row hdst_idx[i]); Phi(0) = cos(phi) is the
+//       same for every destination, so Wq[:, d_hdst:] Phi(0) is folded into the bias
+//       (computed once by the pack kernel, fp64 accumulate) -- K = d_hdst only.
+//   FFN (kFfn = 1): seg0 = r_i (the K|V epilogue writes it split16), seg1 = h_dst.
+// Roles: epilogue warps 0-3 (one row per thread, TMEM lane quarter = warp), MMA 4,
+// descriptors 5, weights 6, loaders 7-10: 352 threads.
+constexpr int kDPAStages = 8;
+constexpr int kDPWStage = 2 * kDPN * 64;               // hi | lo of a 32-column chunk
+constexpr int kDPW = 4;
+constexpr int kDPLoad0 = 7, kDPLoadWarps = 4;
+constexpr int kDPThreads = (kDPLoad0 + kDPLoadWarps) * 32;   // 352
+constexpr int kDPPipeBytes = kDPAStages * kPAStage + kDPW * kDPWStage;
+constexpr int kDPSmem = 1024 + kDPPipeBytes;
+
+struct DPPlan {        // K' = [seg0: dp0 | seg1: dp1], 32-column chunks
+  int d0, d1, dp0, dp1, k, n;
+};
+static DPPlan make_dp_plan(int d0, int d1) {
+  DPPlan p;
+  p.d0 = d0; p.d1 = d1;
+  p.dp0 = pad8h(d0); p.dp1 = pad8h(d1);
+  p.k = p.dp0 + p.dp1;
+  p.n = (p.k + kTC - 1) / kTC;
+  return p;
+}
+
+// W [n_out][ksrc] (columns [c0, c0 + d0) then [c1, c1 + d1)) in the K' order, packed as
+// kv_pre packs [Wk ; Wv] but with N = 104 rows; qfold != nullptr (Q only): bias'[n] =
+// b[n] + sum_j W[n][d_hdst + j] cos(phi_j) (Phi(0), R10: fl(omega * 0 + phi) = phi)
+__global__ void pack_dense_pre_kernel(const float* W, int n_out, int ksrc, int c0, int c1,
+                                      DPPlan p, uint8_t* out, const float* b, const float* phi,
+                                      int d_t, int col_t, float* bias_out) {
+  const int kw = p.n * kTC;
+  const int64_t total = (int64_t)kDPN * kw;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const int n = (int)(x / kw), kp = (int)(x % kw);
+    const int c = kp / kTC, cc = kp % kTC;
+    int src = -1;
+    if (kp < p.dp0) {
+      if (kp < p.d0) src = c0 + kp;
+    } else if (kp < p.k) {
+      if (kp - p.dp0 < p.d1) src = c1 + (kp - p.dp0);
+    }
+    const float v = (n < n_out && src >= 0) ? W[(int64_t)n * ksrc + src] : 0.f;
+    const __nv_bfloat16 hi = __float2bfloat16_rn(v);
+    const __nv_bfloat16 lo = __float2bfloat16_rn(v - __bfloat162float(hi));
+    const int64_t off = (int64_t)c * kDPWStage + (n >> 3) * 512 + sw64_off(n, cc);
+    *reinterpret_cast<__nv_bfloat16*>(out + off) = hi;
+    *reinterpret_cast<__nv_bfloat16*>(out + off + kDPN * 64) = lo;
+  }
+  if (bias_out != nullptr && blockIdx.x == 0) {
+    for (int n = threadIdx.x; n < n_out; n += blockDim.x) {
+      double acc = b[n];
+      if (phi != nullptr)
+        for (int j = 0; j < d_t; ++j)
+          acc += (double)W[(int64_t)n * ksrc + col_t + j] * (double)cosf(phi[j]);
+      bias_out[n] = (float)acc;
+    }
+  }
+}
+
+struct DPBars {
+  uint64_t afull[kDPAStages], aempty[kDPAStages];
+  uint64_t wfull[kDPW], wempty[kDPW];
+  uint64_t dfull[kDSlots], dempty[kDSlots];
+  uint64_t tfull[2], tempty[2];
+};
+struct DPDesc {
+  int row0[kBM];
+  int row1[kBM];
+  int live;
+  int rows;
+  int64_t i0;
+};
+
+template <bool kFfn>
+__global__ void __launch_bounds__(kDPThreads, 1)
+    dense_pre_kernel(const Args a, const DPPlan plan, const uint8_t* __restrict__ wpk,
+                     const float* __restrict__ bias) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* pipe = align1024(smem_raw);
+  __shared__ DPBars B;
+  __shared__ uint32_t s_tmem;
+  __shared__ DPDesc bd[kDSlots];
+  __shared__ float s_v0[kMaxModel], s_v1[kMaxModel], s_v2[kMaxModel];
+  constexpr uint32_t kCols = 128;
+  const tgl_attn_params& P = a.P;
+  const bool split = a.split != 0;
+  const int nch = plan.n;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < kDPAStages; ++s) {
+      mbar_init(&B.afull[s], kDPLoadWarps * 32);
+      mbar_init(&B.aempty[s], 1);
+    }
+    for (int s = 0; s < kDPW; ++s) {
+      mbar_init(&B.wfull[s], 1);
+      mbar_init(&B.wempty[s], 1);
+    }
+    for (int s = 0; s < kDSlots; ++s) {
+      mbar_init(&B.dfull[s], 1);
+      mbar_init(&B.dempty[s], kEpiWarps + kDPLoadWarps + 2);
+    }
+    for (int s = 0; s < 2; ++s) {
+      mbar_init(&B.tfull[s], 1);
+      mbar_init(&B.tempty[s], kEpiWarps);
+    }
+    fence_mbar_init();
+  }
+  if (warp == kMmaWarp) tmem_alloc(&s_tmem, 2 * kCols);
+  for (int j = threadIdx.x; j < P.d_model; j += blockDim.x) {
+    if (kFfn) {
+      s_v0[j] = P.bo[j];
+      s_v1[j] = P.ln_gamma[j];
+      s_v2[j] = P.ln_beta[j];
+    } else {
+      s_v0[j] = bias[j];                               // bq + Wq[:, d_hdst:] Phi(0)
+      s_v1[j] = P.bk[j];
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  pdl_wait();
+  pdl_trigger();
+  const int64_t n = dev_count(a.n_dst_dev, a.n_dst_max);
+  const uint32_t tmem = s_tmem;
+  const uint32_t a_s = smem_u32(pipe);
+  const uint32_t w_s = a_s + kDPAStages * kPAStage;
+  const int64_t ntiles = (n + kBM - 1) / kBM;
+  uint32_t tt = 0;
+  // split16 row tables: seg0 / seg1 base and pitch (bytes)
+  const uint8_t* b0 = reinterpret_cast<const uint8_t*>(kFfn ? (const void*)a.rsplit
+                                                            : (const void*)a.hdst);
+  const int64_t ld0 = kFfn ? 4 * (int64_t)kDPN : 4 * a.ld_hdst;
+  const uint8_t* b1 = reinterpret_cast<const uint8_t*>(a.hdst);
+  const int64_t ld1 = 4 * a.ld_hdst;
+
+  if (warp == kDescWarp) {                           // ---------------- row descriptors
+    for (;; ++tt) {
+      const uint32_t ds = tt % kDSlots;
+      wait_free(&B.dempty[ds], tt / kDSlots);
+      DPDesc& R = bd[ds];
+      const int64_t T = blockIdx.x + (int64_t)tt * gridDim.x;
+      if (T >= ntiles) {
+        if (lane == 0) R.live = 0;
+        warp_arrive(&B.dfull[ds]);
+        break;
+      }
+      const int64_t i0 = T * kBM;
+      const int rows = (int)((n - i0) < kBM ? (n - i0) : kBM);
+#pragma unroll
+      for (int u = 0; u < kBM / 32; ++u) {
+        const int r = lane + 32 * u;
+        int hrow = -1;
+        if (r < rows) hrow = a.hdst_idx ? a.hdst_idx[i0 + r] : (int)(i0 + r);
+        R.row0[r] = kFfn ? (r < rows ? (int)(i0 + r) : -1) : hrow;
+        R.row1[r] = kFfn ? hrow : -1;
+      }
+      if (lane == 0) {
+        R.live = 1;
+        R.rows = rows;
+        R.i0 = i0;
+      }
+      warp_arrive(&B.dfull[ds]);
+    }
+  } else if (warp == kWWarp) {                       // ---------------- weight loader
+    uint32_t k = 0;
+    const uint32_t wbytes = split ? kDPWStage : kDPN * 64;
+    const uint64_t wpol = l2_policy_evict_last();
+    for (;; ++tt) {
+      const uint32_t ds = tt % kDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kDSlots) & 1u);
+      const int live = bd[ds].live;
+      warp_arrive(&B.dempty[ds]);
+      if (!live) break;
+      if (lane == 0) {
+        for (int i = 0; i < nch; ++i, ++k) {
+          const uint32_t sw = k % kDPW;
+          wait_free(&B.wempty[sw], k / kDPW);
+          mbar_arrive_expect_tx(&B.wfull[sw], wbytes);
+          bulk_g2s_hint(pipe + kDPAStages * kPAStage + sw * kDPWStage,
+                        wpk + (size_t)i * kDPWStage, wbytes, &B.wfull[sw], wpol);
+        }
+      }
+      __syncwarp();
+    }
+  } else if (warp >= kDPLoad0 && warp < kDPLoad0 + kDPLoadWarps) {   // ---------- loaders
+    const int lw = warp - kDPLoad0;
+    const int r0 = lw * 32 + (lane >> 3), pc = lane & 7;
+    const bool lo_piece = pc >= 4;
+    const int j = pc & 3;
+    const uint32_t ofs0 = (uint32_t)(r0 >> 3) * 1024 + (lo_piece ? 512 : 0);
+    const bool active = split || !lo_piece;
+    uint32_t g = 0;
+    for (;; ++tt) {
+      const uint32_t ds = tt % kDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kDSlots) & 1u);
+      const DPDesc& R = bd[ds];
+      if (!R.live) {
+        warp_arrive(&B.dempty[ds]);
+        break;
+      }
+      int x0[8], x1[8];
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        x0[k] = R.row0[r0 + 4 * k];
+        x1[k] = R.row1[r0 + 4 * k];
+      }
+      __syncwarp();
+      warp_arrive(&B.dempty[ds]);
+      for (int i = 0; i < nch; ++i, ++g) {
+        const int col = i * kTC + 8 * j;
+        const int ks = (plan.k - i * kTC) > 16 ? 2 : 1;
+        const uint32_t sa = g % kDPAStages;
+        wait_free(&B.aempty[sa], g / kDPAStages);
+        if (active && col < i * kTC + 16 * ks) {
+          const bool s0 = col < plan.dp0;
+          const bool pad = col >= plan.k;
+          const uint8_t* base = s0 ? b0 : b1;
+          const int64_t ldb = s0 ? ld0 : ld1;
+          const int dpw = s0 ? plan.dp0 : plan.dp1;
+          const int lc = s0 ? col : col - plan.dp0;
+          const uint32_t pofs = (uint32_t)(lo_piece ? 2 * dpw : 0) + 2 * lc;
+          const uint32_t dst = a_s + sa * kPAStage + ofs0;
+#pragma unroll
+          for (int k = 0; k < 8; ++k) {
+            const int row = s0 ? x0[k] : x1[k];
+            const int rr = (r0 + 4 * k) & 7;
+            const uint32_t d = dst + (uint32_t)(k >> 1) * 1024 + rr * 64 +
+                               (((j ^ (rr >> 1)) & 3) << 4);
+            const bool ok = row >= 0 && !pad;
+            cp_async16_zfill(d, ok ? base + (int64_t)row * ldb + pofs : b1, ok ? 16u : 0u);
+          }
+        }
+        cp_async_mbar_arrive_noinc(&B.afull[sa]);
+      }
+    }
+  } else if (warp == kMmaWarp) {                     // ---------------- MMA issuer
+    uint32_t g = 0, k = 0;
+    constexpr uint32_t idesc = idesc_bf16(kBM, kDPN);
+    for (;; ++tt) {
+      const uint32_t ds = tt % kDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kDSlots) & 1u);
+      const int live = bd[ds].live;
+      warp_arrive(&B.dempty[ds]);
+      if (!live) break;
+      const uint32_t acc = tmem + (tt & 1u) * kCols;
+      wait_free(&B.tempty[tt & 1u], tt >> 1);
+      tc_fence_after();
+      for (int i = 0; i < nch; ++i, ++g, ++k) {
+        const int nk = (plan.k - i * kTC) > 16 ? 2 : 1;
+        const uint32_t sa = g % kDPAStages, sw = k % kDPW;
+        mbar_wait(&B.afull[sa], (g / kDPAStages) & 1u);
+        mbar_wait(&B.wfull[sw], (k / kDPW) & 1u);
+        tc_fence_after();
+        if (elect_one()) {
+          const uint64_t a0 = desc_sw64(a_s + sa * kPAStage, 1024);
+          const uint64_t w0 = desc_sw64(w_s + sw * kDPWStage, 512);
+#pragma unroll
+          for (int ks = 0; ks < 2; ++ks) {
+            if (ks < nk) {
+              const uint64_t ah = a0 + 2 * ks, bh = w0 + 2 * ks;
+              mma_bf16(acc, ah, bh, idesc, (i | ks) != 0);
+              if (split) {
+                mma_bf16(acc, ah + (512 >> 4), bh, idesc, 1u);
+                mma_bf16(acc, ah, bh + ((kDPN * 64) >> 4), idesc, 1u);
+              }
+            }
+          }
+          mma_commit(&B.aempty[sa]);
+          mma_commit(&B.wempty[sw]);
+        }
+        __syncwarp();
+      }
+      if (elect_one()) mma_commit(&B.tfull[tt & 1u]);
+      __syncwarp();
+    }
+  } else if (warp < kEpiWarps) {                     // ---------------- epilogue
+    const int row = warp * 32 + lane;
+    const int D = P.d_model;
+    for (;; ++tt) {
+      const uint32_t ab = tt & 1u, ds = tt % kDSlots;
+      mbar_wait(&B.dfull[ds], (tt / kDSlots) & 1u);
+      const int live = bd[ds].live;
+      const int rows = bd[ds].rows;
+      const int64_t i0 = bd[ds].i0;
+      warp_arrive(&B.dempty[ds]);
+      if (!live) break;
+      mbar_wait(&B.tfull[ab], (tt >> 1) & 1u);
+      tc_fence_after();
+      const uint32_t ta = tmem + ab * kCols + ((uint32_t)(warp * 32) << 16);
+      float v[32];
+      if (!kFfn) {
+        float* q = a.qbuf + (i0 + row) * kQLd;
+        const int dhq = D / P.n_heads;
+        float qb0 = 0.f, qb1 = 0.f;
+#pragma unroll 1
+        for (int cq = 0; cq < 4; ++cq) {
+          tmem_ld32(ta + cq * 32, v);
+          tmem_wait_ld();
+          if (row < rows) {
+#pragma unroll
+            for (int jj = 0; jj < 32; jj += 4) {
+              const int col = cq * 32 + jj;
+              if (col < D) {
+                float4 o = make_float4(v[jj] + s_v0[col], v[jj + 1] + s_v0[col + 1],
+                                       v[jj + 2] + s_v0[col + 2], v[jj + 3] + s_v0[col + 3]);
+                *reinterpret_cast<float4*>(q + col) = o;
+                const float oq[4] = {o.x, o.y, o.z, o.w};
+#pragma unroll
+                for (int e = 0; e < 4; ++e) {
+                  const float pb = oq[e] * s_v1[col + e];
+                  if (col + e < dhq) qb0 += pb; else qb1 += pb;
+                }
+              }
+            }
+          }
+        }
+        if (row < rows && D + 2 <= kQLd) {
+          q[D] = qb0;
+          q[D + 1] = qb1;
+        }
+      } else {
+        float s = 0.f, s2 = 0.f;
+#pragma unroll 1
+        for (int cq = 0; cq < 4; ++cq) {
+          tmem_ld32(ta + cq * 32, v);
+          tmem_wait_ld();
+#pragma unroll
+          for (int jj = 0; jj < 32; ++jj) {
+            const int col = cq * 32 + jj;
+            if (col < D) {
+              const float y = fmaxf(v[jj] + s_v0[col], 0.f);
+              s += y;
+              s2 = fmaf(y, y, s2);
+            }
+          }
+        }
+        const float mean = s / (float)D;
+        const float var = fmaxf(s2 / (float)D - mean * mean, 0.f);
+        const float inv = rsqrtf(var + P.ln_eps);
+        float* o = a.out + (i0 + row) * D;
+#pragma unroll 1
+        for (int cq = 0; cq < 4; ++cq) {
+          tmem_ld32(ta + cq * 32, v);
+          tmem_wait_ld();
+          if (row < rows) {
+#pragma unroll
+            for (int jj = 0; jj < 32; jj += 4) {
+              const int col = cq * 32 + jj;
+              if (col < D) {
+                float r4[4];
+#pragma unroll
+                for (int e = 0; e < 4; ++e)
+                  r4[e] = (fmaxf(v[jj + e] + s_v0[col + e], 0.f) - mean) * inv * s_v1[col + e] +
+                          s_v2[col + e];
+                *reinterpret_cast<float4*>(o + col) = make_float4(r4[0], r4[1], r4[2], r4[3]);
+              }
+            }
+          }
+        }
+      }
+      tc_fence_before();
+      warp_arrive(&B.tempty[ab]);
+    }
+  }
+  ws_teardown(tmem, 2 * kCols, kMmaWarp);
+}
 
 // ------------------------------------------------------------------ 2-SM pre-split K|V kernel
 // kv_pre2_kernel: kv_pre on a CTA pair (cluster of 2 on one TPC), one
@@ -3162,7 +3609,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
         const bool ovf = (ovf_bins >> (j / bdst)) & 1u;
         if (sg[j + 1] == sg[j] || ovf) {
           const float fill = ovf ? __int_as_float(0x7fc00000) : 0.f;
-          for (int c = lane; c < dm; c += 32) a.rbuf[(d0 + j) * kQLd + c] = fill;
+          fill_r_row(a, d0 + j, fill, lane, dm);
         }
       }
       R.live = 1;
@@ -3454,7 +3901,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
 namespace tca {
 
 struct PackedLayout {
-  size_t oq, okv, oo, okv64, okvc, okvp, okvp2, total;
+  size_t oq, okv, oo, okv64, okvc, okvp, okvp2, oqp, oop, obq, total;
 };
 
 static PackedLayout packed_layout(const tgl_attn_params* P) {
@@ -3470,6 +3917,9 @@ static PackedLayout packed_layout(const tgl_attn_params* P) {
   L.okvc = W.take((size_t)make_plan_contig(P->d_hsrc, P->d_e, P->d_t).n * kTWStage);
   L.okvp = W.take((size_t)make_pre_plan(P->d_hsrc, P->d_e, P->d_t).n * kTWStage);
   L.okvp2 = W.take((size_t)make_pre_plan(P->d_hsrc, P->d_e, P->d_t).n * 2 * kP2WStage);
+  L.oqp = W.take((size_t)make_dp_plan(P->d_hdst, 0).n * kDPWStage);
+  L.oop = W.take((size_t)make_dp_plan(P->d_model, P->d_hdst).n * kDPWStage);
+  L.obq = W.take(sizeof(float) * kDPN);
   L.total = W.off;
   return L;
 }
@@ -3499,7 +3949,17 @@ static tgl_status launch_pack(const tgl_attn_params* P, uint8_t* base, cudaStrea
   pack_kv_pre2_kernel<<<64, 256, 0, s>>>(P->Wk, P->Wv, P->d_model, P->d_hsrc + P->d_e + P->d_t,
                                          make_pre_plan(P->d_hsrc, P->d_e, P->d_t),
                                          base + L.okvp2);
-  return launch_check("pack_kv_pre2");
+  TGL_TRY(launch_check("pack_kv_pre2"));
+  // dense_pre: Q over h_dst only (Phi(0) folded into the bias), FFN over [r | h_dst]
+  pack_dense_pre_kernel<<<64, 256, 0, s>>>(P->Wq, P->d_model, P->d_hdst + P->d_t, 0, 0,
+                                           make_dp_plan(P->d_hdst, 0), base + L.oqp, P->bq,
+                                           P->phi, P->d_t, P->d_hdst,
+                                           reinterpret_cast<float*>(base + L.obq));
+  TGL_TRY(launch_check("pack_dense_pre q"));
+  pack_dense_pre_kernel<<<64, 256, 0, s>>>(P->Wo, P->d_out, P->d_model + P->d_hdst, 0,
+                                           P->d_model, make_dp_plan(P->d_model, P->d_hdst),
+                                           base + L.oop, nullptr, nullptr, 0, 0, nullptr);
+  return launch_check("pack_dense_pre ffn");
 }
 
 }  // namespace tca
@@ -3542,6 +4002,12 @@ static tgl_status set_smem_attrs(int smem_q, int smem_kv, int smem_kvb) {
     if (e == cudaSuccess)
       e = cudaFuncSetAttribute(kv_pre2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                kP2Smem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(dense_pre_kernel<false>,
+                               cudaFuncAttributeMaxDynamicSharedMemorySize, kDPSmem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(dense_pre_kernel<true>,
+                               cudaFuncAttributeMaxDynamicSharedMemorySize, kDPSmem);
     return e;
   }), "smem attributes");
 }
@@ -3600,6 +4066,7 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
   a.out = out;
   a.qbuf = reinterpret_cast<float*>(w + o_q);
   a.rbuf = reinterpret_cast<float*>(w + o_r);
+  a.rsplit = nullptr;
   a.wq = pk + PL.oq;
   a.wkv = pk + PL.okv;
   a.wo = pk + PL.oo;
@@ -3625,7 +4092,23 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
   TGL_TRY(set_smem_attrs(smem_q, smem_kv, smem_kvb));
   const int64_t tiles = ceil_div(n_dst_max, kBM);
   const unsigned gq = (unsigned)(tiles < kNumSMs ? tiles : kNumSMs);
-  launch_pdl(dense_kernel<false>, dim3(gq), dim3(kWsThreads), smem_q, s, a);
+  // split16 h_dst (and so split16 r, written by the K|V epilogue): converter-free Q / FFN
+  const bool dpre = (P->input_layout & TGL_SPLIT_HDST) != 0;
+  const DPPlan qplan = make_dp_plan(P->d_hdst, 0), oplan = make_dp_plan(P->d_model, P->d_hdst);
+  if (dpre) {
+    if (!(P->input_layout & (TGL_SPLIT_HSRC | TGL_SPLIT_E)) ||
+        !rows_16b(hdst, 1, ld_hdst) || ld_hdst < qplan.dp0 || P->d_model != 100 ||
+        qplan.n > kPMaxChunks || oplan.n > kPMaxChunks) {
+      set_error("TGL_SPLIT_HDST needs the pre-split K|V path (TGL_SPLIT_HSRC / _E), a 16-byte "
+                "aligned split16 h_dst table with ld >= round8(d_hdst)");
+      return TGL_EUNSUPPORTED;
+    }
+    a.rsplit = reinterpret_cast<uint8_t*>(a.rbuf);   // r scratch rows hold the split16 rows
+    launch_pdl(dense_pre_kernel<false>, dim3(gq), dim3(kDPThreads), kDPSmem, s, a, qplan,
+               pk + PL.oqp, reinterpret_cast<const float*>(pk + PL.obq));
+  } else {
+    launch_pdl(dense_kernel<false>, dim3(gq), dim3(kWsThreads), smem_q, s, a);
+  }
   TGL_TRY(launch_check("tc q kernel"));
   const int sel = P->kv_kernel;
   if (sel < TGL_KV_AUTO || sel > TGL_KV_PRE2 || sel == TGL_KV_SIMT) {
@@ -3674,7 +4157,11 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
     if (probe && probe->ev_stop)
       TGL_TRY(cuda_check(cudaEventRecord(static_cast<cudaEvent_t>(probe->ev_stop), s),
                          "probe event"));
-    launch_pdl(dense_kernel<true>, dim3(gq), dim3(kWsThreads), smem_q, s, a);
+    if (dpre)
+      launch_pdl(dense_pre_kernel<true>, dim3(gq), dim3(kDPThreads), kDPSmem, s, a, oplan,
+                 pk + PL.oop, nullptr);
+    else
+      launch_pdl(dense_kernel<true>, dim3(gq), dim3(kWsThreads), smem_q, s, a);
     return launch_check("tc ffn kernel");
   }
   const bool binned = max_seg > 0 && max_seg <= 32 && P->n_heads == 2;

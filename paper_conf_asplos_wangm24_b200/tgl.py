@@ -22,7 +22,7 @@ FP32, BF16, FP32_SIMT = 0, 1, 2
 # tgl_attn_params.kv_kernel (include/tgl.h TGL_KV_*)
 KV_KERNEL = {"auto": 0, "split": 1, "split_pad": 2, "async": 3, "bin": 4, "general": 5,
              "pre": 7, "pre2": 8}
-SPLIT_HSRC, SPLIT_E, SPLIT_TABLE = 1, 2, 4
+SPLIT_HSRC, SPLIT_E, SPLIT_TABLE, SPLIT_HDST = 1, 2, 4, 8
 KV_KERNEL_NAME = {1: "kv_split_kernel (contiguous K plan)", 2: "kv_split_kernel (padded K plan)",
                   3: "kv_async_kernel", 4: "kv_bin_kernel", 5: "kv_kernel (general)",
                   6: "kv_attn_kernel (SIMT)", 7: "kv_pre_kernel (pre-split operands)",

@@ -247,15 +247,19 @@ def test_attention_vs_oracle(T, monkeypatch, precision, kv, n_dst, kmax, d_h, d_
     put = cu_pad if kv in ("async", "split", "split_pad") else cu
     nf = put(nfeat)
     hs, efd = nf, (put(ef) if d_e else None)
-    tables = [(None, 0), (tab, 0)]
+    tables = [(None, 0, nf), (tab, 0, nf)]
     if kv in ("pre", "pre2"):  # split16 operand tables (tgl_split_rows), fp32 h_dst
         hs = T.split_rows(nf)
         efd = T.split_rows(efd) if d_e else None
         base = T.SPLIT_HSRC | (T.SPLIT_E if d_e else 0)
-        tables = [(None, base), (tab, base), (T.split_rows(tab), base | T.SPLIT_TABLE)]
-    for table, layout in tables:
+        ts = T.split_rows(tab)
+        tables = [(None, base, nf), (tab, base, nf), (ts, base | T.SPLIT_TABLE, nf),
+                  # split16 h_dst too: converter-free Q / FFN (dense_pre)
+                  (ts, base | T.SPLIT_TABLE | T.SPLIT_HDST, hs),
+                  (None, base | T.SPLIT_HDST, hs)]
+    for table, layout, hd in tables:
         P.struct.input_layout = layout
-        got = T.tblock_attn(P, cu(seg), cu(dst_t), nf, cu(dn), hs, cu(sn),
+        got = T.tblock_attn(P, cu(seg), cu(dst_t), hd, cu(dn), hs, cu(sn),
                             efd, cu(eid) if d_e else None, cu(et),
                             table=table, max_seg=int(np.diff(seg).max()))
         err = np.abs(np_(got)[:n_dst] - exp).max()
