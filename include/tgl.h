@@ -336,6 +336,19 @@ tgl_status tgl_tblock_attn_backward(
     void* stream);
 
 /* ---------------------------------------------------------------------------
+ * N4  preload(): feature tables that live in host memory (graphs whose
+ * features exceed HBM: GDELT's edge features are 142 GB) are read by the GPU
+ * directly from pinned memory, one block at a time: dst row j = src row idx[j]
+ * (row_bytes bytes, any layout: fp32 or split16) for j < n, n = n_dev[n_at ? *n_at : 0]
+ * (NULL n_dev -> n_max; n_at lets n be seg_ptr[U] of a block, both on the device).  src
+ * may be pinned host memory (cudaHostAlloc / cudaHostRegister; the pointer is valid on
+ * the device under UVA) or device memory; dst is device memory; idx NULL = identity.
+ * The TBlock chain then gathers from dst with identity indices.  Errors: EINVAL. */
+tgl_status tgl_preload_rows(int64_t n_max, const int64_t* n_dev, const int64_t* n_at,
+                            const int32_t* idx, const void* src, int64_t src_pitch,
+                            int64_t row_bytes, void* dst, int64_t dst_pitch, void* stream);
+
+/* ---------------------------------------------------------------------------
  * S14  Dedup inverse applied to rows (the hook of P:279 / TGOpt dedup_invert
  * P:179): out[j][:] = table[idx[j]][:] for j < n, n = *n_dev (NULL -> n_max).
  * ------------------------------------------------------------------------- */

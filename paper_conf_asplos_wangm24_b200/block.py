@@ -57,7 +57,7 @@ class TGATPipeline:
                  sampler: TSampler, use_dedup: bool, precompute: bool, window: int = 65536,
                  precision: str = "fp32", staging: bool = False, device=None,
                  cache_capacity: int = 0, shard: tuple | None = None,
-                 layout: str | None = None):
+                 layout: str | None = None, host_features: bool = False):
         """shard = (rank, world): root sharding (S16).  The batch's roots
         (deduped when use_dedup) are formed on every rank; this pipeline computes the
         contiguous slice `rank` of them (tgl_shard_slice) and forward(slot) returns the
@@ -69,7 +69,13 @@ class TGATPipeline:
         from split16 tables (tgl_split_rows: bf16 hi / lo halves, the kv_pre kernel) --
         graph["nfeat_split"] / graph["efeat_split"] when given, else split here once --
         and every inner layer output is split once for the layer above; "fp32" gathers
-        fp32 rows and converts in the SM (kv_split)."""
+        fp32 rows and converts in the SM (kv_split).
+
+        host_features: the operand tables live in pinned host memory (preload(), P:299-301;
+        graphs whose features exceed HBM): every block first copies the rows it gathers --
+        edge rows by eid, and for the tail block node rows by nbr / dst -- into device staging
+        tables with tgl_preload_rows (the GPU reads host memory directly), then runs on them
+        with identity indices.  Device tables passed in are moved to pinned host memory."""
         self.dev = device or torch.device("cuda")
         self.g = graph
         self.tcsr = tcsr
@@ -101,6 +107,17 @@ class TGATPipeline:
         k = sampler.k
         i32, f32, i64 = torch.int32, torch.float32, torch.int64
         z = lambda n, dt: torch.zeros(max(int(n), 1), dtype=dt, device=self.dev)
+        self.host = host_features
+        if host_features:        # N4: operand tables in pinned host memory
+            pin = lambda t: None if t is None else (t if (not t.is_cuda and t.is_pinned())
+                                                    else t.cpu().pin_memory())
+            if self.split:
+                self.nfeat_host, self.efeat_host = pin(self.nfeat_split), pin(self.efeat_split)
+                self.nfeat_split = self.efeat_split = None
+            else:
+                self.nfeat_host = pin(graph["nfeat"])
+                ef = graph.get("efeat")
+                self.efeat_host = pin(ef) if ef is not None and ef.numel() else None
         self.start_dev = torch.zeros(1, dtype=i64, device=self.dev)
         self.blocks = []
         n_max = 3 * batch
@@ -133,6 +150,17 @@ class TGATPipeline:
             self.blocks.append(b)
             n_max = n_max + n_max * k
         self.emb = z(3 * batch * self.attn[0].d_out, f32).view(-1, self.attn[0].d_out)
+        if self.host:            # device staging tables for the preloaded rows, per block
+            cap = max(b.n_max * k for b in self.blocks)
+            self.iota = torch.arange(max(cap, 1), dtype=i32, device=self.dev)
+            for b in self.blocks:
+                if self.efeat_host is not None:
+                    pe = self.efeat_host.shape[1]
+                    b.ws["epre"] = torch.zeros(max(b.n_max * k, 1), pe, dtype=f32, device=self.dev)
+            tail = self.blocks[-1]
+            pv = self.nfeat_host.shape[1]
+            tail.ws["nsrc"] = torch.zeros(max(tail.n_max * k, 1), pv, dtype=f32, device=self.dev)
+            tail.ws["ndst"] = torch.zeros(max(tail.n_max, 1), pv, dtype=f32, device=self.dev)
         if shard is not None:   # the head block writes the slice into send[slot]
             d0 = self.attn[0].d_out
             self.send = [z(self.c_max * d0, f32).view(-1, d0) for _ in range(2)]
@@ -153,6 +181,8 @@ class TGATPipeline:
                      for l in range(self.L)]
         self.launches_per_forward = 1 + sum(per_block) + (1 if use_dedup and shard is None
                                                           else 0)
+        if host_features:        # preload launches: edge rows per block, node rows (tail)
+            self.launches_per_forward += (self.L if self.efeat_host is not None else 0) + 2
         # cache() (TGOpt per-layer store, Listing 1 L23; inference): every
         # block's dst pairs after dedup are looked up in that layer's table; only the
         # misses are sampled and computed, then stored, and the combine hook rebuilds the
@@ -275,6 +305,21 @@ class TGATPipeline:
                 else:
                     hdst_idx = hsrc_idx = None
             ef = self.efeat_split if self.split else g["efeat"]
+            eid = b.eid
+            if self.host:        # N4 preload(): the block's rows from pinned host memory
+                ef = None
+                if self.efeat_host is not None:
+                    ef, eid = b.ws["epre"], self.iota
+                    tgl.preload_rows(b.eid, self.efeat_host, ef, n_max=b.n_max * k,
+                                     n_dev=b.seg_ptr, n_at=b.u_dev, stream=s)
+                if l == self.L - 1:
+                    hsrc, hdst = b.ws["nsrc"], b.ws["ndst"]
+                    tgl.preload_rows(b.nbr, self.nfeat_host, hsrc, n_max=b.n_max * k,
+                                     n_dev=b.seg_ptr, n_at=b.u_dev, stream=s)
+                    tgl.preload_rows(b.uniq_node, self.nfeat_host, hdst, n_max=b.n_max,
+                                     n_dev=b.u_dev, stream=s)
+                    hdst_idx = hsrc_idx = None
+                mark(f"preload{l}")
             ld_e = ef.stride(0) if (ef is not None and ef.dim() == 2 and ef.shape[1] > 0) else 0
             if record is not None:
                 ev = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
@@ -283,7 +328,7 @@ class TGATPipeline:
                      [tgl.C.byref(a.struct), b.n_max, tgl._p(b.u_dev), tgl._p(b.seg_ptr),
                       tgl._p(b.uniq_t), tgl._prow(hdst), tgl._p(hdst_idx), hdst.stride(0),
                       tgl._prow(hsrc), tgl._p(hsrc_idx), tgl._p(off), hsrc.stride(0),
-                      tgl._prow(ef) if ld_e else None, tgl._p(b.eid) if ld_e else None, ld_e,
+                      tgl._prow(ef) if ld_e else None, tgl._p(eid) if ld_e else None, ld_e,
                       tgl._p(b.ts), tgl._p(self.tables[l]),
                       0 if self.tables[l] is None else self.tables[l].shape[0], k,
                       tgl._p(b.out)], b.ws["attn"], s, "tgl_tblock_attn")

@@ -113,6 +113,35 @@ __global__ void scatter_add_rows_kernel(int64_t n_max, const int64_t* n_dev,
   }
 }
 
+// ---------------------------------------------------------------- N4 preload
+// dst row j = src row idx[j] (row_bytes bytes) for j < n; src may be pinned host memory
+// mapped into the device address space (the GPU reads it over the host link).  One warp
+// per row, 16-byte vectors when every pitch and the row size allow.
+__global__ void preload_rows_kernel(int64_t n_max, const int64_t* n_dev, const int64_t* n_at,
+                                    const int32_t* __restrict__ idx, const uint8_t* src,
+                                    int64_t src_pitch, int64_t row_bytes, uint8_t* dst,
+                                    int64_t dst_pitch, bool vec16) {
+  pdl_wait();
+  pdl_trigger();
+  int64_t n = n_max;
+  if (n_dev != nullptr) n = n_dev[n_at ? *n_at : 0];
+  n = n < n_max ? n : n_max;
+  const int lane = threadIdx.x & 31;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t j = blockIdx.x * (int64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); j < n; j += warps) {
+    const int64_t r = idx ? (int64_t)idx[j] : j;
+    const uint8_t* s = src + r * src_pitch;
+    uint8_t* d = dst + j * dst_pitch;
+    if (vec16) {
+      for (int64_t b = 16 * lane; b < row_bytes; b += 16 * 32)
+        *reinterpret_cast<uint4*>(d + b) = *reinterpret_cast<const uint4*>(s + b);
+    } else {
+      for (int64_t b = 4 * lane; b < row_bytes; b += 4 * 32)
+        *reinterpret_cast<uint32_t*>(d + b) = *reinterpret_cast<const uint32_t*>(s + b);
+    }
+  }
+}
+
 // ---------------------------------------------------------------- split16 rows
 // dst row r (pitch ld_dst 4-byte words): bf16 hi of columns [0, dp) then bf16 lo of the
 // same columns, dp = d rounded up to 8 (zero columns past d); hi = RNE(x),
@@ -219,6 +248,25 @@ tgl_status tgl_scatter_add_rows(int64_t n_max, const int64_t* n_dev, const int32
   launch_pdl(scatter_add_rows_kernel, dim3(grid_for(n_max * d, 256)), dim3(256), 0,
              as_stream(stream), n_max, n_dev, idx, src, ld_src, d, out, ld_out);
   return launch_check("scatter_add_rows");
+}
+
+tgl_status tgl_preload_rows(int64_t n_max, const int64_t* n_dev, const int64_t* n_at,
+                            const int32_t* idx, const void* src, int64_t src_pitch,
+                            int64_t row_bytes, void* dst, int64_t dst_pitch, void* stream) {
+  TGL_REQUIRE(n_max >= 0 && row_bytes >= 0 && src_pitch >= row_bytes && dst_pitch >= row_bytes,
+              "bad size");
+  TGL_REQUIRE(row_bytes % 4 == 0, "row_bytes must be a multiple of 4");
+  if (n_max == 0 || row_bytes == 0) return TGL_OK;
+  TGL_REQUIRE(src && dst, "null pointer");
+  const bool vec16 = row_bytes % 16 == 0 && src_pitch % 16 == 0 && dst_pitch % 16 == 0 &&
+                     (reinterpret_cast<uintptr_t>(src) & 15) == 0 &&
+                     (reinterpret_cast<uintptr_t>(dst) & 15) == 0;
+  int64_t g = ceil_div(n_max, 8);
+  if (g > (int64_t)kNumSMs * 16) g = (int64_t)kNumSMs * 16;
+  launch_pdl(preload_rows_kernel, dim3((unsigned)g), dim3(256), 0, as_stream(stream), n_max,
+             n_dev, n_at, idx, static_cast<const uint8_t*>(src), src_pitch, row_bytes,
+             static_cast<uint8_t*>(dst), dst_pitch, vec16);
+  return launch_check("preload_rows");
 }
 
 tgl_status tgl_split_rows(int64_t n_rows, int32_t d, const float* src, int64_t ld_src,

@@ -35,7 +35,8 @@ SYMBOLS = ["tgl_version", "tgl_status_string", "tgl_last_error", "tgl_build_tcsr
            "tgl_time_precompute", "tgl_time_encode", "tgl_tblock_attn", "tgl_gather_rows",
            "tgl_attn_packed_bytes", "tgl_attn_pack", "tgl_cache_lookup", "tgl_cache_store", "tgl_cache_combine",
            "tgl_cache_merge", "tgl_shard_slice", "tgl_shard_gather", "tgl_split_rows",
-           "tgl_tcsr_index", "tgl_tblock_attn_backward", "tgl_scatter_add_rows"]
+           "tgl_tcsr_index", "tgl_tblock_attn_backward", "tgl_scatter_add_rows",
+           "tgl_preload_rows"]
 
 
 class TGLError(RuntimeError):
@@ -74,6 +75,7 @@ def _load():
         "tgl_split_rows": [i64, i32, vp, i64, vp, i64, vp],
         "tgl_tcsr_index": [vp, vp, vp, vp],
         "tgl_scatter_add_rows": [i64, vp, vp, vp, i64, i32, vp, i64, vp],
+        "tgl_preload_rows": [i64, vp, vp, vp, vp, i64, i64, vp, i64, vp],
         "tgl_tblock_attn_backward": [vp, i64, vp, i64, vp, vp, vp, vp, i64, vp, vp, vp, i64, vp,
                                      vp, i64, vp, vp, i64, vp, vp, i64, vp, i64, vp, sz, vp],
     }
@@ -572,4 +574,20 @@ def scatter_add_rows(idx, src, out, n_dev=None, n_max=None, stream=None):
     _check(_lib.tgl_scatter_add_rows(n_max, _p(n_dev), _p(idx), _prow(src), src.stride(0),
                                      src.shape[1], _prow(out), out.stride(0), _s(stream)),
            "tgl_scatter_add_rows")
+    return out
+
+
+# --------------------------------------------------------------------------- N4 preload()
+def preload_rows(idx, src, out, n_max=None, n_dev=None, n_at=None, stream=None):
+    """out[j] = src[idx[j]] for j < n (n = n_dev[*n_at] or *n_dev, on the device); `src` may
+    be a pinned host tensor (read by the GPU over the host link).  Row tables are 2-D with
+    unit column stride; a row is src.shape[1] elements."""
+    assert src.stride(1) == 1 and out.stride(1) == 1
+    assert src.is_cuda or src.is_pinned(), "host tables must be pinned (page-locked)"
+    n_max = (idx.numel() if idx is not None else src.shape[0]) if n_max is None else n_max
+    es = src.element_size()
+    _check(_lib.tgl_preload_rows(n_max, _p(n_dev), _p(n_at), _p(idx), src.data_ptr(),
+                                 src.stride(0) * es, src.shape[1] * es, out.data_ptr(),
+                                 out.stride(0) * out.element_size(), _s(stream)),
+           "tgl_preload_rows")
     return out
