@@ -16,4 +16,5 @@ from .gen import (  # noqa: F401
     make_time_params,
     batch_roots_inputs,
     feature_rows,
+    make_gru_params,
 )

@@ -183,3 +183,15 @@ def model_params(cfg: Config, **kw) -> list:
         d_h = cfg.d_v if l == cfg.n_layers - 1 else cfg.d_model
         out.append(make_layer_params(cfg, l, d_h, d_h, **kw))
     return out
+
+
+def make_gru_params(cfg: Config, d_mem: int = 100, random_phi: bool = True) -> dict:
+    """TGN memory updater (N3): PyTorch-GRUCell-style U(+-1/sqrt(d_mem)) weights for input
+    [mail (2 d_mem + d_e) ; Phi (d_t)], plus the time encoder (Listing 4's GRUMemoryUpdater)."""
+    rng = np.random.default_rng(cfg.seeds["weights"] + 1000)
+    d_x = 2 * d_mem + cfg.d_e + cfg.d_t
+    bound = 1.0 / np.sqrt(d_mem)
+    u = lambda *s: rng.uniform(-bound, bound, s).astype(np.float32)
+    omega, phi = make_time_params(cfg, random_phi, seed=cfg.seeds["weights"] + 1001)
+    return dict(d_mem=d_mem, W_ih=u(3 * d_mem, d_x), W_hh=u(3 * d_mem, d_mem), b_ih=u(3 * d_mem),
+                b_hh=u(3 * d_mem), omega=omega, phi=phi)
