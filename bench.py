@@ -65,6 +65,9 @@ def parse():
                     choices=["auto", "pre", "pre2", "split", "split_pad", "async", "bin",
                              "general"])
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--host-features", action="store_true",
+                    help="N4: feature tables in pinned host memory, preload() per block "
+                         "(the paper's CPU-to-GPU case; configs whose tables fit host RAM)")
     return ap.parse_args()
 
 
@@ -214,6 +217,8 @@ def config_dict(cfg, args, world: int, flush: bool) -> dict:
                                LAYOUT.get(cfg.name, "split") == "fp32" else
                                "split16 (bf16 hi/lo tables, tgl_split_rows)"),
             "cache_slots_per_layer": args.cache,
+            "features": ("pinned host memory, preload() per block (CPU-to-GPU)"
+                         if getattr(args, "host_features", False) else "HBM-resident"),
             "parallelism": (f"root-sharded x{world} (each rank: slice of the batch's roots; "
                             f"NCCL all-gather of root embeddings)" if world > 1 else "single"),
             "l2": ("flushed (256 MiB write) between timed steps, outside per-step events"
@@ -513,7 +518,7 @@ def run_ours(args):
     layout = "fp32" if args.precision == "fp32_simt" else LAYOUT.get(cfg.name, "split")
     pipe = TGATPipeline(dev, tc, params, cfg.batch, sampler, cfg.dedup, cfg.precompute,
                         cfg.window, args.precision, cache_capacity=args.cache, shard=shard,
-                        layout=layout)
+                        layout=layout, host_features=args.host_features)
     for a in pipe.attn:
         a.set_kv_kernel(args.kv_kernel)
     pipe.capture()
@@ -721,7 +726,7 @@ def run_e2e(args, cfg, g, neg, params, dev, tc, sampler, batch_of, world, rank, 
     n0 = 3 * cfg.batch
     pipe_h = TGATPipeline(dev, tc, params, cfg.batch, sampler, cfg.dedup, cfg.precompute,
                           cfg.window, args.precision, staging=True, cache_capacity=args.cache,
-                          shard=shard, layout=layout)
+                          shard=shard, layout=layout, host_features=args.host_features)
     for a in pipe_h.attn:
         a.set_kv_kernel(args.kv_kernel)
     pipe_h.capture()

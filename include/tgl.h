@@ -349,6 +349,57 @@ tgl_status tgl_preload_rows(int64_t n_max, const int64_t* n_dev, const int64_t* 
                             int64_t row_bytes, void* dst, int64_t dst_pitch, void* stream);
 
 /* ---------------------------------------------------------------------------
+ * N3  TGN node memory (eqs 9-11, and the TGN case
+ * study, Listings 3-4).  Reading R25-R27.  The caller owns the
+ * state, all device fp32 row-major:
+ *   mem [n_nodes, d_mem] (s_v), mem_ts [n_nodes] (time of s_v's last update),
+ *   mail [n_nodes, d_mail] with d_mail = 2 d_mem + d_e (the one-slot mailbox: TGN keeps
+ *   only the latest message per node), mail_ts [n_nodes].
+ * ------------------------------------------------------------------------- */
+typedef struct {
+  int64_t n_nodes;
+  int32_t d_mem, d_e;
+  float* mem;
+  float* mem_ts;
+  float* mail;
+  float* mail_ts;
+} tgl_memory;
+
+/* GRU memory updater (eq 11; Listing 4 GRUMemoryUpdater): PyTorch GRUCell
+ * layout, gates (r, z, n) stacked along rows: W_ih [3 d_mem, d_mail + d_t], W_hh
+ * [3 d_mem, d_mem], b_ih / b_hh [3 d_mem]; the time encoder omega / phi [d_t]. */
+typedef struct {
+  int32_t d_t;
+  const float *W_ih, *W_hh, *b_ih, *b_hh, *omega, *phi;
+} tgl_gru_params;
+
+/* save_raw_msgs + mailbox.store (Listing 4 L20-25).  The batch: edges j < B = *B_dev
+ * (NULL -> B_max) with endpoints src[j], dst[j], time t[j] and edge id eid[j] (NULL ->
+ * eid0 + j: consecutive rows of the time-sorted edge list).  Edge j gives src[j] the
+ * message [mem[src] ; mem[dst] ; efeat[eid]] (position j) and dst[j] the message
+ * [mem[dst] ; mem[src] ; efeat[eid]] (position B + j) (eq 9).  coalesce(by='latest')
+ * (eq 10): per node, the message with the largest t, ties -> the larger position (R26);
+ * it is written to mail[node], its t to mail_ts[node].  Outputs (device, capacity
+ * 2 B_max): uniq[i] = the distinct nodes in order of first position, pick[i] = the
+ * position of the kept message, *n_uniq_dev = their count.  mem is only read.
+ * Workspace: a hash table of O(B_max) slots plus scan state.  Errors: EINVAL (nulls,
+ * d_e > 0 without efeat, node ids outside [0, n_nodes) are skipped, not errors). */
+tgl_status tgl_mailbox_store(const tgl_memory* M, int64_t B_max, const int64_t* B_dev,
+                             const int32_t* src, const int32_t* dst, const float* t,
+                             const int32_t* eid, int64_t eid0, const float* efeat,
+                             int64_t ld_e, int32_t* uniq, int64_t* pick, int64_t* n_uniq_dev,
+                             void* ws, size_t* ws_bytes, void* stream);
+
+/* update_memory (Listing 4 L11-17, eq 11) for the n = *n_dev (NULL -> n_max) nodes[i],
+ * which must be distinct (the dedup'ed nodes of a block): dt = fl(mail_ts[v] - mem_ts[v]),
+ * x = [mail[v] ; Phi(dt)] (R10), mem[v] = GRUCell(x, mem[v]), mem_ts[v] = mail_ts[v].
+ * fp32 GEMMs (exact products, fp32 sums).  Workspace: O(n_max (d_mail + d_t + 7 d_mem))
+ * floats.  Errors: EINVAL (nulls, d_mem < 1). */
+tgl_status tgl_memory_update(const tgl_memory* M, const tgl_gru_params* G, int64_t n_max,
+                             const int64_t* n_dev, const int32_t* nodes, void* ws,
+                             size_t* ws_bytes, void* stream);
+
+/* ---------------------------------------------------------------------------
  * S14  Dedup inverse applied to rows (the hook of P:279 / TGOpt dedup_invert
  * P:179): out[j][:] = table[idx[j]][:] for j < n, n = *n_dev (NULL -> n_max).
  * ------------------------------------------------------------------------- */

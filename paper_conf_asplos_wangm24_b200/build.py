@@ -16,7 +16,7 @@ LIB = os.path.join(PKG, "libtgl.so")
 OBJ = os.path.join(ROOT, "build", "obj")
 
 SOURCES = ["api.cu", "tcsr.cu", "sample.cu", "dedup.cu", "time_encode.cu", "attn.cu", "cache.cu",
-           "shard.cu", "attn_bwd.cu", "attn_tc.cu"]
+           "shard.cu", "attn_bwd.cu", "memory.cu", "attn_tc.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 # no --use_fast_math: the time encoder needs the accurate cosf (reading R10)

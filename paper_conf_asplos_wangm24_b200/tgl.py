@@ -36,7 +36,7 @@ SYMBOLS = ["tgl_version", "tgl_status_string", "tgl_last_error", "tgl_build_tcsr
            "tgl_attn_packed_bytes", "tgl_attn_pack", "tgl_cache_lookup", "tgl_cache_store", "tgl_cache_combine",
            "tgl_cache_merge", "tgl_shard_slice", "tgl_shard_gather", "tgl_split_rows",
            "tgl_tcsr_index", "tgl_tblock_attn_backward", "tgl_scatter_add_rows",
-           "tgl_preload_rows"]
+           "tgl_preload_rows", "tgl_mailbox_store", "tgl_memory_update"]
 
 
 class TGLError(RuntimeError):
@@ -76,6 +76,8 @@ def _load():
         "tgl_tcsr_index": [vp, vp, vp, vp],
         "tgl_scatter_add_rows": [i64, vp, vp, vp, i64, i32, vp, i64, vp],
         "tgl_preload_rows": [i64, vp, vp, vp, vp, i64, i64, vp, i64, vp],
+        "tgl_mailbox_store": [vp, i64, vp, vp, vp, vp, vp, i64, vp, i64, vp, vp, vp, vp, sz, vp],
+        "tgl_memory_update": [vp, vp, i64, vp, vp, vp, sz, vp],
         "tgl_tblock_attn_backward": [vp, i64, vp, i64, vp, vp, vp, vp, i64, vp, vp, vp, i64, vp,
                                      vp, i64, vp, vp, i64, vp, vp, i64, vp, i64, vp, sz, vp],
     }
@@ -591,3 +593,64 @@ def preload_rows(idx, src, out, n_max=None, n_dev=None, n_at=None, stream=None):
                                  out.stride(0) * out.element_size(), _s(stream)),
            "tgl_preload_rows")
     return out
+
+
+# --------------------------------------------------------------------------- N3 TGN memory
+class MemoryC(C.Structure):
+    _fields_ = [("n_nodes", C.c_int64), ("d_mem", C.c_int32), ("d_e", C.c_int32),
+                ("mem", C.c_void_p), ("mem_ts", C.c_void_p), ("mail", C.c_void_p),
+                ("mail_ts", C.c_void_p)]
+
+
+class GruParamsC(C.Structure):
+    _fields_ = [("d_t", C.c_int32)] + [(n, C.c_void_p) for n in ("W_ih", "W_hh", "b_ih", "b_hh",
+                                                                  "omega", "phi")]
+
+
+class TGNMemory:
+    """Node memory + one-slot mailbox of TGN (eqs 9-11, Listings 3-4), device fp32
+    state owned here: mem [N, d_mem], mem_ts [N], mail [N, 2 d_mem + d_e], mail_ts [N]
+    (all zero at start, as TGN's reset).  `params` = GRU + time-encoder weights
+    (W_ih, W_hh, b_ih, b_hh, omega, phi as arrays / tensors)."""
+
+    def __init__(self, n_nodes: int, d_mem: int, d_e: int, params: dict, device=None):
+        dev = device or torch.device("cuda")
+        f = lambda a: torch.as_tensor(a, dtype=torch.float32).to(dev).contiguous()
+        self.n_nodes, self.d_mem, self.d_e = n_nodes, d_mem, d_e
+        self.mem = torch.zeros(n_nodes, d_mem, device=dev)
+        self.mem_ts = torch.zeros(n_nodes, device=dev)
+        self.mail = torch.zeros(n_nodes, 2 * d_mem + d_e, device=dev)
+        self.mail_ts = torch.zeros(n_nodes, device=dev)
+        self.p = {k: f(params[k]) for k in ("W_ih", "W_hh", "b_ih", "b_hh", "omega", "phi")}
+        assert self.p["W_ih"].shape[1] == 2 * d_mem + d_e + self.p["omega"].numel()
+        self.struct = MemoryC(n_nodes, d_mem, d_e, self.mem.data_ptr(), self.mem_ts.data_ptr(),
+                              self.mail.data_ptr(), self.mail_ts.data_ptr())
+        self.gru = GruParamsC(self.p["omega"].numel(), *[self.p[k].data_ptr() for k in
+                                                         ("W_ih", "W_hh", "b_ih", "b_hh",
+                                                          "omega", "phi")])
+        self.ws = Workspace(dev)
+
+    def store(self, src, dst, t, efeat=None, eid=None, eid0: int = 0, B_dev=None, B_max=None,
+              out=None, stream=None):
+        """save_raw_msgs (Listing 4 L20-25): coalesce the batch's messages by latest and
+        store them.  Returns (uniq [2B], pick [2B], n_uniq_dev [1])."""
+        B_max = src.numel() if B_max is None else B_max
+        dev = self.mem.device
+        if out is None:
+            out = (torch.empty(max(2 * B_max, 1), dtype=torch.int32, device=dev),
+                   torch.empty(max(2 * B_max, 1), dtype=torch.int64, device=dev),
+                   torch.empty(1, dtype=torch.int64, device=dev))
+        uniq, pick, n_u = out
+        ld_e = efeat.stride(0) if (efeat is not None and self.d_e) else 0
+        _ws_call(_lib.tgl_mailbox_store,
+                 [C.byref(self.struct), B_max, _p(B_dev), _p(src), _p(dst), _p(t), _p(eid), eid0,
+                  _prow(efeat) if ld_e else None, ld_e, _p(uniq), _p(pick), _p(n_u)], self.ws,
+                 _s(stream), "tgl_mailbox_store")
+        return uniq, pick, n_u
+
+    def update(self, nodes, n_dev=None, n_max=None, stream=None):
+        """update_memory (Listing 4 L11-17, eq 11) for distinct nodes."""
+        n_max = nodes.numel() if n_max is None else n_max
+        _ws_call(_lib.tgl_memory_update,
+                 [C.byref(self.struct), C.byref(self.gru), n_max, _p(n_dev), _p(nodes)], self.ws,
+                 _s(stream), "tgl_memory_update")
