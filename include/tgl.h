@@ -104,6 +104,18 @@ typedef struct {
  * tgl_sample; results are bit-identical with or without them. */
 tgl_status tgl_tcsr_index(const tgl_tcsr* g, float* ts_coarse, void* entries, void* stream);
 
+/* tgl_build_tcsr that also writes the sampler indexes above (ts_coarse / entries, either
+ * may be NULL) in the same sweep: the arrays equal tgl_build_tcsr + tgl_tcsr_index bit for
+ * bit.  For M < 2^30 entries the build moves each entry as one 16-byte record through a
+ * stable LSD digit sort (one kernel per 8-bit digit of the owner, plus four of t without
+ * TGL_INPUT_TIME_SORTED), so no output is gathered afterwards; larger graphs take the
+ * index-sort path and then tgl_tcsr_index.  Same arguments, errors and workspace protocol
+ * as tgl_build_tcsr (the workspace holds the records: 16 B per entry for <= 2 passes). */
+tgl_status tgl_build_tcsr_ex(int64_t num_nodes, int64_t num_edges, const int32_t* src,
+                             const int32_t* dst, const float* t, uint32_t flags, int64_t* indptr,
+                             int32_t* nbr, int32_t* eid, float* ts, float* ts_coarse,
+                             void* entries, void* ws, size_t* ws_bytes, void* stream);
+
 /* ---------------------------------------------------------------------------
  * S2  Roots of a batch (head TBlock).  P:235 (L2.8) `head = batch.block(ctx)`;
  * roots are the batch's source and destination nodes plus one negative

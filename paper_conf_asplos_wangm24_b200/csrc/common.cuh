@@ -141,17 +141,20 @@ __device__ __forceinline__ T warp_inclusive_scan(T v, int lane) {
 // Decoupled look-back (Merrill & Garland) tile status: one 64-bit word per tile,
 // flag in bits 62-63 (0 = not published, 1 = aggregate, 2 = inclusive prefix),
 // value in bits 0-61.  Tiles take ids from an atomic ticket so a tile only ever
-// waits on tiles that have already started.
+// waits on tiles that have already started.  Status words are read and written with
+// relaxed gpu-scope accesses: a tile consumes only the status words themselves (no data
+// published alongside them), and acquire loads would invalidate L1 on every poll
+// (CCTL.IVALL in SASS -- the top stall of the T-CSR scatter before this).
 constexpr unsigned long long kFlagAgg = 1ull << 62;
 constexpr unsigned long long kFlagPrefix = 2ull << 62;
 constexpr unsigned long long kValMask = (1ull << 62) - 1;
 
 __device__ __forceinline__ void st_status(unsigned long long* p, unsigned long long v) {
-  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 __device__ __forceinline__ unsigned long long ld_status(const unsigned long long* p) {
   unsigned long long v;
-  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
 }
 

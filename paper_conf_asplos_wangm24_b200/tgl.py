@@ -36,7 +36,7 @@ SYMBOLS = ["tgl_version", "tgl_status_string", "tgl_last_error", "tgl_build_tcsr
            "tgl_attn_packed_bytes", "tgl_attn_pack", "tgl_cache_lookup", "tgl_cache_store", "tgl_cache_combine",
            "tgl_cache_merge", "tgl_shard_slice", "tgl_shard_gather", "tgl_split_rows",
            "tgl_tcsr_index", "tgl_tblock_attn_backward", "tgl_scatter_add_rows",
-           "tgl_preload_rows", "tgl_mailbox_store", "tgl_memory_update"]
+           "tgl_preload_rows", "tgl_mailbox_store", "tgl_memory_update", "tgl_build_tcsr_ex"]
 
 
 class TGLError(RuntimeError):
@@ -56,6 +56,7 @@ def _load():
     lib.tgl_last_error.restype = C.c_char_p
     sig = {
         "tgl_build_tcsr": [i64, i64, vp, vp, vp, u32, vp, vp, vp, vp, vp, sz, vp],
+        "tgl_build_tcsr_ex": [i64, i64, vp, vp, vp, u32, vp, vp, vp, vp, vp, vp, vp, sz, vp],
         "tgl_batch_roots": [i64, i64, vp, vp, vp, vp, vp, vp, vp, vp, vp],
         "tgl_dedup": [i64, vp, vp, vp, vp, vp, vp, vp, vp, sz, vp],
         "tgl_sample": [vp, i64, vp, vp, vp, i32, i32, u64, u32, vp, vp, vp, vp, vp, sz, vp],
@@ -172,14 +173,17 @@ class TemporalCSR:
     """Device-resident T-CSR + the host struct the ABI takes."""
 
     def __init__(self, indptr, nbr, eid, ts, coarse: bool = True, packed: bool = True,
-                 stream=None):
+                 stream=None, ts_coarse=None, entries=None):
         """coarse / packed: build the sampler's fence index (M/32 floats) and the packed
-        16-byte entry records (16 B per entry) with tgl_tcsr_index."""
+        16-byte entry records (16 B per entry) with tgl_tcsr_index, unless they are passed
+        in already built (ts_coarse / entries, as tgl_build_tcsr_ex writes them)."""
         self.indptr, self.nbr, self.eid, self.ts = indptr, nbr, eid, ts
         M = nbr.numel()
-        self.ts_coarse = self.entries = None
-        self.struct = TCSR(indptr.numel() - 1, M, _p(indptr), _p(nbr), _p(eid), _p(ts), None,
-                           None)
+        self.ts_coarse, self.entries = ts_coarse, entries
+        self.struct = TCSR(indptr.numel() - 1, M, _p(indptr), _p(nbr), _p(eid), _p(ts),
+                           _p(ts_coarse), _p(entries))
+        if ts_coarse is not None or entries is not None:
+            return
         if M > 0 and (coarse or packed):
             if coarse:
                 self.ts_coarse = torch.empty((M + 31) // 32, dtype=torch.float32,
@@ -207,9 +211,14 @@ def build_tcsr(num_nodes: int, src, dst, t, undirected=True, time_sorted=False,
     eid = torch.empty(max(M, 1), dtype=torch.int32, device=dev)[:M]
     ts = torch.empty(max(M, 1), dtype=torch.float32, device=dev)[:M]
     flags = (TGL_UNDIRECTED if undirected else 0) | (TGL_INPUT_TIME_SORTED if time_sorted else 0)
-    _ws_call(_lib.tgl_build_tcsr, [num_nodes, E, _p(src), _p(dst), _p(t), flags, _p(indptr),
-                                   _p(nbr), _p(eid), _p(ts)], ws, _s(stream), "tgl_build_tcsr")
-    return TemporalCSR(indptr, nbr, eid, ts, coarse=coarse, packed=packed, stream=stream)
+    # the sampler indexes are written by the same sweep (tgl_build_tcsr_ex)
+    tsc = torch.empty((M + 31) // 32, dtype=torch.float32, device=dev) if coarse and M else None
+    ent = torch.empty(M, 4, dtype=torch.int32, device=dev) if packed and M else None
+    _ws_call(_lib.tgl_build_tcsr_ex, [num_nodes, E, _p(src), _p(dst), _p(t), flags, _p(indptr),
+                                      _p(nbr), _p(eid), _p(ts), _p(tsc), _p(ent)], ws,
+             _s(stream), "tgl_build_tcsr_ex")
+    return TemporalCSR(indptr, nbr, eid, ts, coarse=False, packed=False, stream=stream,
+                       ts_coarse=tsc, entries=ent)
 
 
 # --------------------------------------------------------------------------- S2

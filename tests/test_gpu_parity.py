@@ -57,6 +57,26 @@ def test_tcsr_bit_exact(T, N, E, max_t, undirected, sort):
         assert np.array_equal(a, b)
 
 
+@pytest.mark.parametrize("N,E,max_t,sort", [(20000, 300000, 50, True), (45000, 250000, 10**7, False),
+                                            (256, 70000, 3, True), (257, 70000, 3, True)])
+def test_tcsr_ex_indexes_and_tiles(T, N, E, max_t, sort):
+    """tgl_build_tcsr_ex (one sweep of 16-byte records, indexes written by the last pass)
+    over many 4,096-entry tiles with heavy time ties: T-CSR bit-exact against the oracle,
+    ts_coarse / entries bit-exact against tgl_tcsr_index run on the result, and the
+    one-pass (N <= 256) / two-pass, degree / owner-key indptr variants."""
+    import torch
+    rng = np.random.default_rng(N + E)
+    src, dst, t = rand_graph(rng, N, E, max_t, sort)
+    g = T.build_tcsr(N, cu(src), cu(dst), cu(t), True, sort)
+    exp = oracle.build_tcsr(N, src, dst, t, True)
+    for a, b in zip((g.indptr, g.nbr, g.eid, g.ts), exp):
+        assert np.array_equal(np_(a), b)
+    ref = T.TemporalCSR(g.indptr, g.nbr, g.eid, g.ts, coarse=True, packed=True)
+    torch.cuda.synchronize()
+    assert np.array_equal(np_(g.ts_coarse).view(np.uint32), np_(ref.ts_coarse).view(np.uint32))
+    assert np.array_equal(np_(g.entries), np_(ref.entries))
+
+
 @pytest.mark.parametrize("name", ["WIKI", "REDDIT", "LASTFM"])
 def test_tcsr_full_configs(T, name):
     cfg = synth.get_config(name)
