@@ -64,6 +64,8 @@ def parse():
     ap.add_argument("--kv-kernel", default="auto",
                     choices=["auto", "pre", "pre2", "split", "split_pad", "async", "bin",
                              "general"])
+    ap.add_argument("--node-proj", default="auto", choices=["auto", "on", "off"],
+                    help="the tail block's h projections per node (tgl_node_proj, DESIGN §7)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--host-features", action="store_true",
                     help="N4: feature tables in pinned host memory, preload() per block "
@@ -217,6 +219,7 @@ def config_dict(cfg, args, world: int, flush: bool) -> dict:
                                LAYOUT.get(cfg.name, "split") == "fp32" else
                                "split16 (bf16 hi/lo tables, tgl_split_rows)"),
             "cache_slots_per_layer": args.cache,
+            "node_proj": getattr(args, "node_proj", "auto"),
             "features": ("pinned host memory, preload() per block (CPU-to-GPU)"
                          if getattr(args, "host_features", False) else "HBM-resident"),
             "parallelism": (f"root-sharded x{world} (each rank: slice of the batch's roots; "
@@ -420,14 +423,25 @@ def run_reference(args):
 
 
 # ---------------------------------------------------------------------- our arm
-def algorithmic_kv(cfg, n_dst: float, n_edges: float, d_hsrc: int):
+NODE_PROJ = {"auto": None, "on": True, "off": False}
+
+
+def algorithmic_kv(cfg, n_dst: float, n_edges: float, d_hsrc: int, node_proj: bool = False):
     """Per launch of the K|V attention kernel (S6, S7, S9-S12):
     FLOPs = E * (2 * 2*d_model * K) for [K;V] = W [h ; e ; Phi] (K = d_hs + d_e + d_t)
             + E * 4 * d_model for the logits and the alpha-weighted sum;
     bytes = E * (4 (d_hs + d_e) + 12)  (gathered rows + nbr/eid/ts; Phi computed or
             table-read, counted 0 as in SURVEY §8(d))
-            + n_dst * (8 + 4 + 4 (d_model + 2) + 4 d_model)  (seg_ptr, t, q row, r row)."""
+            + n_dst * (8 + 4 + 4 (d_model + 2) + 4 d_model)  (seg_ptr, t, q row, r row).
+    node_proj (the tail block on tgl_node_proj's Z): the h_src part of [K;V] is one
+    gathered Z row of 2*d_model floats per edge instead of d_hs features and its MMA, so
+    FLOPs = E * (2 * 2*d_model * (d_e + d_t) + 2*d_model + 4*d_model),
+    bytes = E * (4 * (2*d_model + d_e) + 12) + the same per-destination bytes."""
     dm = cfg.d_model
+    if node_proj:
+        flops = n_edges * (2 * 2 * dm * (cfg.d_e + cfg.d_t) + 2 * dm + 4 * dm)
+        bytes_ = n_edges * (4 * (2 * dm + cfg.d_e) + 12) + n_dst * (12 + 4 * (dm + 2) + 4 * dm)
+        return flops, bytes_
     k = d_hsrc + cfg.d_e + cfg.d_t
     flops = n_edges * (2 * 2 * dm * k + 4 * dm)
     bytes_ = n_edges * (4 * (d_hsrc + cfg.d_e) + 12) + n_dst * (12 + 4 * (dm + 2) + 4 * dm)
@@ -518,7 +532,8 @@ def run_ours(args):
     layout = "fp32" if args.precision == "fp32_simt" else LAYOUT.get(cfg.name, "split")
     pipe = TGATPipeline(dev, tc, params, cfg.batch, sampler, cfg.dedup, cfg.precompute,
                         cfg.window, args.precision, cache_capacity=args.cache, shard=shard,
-                        layout=layout, host_features=args.host_features)
+                        layout=layout, host_features=args.host_features,
+                        node_proj=NODE_PROJ[args.node_proj])
     for a in pipe.attn:
         a.set_kv_kernel(args.kv_kernel)
     pipe.capture()
@@ -640,7 +655,7 @@ def run_ours(args):
     U_avg = sum(u for u, _ in shapes) / len(shapes)
     E_avg = sum(e for _, e in shapes) / len(shapes)
     kv_avg = sum(kv_ms) / len(kv_ms)
-    kv_fl, kv_by = algorithmic_kv(cfg, U_avg, E_avg, cfg.d_v)
+    kv_fl, kv_by = algorithmic_kv(cfg, U_avg, E_avg, cfg.d_v, pipe.node_proj)
     peaks = {}
     try:
         peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -652,9 +667,11 @@ def run_ours(args):
     passes = {"fp32": 3, "bf16": 1, "fp32_simt": 0}[args.precision]
     kv_tf = kv_fl / (kv_avg / 1e3) / 1e12
     kv_gbs = kv_by / (kv_avg / 1e3) / 1e9
-    tr = ncu_traffic(cfg.name, args.precision)
+    tr = ncu_traffic(cfg.name, args.precision + ("_node_proj" if pipe.node_proj else ""))
     roofline = {"kernel": f"{tgl.KV_KERNEL_NAME.get(min(kinds), '?')}: K|V attention of the "
-                          f"tail block (S6, S7, S9-S12)",
+                          f"tail block (S6, S7, S9-S12)" +
+                          (" on node projections (h_src part = gathered Z rows)"
+                           if pipe.node_proj else ""),
                 "bound": "hbm", "achieved": kv_gbs, "peak": hbm_peak, "unit": "GB/s",
                 "frac": kv_gbs / hbm_peak,
                 "traffic": tr["dram_bytes_per_launch"] if tr else None,
@@ -726,7 +743,8 @@ def run_e2e(args, cfg, g, neg, params, dev, tc, sampler, batch_of, world, rank, 
     n0 = 3 * cfg.batch
     pipe_h = TGATPipeline(dev, tc, params, cfg.batch, sampler, cfg.dedup, cfg.precompute,
                           cfg.window, args.precision, staging=True, cache_capacity=args.cache,
-                          shard=shard, layout=layout, host_features=args.host_features)
+                          shard=shard, layout=layout, host_features=args.host_features,
+                          node_proj=NODE_PROJ[args.node_proj])
     for a in pipe_h.attn:
         a.set_kv_kernel(args.kv_kernel)
     pipe_h.capture()

@@ -253,6 +253,21 @@ tgl_status tgl_time_encode(int64_t n, const float* dt, int32_t d_t, const float*
 #define TGL_SPLIT_HDST 8    /* hdst is split16 too: the Q / FFN projections gather converter-
                                free operands (Phi(0) folded into the Q bias); needs the
                                pre-split K|V path and d_model == 100 */
+#define TGL_NODE_PROJ 16    /* node projections: P->node_proj holds tgl_node_proj's Z for the
+                               node table that h_src and h_dst both index (the tail block of
+                               a chain, whose inputs are node features); hsrc_idx / hdst_idx
+                               index Z rows, hsrc / hdst are not read.  Needs d_hsrc ==
+                               d_hdst, split16 e (TGL_SPLIT_E), kv_kernel AUTO / PRE */
+
+/* Layout of the node-projection table Z [n_nodes][TGL_NODE_PROJ_LD] fp32 (tgl_node_proj):
+ * columns [K, K+d_model) = Wk[:, :d_h] h_v, [V, V+d_model) = Wv[:, :d_h] h_v,
+ * [Q, Q+d_model) = Wq [h_v ; Phi(0)] + bq and Q+d_model+hd = q^hd . bk^hd (per head),
+ * [O, O+d_model) = Wo[:, d_model:] h_v. */
+#define TGL_NODE_PROJ_LD 512
+#define TGL_NODE_PROJ_K 0
+#define TGL_NODE_PROJ_V 100
+#define TGL_NODE_PROJ_Q 256
+#define TGL_NODE_PROJ_O 384
 
 /* Measurement record (bench.py): when tgl_attn_params.probe != NULL the call records
  * ev_start / ev_stop (cudaEvent_t, created by the caller) on its stream immediately
@@ -282,7 +297,8 @@ typedef struct {
   tgl_kv_probe* probe;            /* optional (NULL): caller-owned measurement record */
   int32_t input_layout;           /* TGL_SPLIT_* bits: hsrc / efeat / tenc_table are
                                      split16 tables (tensor-core precisions, max_seg <= 32,
-                                     2 heads) */
+                                     2 heads); TGL_NODE_PROJ */
+  const float* node_proj;         /* TGL_NODE_PROJ: Z of tgl_node_proj (else unused) */
 } tgl_attn_params;
 
 /* Weight layout transform for the tensor-core path, done once per layer (the
@@ -293,6 +309,19 @@ typedef struct {
  * tensor-core path does not take. */
 size_t tgl_attn_packed_bytes(const tgl_attn_params* P);
 tgl_status tgl_attn_pack(const tgl_attn_params* P, void* packed, size_t bytes, void* stream);
+
+/* Node projections (the TBlock layer of eqs 4, 5, 7 is linear in h before the logits:
+ * q_i = Wq [h_i ; Phi(0)] + bq, k_e = Wk [h_src ; e ; Phi] + bk = Wk[:, :d_h] h_src + ...,
+ * FFN input Wo [r ; h_i] = Wo[:, :d_model] r + Wo[:, d_model:] h_i).  When h_src and h_dst
+ * are rows of one node table with far fewer rows than the block gathers (the tail block:
+ * GDELT 16,682 nodes vs 1.32M sampled edges per batch), the h terms are computed once per
+ * node and gathered, so the per-edge MMAs cover [e | Phi] only.  Writes Z (layout above)
+ * for rows v < n_nodes of hnode (split16, tgl_split_rows; ld >= round_up(d_hsrc, 8) words,
+ * 16-byte aligned).  Same precision modes as tgl_tblock_attn (3-pass fp32 / bf16); Z is
+ * fp32.  Needs P->packed (tgl_attn_pack), d_hsrc == d_hdst, 2 heads.  Z is owned by the
+ * caller, valid until the weights change.  Errors: EINVAL, EUNSUPPORTED. */
+tgl_status tgl_node_proj(const tgl_attn_params* P, int64_t n_nodes, const void* hnode,
+                         int64_t ld, float* Z, void* stream);
 
 tgl_status tgl_tblock_attn(const tgl_attn_params* P, int64_t n_dst_max, const int64_t* n_dst_dev,
                            const int64_t* seg_ptr, const float* dst_t, const float* hdst,

@@ -57,7 +57,8 @@ class TGATPipeline:
                  sampler: TSampler, use_dedup: bool, precompute: bool, window: int = 65536,
                  precision: str = "fp32", staging: bool = False, device=None,
                  cache_capacity: int = 0, shard: tuple | None = None,
-                 layout: str | None = None, host_features: bool = False):
+                 layout: str | None = None, host_features: bool = False,
+                 node_proj: bool | None = None):
         """shard = (rank, world): root sharding (S16).  The batch's roots
         (deduped when use_dedup) are formed on every rank; this pipeline computes the
         contiguous slice `rank` of them (tgl_shard_slice) and forward(slot) returns the
@@ -75,7 +76,13 @@ class TGATPipeline:
         graphs whose features exceed HBM): every block first copies the rows it gathers --
         edge rows by eid, and for the tail block node rows by nbr / dst -- into device staging
         tables with tgl_preload_rows (the GPU reads host memory directly), then runs on them
-        with identity indices.  Device tables passed in are moved to pinned host memory."""
+        with identity indices.  Device tables passed in are moved to pinned host memory.
+
+        node_proj: the tail block's projections of h (eqs 4, 5, 7 are linear in h) are
+        computed once per node per forward (tgl_node_proj into Z [n_nodes, 512]) and
+        gathered, so the tail's per-edge MMAs cover [e | Phi] only and it has no Q launch.
+        None (default) = on when the node table is split16 and device-resident and has
+        fewer rows than the tail block gathers per batch (and Z fits 2 GB)."""
         self.dev = device or torch.device("cuda")
         self.g = graph
         self.tcsr = tcsr
@@ -150,6 +157,21 @@ class TGATPipeline:
             self.blocks.append(b)
             n_max = n_max + n_max * k
         self.emb = z(3 * batch * self.attn[0].d_out, f32).view(-1, self.attn[0].d_out)
+        # node projections for the tail block (its h_src / h_dst are node-feature rows)
+        n_nodes = graph["nfeat"].shape[0] if graph.get("nfeat") is not None else 0
+        tail = self.blocks[-1]
+        np_ok = (self.split and precision in ("fp32", "bf16") and not host_features and
+                 n_nodes > 0 and self.attn[-1].host["n_heads"] == 2)
+        if node_proj is None:
+            node_proj = np_ok and n_nodes <= tail.n_max * k and n_nodes * 2048 <= (2 << 30)
+        assert not node_proj or np_ok, "node_proj needs the split16 device-resident tables"
+        self.node_proj = bool(node_proj)
+        self.zproj = None
+        if self.node_proj:
+            self.zproj = torch.empty(n_nodes, tgl.NODE_PROJ_LD, dtype=f32, device=self.dev)
+            at = self.attn[-1]
+            at.struct.input_layout |= tgl.NODE_PROJ
+            at.struct.node_proj = tgl._p(self.zproj)
         if self.host:            # device staging tables for the preloaded rows, per block
             cap = max(b.n_max * k for b in self.blocks)
             self.iota = torch.arange(max(cap, 1), dtype=i32, device=self.dev)
@@ -175,8 +197,8 @@ class TGATPipeline:
         dedup_launches = [(1 if b.n_max <= 4096 else 3) if use_dedup else 0 for b in self.blocks]
         if shard is not None:   # roots' dedup (before the slice) replaces block 0's + slice
             dedup_launches[0] = ((1 if 3 * batch <= 4096 else 3) if use_dedup else 0) + 1
-        # per block: next_block, dedup, sample (count + scan + pick), Q + K|V + FFN, split
-        per_block = [(1 if l > 0 else 0) + dedup_launches[l] + 3 + 3 + (1 if self.split and l > 0
+        # per block: next_block, dedup, sample (count + pick), Q + K|V + FFN, split
+        per_block = [(1 if l > 0 else 0) + dedup_launches[l] + 2 + 3 + (1 if self.split and l > 0
                                                                          else 0)
                      for l in range(self.L)]
         self.launches_per_forward = 1 + sum(per_block) + (1 if use_dedup and shard is None
@@ -294,6 +316,10 @@ class TGATPipeline:
                 hdst, hdst_idx, hsrc, hsrc_idx, off = g["nfeat"], b.uniq_node, g["nfeat"], b.nbr, None
                 if self.split:
                     hdst = hsrc = self.nfeat_split
+                if self.node_proj:   # Z rows for every node, then the tail indexes them
+                    tgl.node_proj(a, self.nfeat_split, n_nodes=self.zproj.shape[0],
+                                  out=self.zproj, stream=s)
+                    mark("node_proj")
             else:
                 nx = self.blocks[l + 1]
                 hdst = hsrc = nx.ws["cache"]["comb"] if self.cache_on else nx.out

@@ -130,6 +130,14 @@ struct Args {
   int np_q, np_kv, np_o;
   int dpb;
   int split;           // 1 = 3-pass fp32 mode
+  // node projections (TGL_NODE_PROJ, tgl_node_proj): per-node rows of Z [n_nodes][z_ld]
+  // = [h Wk_h^T | h Wv_h^T | pad | q (+ q.b_k) | h Wo_h^T]; the K|V accumulator starts
+  // from zkv[row], the FFN adds zo[row]; the epilogue reads q row q_idx[d] (stride q_ld)
+  const float* zkv;
+  const float* zo;
+  int64_t z_ld;
+  const int32_t* q_idx;
+  int64_t q_ld;
   int dbg;             // TGL_DEBUG_MASK (profiling only): 1 skip epilogue math, 2 skip gathers, 4 skip MMAs
 };
 
@@ -1050,7 +1058,8 @@ __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uin
     const int hi = __ffs(emask & (0xffffffffu << lane));              // last end >= lane, +1
     // this row's q (head columns) and q . bk, fetched before waiting for the accumulator
     // (kLowReg: read piecewise after the wait instead -- 64-register budget)
-    const float* qrow = a.qbuf + (int64_t)(valid ? d : 0) * kQLd;
+    const int64_t qr = valid ? (a.q_idx ? (int64_t)a.q_idx[d] : (int64_t)d) : 0;
+    const float* qrow = a.qbuf + qr * a.q_ld;
     float qv[kLowReg ? 1 : dh];
     if (!kLowReg) {
 #pragma unroll
@@ -2556,8 +2565,10 @@ static PrePlan make_pre_plan(int d0, int d1, int dt) {
   return p;
 }
 
+// col_off: the W column of K' column 0 (d_hsrc for the node-projection plan, whose K'
+// starts at the e columns)
 __global__ void pack_kv_pre_kernel(const float* Wk, const float* Wv, int dm, int ksrc, PrePlan p,
-                                   uint8_t* out) {
+                                   uint8_t* out, int col_off) {
   const int kw = p.n * kTC;
   const int64_t total = (int64_t)kNPkv * kw;
   for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
@@ -2573,6 +2584,7 @@ __global__ void pack_kv_pre_kernel(const float* Wk, const float* Wv, int dm, int
       if (kp - p.dp0 - p.dp1 < p.dt) src = p.d0 + p.d1 + (kp - p.dp0 - p.dp1);
     }
     float v = 0.f;
+    if (src >= 0) src += col_off;
     if (n < 2 * dm && src >= 0)
       v = n < dm ? Wk[(int64_t)n * ksrc + src] : Wv[(int64_t)(n - dm) * ksrc + src];
     const __nv_bfloat16 hi = __float2bfloat16_rn(v);
@@ -2598,6 +2610,7 @@ struct PBars {
   uint64_t wfull[kPW], wempty[kPW];
   uint64_t dfull[kSDSlots], dempty[kSDSlots];
   uint64_t tfull[2], tempty[2];
+  uint64_t zfull[2];    // node projections: the accumulator holds zkv[row] (loaders)
 };
 
 __global__ void __launch_bounds__(kPThreads, 1)
@@ -2617,6 +2630,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
   constexpr int dm = 100;
   const tgl_attn_params& P = a.P;
   const bool split = a.split != 0;
+  const bool np = a.zkv != nullptr;   // TGL_NODE_PROJ: h_src columns come from zkv rows
   const int nch = plan.n;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   // prologue independent of the predecessor grid (PDL): barriers, TMEM, constants
@@ -2636,6 +2650,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
     for (int s = 0; s < 2; ++s) {
       mbar_init(&B.tfull[s], 1);
       mbar_init(&B.tempty[s], kBEpi);
+      mbar_init(&B.zfull[s], kPLoadWarps);
     }
     fence_mbar_init();
   }
@@ -2792,8 +2807,38 @@ __global__ void __launch_bounds__(kPThreads, 1)
         erow[k] = R.erow[r0 + 4 * k];
         trw[k] = (tsplit && R.rdst[r0 + 4 * k] >= 0) ? R.trow[r0 + 4 * k] : -1;
       }
+      const int zn = np ? R.hrow[lw * 32 + lane] : -1;   // this lane's TMEM row
       __syncwarp();
       warp_arrive(&B.dempty[ds]);
+      if (np) {
+        // the row's h_src part of K|V (eq 5) = zkv[node] (tgl_node_proj): it initialises
+        // the accumulator, the MMAs add [e | Phi] W^T on top (padding rows: zeros)
+        wait_free(&B.tempty[tt & 1u], tt >> 1);
+        tc_fence_after();
+        const uint32_t tz = tmem + (tt & 1u) * 256u + ((uint32_t)(lw * 32) << 16);
+        const float* zr = a.zkv + (int64_t)(zn >= 0 ? zn : 0) * a.z_ld;
+#pragma unroll 1
+        for (int c0 = 0; c0 < 2 * 100; c0 += 32) {
+          float zv[32];
+#pragma unroll
+          for (int q = 0; q < 8; ++q) {
+            float4 z4 = make_float4(0.f, 0.f, 0.f, 0.f);
+            if (zn >= 0 && c0 + 4 * q < 200)
+              z4 = __ldg(reinterpret_cast<const float4*>(zr + c0 + 4 * q));
+            zv[4 * q] = z4.x;
+            zv[4 * q + 1] = z4.y;
+            zv[4 * q + 2] = z4.z;
+            zv[4 * q + 3] = z4.w;
+          }
+#pragma unroll
+          for (int q = 0; q < 4; ++q)
+            if (c0 + 8 * q < 200) tmem_st8(tz + c0 + 8 * q, zv + 8 * q);
+        }
+        tmem_wait_st();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&B.zfull[tt & 1u]);
+      }
       for (int i = 0; i < nch; ++i, ++g) {
         const int c = plan.order[chunk_of(tt, i, nch)];
         const int col = c * kTC + 8 * j;             // K' column of this piece
@@ -2945,6 +2990,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
       const uint32_t acc = tmem + (tt & 1u) * kCols;
       TGL_PROF_CLK(mt0);
       wait_free(&B.tempty[tt & 1u], tt >> 1);
+      if (np) mbar_wait(&B.zfull[tt & 1u], (tt >> 1) & 1u);   // zkv rows stored
       TGL_PROF_CLK(mt1);
 #ifdef TGL_KV_PROF
       prof_add(a, 7, mt1 - mt0);                     // MMA: wait for an accumulator
@@ -2977,7 +3023,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
           for (int ks = 0; ks < 2; ++ks) {
             if (ks < nk && !(TGL_DBG(a) & 4)) {
               const uint64_t ah = a0 + 2 * ks, bh = w0 + 2 * ks;
-              mma_bf16(acc, ah, bh, idesc, (i | ks) != 0);
+              mma_bf16(acc, ah, bh, idesc, np || (i | ks) != 0);
               if (split) {
                 mma_bf16(acc, ah + (512 >> 4), bh, idesc, 1u);
                 mma_bf16(acc, ah, bh + (kTWHalf >> 4), idesc, 1u);
@@ -3059,7 +3105,7 @@ __global__ void pack_dense_pre_kernel(const float* W, int n_out, int ksrc, int c
   }
   if (bias_out != nullptr && blockIdx.x == 0) {
     for (int n = threadIdx.x; n < n_out; n += blockDim.x) {
-      double acc = b[n];
+      double acc = b != nullptr ? b[n] : 0.0;
       if (phi != nullptr)
         for (int j = 0; j < d_t; ++j)
           acc += (double)W[(int64_t)n * ksrc + col_t + j] * (double)cosf(phi[j]);
@@ -3074,6 +3120,20 @@ struct DPBars {
   uint64_t dfull[kDSlots], dempty[kDSlots];
   uint64_t tfull[2], tempty[2];
 };
+// what one grid row (blockIdx.y) of dense_pre computes: Q form (kFfn = 0) writes
+// out[i] = A_i W^T + bias (+ q.b_k per head after column D when qbk != null) with row
+// pitch ld; the FFN form writes LayerNorm(ReLU(A_i W^T + b_o [+ zo[node_i]])) rows
+struct DPJob {
+  const uint8_t* wpk;
+  const float* bias;
+  const float* qbk;
+  float* out;
+  int64_t ld;
+};
+struct DPJobs {
+  DPJob j[4];
+};
+
 struct DPDesc {
   int row0[kBM];
   int row1[kBM];
@@ -3084,8 +3144,7 @@ struct DPDesc {
 
 template <bool kFfn>
 __global__ void __launch_bounds__(kDPThreads, 1)
-    dense_pre_kernel(const Args a, const DPPlan plan, const uint8_t* __restrict__ wpk,
-                     const float* __restrict__ bias) {
+    dense_pre_kernel(const Args a, const DPPlan plan, const DPJobs jobs) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* pipe = align1024(smem_raw);
   __shared__ DPBars B;
@@ -3094,6 +3153,8 @@ __global__ void __launch_bounds__(kDPThreads, 1)
   __shared__ float s_v0[kMaxModel], s_v1[kMaxModel], s_v2[kMaxModel];
   constexpr uint32_t kCols = 128;
   const tgl_attn_params& P = a.P;
+  const DPJob& J = jobs.j[blockIdx.y];
+  const uint8_t* __restrict__ wpk = J.wpk;
   const bool split = a.split != 0;
   const int nch = plan.n;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -3123,8 +3184,8 @@ __global__ void __launch_bounds__(kDPThreads, 1)
       s_v1[j] = P.ln_gamma[j];
       s_v2[j] = P.ln_beta[j];
     } else {
-      s_v0[j] = bias[j];                               // bq + Wq[:, d_hdst:] Phi(0)
-      s_v1[j] = P.bk[j];
+      s_v0[j] = J.bias ? J.bias[j] : 0.f;              // bq + Wq[:, d_hdst:] Phi(0)
+      s_v1[j] = J.qbk ? J.qbk[j] : 0.f;
     }
   }
   tc_fence_before();
@@ -3239,7 +3300,7 @@ __global__ void __launch_bounds__(kDPThreads, 1)
             const uint32_t d = dst + (uint32_t)(k >> 1) * 1024 + rr * 64 +
                                (((j ^ (rr >> 1)) & 3) << 4);
             const bool ok = row >= 0 && !pad;
-            cp_async16_zfill(d, ok ? base + (int64_t)row * ldb + pofs : b1, ok ? 16u : 0u);
+            cp_async16_zfill(d, ok ? base + (int64_t)row * ldb + pofs : b0, ok ? 16u : 0u);
           }
         }
         cp_async_mbar_arrive_noinc(&B.afull[sa]);
@@ -3301,7 +3362,7 @@ __global__ void __launch_bounds__(kDPThreads, 1)
       const uint32_t ta = tmem + ab * kCols + ((uint32_t)(warp * 32) << 16);
       float v[32];
       if (!kFfn) {
-        float* q = a.qbuf + (i0 + row) * kQLd;
+        float* q = J.out + (i0 + row) * J.ld;
         const int dhq = D / P.n_heads;
         float qb0 = 0.f, qb1 = 0.f;
 #pragma unroll 1
@@ -3326,16 +3387,32 @@ __global__ void __launch_bounds__(kDPThreads, 1)
             }
           }
         }
-        if (row < rows && D + 2 <= kQLd) {
+        if (row < rows && J.qbk != nullptr && D + 2 <= J.ld) {
           q[D] = qb0;
           q[D + 1] = qb1;
         }
       } else {
+        // node projections: + h_i Wo_h^T, precomputed per node (TGL_NODE_PROJ)
+        const float* zr = nullptr;
+        if (a.zo != nullptr && row < rows)
+          zr = a.zo + (int64_t)(a.hdst_idx ? a.hdst_idx[i0 + row] : (int)(i0 + row)) * a.z_ld;
         float s = 0.f, s2 = 0.f;
 #pragma unroll 1
         for (int cq = 0; cq < 4; ++cq) {
           tmem_ld32(ta + cq * 32, v);
           tmem_wait_ld();
+          if (zr != nullptr) {
+#pragma unroll
+            for (int jj = 0; jj < 32; jj += 4) {
+              if (cq * 32 + jj < D) {
+                const float4 z4 = __ldg(reinterpret_cast<const float4*>(zr + cq * 32 + jj));
+                v[jj] += z4.x;
+                v[jj + 1] += z4.y;
+                v[jj + 2] += z4.z;
+                v[jj + 3] += z4.w;
+              }
+            }
+          }
 #pragma unroll
           for (int jj = 0; jj < 32; ++jj) {
             const int col = cq * 32 + jj;
@@ -3349,11 +3426,23 @@ __global__ void __launch_bounds__(kDPThreads, 1)
         const float mean = s / (float)D;
         const float var = fmaxf(s2 / (float)D - mean * mean, 0.f);
         const float inv = rsqrtf(var + P.ln_eps);
-        float* o = a.out + (i0 + row) * D;
+        float* o = J.out + (i0 + row) * J.ld;
 #pragma unroll 1
         for (int cq = 0; cq < 4; ++cq) {
           tmem_ld32(ta + cq * 32, v);
           tmem_wait_ld();
+          if (zr != nullptr) {
+#pragma unroll
+            for (int jj = 0; jj < 32; jj += 4) {
+              if (cq * 32 + jj < D) {
+                const float4 z4 = __ldg(reinterpret_cast<const float4*>(zr + cq * 32 + jj));
+                v[jj] += z4.x;
+                v[jj + 1] += z4.y;
+                v[jj + 2] += z4.z;
+                v[jj + 3] += z4.w;
+              }
+            }
+          }
           if (row < rows) {
 #pragma unroll
             for (int jj = 0; jj < 32; jj += 4) {
@@ -3510,6 +3599,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t rank = cluster_ctarank();
   const bool leader = rank == 0;
+#ifdef TGL_KV_PROF
+  const long long k0c = clock64();
+#endif
   const int64_t pair = blockIdx.x >> 1, npairs = gridDim.x >> 1;
   if (threadIdx.x == 0) {
     for (int s = 0; s < kP2AStages; ++s) {
@@ -3567,7 +3659,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
     float* stdv = s_td[dw];
     for (tt = dw;; tt += kTDescWarps) {
       const uint32_t ds = tt % kSDSlots;
+      TGL_PROF_CLK(d0c);
       PRE_FREE_SLEEP(&B.dempty[ds], tt / kSDSlots, TGL_SLEEP_DESC);
+#ifdef TGL_KV_PROF
+      if (dw == 0) prof_add(a, 10, clock64() - d0c);  // desc: wait for a slot
+#endif
       TDesc& R = bd[ds];
       const int64_t PT = pair + (int64_t)tt * npairs;
       if (PT >= npt) {
@@ -3649,7 +3745,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
         for (int i = r0; i < nch; ++i) {
           const uint32_t k = wl + (i - r0);
           const uint32_t sw = k % kP2W;
+          TGL_PROF_CLK(w0c);
           PRE_FREE_SLEEP(&B.wempty[sw], k / kP2W, TGL_SLEEP_W);
+#ifdef TGL_KV_PROF
+          prof_add(a, 3, clock64() - w0c);             // weights: wait for a free stage
+#endif
           mbar_arrive_expect_tx(&B.wfull[sw], wbytes);
           bulk_g2s(pipe + kP2AStages * kPAStage + sw * kP2WStage,
                    wkv + (size_t)plan.order[chunk_of(tt, i, nch)] * 2 * kP2WStage +
@@ -3695,8 +3795,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
         const int col = c * kTC + 8 * j;
         const int ks = (plan.k - c * kTC) > 16 ? 2 : 1;
         const uint32_t sa = g % kP2AStages;
+        TGL_PROF_CLK(l0);
         PRE_FREE_SLEEP(&B.aempty[sa], g / kP2AStages, TGL_SLEEP_LOAD);
-        const bool in_k = active && col < c * kTC + 16 * ks;
+#ifdef TGL_KV_PROF
+        if (lw == 0) prof_add(a, 0, clock64() - l0);  // loader: wait for a free stage
+#endif
+        const bool in_k = active && col < c * kTC + 16 * ks && !(TGL_DBG(a) & 2);
         const uint32_t dst = a_s + sa * kPAStage + ofs0;
         if (in_k && col < kt0) {
           const bool seg_h = col < plan.dp0;
@@ -3752,9 +3856,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
         const int c = plan.order[chunk_of(tt, i, nch)];
         const int ks = (plan.k - c * kTC) > 16 ? 2 : 1;
         const uint32_t sa = g % kP2AStages;
-        const bool has_time = (c + 1) * kTC > kt0;
+        const bool has_time = (c + 1) * kTC > kt0 && !(TGL_DBG(a) & 64);
         if (has_time) {
+          TGL_PROF_CLK(t0);
           wait_free(&B.aempty[sa], g / kP2AStages);
+          TGL_PROF_CLK(t1);
+#ifdef TGL_KV_PROF
+          if (tw == 0) prof_add(a, 1, t1 - t0);        // time warp: wait for a free stage
+#endif
           const uint32_t dst = a_s + sa * kPAStage + rofs;
 #pragma unroll
           for (int jj = 0; jj < 4; ++jj) {
@@ -3797,6 +3906,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
           }
           fence_proxy_async_smem();
           __syncwarp();
+#ifdef TGL_KV_PROF
+          if (tw == 0) prof_add(a, 2, clock64() - t1);  // time warp: Phi + split + store
+#endif
           if (lane == 0) mbar_arrive(&B.afull[sa]);
         } else {
           if (lane == 0) {
@@ -3820,11 +3932,17 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
       const int r0 = (tt > 0 && nch >= 4) ? 2 : 0;
       for (int i = 0; i < nch; ++i, ++g) {
         const uint32_t sa = g % kP2AStages;
+        TGL_PROF_CLK(r0c);
         mbar_wait(&B.afull[sa], (g / kP2AStages) & 1u);
+        TGL_PROF_CLK(r1c);
         if (i >= r0) {
           const uint32_t kw = wl + (i - r0);
           mbar_wait(&B.wfull[kw % kP2W], (kw / kP2W) & 1u);
         }
+#ifdef TGL_KV_PROF
+        prof_add(a, 4, r1c - r0c);                     // relay: A wait
+        prof_add(a, 5, clock64() - r1c);               // relay: W wait
+#endif
         if (lane == 0) mbar_arrive_remote(pfull0 + sa * 8);
         __syncwarp();
       }
@@ -3840,15 +3958,22 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
       warp_arrive(&B.dempty[ds]);
       if (!live) break;
       const uint32_t acc = tmem + (tt & 1u) * kCols;
+      TGL_PROF_CLK(mt0);
       if (tt >= 2) mbar_wait_cluster(&B.tempty[tt & 1u], ((tt >> 1) - 1) & 1u);
+#ifdef TGL_KV_PROF
+      prof_add(a, 6, clock64() - mt0);               // MMA: wait for an accumulator
+#endif
       tc_fence_after();
       const int r0 = (tt > 0 && nch >= 4) ? 2 : 0;
       for (int i = 0; i < nch; ++i, ++g) {
         const int c = plan.order[chunk_of(tt, i, nch)];
         const int nk = (plan.k - c * kTC) > 16 ? 2 : 1;
         const uint32_t sa = g % kP2AStages;
+        TGL_PROF_CLK(ma0);
         mbar_wait(&B.afull[sa], (g / kP2AStages) & 1u);
+        TGL_PROF_CLK(ma1);
         mbar_wait_cluster(&B.pfull[sa], (g / kP2AStages) & 1u);
+        TGL_PROF_CLK(ma2);
         uint32_t kw;
         if (i < r0) {
           kw = wl - 1 - i;
@@ -3856,13 +3981,18 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
           kw = wl + (i - r0);
           mbar_wait(&B.wfull[kw % kP2W], (kw / kP2W) & 1u);
         }
+#ifdef TGL_KV_PROF
+        prof_add(a, 7, ma1 - ma0);                     // MMA: local A wait
+        prof_add(a, 8, ma2 - ma1);                     // MMA: peer relay wait
+        prof_add(a, 9, clock64() - ma2);               // MMA: W wait
+#endif
         tc_fence_after();
         if (elect_one()) {
           const uint64_t a0 = desc_sw64(a_s + sa * kPAStage, 1024);
           const uint64_t w0 = desc_sw64(w_s + (kw % kP2W) * kP2WStage, 512);
 #pragma unroll
           for (int ks = 0; ks < 2; ++ks) {
-            if (ks < nk) {
+            if (ks < nk && !(TGL_DBG(a) & 4)) {
               const uint64_t ah = a0 + 2 * ks, bh = w0 + 2 * ks;
               mma_bf16_pair(acc, ah, bh, idesc, (i | ks) != 0);
               if (split) {
@@ -3888,6 +4018,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
   }
   tc_fence_before();
   __syncthreads();
+#ifdef TGL_KV_PROF
+  if (threadIdx.x == 0) prof_add(a, 13, clock64() - k0c);   // whole kernel
+#endif
   cluster_sync_all();                                // the peer's smem / barriers stay valid
   if (warp == kTMma)
     asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem),
@@ -3901,7 +4034,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
 namespace tca {
 
 struct PackedLayout {
-  size_t oq, okv, oo, okv64, okvc, okvp, okvp2, oqp, oop, obq, total;
+  size_t oq, okv, oo, okv64, okvc, okvp, okvp2, oqp, oop, obq;
+  size_t okvn, onk, onv, ono, oor;   // node projections (TGL_NODE_PROJ)
+  size_t total;
 };
 
 static PackedLayout packed_layout(const tgl_attn_params* P) {
@@ -3920,6 +4055,13 @@ static PackedLayout packed_layout(const tgl_attn_params* P) {
   L.oqp = W.take((size_t)make_dp_plan(P->d_hdst, 0).n * kDPWStage);
   L.oop = W.take((size_t)make_dp_plan(P->d_model, P->d_hdst).n * kDPWStage);
   L.obq = W.take(sizeof(float) * kDPN);
+  // node projections: the per-edge K|V plan over [e | Phi] only, the per-node Wk_h / Wv_h /
+  // Wo_h projections (tgl_node_proj) and the FFN over r only
+  L.okvn = W.take((size_t)make_pre_plan(0, P->d_e, P->d_t).n * kTWStage);
+  L.onk = W.take((size_t)make_dp_plan(P->d_hsrc, 0).n * kDPWStage);
+  L.onv = W.take((size_t)make_dp_plan(P->d_hsrc, 0).n * kDPWStage);
+  L.ono = W.take((size_t)make_dp_plan(P->d_hdst, 0).n * kDPWStage);
+  L.oor = W.take((size_t)make_dp_plan(P->d_model, 0).n * kDPWStage);
   L.total = W.off;
   return L;
 }
@@ -3944,8 +4086,26 @@ static tgl_status launch_pack(const tgl_attn_params* P, uint8_t* base, cudaStrea
   TGL_TRY(launch_check("pack_kv64 contiguous"));
   pack_kv_pre_kernel<<<64, 256, 0, s>>>(P->Wk, P->Wv, P->d_model, P->d_hsrc + P->d_e + P->d_t,
                                         make_pre_plan(P->d_hsrc, P->d_e, P->d_t),
-                                        base + L.okvp);
+                                        base + L.okvp, 0);
   TGL_TRY(launch_check("pack_kv_pre"));
+  pack_kv_pre_kernel<<<64, 256, 0, s>>>(P->Wk, P->Wv, P->d_model, P->d_hsrc + P->d_e + P->d_t,
+                                        make_pre_plan(0, P->d_e, P->d_t), base + L.okvn,
+                                        P->d_hsrc);
+  TGL_TRY(launch_check("pack_kv_pre node-proj"));
+  const int kin = P->d_hsrc + P->d_e + P->d_t;
+  pack_dense_pre_kernel<<<64, 256, 0, s>>>(P->Wk, P->d_model, kin, 0, 0,
+                                           make_dp_plan(P->d_hsrc, 0), base + L.onk, nullptr,
+                                           nullptr, 0, 0, nullptr);
+  pack_dense_pre_kernel<<<64, 256, 0, s>>>(P->Wv, P->d_model, kin, 0, 0,
+                                           make_dp_plan(P->d_hsrc, 0), base + L.onv, nullptr,
+                                           nullptr, 0, 0, nullptr);
+  pack_dense_pre_kernel<<<64, 256, 0, s>>>(P->Wo, P->d_out, P->d_model + P->d_hdst, P->d_model,
+                                           0, make_dp_plan(P->d_hdst, 0), base + L.ono, nullptr,
+                                           nullptr, 0, 0, nullptr);
+  pack_dense_pre_kernel<<<64, 256, 0, s>>>(P->Wo, P->d_out, P->d_model + P->d_hdst, 0, 0,
+                                           make_dp_plan(P->d_model, 0), base + L.oor, nullptr,
+                                           nullptr, 0, 0, nullptr);
+  TGL_TRY(launch_check("pack node-proj"));
   pack_kv_pre2_kernel<<<64, 256, 0, s>>>(P->Wk, P->Wv, P->d_model, P->d_hsrc + P->d_e + P->d_t,
                                          make_pre_plan(P->d_hsrc, P->d_e, P->d_t),
                                          base + L.okvp2);
@@ -4067,6 +4227,11 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
   a.qbuf = reinterpret_cast<float*>(w + o_q);
   a.rbuf = reinterpret_cast<float*>(w + o_r);
   a.rsplit = nullptr;
+  a.zkv = nullptr;
+  a.zo = nullptr;
+  a.z_ld = 0;
+  a.q_idx = nullptr;
+  a.q_ld = kQLd;
   a.wq = pk + PL.oq;
   a.wkv = pk + PL.okv;
   a.wo = pk + PL.oo;
@@ -4092,6 +4257,54 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
   TGL_TRY(set_smem_attrs(smem_q, smem_kv, smem_kvb));
   const int64_t tiles = ceil_div(n_dst_max, kBM);
   const unsigned gq = (unsigned)(tiles < kNumSMs ? tiles : kNumSMs);
+  if (P->input_layout & TGL_NODE_PROJ) {
+    // node projections (tgl_node_proj, P->node_proj = Z): q_i, the h_src part of k_e / v_e
+    // and the h_i part of the FFN input are rows of Z (eqs 4, 5, 7 are linear in h); the
+    // per-edge MMAs cover [e | Phi] only, the FFN's cover r only.  No Q launch.
+    const PrePlan plan = make_pre_plan(0, P->d_e, P->d_t);
+    const DPPlan rplan = make_dp_plan(P->d_model, 0);
+    const bool e_ok = P->d_e == 0 || ((P->input_layout & TGL_SPLIT_E) && ld_e >= plan.dp1 &&
+                                      rows_16b(efeat, 1, ld_e));
+    const bool t_ok = !(P->input_layout & TGL_SPLIT_TABLE) || table == nullptr ||
+                      rows_16b(table, 1, plan.dpt);
+    const int sel = P->kv_kernel;
+    if (P->node_proj == nullptr || (reinterpret_cast<uintptr_t>(P->node_proj) & 15) || !e_ok ||
+        !t_ok || !(sel == TGL_KV_AUTO || sel == TGL_KV_PRE) ||
+        !(max_seg > 0 && max_seg <= 32 && P->n_heads == 2) || P->d_hsrc != P->d_hdst ||
+        plan.n > kPMaxChunks || rplan.n > kPMaxChunks) {
+      set_error("TGL_NODE_PROJ: needs P->node_proj (tgl_node_proj output, 16-byte aligned), "
+                "d_hsrc == d_hdst, split16 e / table (input_layout), kv_kernel AUTO/PRE, "
+                "max_seg <= 32, 2 heads");
+      return TGL_EUNSUPPORTED;
+    }
+    a.zkv = P->node_proj;
+    a.zo = P->node_proj + TGL_NODE_PROJ_O;
+    a.z_ld = TGL_NODE_PROJ_LD;
+    a.qbuf = const_cast<float*>(P->node_proj) + TGL_NODE_PROJ_Q;
+    a.q_ld = TGL_NODE_PROJ_LD;
+    a.q_idx = hdst_idx;
+    a.rsplit = reinterpret_cast<uint8_t*>(a.rbuf);   // r rows split16 for the FFN
+    tgl_kv_probe* probe = P->probe;
+    if (probe) {
+      probe->kernel = TGL_KV_PRE;
+      if (probe->ev_start)
+        TGL_TRY(cuda_check(cudaEventRecord(static_cast<cudaEvent_t>(probe->ev_start), s),
+                           "probe event"));
+    }
+    const int bdst = 32 / max_seg;
+    const int64_t ttiles = ceil_div(n_dst_max, 4 * bdst);
+    const unsigned gt = (unsigned)(ttiles < kNumSMs ? (ttiles > 0 ? ttiles : 1) : kNumSMs);
+    launch_pdl(kv_pre_kernel, dim3(gt), dim3(kPThreads), kPSmem, s, a, plan, pk + PL.okvn,
+               bdst);
+    TGL_TRY(launch_check("tc kv pre kernel (node proj)"));
+    if (probe && probe->ev_stop)
+      TGL_TRY(cuda_check(cudaEventRecord(static_cast<cudaEvent_t>(probe->ev_stop), s),
+                         "probe event"));
+    DPJobs jo{};
+    jo.j[0] = DPJob{pk + PL.oor, nullptr, nullptr, a.out, P->d_model};
+    launch_pdl(dense_pre_kernel<true>, dim3(gq), dim3(kDPThreads), kDPSmem, s, a, rplan, jo);
+    return launch_check("tc ffn kernel (node proj)");
+  }
   // split16 h_dst (and so split16 r, written by the K|V epilogue): converter-free Q / FFN
   const bool dpre = (P->input_layout & TGL_SPLIT_HDST) != 0;
   const DPPlan qplan = make_dp_plan(P->d_hdst, 0), oplan = make_dp_plan(P->d_model, P->d_hdst);
@@ -4104,8 +4317,10 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
       return TGL_EUNSUPPORTED;
     }
     a.rsplit = reinterpret_cast<uint8_t*>(a.rbuf);   // r scratch rows hold the split16 rows
-    launch_pdl(dense_pre_kernel<false>, dim3(gq), dim3(kDPThreads), kDPSmem, s, a, qplan,
-               pk + PL.oqp, reinterpret_cast<const float*>(pk + PL.obq));
+    DPJobs jq{};
+    jq.j[0] = DPJob{pk + PL.oqp, reinterpret_cast<const float*>(pk + PL.obq), P->bk, a.qbuf,
+                    kQLd};
+    launch_pdl(dense_pre_kernel<false>, dim3(gq), dim3(kDPThreads), kDPSmem, s, a, qplan, jq);
   } else {
     launch_pdl(dense_kernel<false>, dim3(gq), dim3(kWsThreads), smem_q, s, a);
   }
@@ -4157,9 +4372,11 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
     if (probe && probe->ev_stop)
       TGL_TRY(cuda_check(cudaEventRecord(static_cast<cudaEvent_t>(probe->ev_stop), s),
                          "probe event"));
-    if (dpre)
-      launch_pdl(dense_pre_kernel<true>, dim3(gq), dim3(kDPThreads), kDPSmem, s, a, oplan,
-                 pk + PL.oop, nullptr);
+    if (dpre) {
+      DPJobs jo{};
+      jo.j[0] = DPJob{pk + PL.oop, nullptr, nullptr, a.out, P->d_model};
+      launch_pdl(dense_pre_kernel<true>, dim3(gq), dim3(kDPThreads), kDPSmem, s, a, oplan, jo);
+    }
     else
       launch_pdl(dense_kernel<true>, dim3(gq), dim3(kWsThreads), smem_q, s, a);
     return launch_check("tc ffn kernel");
@@ -4249,6 +4466,50 @@ extern "C" tgl_status tgl_attn_pack(const tgl_attn_params* P, void* packed, size
   }
   TGL_REQUIRE((reinterpret_cast<uintptr_t>(packed) & 255) == 0, "packed must be 256-aligned");
   return tca::launch_pack(P, static_cast<uint8_t*>(packed), as_stream(stream));
+}
+
+extern "C" tgl_status tgl_node_proj(const tgl_attn_params* P, int64_t n_nodes, const void* hnode,
+                                    int64_t ld, float* Z, void* stream) {
+  using namespace tca;
+  TGL_REQUIRE(P != nullptr && Z != nullptr, "null pointer");
+  TGL_REQUIRE(n_nodes >= 0, "n_nodes < 0");
+  if (!tc_attn_supported(P) || P->n_heads != 2 || P->d_hsrc != P->d_hdst ||
+      !(P->precision == TGL_FP32 || P->precision == TGL_BF16)) {
+    set_error("tgl_node_proj: tensor-core precisions, d_model == 100, 2 heads, d_hsrc == d_hdst");
+    return TGL_EUNSUPPORTED;
+  }
+  TGL_REQUIRE(P->packed != nullptr, "tgl_node_proj needs P->packed (tgl_attn_pack)");
+  const DPPlan plan = make_dp_plan(P->d_hsrc, 0);
+  TGL_REQUIRE(plan.n <= kPMaxChunks, "d_hsrc too large");
+  TGL_REQUIRE(!(reinterpret_cast<uintptr_t>(Z) & 15), "Z must be 16-byte aligned");
+  if (n_nodes == 0) return TGL_OK;
+  TGL_REQUIRE(hnode != nullptr && !(reinterpret_cast<uintptr_t>(hnode) & 15) && ld % 4 == 0 &&
+                  ld >= plan.dp0,
+              "hnode: split16 rows, 16-byte aligned, ld >= round8(d_hsrc)");
+  cudaStream_t s = as_stream(stream);
+  TGL_TRY(set_smem_attrs(Pipe<kNPq>::kBytes + 1024, Pipe<kNPkv>::kBytes + 1024 + kKvEpiBytes,
+                         Pipe<kNPkv>::kBytes + 1024 + kBEpi * 32 * 33 * 4));
+  const uint8_t* pk = static_cast<const uint8_t*>(P->packed);
+  const PackedLayout PL = packed_layout(P);
+  Args a{};
+  a.P = *P;
+  a.n_dst_max = n_nodes;
+  a.n_dst_dev = nullptr;
+  a.hdst = static_cast<const float*>(hnode);
+  a.hdst_idx = nullptr;
+  a.ld_hdst = ld;
+  a.q_ld = kQLd;
+  a.split = P->precision == TGL_FP32 ? 1 : 0;
+  DPJobs j{};
+  j.j[0] = DPJob{pk + PL.onk, nullptr, nullptr, Z + TGL_NODE_PROJ_K, TGL_NODE_PROJ_LD};
+  j.j[1] = DPJob{pk + PL.onv, nullptr, nullptr, Z + TGL_NODE_PROJ_V, TGL_NODE_PROJ_LD};
+  j.j[2] = DPJob{pk + PL.oqp, reinterpret_cast<const float*>(pk + PL.obq), P->bk,
+                 Z + TGL_NODE_PROJ_Q, TGL_NODE_PROJ_LD};
+  j.j[3] = DPJob{pk + PL.ono, nullptr, nullptr, Z + TGL_NODE_PROJ_O, TGL_NODE_PROJ_LD};
+  const int64_t tiles = ceil_div(n_nodes, kBM);
+  const unsigned gx = (unsigned)(tiles < kNumSMs ? tiles : kNumSMs);
+  launch_pdl(dense_pre_kernel<false>, dim3(gx, 4), dim3(kDPThreads), kDPSmem, s, a, plan, j);
+  return launch_check("tgl_node_proj");
 }
 
 #ifdef TGL_PROBE

@@ -22,7 +22,8 @@ FP32, BF16, FP32_SIMT = 0, 1, 2
 # tgl_attn_params.kv_kernel (include/tgl.h TGL_KV_*)
 KV_KERNEL = {"auto": 0, "split": 1, "split_pad": 2, "async": 3, "bin": 4, "general": 5,
              "pre": 7, "pre2": 8}
-SPLIT_HSRC, SPLIT_E, SPLIT_TABLE, SPLIT_HDST = 1, 2, 4, 8
+SPLIT_HSRC, SPLIT_E, SPLIT_TABLE, SPLIT_HDST, NODE_PROJ = 1, 2, 4, 8, 16
+NODE_PROJ_LD = 512       # tgl.h TGL_NODE_PROJ_LD: Z row pitch (floats)
 KV_KERNEL_NAME = {1: "kv_split_kernel (contiguous K plan)", 2: "kv_split_kernel (padded K plan)",
                   3: "kv_async_kernel", 4: "kv_bin_kernel", 5: "kv_kernel (general)",
                   6: "kv_attn_kernel (SIMT)", 7: "kv_pre_kernel (pre-split operands)",
@@ -36,7 +37,8 @@ SYMBOLS = ["tgl_version", "tgl_status_string", "tgl_last_error", "tgl_build_tcsr
            "tgl_attn_packed_bytes", "tgl_attn_pack", "tgl_cache_lookup", "tgl_cache_store", "tgl_cache_combine",
            "tgl_cache_merge", "tgl_shard_slice", "tgl_shard_gather", "tgl_split_rows",
            "tgl_tcsr_index", "tgl_tblock_attn_backward", "tgl_scatter_add_rows",
-           "tgl_preload_rows", "tgl_mailbox_store", "tgl_memory_update", "tgl_build_tcsr_ex"]
+           "tgl_preload_rows", "tgl_mailbox_store", "tgl_memory_update", "tgl_build_tcsr_ex",
+           "tgl_node_proj"]
 
 
 class TGLError(RuntimeError):
@@ -67,6 +69,7 @@ def _load():
                             vp, i64, i32, vp, vp, sz, vp],
         "tgl_gather_rows": [i64, vp, vp, vp, i64, i32, vp, i64, vp],
         "tgl_attn_pack": [vp, vp, C.c_size_t, vp],
+        "tgl_node_proj": [vp, i64, vp, i64, vp, vp],
         "tgl_cache_lookup": [vp, i64, vp, vp, vp, vp, vp, vp, vp, vp, sz, vp],
         "tgl_cache_store": [vp, i64, vp, vp, vp, vp, i64, vp],
         "tgl_cache_combine": [vp, i64, vp, vp, vp, i64, vp, i64, vp],
@@ -303,7 +306,7 @@ class AttnParamsC(C.Structure):
                 ("leaky_slope", C.c_float), ("logit_scale", C.c_float),
                 ("precision", C.c_int32), ("packed", C.c_void_p),
                 ("kv_kernel", C.c_int32), ("probe", C.c_void_p),
-                ("input_layout", C.c_int32)]
+                ("input_layout", C.c_int32), ("node_proj", C.c_void_p)]
 
 
 class KvProbeC(C.Structure):
@@ -357,7 +360,7 @@ class AttnParams:
                                   _p(self.t["omega"]), _p(self.t["phi"]),
                                   float(p["leaky_slope"]), float(p["logit_scale"]),
                                   self.precision, None,
-                                  KV_KERNEL.get(kv_kernel, kv_kernel), None, 0)
+                                  KV_KERNEL.get(kv_kernel, kv_kernel), None, 0, None)
         self.packed = None
         if pack and self.precision != FP32_SIMT:
             nb = _lib.tgl_attn_packed_bytes(C.byref(self.struct))
@@ -374,6 +377,17 @@ class AttnParams:
 
     def set_kv_kernel(self, kv_kernel: str | int):
         self.struct.kv_kernel = KV_KERNEL.get(kv_kernel, kv_kernel)
+
+
+def node_proj(P: AttnParams, hnode, n_nodes: int | None = None, out=None, stream=None):
+    """tgl_node_proj: Z [n_nodes, NODE_PROJ_LD] fp32 per-node projections of the split16
+    node table `hnode` (needs P packed).  Attach with P.struct.node_proj + NODE_PROJ."""
+    n = hnode.shape[0] if n_nodes is None else n_nodes
+    if out is None:
+        out = torch.empty(max(n, 1), NODE_PROJ_LD, dtype=torch.float32, device=hnode.device)
+    _check(_lib.tgl_node_proj(C.byref(P.struct), n, _prow(hnode), hnode.stride(0), _p(out),
+                              _s(stream)), "tgl_node_proj")
+    return out
 
 
 def tblock_attn(P: AttnParams, seg_ptr, dst_t, hdst, hdst_idx, hsrc, hsrc_idx, efeat, eid,

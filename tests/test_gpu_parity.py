@@ -374,7 +374,8 @@ def _world(name, n_edges=None, dedup=None, strategy=None):
     return cfg, g, neg, params
 
 
-def _gpu_pipeline(T, cfg, g, neg, params, precision="fp32", dev=None, layout=None):
+def _gpu_pipeline(T, cfg, g, neg, params, precision="fp32", dev=None, layout=None,
+                  node_proj=None):
     from paper_conf_asplos_wangm24_b200 import TGATPipeline, TSampler
     if dev is None:
         dev = {"src": cu(g.src), "dst": cu(g.dst), "t": cu(g.t), "neg": cu(neg),
@@ -382,7 +383,8 @@ def _gpu_pipeline(T, cfg, g, neg, params, precision="fp32", dev=None, layout=Non
     tc = T.build_tcsr(cfg.n_nodes, dev["src"], dev["dst"], dev["t"], True, True)
     pipe = TGATPipeline(dev, tc, params, cfg.batch,
                         TSampler(cfg.k, cfg.strategy, cfg.seeds["sampler"]), cfg.dedup,
-                        cfg.precompute, cfg.window, precision, layout=layout)
+                        cfg.precompute, cfg.window, precision, layout=layout,
+                        node_proj=node_proj)
     return pipe
 
 

@@ -108,7 +108,10 @@ if os.environ.get("PROBE_PROF"):
         call(); torch.cuda.synchronize()
         lib.tgl_debug_prof(host, 0)
         v = np.frombuffer(host, dtype=np.uint64).reshape(148, 16).astype(np.float64)
-        names = (["T:aempty-wait", "T:phi+split+st", "2", "3", "4", "L:aempty-wait", "6",
+        names = (["L:aempty-wait", "T:aempty-wait", "T:work", "W:wempty-wait", "R:afull-wait",
+                  "R:wfull-wait", "M:tempty-wait", "M:afull-wait", "M:pfull-wait", "M:wfull-wait",
+                  "D:slot-wait", "E:acc-wait", "E:work", "total"] if kv == "pre2" else
+                 ["T:aempty-wait", "T:phi+split+st", "2", "3", "4", "L:aempty-wait", "6",
                   "M:tempty-wait", "M:afull-wait(gathered)", "M:afull-wait(time)",
                   "M:wfull-wait", "E:acc-wait", "E:work"] if kv == "pre" else
                  ["C:ffull-wait", "C:lds+phi", "C:bempty-wait", "C:cvt+sts", "C:fence",
@@ -117,8 +120,14 @@ if os.environ.get("PROBE_PROF"):
                  ["P:stage-free", "P:issue", "P:data-wait", "P:convert", "P:fence+arrive",
                  "MMA:A-wait", "MMA:W-wait", "MMA:acc-wait", "MMA:tile", "D:slot-wait",
                  "D:build", "E:acc-wait", "E:work"])
-        med = np.median(v[:, :13], axis=0)
-        print(kv, "cycles per CTA (median):", "  ".join(f"{n} {m:.0f}" for n, m in zip(names, med)))
+        if kv == "pre2":
+            for who, rows in (("leader", v[0::2, :14]), ("peer", v[1::2, :14])):
+                med = np.median(rows, axis=0)
+                print(kv, who, "cycles per CTA (median):",
+                      "  ".join(f"{n} {m:.0f}" for n, m in zip(names, med) if m > 0))
+        else:
+            med = np.median(v[:, :13], axis=0)
+            print(kv, "cycles per CTA (median):", "  ".join(f"{n} {m:.0f}" for n, m in zip(names, med)))
     os.environ["TGL_DEBUG_MASK"] = "0"
 
 if os.environ.get("PROBE_TRACE"):

@@ -32,10 +32,11 @@ def main(path):
             cur.append((name, v))
     # a full step ends with the S14 gather (or, with cache(), the root cache_merge); torch
     # kernels (the bench's per-step counters, outside the timed region) are left out
+    # (steps that end at the next batch's roots are complete by construction)
     done = lambda st: any("gather_rows" in n or "cache_merge" in n for n, _ in st)
     if cur and done(cur):
         steps.append(cur)
-    steps = [[(n, v) for n, v in s if "at::" not in n] for s in steps if done(s)]
+    steps = [[(n, v) for n, v in s if "at::" not in n and "native::" not in n] for s in steps]
     tot = [sum(v for _, v in s) for s in steps]
     med = sorted(range(len(steps)), key=lambda i: tot[i])[len(steps) // 2]
     s = steps[med]

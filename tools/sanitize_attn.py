@@ -42,7 +42,17 @@ for prec in ("fp32", "bf16"):
         o = tgl.tblock_attn(P, cu(seg), cu(dst_t), nfeat, dn, hs, sn, ef, eid, et, max_seg=10)
         torch.cuda.synchronize()
         outs[(prec, kv)] = o[:n_dst].cpu().numpy()
+    # node projections (tgl_node_proj + TGL_NODE_PROJ): Z rows initialise the accumulator
+    P = tgl.AttnParams(p, precision=prec, pack=True)
+    Z = tgl.node_proj(P, tgl.split_rows(nfeat))
+    P.struct.input_layout = tgl.SPLIT_HSRC | tgl.SPLIT_E | tgl.NODE_PROJ
+    P.struct.node_proj = tgl._p(Z)
+    o = tgl.tblock_attn(P, cu(seg), cu(dst_t), nfeat, dn, nfeat, sn, tgl.split_rows(efeat), eid,
+                        et, max_seg=10)
+    torch.cuda.synchronize()
+    outs[(prec, "np")] = o[:n_dst].cpu().numpy()
 for prec in ("fp32", "bf16"):
     d = np.abs(outs[(prec, "pre")] - outs[(prec, "split")]).max()
-    print(f"{prec}: |pre - split| = {d:.2e}")
+    dn_ = np.abs(outs[(prec, "pre")] - outs[(prec, "np")]).max()
+    print(f"{prec}: |pre - split| = {d:.2e}  |pre - node_proj| = {dn_:.2e}")
 print("sanitize_attn done")
