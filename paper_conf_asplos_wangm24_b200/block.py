@@ -81,8 +81,9 @@ class TGATPipeline:
         node_proj: the tail block's projections of h (eqs 4, 5, 7 are linear in h) are
         computed once per node per forward (tgl_node_proj into Z [n_nodes, 512]) and
         gathered, so the tail's per-edge MMAs cover [e | Phi] only and it has no Q launch.
-        None (default) = on when the node table is split16 and device-resident and has
-        fewer rows than the tail block gathers per batch (and Z fits 2 GB)."""
+        None (default) = on when the node table is split16 and device-resident, has at
+        most 1/16 of the rows the tail block gathers per batch, d_h >= 2 d_model (the h
+        columns dominate the projections) and Z fits 2 GB."""
         self.dev = device or torch.device("cuda")
         self.g = graph
         self.tcsr = tcsr
@@ -163,7 +164,13 @@ class TGATPipeline:
         np_ok = (self.split and precision in ("fp32", "bf16") and not host_features and
                  n_nodes > 0 and self.attn[-1].host["n_heads"] == 2)
         if node_proj is None:
-            node_proj = np_ok and n_nodes <= tail.n_max * k and n_nodes * 2048 <= (2 << 30)
+            # a clear win only when the h columns dominate the projections and the node
+            # table is small next to the rows the tail block gathers (measured: GDELT
+            # 7.8e6 -> 1.03e7 emb/s; REDDIT / LASTFM / WIKI, d_v <= 172, lose 3-12 %)
+            d_h = self.attn[-1].host["d_hdst"]
+            node_proj = (np_ok and n_nodes * 16 <= tail.n_max * k and
+                         d_h >= 2 * self.attn[-1].host["d_model"] and
+                         n_nodes * 2048 <= (2 << 30))
         assert not node_proj or np_ok, "node_proj needs the split16 device-resident tables"
         self.node_proj = bool(node_proj)
         self.zproj = None

@@ -2622,6 +2622,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
   __shared__ uint32_t s_tmem;
   __shared__ TDesc bd[kSDSlots];
   __shared__ float s_omega[256], s_phi[256];
+  __shared__ unsigned char s_order[64];      // plan.order (indexed: smem, not a local copy)
   __shared__ float s_bias[2 * kMaxModel];
   __shared__ int64_t s_seg[kTDescWarps][4 * 32 + 1];
   __shared__ float s_td[kTDescWarps][4 * 32];
@@ -2656,6 +2657,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
   }
   TGL_TRACE_RESET();
   if (warp == kTMma) tmem_alloc(&s_tmem, 2 * kCols);
+  for (int j = threadIdx.x; j < 64; j += blockDim.x) s_order[j] = plan.order[j];
   for (int j = threadIdx.x; j < P.d_t; j += blockDim.x) {
     s_omega[j] = P.omega[j];
     s_phi[j] = P.phi[j];
@@ -2767,7 +2769,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
           PRE_FREE_SLEEP(&B.wempty[sw], k / kPW, TGL_SLEEP_W);
           mbar_arrive_expect_tx(&B.wfull[sw], wbytes);
           bulk_g2s_hint(pipe + kPAStages * kPAStage + sw * kTWStage,
-                        wkv + (size_t)plan.order[chunk_of(tt, i, nch)] * kTWStage, wbytes,
+                        wkv + (size_t)s_order[chunk_of(tt, i, nch)] * kTWStage, wbytes,
                         &B.wfull[sw], wpol);
         }
         wl += nch - r0;
@@ -2813,26 +2815,32 @@ __global__ void __launch_bounds__(kPThreads, 1)
       if (np) {
         // the row's h_src part of K|V (eq 5) = zkv[node] (tgl_node_proj): it initialises
         // the accumulator, the MMAs add [e | Phi] W^T on top (padding rows: zeros)
-        wait_free(&B.tempty[tt & 1u], tt >> 1);
-        tc_fence_after();
+        // 16-column rounds, the next round's loads in flight while this one is stored; the
+        // first round is loaded before waiting for the accumulator to be released
         const uint32_t tz = tmem + (tt & 1u) * 256u + ((uint32_t)(lw * 32) << 16);
         const float* zr = a.zkv + (int64_t)(zn >= 0 ? zn : 0) * a.z_ld;
-#pragma unroll 1
-        for (int c0 = 0; c0 < 2 * 100; c0 += 32) {
-          float zv[32];
+        float4 zb[2][4];
 #pragma unroll
-          for (int q = 0; q < 8; ++q) {
-            float4 z4 = make_float4(0.f, 0.f, 0.f, 0.f);
-            if (zn >= 0 && c0 + 4 * q < 200)
-              z4 = __ldg(reinterpret_cast<const float4*>(zr + c0 + 4 * q));
-            zv[4 * q] = z4.x;
-            zv[4 * q + 1] = z4.y;
-            zv[4 * q + 2] = z4.z;
-            zv[4 * q + 3] = z4.w;
+        for (int q = 0; q < 4; ++q)
+          zb[0][q] = zn >= 0 ? __ldg(reinterpret_cast<const float4*>(zr + 4 * q))
+                             : make_float4(0.f, 0.f, 0.f, 0.f);
+        wait_free(&B.tempty[tt & 1u], tt >> 1);
+        tc_fence_after();
+#pragma unroll
+        for (int c0 = 0; c0 < 2 * 100; c0 += 16) {
+          const int cur = (c0 >> 4) & 1;
+          if (c0 + 16 < 2 * 100) {
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+              const int cc = c0 + 16 + 4 * q;
+              zb[cur ^ 1][q] = (zn >= 0 && cc < 200)
+                                   ? __ldg(reinterpret_cast<const float4*>(zr + cc))
+                                   : make_float4(0.f, 0.f, 0.f, 0.f);
+            }
           }
-#pragma unroll
-          for (int q = 0; q < 4; ++q)
-            if (c0 + 8 * q < 200) tmem_st8(tz + c0 + 8 * q, zv + 8 * q);
+          const float* zv = reinterpret_cast<const float*>(&zb[cur][0]);
+          tmem_st8(tz + c0, zv);
+          if (c0 + 8 < 2 * 100) tmem_st8(tz + c0 + 8, zv + 8);
         }
         tmem_wait_st();
         tc_fence_before();
@@ -2840,7 +2848,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
         if (lane == 0) mbar_arrive(&B.zfull[tt & 1u]);
       }
       for (int i = 0; i < nch; ++i, ++g) {
-        const int c = plan.order[chunk_of(tt, i, nch)];
+        const int c = s_order[chunk_of(tt, i, nch)];
         const int col = c * kTC + 8 * j;             // K' column of this piece
         const int ks = (plan.k - c * kTC) > 16 ? 2 : 1;   // K steps the MMA issues
         const uint32_t sa = g % kPAStages;
@@ -2910,7 +2918,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
       __syncwarp();
       warp_arrive(&B.dempty[ds]);
       for (int i = 0; i < nch; ++i, ++g) {
-        const int c = plan.order[chunk_of(tt, i, nch)];
+        const int c = s_order[chunk_of(tt, i, nch)];
         const int ks = (plan.k - c * kTC) > 16 ? 2 : 1;
         const uint32_t sa = g % kPAStages;
         const bool has_time = (c + 1) * kTC > kt0 && !(TGL_DBG(a) & 64);
@@ -2998,7 +3006,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
       tc_fence_after();
       const int r0 = (tt > 0 && nch >= 4) ? kPreReuse : 0;
       for (int i = 0; i < nch; ++i, ++g) {
-        const int c = plan.order[chunk_of(tt, i, nch)];
+        const int c = s_order[chunk_of(tt, i, nch)];
         const int nk = (plan.k - c * kTC) > 16 ? 2 : 1;
         const uint32_t sa = g % kPAStages;
         TGL_PROF_CLK(ma0);
@@ -3058,9 +3066,11 @@ __global__ void __launch_bounds__(kPThreads, 1)
 //   FFN (kFfn = 1): seg0 = r_i (the K|V epilogue writes it split16), seg1 = h_dst.
 // Roles: epilogue warps 0-3 (one row per thread, TMEM lane quarter = warp), MMA 4,
 // descriptors 5, weights 6, loaders 7-10: 352 threads.
-constexpr int kDPAStages = 8;
+constexpr int kDPAStages = 6;
 constexpr int kDPWStage = 2 * kDPN * 64;               // hi | lo of a 32-column chunk
-constexpr int kDPW = 4;
+// 8 weight stages: tgl_node_proj applies 4 weight chunks to every A chunk, so a 4-deep
+// ring could not fetch ahead across A chunks (latency-bound: 36 us for GDELT's nodes)
+constexpr int kDPW = 8;
 constexpr int kDPLoad0 = 7, kDPLoadWarps = 4;
 constexpr int kDPThreads = (kDPLoad0 + kDPLoadWarps) * 32;   // 352
 constexpr int kDPPipeBytes = kDPAStages * kPAStage + kDPW * kDPWStage;
@@ -3119,6 +3129,7 @@ struct DPBars {
   uint64_t wfull[kDPW], wempty[kDPW];
   uint64_t dfull[kDSlots], dempty[kDSlots];
   uint64_t tfull[2], tempty[2];
+  uint64_t zfull[2];    // FFN on node projections: the accumulator holds zo[row] (loaders)
 };
 // what one grid row (blockIdx.y) of dense_pre computes: Q form (kFfn = 0) writes
 // out[i] = A_i W^T + bias (+ q.b_k per head after column D when qbk != null) with row
@@ -3132,6 +3143,7 @@ struct DPJob {
 };
 struct DPJobs {
   DPJob j[4];
+  int n;         // > 1: n jobs share each A chunk (Q form, gridDim.y == 1)
 };
 
 struct DPDesc {
@@ -3150,11 +3162,15 @@ __global__ void __launch_bounds__(kDPThreads, 1)
   __shared__ DPBars B;
   __shared__ uint32_t s_tmem;
   __shared__ DPDesc bd[kDSlots];
-  __shared__ float s_v0[kMaxModel], s_v1[kMaxModel], s_v2[kMaxModel];
+  // Q form with nj > 1 (tgl_node_proj): nj jobs share every A chunk (one accumulator
+  // of 128 columns each, single-buffered); else one job per grid row, double-buffered
+  __shared__ float s_v0[4 * kMaxModel], s_v1[4 * kMaxModel], s_v2[kMaxModel];
   constexpr uint32_t kCols = 128;
   const tgl_attn_params& P = a.P;
-  const DPJob& J = jobs.j[blockIdx.y];
-  const uint8_t* __restrict__ wpk = J.wpk;
+  const int nj = (!kFfn && jobs.n > 1) ? jobs.n : 1;
+  const bool zo = kFfn && a.zo != nullptr;   // FFN on node projections (TGL_NODE_PROJ)
+  const DPJob& J = jobs.j[nj > 1 ? 0 : blockIdx.y];
+  const uint32_t tcols = nj > 1 ? 512u : 2u * kCols;
   const bool split = a.split != 0;
   const int nch = plan.n;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -3174,18 +3190,22 @@ __global__ void __launch_bounds__(kDPThreads, 1)
     for (int s = 0; s < 2; ++s) {
       mbar_init(&B.tfull[s], 1);
       mbar_init(&B.tempty[s], kEpiWarps);
+      mbar_init(&B.zfull[s], kDPLoadWarps);
     }
     fence_mbar_init();
   }
-  if (warp == kMmaWarp) tmem_alloc(&s_tmem, 2 * kCols);
+  if (warp == kMmaWarp) tmem_alloc(&s_tmem, tcols);
   for (int j = threadIdx.x; j < P.d_model; j += blockDim.x) {
     if (kFfn) {
       s_v0[j] = P.bo[j];
       s_v1[j] = P.ln_gamma[j];
       s_v2[j] = P.ln_beta[j];
     } else {
-      s_v0[j] = J.bias ? J.bias[j] : 0.f;              // bq + Wq[:, d_hdst:] Phi(0)
-      s_v1[j] = J.qbk ? J.qbk[j] : 0.f;
+      for (int jj = 0; jj < nj; ++jj) {
+        const DPJob& Jj = jobs.j[nj > 1 ? jj : blockIdx.y];
+        s_v0[jj * kMaxModel + j] = Jj.bias ? Jj.bias[j] : 0.f;   // bq + Wq[:, d_hdst:] Phi(0)
+        s_v1[jj * kMaxModel + j] = Jj.qbk ? Jj.qbk[j] : 0.f;
+      }
     }
   }
   tc_fence_before();
@@ -3245,12 +3265,15 @@ __global__ void __launch_bounds__(kDPThreads, 1)
       warp_arrive(&B.dempty[ds]);
       if (!live) break;
       if (lane == 0) {
-        for (int i = 0; i < nch; ++i, ++k) {
-          const uint32_t sw = k % kDPW;
-          wait_free(&B.wempty[sw], k / kDPW);
-          mbar_arrive_expect_tx(&B.wfull[sw], wbytes);
-          bulk_g2s_hint(pipe + kDPAStages * kPAStage + sw * kDPWStage,
-                        wpk + (size_t)i * kDPWStage, wbytes, &B.wfull[sw], wpol);
+        for (int i = 0; i < nch; ++i) {
+          for (int jj = 0; jj < nj; ++jj, ++k) {
+            const uint32_t sw = k % kDPW;
+            wait_free(&B.wempty[sw], k / kDPW);
+            mbar_arrive_expect_tx(&B.wfull[sw], wbytes);
+            bulk_g2s_hint(pipe + kDPAStages * kPAStage + sw * kDPWStage,
+                          jobs.j[nj > 1 ? jj : blockIdx.y].wpk + (size_t)i * kDPWStage, wbytes,
+                          &B.wfull[sw], wpol);
+          }
         }
       }
       __syncwarp();
@@ -3277,8 +3300,43 @@ __global__ void __launch_bounds__(kDPThreads, 1)
         x0[k] = R.row0[r0 + 4 * k];
         x1[k] = R.row1[r0 + 4 * k];
       }
+      const int tq = warp & 3;                       // this warp's TMEM lane quarter
+      const int zn = zo ? R.row1[tq * 32 + lane] : -1;
       __syncwarp();
       warp_arrive(&B.dempty[ds]);
+      if (zo) {
+        // h_i Wo_h^T = zo[node_i] (tgl_node_proj) initialises the accumulator; the MMAs
+        // add r_i Wo_r^T.  16-column rounds, the next round's loads in flight.
+        const uint32_t tz = tmem + (tt & 1u) * kCols + ((uint32_t)(tq * 32) << 16);
+        const float* zr = a.zo + (int64_t)(zn >= 0 ? zn : 0) * a.z_ld;
+        float4 zb[2][4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          zb[0][q] = zn >= 0 ? __ldg(reinterpret_cast<const float4*>(zr + 4 * q))
+                             : make_float4(0.f, 0.f, 0.f, 0.f);
+        wait_free(&B.tempty[tt & 1u], tt >> 1);
+        tc_fence_after();
+#pragma unroll
+        for (int c0 = 0; c0 < kDPN; c0 += 16) {
+          const int cur = (c0 >> 4) & 1;
+          if (c0 + 16 < kDPN) {
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+              const int cc = c0 + 16 + 4 * q;
+              zb[cur ^ 1][q] = (zn >= 0 && cc < P.d_model)
+                                   ? __ldg(reinterpret_cast<const float4*>(zr + cc))
+                                   : make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+          }
+          const float* zv = reinterpret_cast<const float*>(&zb[cur][0]);
+          tmem_st8(tz + c0, zv);
+          if (c0 + 8 < kDPN) tmem_st8(tz + c0 + 8, zv + 8);
+        }
+        tmem_wait_st();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&B.zfull[tt & 1u]);
+      }
       for (int i = 0; i < nch; ++i, ++g) {
         const int col = i * kTC + 8 * j;
         const int ks = (plan.k - i * kTC) > 16 ? 2 : 1;
@@ -3315,54 +3373,66 @@ __global__ void __launch_bounds__(kDPThreads, 1)
       const int live = bd[ds].live;
       warp_arrive(&B.dempty[ds]);
       if (!live) break;
-      const uint32_t acc = tmem + (tt & 1u) * kCols;
-      wait_free(&B.tempty[tt & 1u], tt >> 1);
+      const uint32_t ab = nj > 1 ? 0u : (tt & 1u);
+      const uint32_t acc0 = tmem + ab * kCols;
+      if (nj > 1) wait_free(&B.tempty[0], tt);
+      else wait_free(&B.tempty[ab], tt >> 1);
+      if (zo) mbar_wait(&B.zfull[ab], (tt >> 1) & 1u);   // zo rows stored
       tc_fence_after();
-      for (int i = 0; i < nch; ++i, ++g, ++k) {
+      for (int i = 0; i < nch; ++i, ++g) {
         const int nk = (plan.k - i * kTC) > 16 ? 2 : 1;
-        const uint32_t sa = g % kDPAStages, sw = k % kDPW;
+        const uint32_t sa = g % kDPAStages;
         mbar_wait(&B.afull[sa], (g / kDPAStages) & 1u);
-        mbar_wait(&B.wfull[sw], (k / kDPW) & 1u);
-        tc_fence_after();
-        if (elect_one()) {
-          const uint64_t a0 = desc_sw64(a_s + sa * kPAStage, 1024);
-          const uint64_t w0 = desc_sw64(w_s + sw * kDPWStage, 512);
+        for (int jj = 0; jj < nj; ++jj, ++k) {
+          const uint32_t sw = k % kDPW;
+          const uint32_t acc = acc0 + (uint32_t)jj * kCols;
+          mbar_wait(&B.wfull[sw], (k / kDPW) & 1u);
+          tc_fence_after();
+          if (elect_one()) {
+            const uint64_t a0 = desc_sw64(a_s + sa * kPAStage, 1024);
+            const uint64_t w0 = desc_sw64(w_s + sw * kDPWStage, 512);
 #pragma unroll
-          for (int ks = 0; ks < 2; ++ks) {
-            if (ks < nk) {
-              const uint64_t ah = a0 + 2 * ks, bh = w0 + 2 * ks;
-              mma_bf16(acc, ah, bh, idesc, (i | ks) != 0);
-              if (split) {
-                mma_bf16(acc, ah + (512 >> 4), bh, idesc, 1u);
-                mma_bf16(acc, ah, bh + ((kDPN * 64) >> 4), idesc, 1u);
+            for (int ks = 0; ks < 2; ++ks) {
+              if (ks < nk) {
+                const uint64_t ah = a0 + 2 * ks, bh = w0 + 2 * ks;
+                mma_bf16(acc, ah, bh, idesc, zo || (i | ks) != 0);
+                if (split) {
+                  mma_bf16(acc, ah + (512 >> 4), bh, idesc, 1u);
+                  mma_bf16(acc, ah, bh + ((kDPN * 64) >> 4), idesc, 1u);
+                }
               }
             }
+            mma_commit(&B.wempty[sw]);
+            if (jj == nj - 1) mma_commit(&B.aempty[sa]);
           }
-          mma_commit(&B.aempty[sa]);
-          mma_commit(&B.wempty[sw]);
+          __syncwarp();
         }
-        __syncwarp();
       }
-      if (elect_one()) mma_commit(&B.tfull[tt & 1u]);
+      if (elect_one()) mma_commit(&B.tfull[ab]);
       __syncwarp();
     }
   } else if (warp < kEpiWarps) {                     // ---------------- epilogue
     const int row = warp * 32 + lane;
     const int D = P.d_model;
     for (;; ++tt) {
-      const uint32_t ab = tt & 1u, ds = tt % kDSlots;
+      const uint32_t ab = nj > 1 ? 0u : (tt & 1u), ds = tt % kDSlots;
       mbar_wait(&B.dfull[ds], (tt / kDSlots) & 1u);
       const int live = bd[ds].live;
       const int rows = bd[ds].rows;
       const int64_t i0 = bd[ds].i0;
       warp_arrive(&B.dempty[ds]);
       if (!live) break;
-      mbar_wait(&B.tfull[ab], (tt >> 1) & 1u);
+      mbar_wait(&B.tfull[ab], (nj > 1 ? tt : (tt >> 1)) & 1u);
       tc_fence_after();
-      const uint32_t ta = tmem + ab * kCols + ((uint32_t)(warp * 32) << 16);
       float v[32];
       if (!kFfn) {
-        float* q = J.out + (i0 + row) * J.ld;
+#pragma unroll 1
+       for (int jb = 0; jb < nj; ++jb) {
+        const DPJob& Jj = jobs.j[nj > 1 ? jb : blockIdx.y];
+        const float* sb = s_v0 + jb * kMaxModel;
+        const float* sk = s_v1 + jb * kMaxModel;
+        const uint32_t ta = tmem + (ab + (uint32_t)jb) * kCols + ((uint32_t)(warp * 32) << 16);
+        float* q = Jj.out + (i0 + row) * Jj.ld;
         const int dhq = D / P.n_heads;
         float qb0 = 0.f, qb1 = 0.f;
 #pragma unroll 1
@@ -3374,45 +3444,32 @@ __global__ void __launch_bounds__(kDPThreads, 1)
             for (int jj = 0; jj < 32; jj += 4) {
               const int col = cq * 32 + jj;
               if (col < D) {
-                float4 o = make_float4(v[jj] + s_v0[col], v[jj + 1] + s_v0[col + 1],
-                                       v[jj + 2] + s_v0[col + 2], v[jj + 3] + s_v0[col + 3]);
+                float4 o = make_float4(v[jj] + sb[col], v[jj + 1] + sb[col + 1],
+                                       v[jj + 2] + sb[col + 2], v[jj + 3] + sb[col + 3]);
                 *reinterpret_cast<float4*>(q + col) = o;
                 const float oq[4] = {o.x, o.y, o.z, o.w};
 #pragma unroll
                 for (int e = 0; e < 4; ++e) {
-                  const float pb = oq[e] * s_v1[col + e];
+                  const float pb = oq[e] * sk[col + e];
                   if (col + e < dhq) qb0 += pb; else qb1 += pb;
                 }
               }
             }
           }
         }
-        if (row < rows && J.qbk != nullptr && D + 2 <= J.ld) {
+        if (row < rows && Jj.qbk != nullptr && D + 2 <= Jj.ld) {
           q[D] = qb0;
           q[D + 1] = qb1;
         }
+       }
       } else {
-        // node projections: + h_i Wo_h^T, precomputed per node (TGL_NODE_PROJ)
-        const float* zr = nullptr;
-        if (a.zo != nullptr && row < rows)
-          zr = a.zo + (int64_t)(a.hdst_idx ? a.hdst_idx[i0 + row] : (int)(i0 + row)) * a.z_ld;
+        // (node projections: the accumulator already holds + h_i Wo_h^T, see the loaders)
+        const uint32_t ta = tmem + ab * kCols + ((uint32_t)(warp * 32) << 16);
         float s = 0.f, s2 = 0.f;
 #pragma unroll 1
         for (int cq = 0; cq < 4; ++cq) {
           tmem_ld32(ta + cq * 32, v);
           tmem_wait_ld();
-          if (zr != nullptr) {
-#pragma unroll
-            for (int jj = 0; jj < 32; jj += 4) {
-              if (cq * 32 + jj < D) {
-                const float4 z4 = __ldg(reinterpret_cast<const float4*>(zr + cq * 32 + jj));
-                v[jj] += z4.x;
-                v[jj + 1] += z4.y;
-                v[jj + 2] += z4.z;
-                v[jj + 3] += z4.w;
-              }
-            }
-          }
 #pragma unroll
           for (int jj = 0; jj < 32; ++jj) {
             const int col = cq * 32 + jj;
@@ -3431,18 +3488,6 @@ __global__ void __launch_bounds__(kDPThreads, 1)
         for (int cq = 0; cq < 4; ++cq) {
           tmem_ld32(ta + cq * 32, v);
           tmem_wait_ld();
-          if (zr != nullptr) {
-#pragma unroll
-            for (int jj = 0; jj < 32; jj += 4) {
-              if (cq * 32 + jj < D) {
-                const float4 z4 = __ldg(reinterpret_cast<const float4*>(zr + cq * 32 + jj));
-                v[jj] += z4.x;
-                v[jj + 1] += z4.y;
-                v[jj + 2] += z4.z;
-                v[jj + 3] += z4.w;
-              }
-            }
-          }
           if (row < rows) {
 #pragma unroll
             for (int jj = 0; jj < 32; jj += 4) {
@@ -3463,7 +3508,7 @@ __global__ void __launch_bounds__(kDPThreads, 1)
       warp_arrive(&B.tempty[ab]);
     }
   }
-  ws_teardown(tmem, 2 * kCols, kMmaWarp);
+  ws_teardown(tmem, tcols, kMmaWarp);
 }
 
 // ------------------------------------------------------------------ 2-SM pre-split K|V kernel
@@ -4506,9 +4551,10 @@ extern "C" tgl_status tgl_node_proj(const tgl_attn_params* P, int64_t n_nodes, c
   j.j[2] = DPJob{pk + PL.oqp, reinterpret_cast<const float*>(pk + PL.obq), P->bk,
                  Z + TGL_NODE_PROJ_Q, TGL_NODE_PROJ_LD};
   j.j[3] = DPJob{pk + PL.ono, nullptr, nullptr, Z + TGL_NODE_PROJ_O, TGL_NODE_PROJ_LD};
+  j.n = 4;                                    // the four share every gathered A chunk
   const int64_t tiles = ceil_div(n_nodes, kBM);
   const unsigned gx = (unsigned)(tiles < kNumSMs ? tiles : kNumSMs);
-  launch_pdl(dense_pre_kernel<false>, dim3(gx, 4), dim3(kDPThreads), kDPSmem, s, a, plan, j);
+  launch_pdl(dense_pre_kernel<false>, dim3(gx, 1), dim3(kDPThreads), kDPSmem, s, a, plan, j);
   return launch_check("tgl_node_proj");
 }
 

@@ -192,6 +192,22 @@ __device__ __forceinline__ void tmem_st8(uint32_t taddr, const float* v) {
       "r"(__float_as_uint(v[6])), "r"(__float_as_uint(v[7]))
       : "memory");
 }
+// no-swizzle K-major operand descriptor (core matrices of 8 rows x 16 B, rows 16 B
+// apart): SBO = byte distance between 8-row groups, LBO unused for a 16-byte-wide matrix
+__device__ __forceinline__ uint64_t desc_none(uint32_t saddr, uint32_t sbo) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr >> 4) & 0x3FFFu);
+  d |= (uint64_t)1u << 16;
+  d |= (uint64_t)((sbo >> 4) & 0x3FFFu) << 32;
+  d |= (uint64_t)1u << 46;
+  return d;
+}
+// smem (128 rows x 16 B) -> TMEM lanes 0-127, 4 fp32 columns at taddr; asynchronous,
+// executes in issue order with the same thread's tcgen05.mma (tracked by tcgen05.commit)
+__device__ __forceinline__ void tmem_cp_128x128b(uint32_t taddr, uint64_t sdesc) {
+  asm volatile("tcgen05.cp.cta_group::1.128x128b [%0], %1;" ::"r"(taddr), "l"(sdesc)
+               : "memory");
+}
 __device__ __forceinline__ void tmem_wait_st() {
   asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
 }

@@ -1,0 +1,17 @@
+# node projections via tcgen05.cp Z chunks: parity, bench on/off, sanitizer, role counters
+O=gpurun_out/np2; mkdir -p $O
+python -c "import __graft_entry__ as g; g.build()" > $O/build.log 2>&1 || { tail -30 $O/build.log; exit 1; }
+timeout 900 python -m pytest tests/test_gpu_nodeproj.py -x -q -p no:cacheprovider > $O/pytest_np.log 2>&1; echo "rc=$?" >> $O/pytest_np.log
+tail -15 $O/pytest_np.log
+for np in on off; do for c in GDELT REDDIT; do
+timeout 600 python bench.py --config $c --node-proj $np --no-cpu-baseline --no-e2e > $O/bench_${c}_$np.log 2>&1
+grep metric $O/bench_${c}_$np.log | python -c "
+import json,sys
+d=json.loads(sys.stdin.read()); r=d['roofline']; print('$c $np', round(d['value']), round(d['ms_per_step'],4), 'kv', round(r['per_launch_ms'],4), 'frac', round(r['frac'],3), {k: round(v,3) for k,v in d.get('breakdown_ms_eager').items()})" || tail -5 $O/bench_${c}_$np.log
+done; done
+timeout 600 compute-sanitizer --tool memcheck python tools/sanitize_attn.py > $O/memcheck.log 2>&1; tail -3 $O/memcheck.log
+timeout 600 compute-sanitizer --tool synccheck python tools/sanitize_attn.py > $O/synccheck.log 2>&1; tail -2 $O/synccheck.log
+TGL_NVCC_EXTRA="-DTGL_PROBE -DTGL_KV_PROF" python -c "import __graft_entry__ as g; g.build()" > $O/buildp.log 2>&1 || { tail -30 $O/buildp.log; exit 1; }
+CFG=GDELT PROBE_KV=pre PROBE_MASKS=0,2,4,64,66,70,71 PROBE_PROF=1 PROBE_PROF_KV=pre timeout 300 python tools/kv_probe.py fp32 > $O/probe.log 2>&1
+tail -9 $O/probe.log
+python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1

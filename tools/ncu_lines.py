@@ -15,8 +15,11 @@ def main():
     lo = int(sys.argv[2]) if len(sys.argv) > 3 else 0
     hi = int(sys.argv[3]) if len(sys.argv) > 3 else 10 ** 9
     top = int(sys.argv[4]) if len(sys.argv) > 4 else 60
+    import os
+    kid = os.environ.get("NCU_KERNEL_ID")        # e.g. ":::2" = the 2nd captured launch
     out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source",
-                          "cuda,sass"], capture_output=True, text=True).stdout
+                          "cuda,sass"] + (["--kernel-id", kid] if kid else []),
+                         capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(out)))
     h = rows[2]
     ci, si = h.index("Instructions Executed"), h.index("Warp Stall Sampling (All Samples)")
