@@ -58,6 +58,9 @@ def parse():
                     help="budget of the --impl reference timed steps (sizes its sample)")
     ap.add_argument("--dedup", default="config", choices=["config", "on", "off"],
                     help="override the config's dedup setting (ablation only)")
+    ap.add_argument("--precompute", default="config", choices=["config", "on", "off"],
+                    help="time-precompute table override (ablation; the window covers every "
+                         "integer dt <= max t, capped at 2^22 rows)")
     ap.add_argument("--cache", type=int, default=0,
                     help="cache() table slots per layer (0 = off, the BASELINE configs)")
     ap.add_argument("--l2-flush", default="auto", choices=["auto", "on", "off"])
@@ -367,9 +370,7 @@ def run_reference(args):
     import oracle
     import synth
     cfg = synth.get_config(args.config.upper())
-    if args.dedup != "config":
-        from dataclasses import replace
-        cfg = replace(cfg, dedup=args.dedup == "on")
+    cfg = config_overrides(cfg, args)
     flush = FLUSH_DEFAULT[cfg.name] if args.l2_flush == "auto" else args.l2_flush == "on"
     g, neg = host_graph_for_reference(cfg)
     params = synth.gen.model_params(cfg)
@@ -424,6 +425,21 @@ def run_reference(args):
 
 # ---------------------------------------------------------------------- our arm
 NODE_PROJ = {"auto": None, "on": True, "off": False}
+
+
+def config_overrides(cfg, args):
+    """--dedup / --precompute / --cache ablations on top of the config's own settings."""
+    from dataclasses import replace
+    if args.dedup != "config" or (args.cache and not cfg.dedup):
+        # cache() sits behind each block's dedup (P:578 pairs them)
+        cfg = replace(cfg, dedup=args.dedup == "on" or bool(args.cache))
+    pc = getattr(args, "precompute", "config")
+    if pc != "config":
+        w = 1
+        while w <= cfg.max_t and w < (1 << 22):
+            w <<= 1
+        cfg = replace(cfg, precompute=pc == "on", window=max(cfg.window, w))
+    return cfg
 
 
 def algorithmic_kv(cfg, n_dst: float, n_edges: float, d_hsrc: int, node_proj: bool = False):
@@ -496,9 +512,7 @@ def run_ours(args):
         cfg, g, neg, params = load_world(name)
         dev = {"src": cu(g.src), "dst": cu(g.dst), "t": cu(g.t), "neg": cu(neg),
                "nfeat": cu(g.nfeat), "efeat": cu(g.efeat)}
-    if args.dedup != "config" or (args.cache and not cfg.dedup):
-        from dataclasses import replace              # cache() sits behind each block's dedup
-        cfg = replace(cfg, dedup=args.dedup == "on" or bool(args.cache))   # (P:578 pairs them)
+    cfg = config_overrides(cfg, args)
     flush = FLUSH_DEFAULT[cfg.name] if args.l2_flush == "auto" else args.l2_flush == "on"
     want_cpu = rank == 0 and world == 1 and not args.no_cpu_baseline
 

@@ -507,3 +507,31 @@ def test_host_stream_matches_graph(T):
     for b, e in zip(batches, got):
         exp = np_(ref.run_graph(b * cfg.batch))[:n0]
         assert np.array_equal(e, exp), b
+
+
+@pytest.mark.parametrize("d_h,d_e", [(172, 172), (413, 186)])
+def test_fused_phi_matches_exact_table(T, d_h, d_e):
+    """The K|V kernels evaluate Phi in the SM (reduced argument + SFU cosine, abs error
+    < 2e-6, DESIGN R10 / tenc.cuh); the precompute table holds the exact R10 values
+    (bit-identical to tgl_time_encode).  With every dt an integer inside the window, the
+    same call with and without the table differs only by the fused Phi's error: pinned
+    here at 3e-5 on the outputs -- 30x tighter than the 1e-3 parity bound, so a Phi bug
+    that stays under that bound still fails here."""
+    rng = np.random.default_rng(d_h + d_e)
+    p, seg, dst_t, nfeat, dn, sn, ef, eid, et = attn_case(rng, 1500, 10, d_h, d_e)
+    P = T.AttnParams(p, precision="fp32", pack=True, kv_kernel="pre")
+    dt = np.repeat(dst_t, np.diff(seg)) - et
+    assert (dt == np.round(dt)).all() and dt.min() >= 0 and dt.max() < (1 << 18)
+    tab = T.split_rows(T.time_precompute(1 << 18, P.t["omega"], P.t["phi"]))
+    nf = cu(nfeat)
+    hs, efd = T.split_rows(nf), T.split_rows(cu(ef))
+    base = T.SPLIT_HSRC | T.SPLIT_E
+    outs = []
+    for table, layout in ((None, base), (tab, base | T.SPLIT_TABLE)):
+        P.struct.input_layout = layout
+        got = T.tblock_attn(P, cu(seg), cu(dst_t), nf, cu(dn), hs, cu(sn), efd, cu(eid),
+                            cu(et), table=table, max_seg=10)
+        outs.append(np_(got)[:1500].copy())
+    exp = oracle.tblock_attn(p, seg, dst_t, nfeat, dn, nfeat, sn, ef, eid, et)
+    assert np.abs(outs[1] - exp).max() <= 1e-3
+    assert np.abs(outs[0] - outs[1]).max() <= 3e-5, np.abs(outs[0] - outs[1]).max()
