@@ -179,6 +179,12 @@ class TGATPipeline:
             at = self.attn[-1]
             at.struct.input_layout |= tgl.NODE_PROJ
             at.struct.node_proj = tgl._p(self.zproj)
+            # Z depends on the weights and the node table only: it is computed on a side
+            # stream that forks at the start of a forward and joins before the tail block,
+            # so it overlaps the latency-bound roots / dedup / sampling launches
+            self.np_stream = torch.cuda.Stream(device=self.dev)
+            self.np_fork = torch.cuda.Event()
+            self.np_join = torch.cuda.Event()
         if self.host:            # device staging tables for the preloaded rows, per block
             cap = max(b.n_max * k for b in self.blocks)
             self.iota = torch.arange(max(cap, 1), dtype=i32, device=self.dev)
@@ -281,9 +287,20 @@ class TGATPipeline:
         mark("roots")
         return self._chain(s, record, mark)
 
+    def _node_proj_fork(self, s):
+        """Enqueue tgl_node_proj on the side stream, ordered after the work already on s."""
+        cur = s if s is not None else torch.cuda.current_stream()
+        self.np_fork.record(cur)
+        self.np_stream.wait_event(self.np_fork)
+        tgl.node_proj(self.attn[-1], self.nfeat_split, n_nodes=self.zproj.shape[0],
+                      out=self.zproj, stream=self.np_stream)
+        self.np_join.record(self.np_stream)
+
     def _chain(self, s, record, mark):
         """S3-S15 from block 0's dst pairs to the head output (b0.out / the roots)."""
         g, k = self.g, self.sampler.k
+        if self.node_proj and record is None:
+            self._node_proj_fork(s)
         b0 = self.blocks[0]
         for l, b in enumerate(self.blocks):
             if l > 0:  # S5 next_block (R14): [dst after dedup ; sampled src]
@@ -324,9 +341,13 @@ class TGATPipeline:
                 if self.split:
                     hdst = hsrc = self.nfeat_split
                 if self.node_proj:   # Z rows for every node, then the tail indexes them
-                    tgl.node_proj(a, self.nfeat_split, n_nodes=self.zproj.shape[0],
-                                  out=self.zproj, stream=s)
-                    mark("node_proj")
+                    if record is None:           # join the side stream (forked above)
+                        (s if s is not None else torch.cuda.current_stream()).wait_event(
+                            self.np_join)
+                    else:                        # eager timing: in line, its own mark
+                        tgl.node_proj(a, self.nfeat_split, n_nodes=self.zproj.shape[0],
+                                      out=self.zproj, stream=s)
+                        mark("node_proj")
             else:
                 nx = self.blocks[l + 1]
                 hdst = hsrc = nx.ws["cache"]["comb"] if self.cache_on else nx.out
