@@ -331,8 +331,14 @@ template <bool kFirst, bool kLast>
 __global__ void __launch_bounds__(kSwThreads, 2)
 sw_scatter_kernel(SwArgs a, int p, const uint4* __restrict__ in, SwOut o,
                   uint32_t* __restrict__ status, unsigned int* ticket) {
+  // the tile's records are staged in shared memory in (digit, rank) order, then written
+  // out by consecutive threads: each digit's run of the tile lands as one contiguous,
+  // coalesced stretch (instead of 16-byte / 4-byte stores scattered over 256 buckets)
+  extern __shared__ uint4 s_rec[];              // [kSwTile]
   __shared__ uint32_t s_wrun[kSwWarps][256];
   __shared__ uint32_t s_base[256];
+  __shared__ uint32_t s_loff[256];              // tile-local start of each digit's run
+  __shared__ uint32_t s_wsum[kSwWarps];
   __shared__ int64_t s_tile;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
 #pragma unroll
@@ -379,6 +385,19 @@ sw_scatter_kernel(SwArgs a, int p, const uint4* __restrict__ in, SwOut o,
       s_wrun[w][d] = tot;
       tot += x;
     }
+    {   // exclusive scan of the tile's digit totals (one digit per thread)
+      uint32_t v = tot;
+#pragma unroll
+      for (int o2 = 1; o2 < 32; o2 <<= 1) {
+        const uint32_t n = __shfl_up_sync(0xffffffffu, v, o2);
+        if (lane >= o2) v += n;
+      }
+      if (lane == 31) s_wsum[warp] = v;
+      __syncthreads();
+      uint32_t wo = 0;
+      for (int w = 0; w < warp; ++w) wo += s_wsum[w];
+      s_loff[d] = wo + v - tot;
+    }
     uint32_t* st = status + tile * 256 + d;
     uint32_t excl = 0;
     if (tile == 0) {
@@ -424,16 +443,24 @@ sw_scatter_kernel(SwArgs a, int p, const uint4* __restrict__ in, SwOut o,
     const int64_t i = wbase + r * 32 + lane;
     if (i >= a.M) continue;
     const uint32_t d = sw_digit(rec[r], field, shift);
-    const int64_t pos = (int64_t)s_base[d] + s_wrun[warp][d] + rank[r];
+    s_rec[s_loff[d] + s_wrun[warp][d] + rank[r]] = rec[r];
+  }
+  __syncthreads();
+  const int64_t t0 = tile * kSwTile;
+  const int nv = (int)((a.M - t0) < kSwTile ? (a.M - t0) : kSwTile);
+  for (int x = threadIdx.x; x < nv; x += kSwThreads) {
+    const uint4 rr = s_rec[x];
+    const uint32_t d = sw_digit(rr, field, shift);
+    const int64_t pos = (int64_t)s_base[d] + (uint32_t)(x - (int)s_loff[d]);
     if (!kLast) {
-      o.rec[pos] = rec[r];
+      o.rec[pos] = rr;
     } else {
-      o.nbr[pos] = (int32_t)rec[r].y;
-      o.eid[pos] = (int32_t)rec[r].z;
-      o.ts[pos] = __uint_as_float(rec[r].w);
-      if (o.keys) o.keys[pos] = rec[r].x;
-      if (o.coarse && (pos & 31) == 0) o.coarse[pos >> 5] = __uint_as_float(rec[r].w);
-      if (o.entries) o.entries[pos] = make_int4((int)rec[r].y, (int)rec[r].z, (int)rec[r].w, 0);
+      o.nbr[pos] = (int32_t)rr.y;
+      o.eid[pos] = (int32_t)rr.z;
+      o.ts[pos] = __uint_as_float(rr.w);
+      if (o.keys) o.keys[pos] = rr.x;
+      if (o.coarse && (pos & 31) == 0) o.coarse[pos >> 5] = __uint_as_float(rr.w);
+      if (o.entries) o.entries[pos] = make_int4((int)rr.y, (int)rr.z, (int)rr.w, 0);
     }
   }
 }
@@ -497,6 +524,25 @@ static tgl_status build_onesweep(int64_t num_nodes, int64_t num_edges, const int
                                                      (int)(kSwDegSmemNodes * 4));
                        }), "sw_hist smem attr"));
   }
+  {
+    static PerDeviceOnce once2;
+    TGL_TRY(cuda_check(once2.run([] {
+                         const int b = (int)(sizeof(uint4) * kSwTile);
+                         cudaError_t e = cudaFuncSetAttribute(
+                             sw_scatter_kernel<true, true>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+                         if (e == cudaSuccess)
+                           e = cudaFuncSetAttribute(sw_scatter_kernel<true, false>,
+                                                    cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+                         if (e == cudaSuccess)
+                           e = cudaFuncSetAttribute(sw_scatter_kernel<false, true>,
+                                                    cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+                         if (e == cudaSuccess)
+                           e = cudaFuncSetAttribute(sw_scatter_kernel<false, false>,
+                                                    cudaFuncAttributeMaxDynamicSharedMemorySize, b);
+                         return e;
+                       }), "sw_scatter smem attr"));
+  }
   const int hist_ctas = dsmem <= 100 * 1024 ? 2 * kNumSMs : kNumSMs;
   sw_hist_kernel<<<hist_ctas, 1024, dsmem, s>>>(a, num_edges);
   TGL_TRY(launch_check("tcsr sw_hist"));
@@ -519,14 +565,15 @@ static tgl_status build_onesweep(int64_t num_nodes, int64_t num_edges, const int
     uint32_t* status = reinterpret_cast<uint32_t*>(w + o_status) + (size_t)p * 256 * tiles;
     unsigned int* ticket = reinterpret_cast<unsigned int*>(w + o_ticket) + p;
     const dim3 grid((unsigned)tiles);
+    const size_t rsm = sizeof(uint4) * kSwTile;    // the staged tile (64 KB)
     if (first && last)
-      sw_scatter_kernel<true, true><<<grid, kSwThreads, 0, s>>>(a, p, in, o, status, ticket);
+      sw_scatter_kernel<true, true><<<grid, kSwThreads, rsm, s>>>(a, p, in, o, status, ticket);
     else if (first)
-      sw_scatter_kernel<true, false><<<grid, kSwThreads, 0, s>>>(a, p, in, o, status, ticket);
+      sw_scatter_kernel<true, false><<<grid, kSwThreads, rsm, s>>>(a, p, in, o, status, ticket);
     else if (last)
-      sw_scatter_kernel<false, true><<<grid, kSwThreads, 0, s>>>(a, p, in, o, status, ticket);
+      sw_scatter_kernel<false, true><<<grid, kSwThreads, rsm, s>>>(a, p, in, o, status, ticket);
     else
-      sw_scatter_kernel<false, false><<<grid, kSwThreads, 0, s>>>(a, p, in, o, status, ticket);
+      sw_scatter_kernel<false, false><<<grid, kSwThreads, rsm, s>>>(a, p, in, o, status, ticket);
     TGL_TRY(launch_check("tcsr sw_scatter"));
   }
   if (!deg) {
