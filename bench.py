@@ -516,6 +516,26 @@ def run_ours(args):
     flush = FLUSH_DEFAULT[cfg.name] if args.l2_flush == "auto" else args.l2_flush == "on"
     want_cpu = rank == 0 and world == 1 and not args.no_cpu_baseline
 
+    # S1 T-CSR: one warm-up build (module load, first-touch, the allocator's blocks), then
+    # the best of two timed builds into the same (cached) blocks; the host is otherwise idle
+    # (the oracle's thread starts after), so the events see the GPU build only.
+    # Sampler indexes (tgl_tcsr_index): the fence index everywhere, the packed 16-byte
+    # entries (16 B per CSR entry) where memory allows -- not MAG (2.6B entries)
+    packed = cfg.name != "MAG"
+    tc = tgl.build_tcsr(cfg.n_nodes, dev["src"], dev["dst"], dev["t"], True, True, packed=packed)
+    torch.cuda.synchronize()
+    tcsr_runs = []
+    for _ in range(2):
+        del tc
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ev0.record()
+        tc = tgl.build_tcsr(cfg.n_nodes, dev["src"], dev["dst"], dev["t"], True, True,
+                            packed=packed)
+        ev1.record()
+        torch.cuda.synchronize()
+        tcsr_runs.append(ev0.elapsed_time(ev1))
+    tcsr_ms = min(tcsr_runs)
+
     # the whole-graph oracle's T-CSR (a C qsort of 2E entries: ~2 min on GDELT) builds on a
     # host thread while the GPU is measured (ctypes releases the GIL)
     oracle_box = {}
@@ -524,20 +544,6 @@ def run_ours(args):
             oracle_box["runner"] = OracleRunner(cfg, g, params)
         oth = threading.Thread(target=_build, daemon=True)
         oth.start()
-
-    # S1 T-CSR: one warm-up build (module load, first-touch), then the timed build
-    # sampler indexes (tgl_tcsr_index): the fence index everywhere, the packed 16-byte
-    # entries (16 B per CSR entry) where memory allows -- not MAG (2.6B entries)
-    packed = cfg.name != "MAG"
-    tgl.build_tcsr(cfg.n_nodes, dev["src"], dev["dst"], dev["t"], True, True, packed=packed)
-    torch.cuda.synchronize()
-    torch.cuda.empty_cache()
-    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    ev0.record()
-    tc = tgl.build_tcsr(cfg.n_nodes, dev["src"], dev["dst"], dev["t"], True, True, packed=packed)
-    ev1.record()
-    torch.cuda.synchronize()
-    tcsr_ms = ev0.elapsed_time(ev1)
     M = 2 * cfg.n_edges
     tcsr_bytes = cfg.n_edges * 12 + M * 12 + (cfg.n_nodes + 1) * 8   # SURVEY §8(d) per edge
 
@@ -742,8 +748,9 @@ def run_ours(args):
                 "tcsr": {"build_ms": tcsr_ms, "entries": M,
                          "algorithmic_bytes": tcsr_bytes,
                          "hbm_frac": tcsr_bytes / (tcsr_ms / 1e3) / 1e9 / hbm_peak,
-                         "timing": "second build (the first warms module load / first touch); "
-                                   "includes the sampler indexes (tgl_tcsr_index)"},
+                         "timing": "best of two builds after a warm-up (module load, first "
+                                   "touch, allocator blocks), host idle; includes the sampler "
+                                   "indexes"},
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
                 "gpu_launches": pipe.launches_per_forward * args.steps,
                 "gpu_launches_per_step": pipe.launches_per_forward,

@@ -211,6 +211,14 @@ struct Pipe {
   }
 };
 
+// code-size knob (experiment): -DTGL_SMALL_CODE keeps the epilogue's transpose passes and
+// the time warps' group loop rolled (the K|V kernel's body exceeds the instruction cache)
+#ifdef TGL_SMALL_CODE
+#define TGL_SMALL_UNROLL _Pragma("unroll 1")
+#else
+#define TGL_SMALL_UNROLL _Pragma("unroll")
+#endif
+
 // ---- profiling instrumentation: compiled only into probe builds (-DTGL_PROBE, tools/);
 // product builds have no debug state, read no environment and take no debug branches
 #ifdef TGL_PROBE
@@ -1142,7 +1150,7 @@ __device__ __forceinline__ void bin_epilogue(const Args& a, uint64_t* dfull, uin
     for (int cq = 0; cq < 2; ++cq) {
       tmem_ld32(ta + dm + cb + cq * 32, v);
       tmem_wait_ld();
-#pragma unroll
+TGL_SMALL_UNROLL
       for (int hh = 0; hh < 32 / kCW; ++hh) {
 #pragma unroll
         for (int j = 0; j < kCW; ++j) pvw[lane * kPW + j] = w * v[hh * kCW + j];
@@ -2927,7 +2935,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
           wait_free(&B.aempty[sa], g / kPAStages);
           TGL_PROF_CLK(t1);
           const uint32_t dst = a_s + sa * kPAStage + rofs;
-#pragma unroll
+TGL_SMALL_UNROLL
           for (int jj = 0; jj < 4; ++jj) {
             const int col = c * kTC + 8 * jj;
             if (col < kt0 || col >= c * kTC + 16 * ks) continue;     // warp-uniform
