@@ -40,7 +40,7 @@ BIG = ("GDELT", "MAG")            # generated on the device (synth.gpu)
 FLUSH_DEFAULT = {"WIKI": True, "REDDIT": True, "LASTFM": True, "GDELT": False, "MAG": False}
 # operand layout of the K|V gathers: split16 tables (kv_pre) everywhere but MAG, whose 62 GB
 # node table cannot be held twice next to its 32 GB T-CSR (fp32 rows, converted in the SM)
-LAYOUT = {"MAG": "fp32"}
+LAYOUT = {}      # every config on split16 operand tables (kv_pre); MAG keeps only those
 
 
 def parse():
@@ -169,18 +169,25 @@ def load_world_device(cfg_name: str):
     src, dst, t = sg.device_graph(cfg, d)
     neg = sg.device_negatives(cfg, d)
     from paper_conf_asplos_wangm24_b200 import tgl
-    # node features: fp32 rows with a 16-byte pitch (h_dst of the Q / FFN kernels) and the
-    # split16 operand table the K|V kernel gathers; edge features: split16 only, built
-    # chunk by chunk from the same counter-based values (the fp32 table never exists)
-    nfeat = sg.device_feature_table(cfg.seeds["feat"], cfg.n_nodes, cfg.d_v, d, pitch_mult=4)
-    dev = {"src": src, "dst": dst, "t": t, "neg": neg, "nfeat": nfeat, "efeat": None}
-    if LAYOUT.get(cfg.name, "split") == "split":
-        dev["nfeat_split"] = tgl.split_rows(nfeat)
+    # node features: the split16 operand table the kernels gather (K|V, Q, FFN), plus fp32
+    # rows with a 16-byte pitch where they fit beside it (GDELT: 28 MB); MAG's 62 GB node
+    # table exists only split16, built chunk by chunk (a second copy would not fit next to
+    # its 32 GB T-CSR); edge features: split16 only, the same way (the fp32 table never
+    # exists)
+    rows_fn = lambda seed, dim: (lambda r0, r1: sg.feature_rows_torch(
+        seed, torch.arange(r0, r1, device=d), dim))
+    if cfg.name == "MAG":
+        nfeat = None
+        nsplit = tgl.split_table(cfg.n_nodes, cfg.d_v, rows_fn(cfg.seeds["feat"], cfg.d_v))
+    else:
+        nfeat = sg.device_feature_table(cfg.seeds["feat"], cfg.n_nodes, cfg.d_v, d,
+                                        pitch_mult=4)
+        nsplit = tgl.split_rows(nfeat)
+    dev = {"src": src, "dst": dst, "t": t, "neg": neg, "nfeat": nfeat, "efeat": None,
+           "nfeat_split": nsplit}
     if cfg.d_e:
-        dev["efeat_split"] = tgl.split_table(
-            cfg.n_edges, cfg.d_e,
-            lambda r0, r1: sg.feature_rows_torch(cfg.seeds["feat"] + 7919,
-                                                 torch.arange(r0, r1, device=d), cfg.d_e))
+        dev["efeat_split"] = tgl.split_table(cfg.n_edges, cfg.d_e,
+                                             rows_fn(cfg.seeds["feat"] + 7919, cfg.d_e))
     torch.cuda.synchronize()
     g = HostGraph(cfg, src.cpu().numpy(), dst.cpu().numpy(), t.cpu().numpy())
     neg_h = neg.cpu().numpy()

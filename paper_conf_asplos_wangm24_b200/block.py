@@ -159,7 +159,8 @@ class TGATPipeline:
             n_max = n_max + n_max * k
         self.emb = z(3 * batch * self.attn[0].d_out, f32).view(-1, self.attn[0].d_out)
         # node projections for the tail block (its h_src / h_dst are node-feature rows)
-        n_nodes = graph["nfeat"].shape[0] if graph.get("nfeat") is not None else 0
+        nft = graph.get("nfeat") if graph.get("nfeat") is not None else graph.get("nfeat_split")
+        n_nodes = nft.shape[0] if nft is not None else 0
         tail = self.blocks[-1]
         np_ok = (self.split and precision in ("fp32", "bf16") and not host_features and
                  n_nodes > 0 and self.attn[-1].host["n_heads"] == 2)

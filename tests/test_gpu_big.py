@@ -95,25 +95,30 @@ def _run(name, host_gb, dev_gb):
     segs = _check_tcsr(cfg, src, dst, t, tc, src_h, dst_h, t_h, rng)
     torch.cuda.empty_cache()
 
-    # the bench's layout (bench.load_world_device): fp32 node rows with a 16-byte pitch
-    # for h_dst, split16 operand tables for the K|V gathers (edge features built chunk by
-    # chunk: the fp32 table never exists), so the kernel the bench times runs here
-    split = name != "MAG"     # MAG: fp32 rows (no room for a second 62 GB node table)
-    nfeat = sg.device_feature_table(cfg.seeds["feat"], cfg.n_nodes, cfg.d_v, dev, pitch_mult=4)
+    # the bench's layout (bench.load_world_device): split16 operand tables for every gather
+    # (edge features, and MAG's node table, built chunk by chunk: those fp32 tables never
+    # exist), fp32 node rows beside them where they fit (GDELT), so the kernels the bench
+    # times run here
+    rows_fn = lambda seed, dim: (lambda r0, r1: sg.feature_rows_torch(
+        seed, torch.arange(r0, r1, device=dev), dim))
+    if name == "MAG":
+        nfeat = None
+        nsplit = tgl.split_table(cfg.n_nodes, cfg.d_v, rows_fn(cfg.seeds["feat"], cfg.d_v))
+    else:
+        nfeat = sg.device_feature_table(cfg.seeds["feat"], cfg.n_nodes, cfg.d_v, dev,
+                                        pitch_mult=4)
+        nsplit = tgl.split_rows(nfeat)
     efeat = None
-    efeat_split = (tgl.split_table(cfg.n_edges, cfg.d_e,
-                                   lambda r0, r1: sg.feature_rows_torch(
-                                       cfg.seeds["feat"] + 7919, torch.arange(r0, r1, device=dev),
-                                       cfg.d_e))
+    efeat_split = (tgl.split_table(cfg.n_edges, cfg.d_e, rows_fn(cfg.seeds["feat"] + 7919, cfg.d_e))
                    if cfg.d_e else None)
     rows = rng.integers(0, cfg.n_nodes, 5)
-    assert np.array_equal(nfeat[torch.from_numpy(rows).to(dev)].cpu().numpy(),
-                          synth.feature_rows(cfg.seeds["feat"], rows, cfg.d_v))
+    want_rows = torch.from_numpy(synth.feature_rows(cfg.seeds["feat"], rows, cfg.d_v)).to(dev)
+    got_rows = nsplit[torch.from_numpy(rows).to(dev)].contiguous().view(torch.int32)
+    assert torch.equal(got_rows, tgl.split_rows(want_rows).contiguous().view(torch.int32))
     params = synth.gen.model_params(cfg)
     graph = {"src": src, "dst": dst, "t": t, "neg": neg, "nfeat": nfeat, "efeat": efeat,
-             "nfeat_split": tgl.split_rows(nfeat) if split else None,
-             "efeat_split": efeat_split}
-    layout = "split" if split else "fp32"
+             "nfeat_split": nsplit, "efeat_split": efeat_split}
+    layout = "split"
     pipe = TGATPipeline(graph, tc, params, cfg.batch,
                         TSampler(cfg.k, cfg.strategy, cfg.seeds["sampler"]), cfg.dedup,
                         cfg.precompute, cfg.window, "fp32", layout=layout)
@@ -130,7 +135,7 @@ def _run(name, host_gb, dev_gb):
     pipe.forward()
     torch.cuda.synchronize()
     pipe.attn[tail].attach_probe(None)
-    want = "pre" if split else ("split" if cfg.d_v % 4 == 0 else "split_pad")
+    want = "pre"
     assert probe.kernel == tgl.KV_KERNEL[want], (probe.kernel, want)
 
     class _G:   # host view for batch slicing
@@ -172,7 +177,7 @@ def _run(name, host_gb, dev_gb):
         torch.cuda.synchronize()
         err16 = np.abs(e16.cpu().numpy()[pick] - exp).max()
         assert err16 <= 5e-2, err16
-    del pipe, pipe16, graph, nfeat, efeat, efeat_split, tc, src, dst, t, neg
+    del pipe, pipe16, graph, nfeat, nsplit, efeat, efeat_split, tc, src, dst, t, neg
     torch.cuda.empty_cache()
 
 
