@@ -114,3 +114,39 @@ def test_shard_validation_errors():
     # c_max smaller than ceil(u_max / world)
     st = lib.tgl_shard_gather(10, None, None, 10, None, 4, None, 2, 100, None, 100, None)
     assert st == -1 and b"c_max" in lib.tgl_last_error()
+
+
+def test_node_proj_validation_errors():
+    """tgl_node_proj rejects shapes / arguments before any launch (no GPU needed)."""
+    lib = tgl.lib()
+    # d_model != 100 -> EUNSUPPORTED
+    p = tgl.AttnParamsC(172, 172, 172, 100, 64, 2, 64)
+    st = lib.tgl_node_proj(C.byref(p), 10, None, 176, C.c_void_p(256), None)
+    assert st == -5
+    # d_hsrc != d_hdst (the tail block indexes one node table) -> EUNSUPPORTED
+    p = tgl.AttnParamsC(172, 128, 172, 100, 100, 2, 100)
+    st = lib.tgl_node_proj(C.byref(p), 10, None, 176, C.c_void_p(256), None)
+    assert st == -5
+    # no packed weights -> EINVAL
+    p = tgl.AttnParamsC(172, 172, 172, 100, 100, 2, 100)
+    st = lib.tgl_node_proj(C.byref(p), 10, None, 176, C.c_void_p(256), None)
+    assert st == -1 and b"packed" in lib.tgl_last_error()
+    # null Z -> EINVAL
+    st = lib.tgl_node_proj(C.byref(p), 10, None, 176, None, None)
+    assert st == -1
+
+
+def test_bench_node_proj_accounting():
+    """bench.algorithmic_kv: the node-projection plan counts what its kernel reads per edge
+    (a Z row of 2 d_model floats + the e row + 12 B) and the MMAs over [e ; Phi] only."""
+    import bench
+    import synth
+    cfg = synth.get_config("GDELT")
+    f0, b0 = bench.algorithmic_kv(cfg, 132000, 1.32e6, cfg.d_v)
+    f1, b1 = bench.algorithmic_kv(cfg, 132000, 1.32e6, cfg.d_v, node_proj=True)
+    dm = cfg.d_model
+    per_dst = 12 + 4 * (dm + 2) + 4 * dm
+    assert b0 == 1.32e6 * (4 * (cfg.d_v + cfg.d_e) + 12) + 132000 * per_dst
+    assert b1 == 1.32e6 * (4 * (2 * dm + cfg.d_e) + 12) + 132000 * per_dst
+    assert f1 == 1.32e6 * (4 * dm * (cfg.d_e + cfg.d_t) + 6 * dm)
+    assert f1 < f0 and b1 < b0
