@@ -2974,23 +2974,31 @@ TGL_SMALL_UNROLL
             st_shared_v4(dst + po, h[0], h[1], h[2], h[3]);
             if (split) st_shared_v4(dst + 512 + po, l[0], l[1], l[2], l[3]);
           }
+          TGL_PROF_CLK(t2);
           fence_proxy_async_smem();
+          TGL_PROF_CLK(t3);
           __syncwarp();
 #ifdef TGL_KV_PROF
           if (tw == 0) {
             prof_add(a, 0, t1 - t0);                   // time warp: wait for a free stage
             prof_add(a, 1, clock64() - t1);            // time warp: Phi + split + store
+            prof_add(a, 2, t2 - t1);                   //   of which Phi + split + st.shared
+            prof_add(a, 3, t3 - t2);                   //   of which fence.proxy.async
           }
 #endif
           if (lane == 0) mbar_arrive(&B.afull[sa]);
         } else {
           // no time columns: arrive once the stage's previous use is released, so the
           // arrival counts toward this chunk's phase
+          TGL_PROF_CLK(n0);
           if (lane == 0) {
             wait_free(&B.aempty[sa], g / kPAStages);
             mbar_arrive(&B.afull[sa]);
           }
           __syncwarp();
+#ifdef TGL_KV_PROF
+          if (tw == 0) prof_add(a, 4, clock64() - n0);  // time warp: non-time chunk pass
+#endif
         }
       }
     }

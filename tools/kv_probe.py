@@ -51,6 +51,7 @@ if os.environ.get("PROBE_WINDOW"):          # 0 = direct evaluation, else a smal
 
 
 hs = pipe.nfeat_split if pipe.split else nf          # operand tables of the pipeline layout
+hd = hs if pipe.split else nf                         # (split layouts: h_dst split16 too)
 if pipe.split:
     ef = pipe.efeat_split
 
@@ -58,7 +59,7 @@ if pipe.split:
 def call():
     _call_ws(lib.tgl_tblock_attn,
              [tgl.C.byref(a.struct), b.n_max, tgl._p(b.u_dev), tgl._p(b.seg_ptr), tgl._p(b.uniq_t),
-              tgl._prow(nf), tgl._p(b.uniq_node), nf.stride(0), tgl._prow(hs), tgl._p(b.nbr), None,
+              tgl._prow(hd), tgl._p(b.uniq_node), hd.stride(0), tgl._prow(hs), tgl._p(b.nbr), None,
               hs.stride(0), tgl._prow(ef), tgl._p(b.eid), ef.stride(0), tgl._p(b.ts),
               tgl._p(tab), 0 if tab is None else tab.shape[0], cfg.k, tgl._p(b.out)],
              b.ws["attn"], None, "tail attn")
@@ -111,7 +112,8 @@ if os.environ.get("PROBE_PROF"):
         names = (["L:aempty-wait", "T:aempty-wait", "T:work", "W:wempty-wait", "R:afull-wait",
                   "R:wfull-wait", "M:tempty-wait", "M:afull-wait", "M:pfull-wait", "M:wfull-wait",
                   "D:slot-wait", "E:acc-wait", "E:work", "total"] if kv == "pre2" else
-                 ["T:aempty-wait", "T:phi+split+st", "2", "3", "4", "L:aempty-wait", "6",
+                 ["T:aempty-wait", "T:phi+split+st", "T:compute+sts", "T:fence", "T:nontime-pass",
+                  "L:aempty-wait", "6",
                   "M:tempty-wait", "M:afull-wait(gathered)", "M:afull-wait(time)",
                   "M:wfull-wait", "E:acc-wait", "E:work"] if kv == "pre" else
                  ["C:ffull-wait", "C:lds+phi", "C:bempty-wait", "C:cvt+sts", "C:fence",
