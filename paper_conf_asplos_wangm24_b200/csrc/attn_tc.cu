@@ -2629,7 +2629,8 @@ __global__ void __launch_bounds__(kPThreads, 1)
   __shared__ PBars B;
   __shared__ uint32_t s_tmem;
   __shared__ TDesc bd[kSDSlots];
-  __shared__ float s_omega[256], s_phi[256];
+  __shared__ __align__(16) float s_omega[256];
+  __shared__ __align__(16) float s_phi[256];
   __shared__ unsigned char s_order[64];      // plan.order (indexed: smem, not a local copy)
   __shared__ float s_bias[2 * kMaxModel];
   __shared__ int64_t s_seg[kTDescWarps][4 * 32 + 1];
@@ -2943,10 +2944,20 @@ TGL_SMALL_UNROLL
             if (tsplit && mode == 1 && col < plan.k) continue;   // gathered from the table
             float x[8];
             if (mode == 0) {
+              // omega / phi of the group as four 16-byte loads (tc is a multiple of 8): the
+              // shared-memory pipe is busy with the tensor core's operand reads, so each
+              // scalar load waited its turn (the group's 16 of them, not the cosine, were
+              // the time warps' cost)
+              float om[8], ph[8];
+              *reinterpret_cast<float4*>(om) = *reinterpret_cast<const float4*>(s_omega + tc);
+              *reinterpret_cast<float4*>(om + 4) =
+                  *reinterpret_cast<const float4*>(s_omega + tc + 4);
+              *reinterpret_cast<float4*>(ph) = *reinterpret_cast<const float4*>(s_phi + tc);
+              *reinterpret_cast<float4*>(ph + 4) = *reinterpret_cast<const float4*>(s_phi + tc + 4);
               bool bad = false;
 #pragma unroll
               for (int e = 0; e < 8; ++e) {
-                const float bb = __fadd_rn(__fmul_rn(s_omega[tc + e], dtr), s_phi[tc + e]);
+                const float bb = __fadd_rn(__fmul_rn(om[e], dtr), ph[e]);
                 bad |= !(fabsf(bb) < 1e9f);
                 x[e] = tenc_cos_reduced(bb);
               }
