@@ -2982,8 +2982,8 @@ TGL_SMALL_UNROLL
 #pragma unroll
             for (int e = 0; e < 4; ++e) split2(x[2 * e], x[2 * e + 1], h[e], l[e]);
             const uint32_t po = (uint32_t)(((jj ^ (rr >> 1)) & 3) << 4);
-            st_shared_v4(dst + po, h[0], h[1], h[2], h[3]);
-            if (split) st_shared_v4(dst + 512 + po, l[0], l[1], l[2], l[3]);
+            st_shared_v4_nc(dst + po, h[0], h[1], h[2], h[3]);
+            if (split) st_shared_v4_nc(dst + 512 + po, l[0], l[1], l[2], l[3]);
           }
           TGL_PROF_CLK(t2);
           fence_proxy_async_smem();

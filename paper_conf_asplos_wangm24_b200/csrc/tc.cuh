@@ -236,6 +236,14 @@ __device__ __forceinline__ uint32_t sw128_off(int r, int j) {
   return (uint32_t)((r >> 3) * 1024 + (r & 7) * 128 + ((j ^ (r & 7)) << 4));
 }
 
+// the same store without a compiler memory clobber: for stage writes that only the async
+// proxy reads (behind a volatile fence.proxy.async + mbarrier arrive, which stay ordered),
+// so the compiler may hoist the next group's loads above it
+__device__ __forceinline__ void st_shared_v4_nc(uint32_t addr, uint32_t a, uint32_t b,
+                                                uint32_t c, uint32_t d) {
+  asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(a), "r"(b), "r"(c),
+               "r"(d));
+}
 __device__ __forceinline__ void st_shared_v4(uint32_t addr, uint32_t a, uint32_t b, uint32_t c,
                                              uint32_t d) {
   asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(a), "r"(b), "r"(c),
