@@ -2520,11 +2520,14 @@ __global__ void __launch_bounds__(kSThreads, 1)
 // In bf16 mode only the hi halves are loaded (half the gather bytes).
 // Roles: epilogue warps 0-7 (bin_epilogue), MMA 8, weights 9, tile descriptors 10-11,
 // loaders 12-15, time warps 16-19: 640 threads.
+// 4 A stages, 5 weight stages, 4 weight chunks kept across a tile boundary (measured on
+// GDELT with node projections: K|V 0.823 -> 0.789 ms against 7 / 3 / 2 -- fewer weight
+// refills beat a deeper A ring; the shared-memory budget allows no more)
 #ifndef TGL_KV_PRE_ASTAGES
-#define TGL_KV_PRE_ASTAGES 7
+#define TGL_KV_PRE_ASTAGES 4
 #endif
 #ifndef TGL_KV_PRE_WSTAGES
-#define TGL_KV_PRE_WSTAGES 3
+#define TGL_KV_PRE_WSTAGES 5
 #endif
 constexpr int kPAStages = TGL_KV_PRE_ASTAGES;         // A stages (hi | lo, 16 KB each)
 constexpr int kPAStage = kBM * kTC * 4;                // 16 KB
@@ -2535,9 +2538,10 @@ constexpr int kPW = TGL_KV_PRE_WSTAGES;
 // weight chunks kept across a tile boundary (the K order alternates per tile).  Kept
 // chunks pin weight stages at the boundary, so the next loads queue behind them.
 #ifndef TGL_KV_PRE_REUSE
-#define TGL_KV_PRE_REUSE 2
+#define TGL_KV_PRE_REUSE 4
 #endif
 constexpr int kPreReuse = TGL_KV_PRE_REUSE;
+static_assert(kPreReuse < kPW, "kept weight chunks must leave a weight stage to stream into");
 constexpr int kPLoad0 = 12, kPLoadWarps = 4;
 constexpr int kPTime0 = 16, kPTimeWarps = 4;
 constexpr int kPThreads = (kPTime0 + kPTimeWarps) * 32;   // 640
@@ -2613,20 +2617,32 @@ __global__ void pack_kv_pre_kernel(const float* Wk, const float* Wv, int dm, int
 #define PRE_FREE_SLEEP(bar, u, ns) wait_free_sleep(bar, u, ns)
 #endif
 
+// ring depths as template parameters: <4, 5, 4> (the default) keeps 4 weight chunks across
+// a tile boundary; <7, 3, 2> (a deeper A ring) serves k > 16 (LASTFM: one destination per
+// 32-row bin, so a tile holds few rows and its gathers need more stages in flight)
+template <int AS, int WS>
+constexpr int pre_smem_bytes() {
+  return 1024 + AS * kPAStage + WS * kTWStage + kBEpi * 32 * kSPW * 4;
+}
+template <int AS, int WS>
 struct PBars {
-  uint64_t afull[kPAStages], aempty[kPAStages];
-  uint64_t wfull[kPW], wempty[kPW];
+  uint64_t afull[AS], aempty[AS];
+  uint64_t wfull[WS], wempty[WS];
   uint64_t dfull[kSDSlots], dempty[kSDSlots];
   uint64_t tfull[2], tempty[2];
   uint64_t zfull[2];    // node projections: the accumulator holds zkv[row] (loaders)
 };
 
+template <int AS, int WS, int RU>
 __global__ void __launch_bounds__(kPThreads, 1)
     kv_pre_kernel(const Args a, const PrePlan plan, const uint8_t* __restrict__ wkv,
                   const int bdst) {
+  constexpr int kPAStages = AS, kPW = WS, kPreReuse = RU;
+  constexpr int kPPipeBytes = AS * kPAStage + WS * kTWStage;
+  static_assert(RU < WS, "kept weight chunks must leave a weight stage to stream into");
   extern __shared__ uint8_t smem_raw[];
   uint8_t* pipe = align1024(smem_raw);
-  __shared__ PBars B;
+  __shared__ PBars<AS, WS> B;
   __shared__ uint32_t s_tmem;
   __shared__ TDesc bd[kSDSlots];
   __shared__ __align__(16) float s_omega[256];
@@ -2642,6 +2658,9 @@ __global__ void __launch_bounds__(kPThreads, 1)
   const bool split = a.split != 0;
   const bool np = a.zkv != nullptr;   // TGL_NODE_PROJ: h_src columns come from zkv rows
   const int nch = plan.n;
+  // weight chunks kept across a tile boundary: the alternating K order maps tile t+1's
+  // chunk i to tile t's stage only while no kept chunk was itself kept (nch >= 2 reuse)
+  const int reuse = nch < 4 ? 0 : (nch / 2 < kPreReuse ? nch / 2 : kPreReuse);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   // prologue independent of the predecessor grid (PDL): barriers, TMEM, constants
   if (threadIdx.x == 0) {
@@ -2771,7 +2790,7 @@ __global__ void __launch_bounds__(kPThreads, 1)
       warp_arrive(&B.dempty[ds]);
       if (!live) break;
       if (lane == 0) {
-        const int r0 = (tt > 0 && nch >= 4) ? kPreReuse : 0;
+        const int r0 = tt > 0 ? reuse : 0;
         for (int i = r0; i < nch; ++i) {
           const uint32_t k = wl + (i - r0);
           const uint32_t sw = k % kPW;
@@ -3031,7 +3050,7 @@ TGL_SMALL_UNROLL
       prof_add(a, 7, mt1 - mt0);                     // MMA: wait for an accumulator
 #endif
       tc_fence_after();
-      const int r0 = (tt > 0 && nch >= 4) ? kPreReuse : 0;
+      const int r0 = tt > 0 ? reuse : 0;
       for (int i = 0; i < nch; ++i, ++g) {
         const int c = s_order[chunk_of(tt, i, nch)];
         const int nk = (plan.k - c * kTC) > 16 ? 2 : 1;
@@ -3065,7 +3084,7 @@ TGL_SMALL_UNROLL
               }
             }
           }
-          const bool keep = (nch >= 4) && (i >= nch - kPreReuse);   // reused by the next tile
+          const bool keep = reuse > 0 && i >= nch - reuse;   // reused by the next tile
           mma_commit(&B.aempty[sa]);
           if (!keep) mma_commit(&B.wempty[kw % kPW]);
         }
@@ -4229,8 +4248,12 @@ static tgl_status set_smem_attrs(int smem_q, int smem_kv, int smem_kvb) {
       e = cudaFuncSetAttribute(kv_split_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                kSSmem);
     if (e == cudaSuccess)
-      e = cudaFuncSetAttribute(kv_pre_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               kPSmem);
+      e = cudaFuncSetAttribute(kv_pre_kernel<kPAStages, kPW, kPreReuse>,
+                               cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               pre_smem_bytes<kPAStages, kPW>());
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(kv_pre_kernel<7, 3, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               pre_smem_bytes<7, 3>());
     if (e == cudaSuccess)
       e = cudaFuncSetAttribute(kv_pre2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                kP2Smem);
@@ -4366,8 +4389,12 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
     const int bdst = 32 / max_seg;
     const int64_t ttiles = ceil_div(n_dst_max, 4 * bdst);
     const unsigned gt = (unsigned)(ttiles < kNumSMs ? (ttiles > 0 ? ttiles : 1) : kNumSMs);
-    launch_pdl(kv_pre_kernel, dim3(gt), dim3(kPThreads), kPSmem, s, a, plan, pk + PL.okvn,
-               bdst);
+    if (max_seg > 16)     // few destinations per tile: the deeper A ring
+      launch_pdl(kv_pre_kernel<7, 3, 2>, dim3(gt), dim3(kPThreads), pre_smem_bytes<7, 3>(), s, a,
+                 plan, pk + PL.okvn, bdst);
+    else
+      launch_pdl(kv_pre_kernel<kPAStages, kPW, kPreReuse>, dim3(gt), dim3(kPThreads),
+                 pre_smem_bytes<kPAStages, kPW>(), s, a, plan, pk + PL.okvn, bdst);
     TGL_TRY(launch_check("tc kv pre kernel (node proj)"));
     if (probe && probe->ev_stop)
       TGL_TRY(cuda_check(cudaEventRecord(static_cast<cudaEvent_t>(probe->ev_stop), s),
@@ -4437,8 +4464,12 @@ tgl_status tc_attn_launch(const tgl_attn_params* P, int64_t n_dst_max, const int
       launch_pdl(kv_pre2_kernel, dim3(gp), dim3(kPThreads), kP2Smem, s, a, plan, pk + PL.okvp2,
                  bdst);
     } else {
-      launch_pdl(kv_pre_kernel, dim3(gt), dim3(kPThreads), kPSmem, s, a, plan, pk + PL.okvp,
-                 bdst);
+      if (max_seg > 16)   // few destinations per tile: the deeper A ring
+        launch_pdl(kv_pre_kernel<7, 3, 2>, dim3(gt), dim3(kPThreads), pre_smem_bytes<7, 3>(), s,
+                   a, plan, pk + PL.okvp, bdst);
+      else
+        launch_pdl(kv_pre_kernel<kPAStages, kPW, kPreReuse>, dim3(gt), dim3(kPThreads),
+                   pre_smem_bytes<kPAStages, kPW>(), s, a, plan, pk + PL.okvp, bdst);
     }
     TGL_TRY(launch_check("tc kv pre kernel"));
     if (probe && probe->ev_stop)
